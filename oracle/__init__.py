@@ -1,0 +1,17 @@
+"""CPU oracle for the nested-pattern hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` / ``--impl reference``
+legs may import this package.  It shares no code with ``paper_conf_micro_leebsro14_b200`` (the CUDA
+path): no kernels, headers, helpers, tables or constants; both follow DESIGN.md.  Everything here is
+plain and slow on purpose: fp64 / exact Python integers, NumPy used only as a library primitive
+(a reduction), every function citing the PAPER.md passage it follows.
+
+Modules
+  sums    — sumRows / sumCols / Split(k) partials / weighted variants   (Fig 1 L68-70, L542-550, Fig 15)
+  select  — nest descriptors, constraints, Algorithm 1, ControlDOP, R2  (§IV)
+  kmeans  — k-means assignment (argmin of squared distances)            (BASELINE.json config 4)
+  logreg  — batched logistic-regression gradient                        (BASELINE.json config 5)
+
+Parity unpinned: the soft-constraint intrinsic weights, the tie-break key and the R2
+runtime rule are pinned only by DESIGN.md, not by printed values in the paper.
+"""

@@ -1,0 +1,390 @@
+"""Oracle: brute-force mapping selector — TEST INFRASTRUCTURE ONLY (see oracle/__init__).
+
+Follows PAPER.md §IV step by step, with the readings of DESIGN.md §2/§3 where the paper is silent:
+  nest descriptor (levels, sync, accesses)   §IV intro L396-403, L454-455; Fig 8 L683-692   (S1)
+  candidate space Dim × Size × Span          Alg 1 L748-753, L772-777                        (S2)
+  hard constraints (HL, HG, HW limits)       Table II; L642-662                      (S3)
+  soft constraints and derived weights       Table II; L664-716                               (S4)
+  best = max score, then DOP, then …         L734-741, Alg 1 L790-792                         (S5)
+  ControlDOP                                 Alg 1; L798-809                         (S6)
+  forced 1D / thread-block-thread / warp     L99-115; Fig 7; L1052-1055    (S7)
+  runtime parameter step (AUTO)              L810-817                                         (S8)
+Written as plain nested loops over the whole candidate space (no pruning, no memoisation).
+
+Parity unpinned vs the paper: W_C/W_B, the tie-break key and R2.
+"""
+from __future__ import annotations
+
+import itertools
+
+# logical dims (S2): x varies fastest
+X, Y, Z = 0, 1, 2
+# span codes (S9 / record)
+ONE, ALL, SPAN_N, SPLIT = 0, 1, 2, 3
+# kernel classes (S9)
+RX, MX, KM, LR = 0, 1, 2, 3
+
+SIZE_SET = [1 << i for i in range(11)]          # {1,2,4,...,1024}  Alg 1
+W_C, W_B = 8, 1                                  # DESIGN.md G3
+MIN_BLOCK_SIZE = 64                              # Table II SG, L563; G5
+UNKNOWN_SIZE = 1000                              # L699-700; G17
+T_BLOCK, U_MIN = 256, 8                          # DESIGN.md S8
+MAX_GRID = (1 << 31) - 1                         # DESIGN.md S3 H6
+
+PATTERNS = ("SUM_ROWS", "SUM_COLS", "KMEANS_ASSIGN", "LOGREG_GRAD",
+            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS")
+DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8}
+
+B200 = dict(sm_count=148, max_threads_per_sm=2048, max_threads_per_block=1024,
+            max_block_dim=(1024, 1024, 64), warp_size=32, max_blocks_per_sm=32,
+            regs_per_sm=65536, regs_per_block=65536, regs_per_thread=32,
+            smem_per_block=232448)
+# Tesla K20c: 13 SMs x 2048 threads
+K20C = dict(sm_count=13, max_threads_per_sm=2048, max_threads_per_block=1024,
+            max_block_dim=(1024, 1024, 64), warp_size=32, max_blocks_per_sm=16,
+            regs_per_sm=65536, regs_per_block=65536, regs_per_thread=32,
+            smem_per_block=49152)
+
+
+class NoFeasibleMapping(Exception):
+    pass
+
+
+class Unsupported(Exception):
+    pass
+
+
+def cdiv(a: int, b: int) -> int:
+    return -(-a // b)
+
+
+def pow2ceil(v: int) -> int:
+    p = 1
+    while p < v:
+        p *= 2
+    return p
+
+
+def prod(xs) -> int:
+    r = 1
+    for v in xs:
+        r *= v
+    return r
+
+
+# ------------------------------------------------------------------ S1 nest descriptor
+
+def build_nest(pattern: str, shape) -> dict:
+    """Levels (N, sync) outermost first and accesses (contig level, exec-count mask)."""
+    if pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS"):
+        R, C = shape
+        levels = [(R, False), (C, True)]            # Map rows / Reduce row (Fig 1 L70)
+        acc = [(0, (0,)), (1, (0, 1))]              # out[r], m[r,c]
+        if pattern == "SUM_WEIGHTED_ROWS":
+            acc.append((1, (0, 1)))                 # v[c]
+    elif pattern in ("SUM_COLS", "SUM_WEIGHTED_COLS"):
+        R, C = shape
+        levels = [(C, False), (R, True)]            # Map cols / Reduce column (Fig 1 L69)
+        acc = [(0, (0,)), (0, (0, 1))]              # out[c], m[r,c] (stride-1 index is c = L0)
+        if pattern == "SUM_WEIGHTED_COLS":
+            acc.append((1, (0, 1)))                 # v[r]
+    elif pattern == "KMEANS_ASSIGN":
+        N, D, K = shape
+        levels = [(N, False), (K, True), (D, True)]
+        acc = [(0, (0,)), (2, (0, 1, 2)), (2, (0, 1, 2))]   # a[i], x[i,d], c[k,d]
+    elif pattern == "LOGREG_GRAD":
+        B, Rb, C = shape
+        levels = [(B, False), (Rb, True), (C, True)]       # L2 holds Map_j and Reduce_k (HG)
+        acc = [(1, (0, 1)), (2, (0, 1, 2)), (2, (0, 1, 2)), (2, (0, 1, 2)), (2, (0, 2))]
+    else:
+        raise ValueError(pattern)
+    return {"pattern": pattern, "levels": levels, "accesses": acc}
+
+
+def _eff(n: int) -> int:
+    return UNKNOWN_SIZE if n < 0 else n
+
+
+# ------------------------------------------------------------------ S6 DOP (G7)
+
+def level_dop(n: int, b: int, span: int, factor: int) -> int:
+    n = _eff(n)
+    if span == ONE:
+        return n
+    if span == ALL:
+        return min(b, n)
+    if span == SPAN_N:
+        return cdiv(n, factor)
+    return factor * min(b, cdiv(n, factor))          # SPLIT
+
+
+def mapping_dop(nest, blocks, spans, factors) -> int:
+    return prod(level_dop(nest["levels"][l][0], blocks[l], spans[l], factors[l])
+                for l in range(len(blocks)))
+
+
+def level_blocks(n: int, b: int, span: int, factor: int, vec: int = 1) -> int:
+    """Blocks along a level (Fig 6 caption L450-452): ONE ⌈N/b⌉, Span(n) ⌈N/(b·n)⌉, ALL 1, Split ⌈N/⌈N/k⌉⌉."""
+    return cdiv(_eff(n), level_chunk(n, b, span, factor, vec))
+
+
+def level_chunk(n: int, b: int, span: int, factor: int, vec: int = 1) -> int:
+    n = _eff(n)
+    if span == ONE:
+        return b * vec
+    if span == SPAN_N:
+        return b * vec * factor
+    if span == ALL:
+        return max(n, 1)
+    return cdiv(n, factor)
+
+
+# ------------------------------------------------------------------ S3 hard constraints
+
+def acc_bytes(pattern: str, dtype: str) -> int:
+    if pattern in ("KMEANS_ASSIGN", "LOGREG_GRAD"):
+        return 8
+    return 4 if dtype == "i32" else 8
+
+
+def staging_bytes(nest) -> int:
+    if nest["pattern"] == "KMEANS_ASSIGN":
+        (N, _), (K, _), (D, _) = nest["levels"]
+        return 4 * _eff(K) * _eff(D) + 4 * _eff(K)
+    return 0
+
+
+def smem_model(nest, dtype, blocks) -> int:
+    par_reduce = any(sync and b > 1 for (n, sync), b in zip(nest["levels"], blocks))
+    return (prod(blocks) * acc_bytes(nest["pattern"], dtype) if par_reduce else 0) + staging_bytes(nest)
+
+
+def hard_ok(nest, dtype, lim, dims, blocks, spans) -> bool:
+    for (n, sync), s in zip(nest["levels"], spans):
+        if sync and s != ALL:                               # H1: HL (Table II), HG (L651-656)
+            return False
+    tb = prod(blocks)
+    if tb > lim["max_threads_per_block"]:                    # H2 (L661-662)
+        return False
+    for d, b in zip(dims, blocks):
+        if b > lim["max_block_dim"][d]:                     # H3 (L661-662)
+            return False
+    if tb * lim["regs_per_thread"] > lim["regs_per_block"]:  # H4 (north_star: registers)
+        return False
+    if smem_model(nest, dtype, blocks) > lim["smem_per_block"]:  # H5 (north_star: shared memory)
+        return False
+    grid = prod(level_blocks(n, b, s, 1) for (n, _), b, s in zip(nest["levels"], blocks, spans))
+    if grid > MAX_GRID:                                      # H6
+        return False
+    return True
+
+
+# ------------------------------------------------------------------ S4 soft constraints
+
+def score(nest, lim, dims, blocks) -> int:
+    total = 0
+    for contig, mask in nest["accesses"]:
+        if contig < 0:
+            continue
+        weight = W_C * prod(_eff(nest["levels"][l][0]) for l in mask)
+        # SL: sequential accesses -> Dim(x) and block size multiple of WARP_SIZE (Table II)
+        if dims[contig] == X and blocks[contig] % lim["warp_size"] == 0:
+            total += weight
+    # SG: threads in block >= MIN_BLOCK_SIZE (Table II), weighted by the whole nest's execution count
+    if prod(blocks) >= MIN_BLOCK_SIZE:
+        total += W_B * prod(_eff(n) for n, _ in nest["levels"])
+    return total
+
+
+# ------------------------------------------------------------------ S2 + S5 search (Algorithm 1)
+
+def search(nest, dtype, lim, restrict_1d=False):
+    """Brute force over CandSet (Alg 1) with the S5 key; returns (dims, blocks, spans, score)."""
+    L = len(nest["levels"])
+    best = None
+    best_key = None
+    for dims in itertools.permutations(range(L)):             # lexicographic
+        for blocks in itertools.product(SIZE_SET, repeat=L):
+            if restrict_1d and any(b != 1 for b in blocks[1:]):
+                continue
+            for spans in itertools.product((ONE, ALL), repeat=L):
+                if restrict_1d and any(s != ALL for s in spans[1:]):
+                    continue
+                if not hard_ok(nest, dtype, lim, dims, blocks, spans):
+                    continue
+                sc = score(nest, lim, dims, blocks)
+                dop = mapping_dop(nest, blocks, spans, [1] * L)
+                key = (sc, dop, -prod(blocks))
+                if best_key is None or key > best_key:           # strict: first (lex-smallest) wins ties
+                    best_key, best = key, (tuple(dims), tuple(blocks), tuple(spans), sc)
+    if best is None:
+        raise NoFeasibleMapping(nest["pattern"])
+    return best
+
+
+# ------------------------------------------------------------------ S6 ControlDOP
+
+def control_dop(nest, lim, blocks, spans):
+    L = len(blocks)
+    spans = list(spans)
+    factors = [1] * L
+    min_dop = lim["sm_count"] * lim["max_threads_per_sm"]      # L799-801
+    max_dop = 100 * min_dop                                    # L801-803
+    dop = mapping_dop(nest, blocks, spans, factors)
+    if dop < min_dop:                                          # Alg 1
+        best_l, best_nb = -1, 1
+        for l in range(L):
+            n, sync = nest["levels"][l]
+            nb = cdiv(_eff(n), blocks[l])
+            if sync and spans[l] == ALL and nb >= 2 and nb > best_nb:
+                best_l, best_nb = l, nb
+        if best_l >= 0:
+            k = min(cdiv(min_dop, dop), best_nb)
+            if k >= 2:
+                spans[best_l], factors[best_l] = SPLIT, k
+    elif dop > max_dop:                                        # Alg 1
+        for l in range(L):
+            if spans[l] == ONE:
+                n = min(cdiv(dop, max_dop), cdiv(_eff(nest["levels"][l][0]), blocks[l]))
+                if n >= 2:
+                    spans[l], factors[l] = SPAN_N, n
+                break
+    return spans, factors
+
+
+def min_max_dop(lim):
+    m = lim["sm_count"] * lim["max_threads_per_sm"]
+    return m, 100 * m
+
+
+# ------------------------------------------------------------------ S7 forced strategies
+
+def forced(nest, dtype, lim, strategy):
+    if len(nest["levels"]) != 2:
+        raise Unsupported(strategy)
+    if strategy == "1D":
+        dims, blocks, spans, _ = search(nest, dtype, lim, restrict_1d=True)
+    elif strategy == "TB_T":                                   # Fig 7a
+        dims, blocks, spans = (Y, X), (1, min(1024, pow2ceil(_eff(nest["levels"][1][0])))), (ONE, ALL)
+    elif strategy == "WARP":                                   # Fig 7b, fn 4 L621-622
+        dims, blocks, spans = (Y, X), (16, 32), (ONE, ALL)
+    else:
+        raise ValueError(strategy)
+    if not hard_ok(nest, dtype, lim, dims, blocks, spans):
+        raise NoFeasibleMapping(strategy)
+    return dims, blocks, spans
+
+
+# ------------------------------------------------------------------ S8 runtime step (R2)
+
+def slots(lim, threads_per_block: int) -> int:
+    per_sm = min(lim["max_blocks_per_sm"], lim["max_threads_per_sm"] // threads_per_block,
+                 lim["regs_per_sm"] // (threads_per_block * lim["regs_per_thread"]))
+    return lim["sm_count"] * max(1, per_sm)
+
+
+def r2_sums(nest, dtype, lim, dims):
+    """DESIGN.md S8 for the 2-level sums: returns (blocks, spans, factors, vec, chunks)."""
+    pattern = nest["pattern"]
+    O, I = nest["levels"][0][0], nest["levels"][1][0]
+    C = I if pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS") else O
+    contig_level = 1 if pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS") else 0
+    x_level = 0 if dims[0] == X else 1
+    v0 = 16 // DTYPE_SIZE[dtype]
+    vec = v0 if (x_level == contig_level and C % v0 == 0) else 1
+    S = slots(lim, T_BLOCK)
+    if x_level == 1:                                           # class RX
+        bx = min(32, pow2ceil(cdiv(I, vec)))
+        by = T_BLOCK // bx
+        g = cdiv(O, by)
+        if g >= S:
+            k, n = 1, cdiv(g, S)
+        else:
+            n = 1
+            k = max(1, min(S // g, cdiv(I, bx * vec * U_MIN)))
+        chunk_i = vec * cdiv(cdiv(I, k), vec)
+        k = cdiv(I, chunk_i)
+        blocks = (by, bx)
+        spans = (ONE if n == 1 else SPAN_N, ALL if k == 1 else SPLIT)
+        factors = (n, k)
+        chunks = (by * n, chunk_i if k > 1 else I)
+    else:                                                      # class MX
+        bx = min(32, pow2ceil(cdiv(O, vec)))
+        by = T_BLOCK // bx
+        g = cdiv(O, bx * vec)
+        if g >= S:
+            k, n = 1, cdiv(g, S)
+        else:
+            n = 1
+            k = max(1, min(S // g, cdiv(I, by * U_MIN)))
+        chunk_i = cdiv(I, k)
+        k = cdiv(I, chunk_i)
+        blocks = (bx, by)
+        spans = (ONE if n == 1 else SPAN_N, ALL if k == 1 else SPLIT)
+        factors = (n, k)
+        chunks = (bx * vec * n, chunk_i if k > 1 else I)
+    return blocks, spans, factors, vec, chunks
+
+
+# ------------------------------------------------------------------ S9 record
+
+def kernel_class(pattern, dims):
+    if pattern == "KMEANS_ASSIGN":
+        return KM
+    if pattern == "LOGREG_GRAD":
+        return LR
+    return RX if dims[1] == X else MX
+
+
+def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chunks=None):
+    L = len(blocks)
+    levels = []
+    for l in range(L):
+        n = nest["levels"][l][0]
+        v = vec if dims[l] == X else 1
+        ch = chunks[l] if chunks is not None else level_chunk(n, blocks[l], spans[l], factors[l], v)
+        levels.append(dict(dim=dims[l], block=blocks[l], span=spans[l],
+                           factor=(factors[l] if spans[l] in (SPAN_N, SPLIT) else 1),
+                           chunk=ch, grid=cdiv(_eff(n), ch)))
+    grid = prod(lv["grid"] for lv in levels)
+    block3 = [1, 1, 1]
+    for l in range(L):
+        block3[dims[l]] = blocks[l]
+    rec = dict(nlevels=L, kernel_class=kernel_class(nest["pattern"], dims), vec=vec, levels=levels,
+               score=score_, dop=mapping_dop(nest, blocks, spans, factors),
+               threads=grid * prod(blocks), grid=grid, block=block3,
+               smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0)
+    if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
+        if levels[1]["grid"] >= 2:
+            O = _eff(nest["levels"][0][0])
+            part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
+            tick = levels[0]["grid"] * 4
+            rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
+    return rec
+
+
+# ------------------------------------------------------------------ entry point
+
+def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -> dict:
+    """The mapping record for (pattern, shape, dtype, limits, strategy) per DESIGN.md §3."""
+    nest = build_nest(pattern, shape)
+    L = len(nest["levels"])
+    if any(n == 0 or n < -1 for n, _ in nest["levels"]):
+        raise ValueError("sizes must be >= 1 (or -1 = unknown)")
+    unknown = any(n < 0 for n, _ in nest["levels"])
+    if strategy in ("1D", "TB_T", "WARP"):
+        dims, blocks, spans = forced(nest, dtype, lim, strategy)
+        return make_record(nest, dtype, lim, dims, blocks, spans, [1] * L, 1,
+                           score(nest, lim, dims, blocks))
+    dims, blocks, spans, sc = search(nest, dtype, lim)
+    spans, factors = control_dop(nest, lim, blocks, spans)
+    if strategy == "LITERAL":
+        return make_record(nest, dtype, lim, dims, blocks, spans, factors, 1, sc)
+    if strategy != "AUTO":
+        raise ValueError(strategy)
+    if unknown:
+        raise Unsupported("AUTO needs known sizes")
+    if L != 2:
+        raise Unsupported("R2 for 3-level nests")
+    b2, s2, f2, vec, chunks = r2_sums(nest, dtype, lim, dims)
+    return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks)

@@ -1,0 +1,120 @@
+"""Pins for oracle/kmeans.py and oracle/logreg.py (closed forms, special cases, library routines)."""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import kmeans, logreg
+from synth import gen
+
+
+# ------------------------------------------------------------------ k-means assignment
+
+def test_points_equal_to_centroids():
+    _, c = gen.kmeans_inputs(4, 16, 8)
+    c = c.numpy()
+    perm = np.array([3, 1, 7, 0, 0, 5, 2, 6, 4])
+    x = c[perm]
+    assert kmeans.assign(x, c).tolist() == perm.tolist()
+    assert kmeans.assign_literal(x, c) == perm.tolist()
+
+
+def test_single_centroid():
+    x, c = gen.kmeans_inputs(50, 5, 1)
+    assert kmeans.assign(x.numpy(), c.numpy()).tolist() == [0] * 50
+
+
+def test_one_dimension_nearest():
+    c = np.array([[-3.0], [0.5], [2.0], [7.0]], dtype=np.float32)
+    x = np.array([[-10.0], [-1.25], [-1.0], [1.0], [1.25], [1.5], [4.5], [4.75], [100.0]], dtype=np.float32)
+    # midpoints -1.25, 1.25, 4.5 are ties -> lowest index
+    assert kmeans.assign(x, c).tolist() == [0, 0, 1, 1, 1, 2, 2, 3, 3]
+    assert kmeans.assign_literal(x, c) == [0, 0, 1, 1, 1, 2, 2, 3, 3]
+
+
+def test_tie_goes_to_lowest_index():
+    c = np.array([[1, 0], [0, 1], [-1, 0], [0, -1]], dtype=np.float32)
+    x = np.zeros((1, 2), dtype=np.float32)
+    assert kmeans.assign(x, c).tolist() == [0]
+    x2 = np.array([[0.0, -1.0]], dtype=np.float32)
+    c2 = np.array([[5, 5], [0, -1], [0, -1]], dtype=np.float32)
+    assert kmeans.assign_literal(x2, c2) == [1]
+
+
+def test_integer_data_exact_and_library():
+    x, c = gen.kmeans_inputs(300, 12, 7, integer=True)
+    x, c = x.numpy(), c.numpy()
+    a = kmeans.assign(x, c)
+    assert a.tolist() == kmeans.assign_literal(x, c)
+    d = torch.cdist(torch.from_numpy(x).double(), torch.from_numpy(c).double()) ** 2
+    # squared integer distances are exact: recompute with exact ints and compare argmin with ties
+    xi, ci = x.astype(np.int64), c.astype(np.int64)
+    exact = ((xi[:, None, :] - ci[None, :, :]) ** 2).sum(-1)
+    assert a.tolist() == np.argmin(exact, axis=1).tolist()
+    assert np.allclose(d.numpy(), exact, rtol=1e-12)
+
+
+def test_random_data_vs_cdist():
+    x, c = gen.kmeans_inputs(2000, 64, 32)
+    x, c = x.numpy(), c.numpy()
+    a = kmeans.assign(x, c)
+    d = torch.cdist(torch.from_numpy(x).double(), torch.from_numpy(c).double())
+    assert a.tolist() == torch.argmin(d, dim=1).tolist()
+    assert kmeans.assign_literal(x[:40], c) == a[:40].tolist()
+
+
+# ------------------------------------------------------------------ logistic-regression gradient
+
+def test_w_zero_closed_form():
+    B, Rb, C = 3, 20, 9
+    x, y, _ = gen.logreg_inputs(B, Rb, C)
+    x, y = x.numpy(), y.numpy()
+    w = np.zeros(C, dtype=np.float32)
+    g = logreg.grad(x, y, w, B)
+    ref = (x.astype(np.float64) * (0.5 - y.astype(np.float64))[:, None]).reshape(B, Rb, C).sum(1)
+    assert np.allclose(g, ref, rtol=1e-14, atol=0)
+
+
+def test_all_ones_symmetry():
+    B, Rb, C = 2, 10, 7
+    x = np.ones((B * Rb, C), dtype=np.float32)
+    _, y, w = gen.logreg_inputs(B, Rb, C)
+    g = logreg.grad(x, y.numpy(), w.numpy(), B)
+    for b in range(B):
+        assert np.allclose(g[b], g[b][0], rtol=1e-15)
+    # sigma(sum w) - y summed over rows
+    s = 1.0 / (1.0 + math.exp(-float(w.double().sum())))
+    assert math.isclose(g[0][0], sum(s - float(v) for v in y[:Rb]), rel_tol=1e-12)
+
+
+@pytest.mark.parametrize("B", [1, 3])
+def test_autograd_and_literal(B):
+    Rb, C = 8, 11
+    x, y, w = gen.logreg_inputs(B, Rb, C, seed=12)
+    g = logreg.grad(x.numpy(), y.numpy(), w.numpy(), B)
+    assert np.allclose(g, np.array(logreg.grad_literal(x.numpy(), y.numpy(), w.numpy(), B)), rtol=1e-13)
+    for b in range(B):
+        wt = w.double().clone().requires_grad_(True)
+        xb, yb = x[b * Rb:(b + 1) * Rb].double(), y[b * Rb:(b + 1) * Rb].double()
+        z = xb @ wt
+        loss = (torch.nn.functional.softplus(z) - yb * z).sum()
+        loss.backward()
+        assert np.allclose(g[b], wt.grad.numpy(), rtol=1e-12, atol=1e-14)
+
+
+def test_finite_differences():
+    Rb, C = 6, 5
+    x, y, w = gen.logreg_inputs(1, Rb, C, seed=13)
+    x64, y64, w64 = x.double().numpy(), y.double().numpy(), w.double().numpy()
+
+    def loss(wv):
+        z = x64 @ wv
+        return float(np.sum(np.logaddexp(0.0, z) - y64 * z))
+    g = logreg.grad(x.numpy(), y.numpy(), w.numpy(), 1)[0]
+    h = 1e-6
+    for j in range(C):
+        e = np.zeros(C)
+        e[j] = h
+        fd = (loss(w64 + e) - loss(w64 - e)) / (2 * h)
+        assert math.isclose(fd, g[j], rel_tol=1e-6, abs_tol=1e-9)

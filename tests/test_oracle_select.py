@@ -1,0 +1,214 @@
+"""Pins for oracle/select.py: values printed in PAPER.md (tests/golden/paper_pins.json), the paper's
+qualitative claims, and the DESIGN.md spec (Appendix-A style vectors, marked 'spec')."""
+import itertools
+import json
+import os
+
+import pytest
+
+from oracle import select as S
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "paper_pins.json")))
+PAPER_SHAPES = [(65536, 1024), (8192, 8192), (1024, 65536)]
+
+
+def _rec(pattern, shape, strategy="LITERAL", lim=S.B200, dtype="f32"):
+    return S.select(pattern, shape, dtype, lim, strategy)
+
+
+def _lv(r):
+    return [(l["dim"], l["block"], l["span"], l["factor"]) for l in r["levels"]]
+
+
+# ------------------------------------------------------------ Fig 6 (L450-452, L541, L549-550)
+
+@pytest.mark.parametrize("M,N", [(192, 32), (640, 96), (1024, 4096)])
+def test_fig6_blocks_and_dop(M, N):
+    bx, by = GOLD["fig6"]["block"]["x"], GOLD["fig6"]["block"]["y"]
+    # (a) Span(1) on both: M/64 x N/16 blocks, DOP M x N
+    a_blocks = S.level_blocks(M, bx, S.ONE, 1) * S.level_blocks(N, by, S.ONE, 1)
+    assert a_blocks == (M // 64) * (N // 16)
+    assert S.level_dop(M, bx, S.ONE, 1) * S.level_dop(N, by, S.ONE, 1) == M * N
+    # (b) Span(all) on x, Span(2) on y: N/32 blocks, DOP 64 x N/2 = 32N
+    b_blocks = S.level_blocks(M, bx, S.ALL, 1) * S.level_blocks(N, by, S.SPAN_N, 2)
+    assert b_blocks == N // 32
+    assert S.level_dop(M, bx, S.ALL, 1) * S.level_dop(N, by, S.SPAN_N, 2) == 32 * N
+    # (c) Split(3) on x, Span(2) on y: 3 x N/32 blocks, DOP x3 = 96N
+    c_blocks = S.level_blocks(M, bx, S.SPLIT, 3) * S.level_blocks(N, by, S.SPAN_N, 2)
+    assert c_blocks == 3 * N // 32
+    assert S.level_dop(M, bx, S.SPLIT, 3) * S.level_dop(N, by, S.SPAN_N, 2) == 96 * N
+
+
+# ------------------------------------------------------------ Fig 7 (L573-583)
+
+@pytest.mark.parametrize("I,J", [(100, 50), (1024, 1024), (64, 4000), (65536, 1024), (8, 70000)])
+def test_fig7_prior_mappings(I, J):
+    tbt = _rec("SUM_ROWS", (I, J), "TB_T")
+    assert [l["dim"] for l in tbt["levels"]] == [S.Y, S.X]
+    assert tbt["levels"][0]["block"] == 1 and tbt["levels"][0]["span"] == S.ONE
+    assert tbt["levels"][1]["span"] == S.ALL
+    assert tbt["dop"] == I * min(J, GOLD["fig7"]["max_block_size"])
+    warp = _rec("SUM_ROWS", (I, J), "WARP")
+    assert [(l["dim"], l["block"]) for l in warp["levels"]] == [(S.Y, 16), (S.X, 32)]
+    assert warp["dop"] == I * min(J, GOLD["fig7"]["warp_size"])
+
+
+# ------------------------------------------------------------ ControlDOP constants (L799-803)
+
+def test_k20c_min_max_dop():
+    g = GOLD["controldop_k20c"]
+    assert S.K20C["sm_count"] == g["sm_count"] and S.K20C["max_threads_per_sm"] == g["max_threads_per_sm"]
+    assert S.min_max_dop(S.K20C) == (g["min_dop"], g["max_dop"])
+    assert S.min_max_dop(S.B200) == (148 * 2048, 100 * 148 * 2048)
+
+
+def test_search_space_base():
+    g = GOLD["search_space"]
+    assert S.SIZE_SET == g["sizeset"]
+    assert len(g["dimset"]) * len(S.SIZE_SET) * len((S.ONE, S.ALL)) == g["base"] < 100
+
+
+# ------------------------------------------------------------ hard constraints (Table II)
+
+def test_hard_local_reduce_needs_span_all():
+    nest = S.build_nest("SUM_ROWS", (100, 100))
+    assert not S.hard_ok(nest, "f32", S.B200, (S.Y, S.X), (1, 64), (S.ONE, S.ONE))
+    assert S.hard_ok(nest, "f32", S.B200, (S.Y, S.X), (1, 64), (S.ONE, S.ALL))
+
+
+def test_hard_global_map_and_reduce_same_level():
+    # LOGREG L2 holds a Map and a Reduce (dot): the level takes the conservative Span(all) (L655-656)
+    r = _rec("LOGREG_GRAD", (16, 64, 256))
+    assert r["levels"][2]["span"] == S.ALL
+
+
+def test_fig9_mapping_is_infeasible():
+    g = GOLD["fig9"]
+    nest = S.build_nest("SUM_ROWS", (8192, 8192))
+    assert 64 * 32 == g["threads"]
+    assert not S.hard_ok(nest, "f32", S.B200, (S.Y, S.X), (64, 32), (S.ONE, S.ALL))
+    assert S.hard_ok(nest, "f32", S.B200, (S.Y, S.X), (32, 32), (S.ONE, S.ALL))   # fails only by size
+
+
+def test_hw_dim_limits():
+    nest = S.build_nest("KMEANS_ASSIGN", (1000, 64, 32))
+    # z is limited to 64 threads (max_block_dim)
+    assert not S.hard_ok(nest, "f32", S.B200, (S.Y, S.Z, S.X), (1, 128, 8), (S.ONE, S.ALL, S.ALL))
+    assert S.hard_ok(nest, "f32", S.B200, (S.Y, S.Z, S.X), (1, 16, 64), (S.ONE, S.ALL, S.ALL))
+
+
+def test_register_and_smem_constraints_bind_on_tiny_device():
+    tiny = dict(S.B200, regs_per_thread=128, smem_per_block=2048)
+    nest = S.build_nest("SUM_ROWS", (1000, 1000))
+    assert not S.hard_ok(nest, "f32", tiny, (S.Y, S.X), (1, 1024), (S.ONE, S.ALL))   # 128*1024 regs > 64K
+    assert not S.hard_ok(nest, "f32", tiny, (S.Y, S.X), (1, 512), (S.ONE, S.ALL))    # 512*8 B smem > 2048
+    assert S.hard_ok(nest, "f32", tiny, (S.Y, S.X), (1, 256), (S.ONE, S.ALL))
+    r = _rec("SUM_ROWS", (1000, 1000), lim=tiny)
+    assert r["levels"][1]["block"] == 256
+
+
+# ------------------------------------------------------------ soft constraints / weights (Fig 8)
+
+def test_fig8_inner_access_weight_dominates():
+    I, J = 300, 500
+    nest = S.build_nest("SUM_ROWS", (I, J))     # array1D(i) at L0, array2D(i,j) at L1 — Fig 8
+    outer_x = S.score(nest, S.B200, (S.X, S.Y), (32, 32))
+    inner_x = S.score(nest, S.B200, (S.Y, S.X), (32, 32))
+    sg = I * J
+    assert outer_x == S.W_C * I + sg            # α·I
+    assert inner_x == S.W_C * I * J + sg        # α·I·J
+    assert inner_x > outer_x
+
+
+@pytest.mark.parametrize("shape", PAPER_SHAPES + [(1024, 1024), (100, 3000), (3000, 100)])
+def test_coalescing_dims(shape):
+    # sumCols assigns the outer (column) pattern to x; sumRows the inner one (L596-600, L1036-1044)
+    assert _rec("SUM_COLS", shape)["levels"][0]["dim"] == S.X
+    assert _rec("SUM_ROWS", shape)["levels"][1]["dim"] == S.X
+    for strat in ("LITERAL", "AUTO"):
+        r = _rec("SUM_COLS", shape, strat)
+        assert r["levels"][0]["block"] * r["vec"] % 32 == 0 or shape[1] < 32
+
+
+def test_split_only_on_sync_span_all_levels():
+    for pat in ("SUM_ROWS", "SUM_COLS"):
+        for R in (1, 7, 100, 1024, 4096, 65536, 1 << 20):
+            for C in (1, 3, 64, 1000, 4096, 65536):
+                if R * C > 1 << 32:
+                    continue
+                for lim in (S.B200, S.K20C):
+                    nest = S.build_nest(pat, (R, C))
+                    r = _rec(pat, (R, C), lim=lim)
+                    for l, lv in enumerate(r["levels"]):
+                        if lv["span"] == S.SPLIT:
+                            assert nest["levels"][l][1]            # a Reduce level
+                        if lv["span"] == S.SPAN_N:
+                            assert not nest["levels"][l][1]
+
+
+def test_search_is_the_argmax():
+    # independent re-enumeration on small nests: no feasible candidate beats the chosen key
+    for pat, shape in [("SUM_ROWS", (40, 70)), ("SUM_COLS", (70, 40)), ("SUM_COLS", (5, 3))]:
+        nest = S.build_nest(pat, shape)
+        dims, blocks, spans, sc = S.search(nest, "f32", S.B200)
+        best = (sc, S.mapping_dop(nest, blocks, spans, [1, 1]), -blocks[0] * blocks[1])
+        for d in itertools.permutations(range(2)):
+            for b in itertools.product(S.SIZE_SET, repeat=2):
+                for s in itertools.product((S.ONE, S.ALL), repeat=2):
+                    if S.hard_ok(nest, "f32", S.B200, d, b, s):
+                        key = (S.score(nest, S.B200, d, b), S.mapping_dop(nest, b, s, [1, 1]), -b[0] * b[1])
+                        assert key <= best
+
+
+def test_no_feasible_mapping():
+    broken = dict(S.B200, max_threads_per_block=0)
+    with pytest.raises(S.NoFeasibleMapping):
+        _rec("SUM_ROWS", (10, 10), lim=broken)
+
+
+# ------------------------------------------------------------ spec vectors (not paper values)
+
+def test_spec_literal_vectors_b200():
+    assert _lv(_rec("SUM_ROWS", (1024, 1024))) == [(S.Y, 1, S.ONE, 1), (S.X, 1024, S.ALL, 1)]
+    assert _lv(_rec("SUM_ROWS", (65536, 1024))) == [(S.Y, 1, S.SPAN_N, 3), (S.X, 1024, S.ALL, 1)]
+    assert _lv(_rec("SUM_ROWS", (1 << 20, 4096))) == [(S.Y, 1, S.SPAN_N, 36), (S.X, 1024, S.ALL, 1)]
+    assert _lv(_rec("SUM_COLS", (65536, 1024))) == [(S.X, 32, S.ONE, 1), (S.Y, 32, S.SPLIT, 10)]
+    assert _rec("SUM_COLS", (65536, 1024))["grid"] == 320
+    assert _lv(_rec("SUM_COLS", (8192, 8192))) == [(S.X, 32, S.ONE, 1), (S.Y, 32, S.SPLIT, 2)]
+    assert _lv(_rec("SUM_COLS", (1024, 65536))) == [(S.X, 32, S.ONE, 1), (S.Y, 32, S.ALL, 1)]
+    assert _lv(_rec("SUM_COLS", (1 << 20, 4096))) == [(S.X, 32, S.ONE, 1), (S.Y, 32, S.SPLIT, 3)]
+    assert _lv(_rec("KMEANS_ASSIGN", (1 << 22, 64, 32))) == [
+        (S.Y, 1, S.SPAN_N, 142), (S.Z, 16, S.ALL, 1), (S.X, 64, S.ALL, 1)]
+    assert _lv(_rec("LOGREG_GRAD", (4096, 4096, 256))) == [
+        (S.Y, 1, S.ONE, 1), (S.Z, 4, S.ALL, 1), (S.X, 256, S.ALL, 1)]
+
+
+def test_spec_literal_vectors_k20c():
+    assert _lv(_rec("SUM_ROWS", (65536, 1024), lim=S.K20C))[0] == (S.Y, 1, S.SPAN_N, 26)
+    assert _lv(_rec("SUM_ROWS", (8192, 8192), lim=S.K20C))[0] == (S.Y, 1, S.SPAN_N, 4)
+    assert _lv(_rec("SUM_COLS", (65536, 1024), lim=S.K20C))[1] == (S.Y, 32, S.ALL, 1)
+
+
+def test_spec_forced_1d():
+    r = _rec("SUM_COLS", (65536, 1024), "1D")
+    assert _lv(r) == [(S.X, 64, S.ONE, 1), (S.Y, 1, S.ALL, 1)] and r["dop"] == 1024 and r["grid"] == 16
+    r = _rec("SUM_ROWS", (1024, 65536), "1D")
+    assert _lv(r) == [(S.X, 64, S.ONE, 1), (S.Y, 1, S.ALL, 1)] and r["dop"] == 1024
+
+
+# ------------------------------------------------------------ R2 invariants (S8)
+
+@pytest.mark.parametrize("pat", ["SUM_ROWS", "SUM_COLS"])
+@pytest.mark.parametrize("shape", PAPER_SHAPES + [(1, 1), (3, 5), (1000, 999), (1 << 20, 4096), (7, 100000)])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+def test_r2_invariants(pat, shape, dtype):
+    r = _rec(pat, shape, "AUTO", dtype=dtype)
+    nest = S.build_nest(pat, shape)
+    S_slots = S.slots(S.B200, S.T_BLOCK)
+    assert r["grid"] <= S_slots and r["block"][0] * r["block"][1] == S.T_BLOCK
+    for l, lv in enumerate(r["levels"]):
+        n = nest["levels"][l][0]
+        assert lv["grid"] == -(-n // lv["chunk"])
+        if lv["dim"] == S.X and lv["span"] == S.SPLIT:
+            assert lv["chunk"] % r["vec"] == 0
+    assert r["vec"] in (1, 16 // S.DTYPE_SIZE[dtype])
