@@ -1,0 +1,397 @@
+#!/usr/bin/env python
+"""Benchmark of the nested-pattern hot path (BASELINE.json metric: achieved HBM GB/s for sumRows /
+sumCols per shape, 1/2/4/8 GPU).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload paper|sumcols_1m4k]
+                    [--strategy AUTO|LITERAL|1D|TB_T|WARP] [--impl reference] [--no-mappings]
+
+A step (workload `paper`, the default) = sumRows and sumCols, AUTO mapping, at the paper's three shapes
+[64K,1K], [8K,8K], [1K,64K] fp32 (Fig 3; BASELINE.json configs[1]) — six launches on six
+distinct 256 MiB buffers, so every launch streams from HBM (inputs > L2, no flush needed).
+At N > 1 each rank owns a row shard of [N*R, C] matrices (weak scaling): sumRows shards need no
+exchange, sumCols partial column sums are all-reduced over NCCL (the one real exchange step).
+
+Output: one JSON line on rank 0 (see DESIGN.md §9 for every key).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PAPER_SHAPES = [(65536, 1024), (8192, 8192), (1024, 65536)]
+METRIC = "achieved HBM GB/s (% of B200 peak) for sumRows/sumCols per shape, 1/2/4/8 GPU"
+
+
+def _fmt_shape(s):
+    def k(v):
+        return f"{v // 1048576}M" if v % 1048576 == 0 else (f"{v // 1024}K" if v % 1024 == 0 else str(v))
+    return f"[{k(s[0])},{k(s[1])}]"
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs: torch copy, read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    return json.load(open(p)) if os.path.exists(p) else {}
+
+
+# ------------------------------------------------------------------------- clocks (NVML, sampled live)
+
+class ClockSampler:
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index: int, period_s: float = 0.002):
+        self.period = period_s
+        self.samples, self.reasons = [], 0
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # noqa: BLE001
+            self.err = str(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                self.reasons |= int(nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
+        names = [n for bit, n in self.REASONS.items() if self.reasons & bit and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------- distributed plumbing
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ------------------------------------------------------------------------- workloads
+
+class Item:
+    """One launch of the step: a plan, its device inputs/outputs, and its algorithmic bytes."""
+
+    def __init__(self, name, plan, ins, out, algo_bytes):
+        self.name, self.plan, self.ins, self.out, self.bytes = name, plan, ins, out, algo_bytes
+
+    def run(self, stream):
+        self.plan.execute(self.ins, self.out, stream=stream)
+
+
+def build_paper(npp, gen, torch, rank, world, strategy, device):
+    items, reduce_views = [], []
+    col_total = sum(C for _, C in PAPER_SHAPES)
+    col_buf = torch.empty(col_total, dtype=torch.float32, device=device)
+    off = 0
+    for si, (R, C) in enumerate(PAPER_SHAPES):
+        for pattern in ("SUM_ROWS", "SUM_COLS"):
+            seed = 300 + 2 * si + (pattern == "SUM_COLS")
+            # rank r owns rows [r*R, (r+1)*R) of a [world*R, C] matrix (counter-based inputs)
+            m = gen.uniform_f32(seed, (R, C), offset=rank * R * C, device=device)
+            plan = npp.Plan(pattern, (R, C), "f32", strategy, device=device)
+            if pattern == "SUM_COLS":
+                out = col_buf[off:off + C]
+                off += C
+            else:
+                out = plan.new_out()
+            nbytes = R * C * 4 + out.numel() * 4
+            items.append(Item(f"{pattern.lower()}{_fmt_shape((R, C))}", plan, [m], out, nbytes))
+    if world > 1:
+        reduce_views.append(col_buf)
+    desc = "sumRows+sumCols fp32 @ [64K,1K],[8K,8K],[1K,64K] (paper shapes, Fig 3)"
+    return items, reduce_views, desc
+
+
+def build_sumcols_1m4k(npp, gen, torch, rank, world, strategy, device):
+    R, C = 1 << 20, 4096
+    r_local = R // world
+    m = gen.uniform_f32(4, (r_local, C), offset=rank * r_local * C, device=device)
+    plan = npp.Plan("SUM_COLS", (r_local, C), "f32", strategy, device=device)
+    out = plan.new_out()
+    items = [Item(f"sum_cols{_fmt_shape((r_local, C))}", plan, [m], out, r_local * C * 4 + C * 4)]
+    return items, ([out] if world > 1 else []), "sumCols fp32 [1M,4K] row-sharded + NCCL all-reduce (strong)"
+
+
+WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k}
+
+
+# ------------------------------------------------------------------------- reference arm (the oracle)
+
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    import numpy as np
+    import torch
+    from oracle import sums
+    from synth import gen
+    shapes = PAPER_SHAPES if args.workload == "paper" else [(1 << 20, 4096)]
+    # bounded sample per step: the first rows of each matrix, 4M elements per (pattern, shape)
+    sample_elems = 1 << 22
+    mats = []
+    for si, (R, C) in enumerate(shapes):
+        rows = max(1, min(R, sample_elems // C))
+        for pattern in (("SUM_ROWS", "SUM_COLS") if args.workload == "paper" else ("SUM_COLS",)):
+            seed = 300 + 2 * si + (pattern == "SUM_COLS")
+            mats.append((pattern, gen.uniform_f32(seed, (rows, C)).numpy()))
+    step_bytes = sum(m.size * 4 + (m.shape[0] if p == "SUM_ROWS" else m.shape[1]) * 4 for p, m in mats)
+
+    def step():
+        for p, m in mats:
+            (sums.sum_rows if p == "SUM_ROWS" else sums.sum_cols)(m)
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = (time.perf_counter() - t0) / args.steps
+    value = step_bytes / dt / 1e9
+    line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "impl": "reference",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": config_for(args, "oracle (NumPy fp64) on host cores"),
+            "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": f"first {sample_elems} elements of each of {len(mats)} matrices per step"},
+            "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_for(args, extra):
+    if args.workload == "paper":
+        wl = "sumRows+sumCols fp32 @ [64K,1K],[8K,8K],[1K,64K] (paper shapes, BASELINE.json configs[1])"
+    else:
+        wl = "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])"
+    return {"workload": wl, "strategy": args.strategy, "impl_detail": extra,
+            "parallelism": f"row shards x{args.gpus}",
+            "l2": "inputs larger than L2 (distinct 256 MiB buffers per launch, 1.5 GiB per step); no flush"}
+
+
+# ------------------------------------------------------------------------- CPU baseline (oracle, bounded)
+
+def cpu_baseline(items, budget_s=12.0):
+    import numpy as np  # noqa: F401
+    from oracle import sums
+    done_bytes, t_total, n = 0, 0.0, 0
+    samples = []
+    for it in items:
+        m = it.ins[0].cpu().numpy()
+        samples.append((it.name, m))
+    t_end = time.perf_counter() + budget_s
+    while time.perf_counter() < t_end:
+        for name, m in samples:
+            t0 = time.perf_counter()
+            (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(m)
+            t_total += time.perf_counter() - t0
+            done_bytes += m.size * 4
+            n += 1
+    return {"value": round(done_bytes / t_total / 1e9, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n} oracle sums over the step's full matrices ({len(samples)} per pass), "
+                      f"{t_total:.1f} s of single-threaded NumPy fp64"}
+
+
+# ------------------------------------------------------------------------- main arm
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="paper", choices=sorted(WORKLOADS))
+    ap.add_argument("--strategy", default="AUTO")
+    ap.add_argument("--impl", default="npp", choices=["npp", "reference"])
+    ap.add_argument("--no-mappings", action="store_true", help="skip the baseline-mapping table")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_micro_leebsro14_b200 import npp
+    from synth import gen
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    device = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=device)
+    items, reduce_bufs, _ = WORKLOADS[args.workload](npp, gen, torch, rank, world, args.strategy, device)
+    stream = torch.cuda.current_stream()
+
+    def step(evs=None):
+        for i, it in enumerate(items):
+            if evs is not None:
+                evs[i].record(stream)
+            it.run(stream)
+        if evs is not None:
+            evs[len(items)].record(stream)
+        for b in reduce_bufs:
+            dist.all_reduce(b)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(items) + 1)] for _ in range(args.steps)]
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(local)
+    with sampler:
+        torch.cuda.synchronize()
+        t_start.record(stream)
+        for k in range(args.steps):
+            step(evs[k])
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms_total = t_start.elapsed_time(t_end)
+    if world > 1:
+        t = torch.tensor([ms_total], dtype=torch.float64, device=device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    per_kernel_ms = [statistics.mean(evs[k][i].elapsed_time(evs[k][i + 1]) for k in range(args.steps))
+                     for i in range(len(items))]
+    step_bytes = sum(it.bytes for it in items)
+    value = step_bytes * world / (ms_step * 1e-3) / 1e9
+    peak, peak_src = measured_peaks()
+    dom = max(range(len(items)), key=lambda i: per_kernel_ms[i])
+    dom_gbs = items[dom].bytes / (per_kernel_ms[dom] * 1e-3) / 1e9
+    traffic = ncu_traffic().get(items[dom].name)
+    per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9, 1),
+                           "frac_of_measured": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9 / peak, 4),
+                           "frac_of_8TBs": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9 / 8000.0, 4),
+                           "us": round(per_kernel_ms[i] * 1e3, 2),
+                           "mapping": mapping_brief(it.plan.mapping)}
+                 for i, it in enumerate(items)}
+
+    out = {"metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
+           "scaling": "weak" if args.workload == "paper" else "strong", "vs_baseline": None, "dtype": "f32",
+           "data": "synthetic (counter-based U[0,1) fp32, seeded)",
+           "config": config_for(args, "libnpp.so sm_100a"),
+           "per_shape": per_shape,
+           "roofline": {"bound": "hbm", "kernel": items[dom].name, "achieved": round(dom_gbs, 1),
+                        "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": round(dom_gbs / peak, 4),
+                        "traffic": traffic, "algorithmic_bytes": items[dom].bytes},
+           "clocks": sampler.summary(),
+           "gpu_launches": args.steps * sum(it.plan.launches for it in items)}
+
+    # e2e: same metric through the C-ABI with HOST buffers (H2D of the inputs + D2H of the result inside)
+    out["e2e"] = None if args.no_e2e else e2e_host(items, torch, stream, world, dist)
+    if rank == 0 and not args.no_mappings and args.workload == "paper":
+        out["mappings"] = mapping_table(npp, torch, gen, device, stream)
+    if rank == 0 and world == 1 and not args.no_cpu:
+        out["cpu_baseline"] = cpu_baseline(items)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def mapping_brief(m):
+    sp = {0: "Span(1)", 1: "Span(all)", 2: "Span(n)", 3: "Split(k)"}
+    dims = "xyz"
+    return "; ".join(f"L{i}:{dims[l['dim']]},{l['block']},{sp[l['span']].replace('n', str(l['factor'])) if l['span'] == 2 else sp[l['span']].replace('k', str(l['factor']))}"
+                     for i, l in enumerate(m["levels"])) + f"; vec={m['vec']}; grid={m['grid']}"
+
+
+def e2e_host(items, torch, stream, world, dist, steps=3):
+    host_ins = [it.ins[0].cpu().pin_memory() for it in items]
+    host_outs = [torch.empty(it.out.shape, dtype=it.out.dtype).pin_memory() for it in items]
+    h2d = sum(h.numel() * h.element_size() for h in host_ins)
+    d2h = sum(h.numel() * h.element_size() for h in host_outs)
+
+    def one():
+        for it, hi, ho in zip(items, host_ins, host_outs):
+            it.plan.execute_host([hi], ho, it.ins, it.out, stream=stream)
+    one()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        one()
+    dt = (time.perf_counter() - t0) / steps
+    if world > 1:
+        t = torch.tensor([dt], dtype=torch.float64, device=items[0].out.device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dt = float(t.item())
+    value = sum(it.bytes for it in items) * world / dt / 1e9
+    return {"value": round(value, 2), "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "steps": steps, "api": "npp_execute_host (pinned host buffers, blocking)"}
+
+
+def mapping_table(npp, torch, gen, device, stream, iters=5):
+    """The paper's Fig 3 comparison on B200: every strategy at every paper shape (GB/s, events)."""
+    table = {}
+    for si, (R, C) in enumerate(PAPER_SHAPES):
+        m = gen.uniform_f32(300 + 2 * si, (R, C), device=device)
+        for pattern in ("SUM_ROWS", "SUM_COLS"):
+            for strat in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
+                p = npp.Plan(pattern, (R, C), "f32", strat, device=device)
+                out = p.new_out()
+                for _ in range(2):
+                    p.execute([m], out, stream=stream)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                for _ in range(iters):
+                    p.execute([m], out, stream=stream)
+                b.record(stream)
+                torch.cuda.synchronize()
+                us = a.elapsed_time(b) * 1e3 / iters
+                gbs = (R * C * 4 + out.numel() * 4) / (us * 1e-6) / 1e9
+                table[f"{pattern.lower()}{_fmt_shape((R, C))}/{strat}"] = {
+                    "GB/s": round(gbs, 1), "us": round(us, 1), "mapping": mapping_brief(p.mapping)}
+        del m
+    return table
+
+
+if __name__ == "__main__":
+    sys.exit(main())

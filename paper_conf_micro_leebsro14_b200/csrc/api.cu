@@ -1,0 +1,390 @@
+// api.cu — the C ABI of include/npp.h: limits query, plans, execution.
+//
+// npp_plan runs the CUDA-free selector (select.cpp: nest -> constraints -> Algorithm 1 -> ControlDOP
+// -> R2) once per (pattern, shape, dtype, strategy) and freezes the mapping record; npp_execute only
+// translates that record into one kernel launch of the matching family (§IV-E) — the
+// paper's split between a static decision and launch-time parameters.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <string>
+
+#include "kernels.hpp"
+#include "select.hpp"
+
+namespace npp {
+extern thread_local std::string g_error;
+}
+
+struct npp_plan_s {
+  int pattern = 0;
+  int dtype = 0;
+  int strategy = 0;
+  int ndim = 0;
+  int64_t shape[3] = {0, 0, 0};
+  bool empty = false;
+  npp_mapping map{};
+  npp_limits lim{};
+};
+
+namespace {
+
+using npp::set_error;
+
+int cuda_fail(const char* what, cudaError_t e) {
+  char buf[256];
+  std::snprintf(buf, sizeof buf, "%s: %s", what, cudaGetErrorString(e));
+  set_error(buf);
+  return NPP_ERR_CUDA;
+}
+
+int n_inputs(int pattern) {
+  switch (pattern) {
+    case NPP_SUM_ROWS:
+    case NPP_SUM_COLS: return 1;
+    case NPP_SUM_WEIGHTED_ROWS:
+    case NPP_SUM_WEIGHTED_COLS:
+    case NPP_KMEANS_ASSIGN: return 2;
+    case NPP_LOGREG_GRAD: return 3;
+    default: return -1;
+  }
+}
+
+// bytes of input k and of the output, for npp_execute_host
+int64_t input_bytes(const npp_plan_s* p, int k) {
+  const int64_t es = npp::dtype_size(p->dtype);
+  const int64_t* s = p->shape;
+  switch (p->pattern) {
+    case NPP_SUM_ROWS:
+    case NPP_SUM_COLS: return s[0] * s[1] * es;
+    case NPP_SUM_WEIGHTED_ROWS: return k == 0 ? s[0] * s[1] * es : s[1] * es;
+    case NPP_SUM_WEIGHTED_COLS: return k == 0 ? s[0] * s[1] * es : s[0] * es;
+    case NPP_KMEANS_ASSIGN: return k == 0 ? s[0] * s[1] * 4 : s[2] * s[1] * 4;
+    case NPP_LOGREG_GRAD: return k == 0 ? s[0] * s[1] * s[2] * 4 : (k == 1 ? s[0] * s[1] * 4 : s[2] * 4);
+    default: return 0;
+  }
+}
+
+int64_t output_bytes(const npp_plan_s* p) {
+  const int64_t es = npp::dtype_size(p->dtype);
+  const int64_t* s = p->shape;
+  switch (p->pattern) {
+    case NPP_SUM_ROWS:
+    case NPP_SUM_WEIGHTED_ROWS: return s[0] * es;
+    case NPP_SUM_COLS:
+    case NPP_SUM_WEIGHTED_COLS: return s[1] * es;
+    case NPP_KMEANS_ASSIGN: return s[0] * 4;
+    case NPP_LOGREG_GRAD: return s[0] * s[2] * 4;
+    default: return 0;
+  }
+}
+
+int validate_request(int pattern, const int64_t* shape, int ndim, int dtype, bool* empty) {
+  if (!shape || ndim < 1 || ndim > 3) {
+    set_error("shape must hold 2 or 3 sizes");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (dtype < NPP_F32 || dtype > NPP_I64) {
+    set_error("unknown dtype");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (n_inputs(pattern) < 0) {
+    set_error("unknown pattern");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) && dtype != NPP_F32) {
+    set_error("k-means and logreg are defined for f32");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  *empty = false;
+  for (int d = 0; d < ndim; ++d) {
+    if (shape[d] < 0) {
+      set_error("npp_plan needs known, non-negative sizes");
+      return NPP_ERR_INVALID_ARG;
+    }
+    if (shape[d] == 0) *empty = true;
+  }
+  return NPP_OK;
+}
+
+int get_limits(const npp_limits* limits, npp_limits* out) {
+  if (limits) {
+    *out = *limits;
+    return npp::check_limits(out);
+  }
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail("cudaGetDevice", e);
+  return npp_limits_query(dev, out);
+}
+
+inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+}  // namespace
+
+extern "C" {
+
+int npp_version(void) { return NPP_VERSION; }
+
+const char* npp_last_error(void) { return npp::g_error.c_str(); }
+
+int npp_limits_query(int device, npp_limits* out) {
+  if (!out) {
+    set_error("out is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  cudaDeviceProp prop;
+  cudaError_t e = cudaGetDeviceProperties(&prop, device);
+  if (e != cudaSuccess) return cuda_fail("cudaGetDeviceProperties", e);
+  npp_limits l{};
+  l.sm_count = prop.multiProcessorCount;
+  l.max_threads_per_sm = prop.maxThreadsPerMultiProcessor;
+  l.max_threads_per_block = prop.maxThreadsPerBlock;
+  l.max_block_dim[0] = prop.maxThreadsDim[0];
+  l.max_block_dim[1] = prop.maxThreadsDim[1];
+  l.max_block_dim[2] = prop.maxThreadsDim[2];
+  l.warp_size = prop.warpSize;
+  l.max_blocks_per_sm = prop.maxBlocksPerMultiProcessor;
+  l.regs_per_sm = prop.regsPerMultiprocessor;
+  l.regs_per_block = prop.regsPerBlock;
+  l.smem_per_block = int64_t(prop.sharedMemPerBlockOptin);
+  int regs = npp::sum_kernels_max_regs();
+  l.regs_per_thread = regs > 0 ? regs : 1;
+  *out = l;
+  return NPP_OK;
+}
+
+int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strategy, const npp_limits* limits,
+             npp_plan_t* out) {
+  if (!out) {
+    set_error("out is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  *out = nullptr;
+  bool empty = false;
+  int st = validate_request(pattern, shape, ndim, dtype, &empty);
+  if (st) return st;
+  npp_plan_s* p = new npp_plan_s();
+  p->pattern = pattern;
+  p->dtype = dtype;
+  p->strategy = strategy;
+  p->ndim = ndim;
+  for (int d = 0; d < ndim; ++d) p->shape[d] = shape[d];
+  p->empty = empty;
+  if (empty) {
+    p->map = npp_mapping{};
+    p->map.kernel_class = NPP_CLASS_EMPTY;
+    *out = p;
+    return NPP_OK;
+  }
+  st = get_limits(limits, &p->lim);
+  if (!st) st = npp_select(pattern, shape, ndim, dtype, &p->lim, strategy, &p->map);
+  if (st) {
+    delete p;
+    return st;
+  }
+  if (p->map.kernel_class == NPP_CLASS_KMEANS || p->map.kernel_class == NPP_CLASS_LOGREG) {
+    delete p;
+    set_error("this build executes the 2-level sum families only");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  *out = p;
+  return NPP_OK;
+}
+
+int npp_plan_with_mapping(int pattern, const int64_t* shape, int ndim, int dtype, const npp_mapping* forced,
+                          const npp_limits* limits, npp_plan_t* out) {
+  if (!out || !forced) {
+    set_error("out/forced is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  *out = nullptr;
+  bool empty = false;
+  int st = validate_request(pattern, shape, ndim, dtype, &empty);
+  if (st) return st;
+  if (empty) {
+    set_error("npp_plan_with_mapping needs non-empty sizes");
+    return NPP_ERR_INVALID_ARG;
+  }
+  npp_limits lim{};
+  st = get_limits(limits, &lim);
+  if (st) return st;
+  npp::Nest nest;
+  st = npp::build_nest(pattern, shape, ndim, &nest);
+  if (st) return st;
+  if (forced->nlevels != nest.L) {
+    set_error("forced mapping has the wrong number of levels");
+    return NPP_ERR_INVALID_ARG;
+  }
+  npp::Choice c;
+  bool seen[3] = {false, false, false};
+  for (int l = 0; l < nest.L; ++l) {
+    const npp_level& lv = forced->level[l];
+    if (lv.dim < 0 || lv.dim >= nest.L || seen[lv.dim] || lv.span < 0 || lv.span > 3 || lv.block < 1 ||
+        lv.factor < 1) {
+      set_error("forced mapping: dims must be an injective assignment of the first L dims; spans 0..3;"
+                " blocks and factors >= 1");
+      return NPP_ERR_INVALID_ARG;
+    }
+    seen[lv.dim] = true;
+    c.dims[l] = lv.dim;
+    c.blocks[l] = lv.block;
+    c.spans[l] = lv.span;
+    c.factors[l] = lv.factor;
+    if (lv.span == NPP_SPLIT_K && !nest.sync[l]) {
+      set_error("Split(k) applies only where Span(all) was forced by a Reduce (P:L545-546)");
+      return NPP_ERR_NO_FEASIBLE_MAPPING;
+    }
+  }
+  if (!npp::hard_ok(nest, dtype, lim, c)) {
+    set_error("forced mapping violates a hard constraint (Table II / device limits)");
+    return NPP_ERR_NO_FEASIBLE_MAPPING;
+  }
+  if (!npp::is_sum_pattern(pattern)) {
+    set_error("explicit mappings are executable for the 2-level sum families only");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  // vector width: only on the x level when it is the stride-1 level of m and C % vec == 0
+  const int v0 = 16 / npp::dtype_size(dtype);
+  const bool rows = pattern == NPP_SUM_ROWS || pattern == NPP_SUM_WEIGHTED_ROWS;
+  const int x_level = c.dims[0] == NPP_DIM_X ? 0 : 1;
+  c.vec = forced->vec <= 1 ? 1 : forced->vec;
+  if (c.vec != 1 && (c.vec != v0 || x_level != (rows ? 1 : 0) || nest.cols % v0 != 0)) {
+    set_error("vec must be 1, or 16/sizeof(dtype) on the stride-1 x level with C % vec == 0");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  npp_plan_s* p = new npp_plan_s();
+  p->pattern = pattern;
+  p->dtype = dtype;
+  p->strategy = -1;
+  p->ndim = ndim;
+  for (int d = 0; d < ndim; ++d) p->shape[d] = shape[d];
+  p->lim = lim;
+  npp::record_from_choice(nest, dtype, lim, c, npp::score(nest, lim, c), &p->map);
+  *out = p;
+  return NPP_OK;
+}
+
+int npp_plan_mapping(npp_plan_t plan, npp_mapping* out) {
+  if (!plan || !out) {
+    set_error("plan/out is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  *out = plan->map;
+  return NPP_OK;
+}
+
+int64_t npp_plan_workspace_bytes(npp_plan_t plan) { return plan ? plan->map.workspace_bytes : 0; }
+
+int npp_plan_launches(npp_plan_t plan) {
+  if (!plan) return 0;
+  if (plan->empty) return output_bytes(plan) > 0 ? 1 : 0;
+  return 1;
+}
+
+void npp_plan_destroy(npp_plan_t plan) { delete plan; }
+
+int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream) {
+  if (!plan) {
+    set_error("plan is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (plan->empty) {
+    const int64_t ob = output_bytes(plan);
+    if (ob > 0) {
+      if (!out) {
+        set_error("out is NULL");
+        return NPP_ERR_INVALID_ARG;
+      }
+      cudaError_t e = cudaMemsetAsync(out, 0, size_t(ob), st);
+      if (e != cudaSuccess) return cuda_fail("cudaMemsetAsync", e);
+    }
+    return NPP_OK;
+  }
+  const int need = n_inputs(plan->pattern);
+  if (!ins || n_in != need || !out) {
+    set_error("wrong number of inputs or NULL pointer");
+    return NPP_ERR_INVALID_ARG;
+  }
+  for (int k = 0; k < need; ++k)
+    if (!ins[k]) {
+      set_error("input pointer is NULL");
+      return NPP_ERR_INVALID_ARG;
+    }
+  const npp_mapping& m = plan->map;
+  if (m.workspace_bytes > 0 && !workspace) {
+    set_error("this plan needs a workspace (npp_plan_workspace_bytes)");
+    return NPP_ERR_WORKSPACE;
+  }
+  if (m.vec > 1) {
+    for (int k = 0; k < need; ++k)
+      if (!aligned16(ins[k])) {
+        set_error("vectorised plan: inputs must be 16-byte aligned");
+        return NPP_ERR_ALIGNMENT;
+      }
+  }
+  if (!npp::is_sum_pattern(plan->pattern)) {
+    set_error("pattern not executable in this build");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  const bool rows = plan->pattern == NPP_SUM_ROWS || plan->pattern == NPP_SUM_WEIGHTED_ROWS;
+  const bool weighted = plan->pattern == NPP_SUM_WEIGHTED_ROWS || plan->pattern == NPP_SUM_WEIGHTED_COLS;
+  const int64_t R = plan->shape[0], C = plan->shape[1];
+  npp::SumArgs a{};
+  a.m = ins[0];
+  a.v = weighted ? ins[1] : nullptr;
+  a.out = out;
+  a.O = rows ? R : C;
+  a.I = rows ? C : R;
+  a.so = rows ? C : 1;
+  a.si = rows ? 1 : C;
+  const npp_level& lo = m.level[0];
+  const npp_level& li = m.level[1];
+  a.bo = lo.block;
+  a.bi = li.block;
+  a.co = lo.chunk;
+  a.ci = li.chunk;
+  a.go = lo.grid;
+  a.gi = li.grid;
+  if (a.gi > 1) {
+    const int acc = plan->dtype == NPP_I32 ? 4 : 8;
+    const int64_t part = ((a.gi * a.O * acc + 255) / 256) * 256;
+    a.partials = workspace;
+    a.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + part);
+  }
+  cudaError_t e = npp::launch_sum(plan->dtype, m.kernel_class, m.vec, weighted, a, st);
+  if (e != cudaSuccess) return cuda_fail("kernel launch", e);
+  return NPP_OK;
+}
+
+int npp_execute_host(npp_plan_t plan, const void* const* host_ins, int n_in, void* host_out,
+                     void* const* dev_ins, void* dev_out, void* workspace, void* stream) {
+  if (!plan || !host_out || !dev_out || (n_in > 0 && (!host_ins || !dev_ins))) {
+    set_error("NULL argument");
+    return NPP_ERR_INVALID_ARG;
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (!plan->empty) {
+    if (n_in != n_inputs(plan->pattern)) {
+      set_error("wrong number of inputs");
+      return NPP_ERR_INVALID_ARG;
+    }
+    for (int k = 0; k < n_in; ++k) {
+      cudaError_t e = cudaMemcpyAsync(dev_ins[k], host_ins[k], size_t(input_bytes(plan, k)),
+                                      cudaMemcpyHostToDevice, st);
+      if (e != cudaSuccess) return cuda_fail("cudaMemcpyAsync H2D", e);
+    }
+  }
+  int rc = npp_execute(plan, const_cast<const void* const*>(reinterpret_cast<void* const*>(dev_ins)), n_in,
+                       dev_out, workspace, stream);
+  if (rc) return rc;
+  cudaError_t e = cudaMemcpyAsync(host_out, dev_out, size_t(output_bytes(plan)), cudaMemcpyDeviceToHost, st);
+  if (e != cudaSuccess) return cuda_fail("cudaMemcpyAsync D2H", e);
+  e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail("cudaStreamSynchronize", e);
+  return NPP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,529 @@
+// select.cpp — the mapping analysis of PAPER.md §IV as deterministic integer logic (CUDA-free).
+//
+//   S1 nest descriptor            §IV intro P:L396-403, L454-455; Fig 8
+//   S2 candidate space            Algorithm 1
+//   S3 hard constraints           Table II P:L559-565 (HL, HG); P:L658-662 (GPU limits)
+//   S4 soft constraints, weights  Table II (SL, SG)
+//   S5 selection key              P:L734-741; Alg 1 P:L790-792 (ties made deterministic, G2)
+//   S6 ControlDOP                 Alg 1
+//   S7 forced prior-work mappings P:L99-115; Fig 7
+//   S8 runtime step R2            P:L810-817 ("block sizes and span/split factors can be
+//                                 dynamically changed without recompiling the code")
+//   S9 mapping record             grid/chunk/workspace for the kernel families (§IV-E)
+// Every rule is spelled out in DESIGN.md §3; oracle/select.py implements the same document
+// independently and tests/test_select_parity.py compares the two records field by field.
+#include "select.hpp"
+
+#include <algorithm>
+#include <climits>
+#include <cstdio>
+
+namespace npp {
+
+namespace {
+
+constexpr int kSizeSetLen = 11;          // {1,2,...,1024}  Alg 1
+constexpr int64_t kWC = 8;               // coalescing intrinsic weight (G3)
+constexpr int64_t kWB = 1;               // min-block-size intrinsic weight (G3)
+constexpr int kMinBlockSize = 64;        // Table II SG (G5)
+constexpr int64_t kUnknownSize = 1000;   // P:L699-700 (G17)
+constexpr int kTBlock = 256;             // R2 threads per block (S8)
+constexpr int64_t kUMin = 8;             // R2 minimum loads per lane per chunk (S8)
+constexpr int64_t kMaxGrid = (int64_t(1) << 31) - 1;  // H6
+
+inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline int64_t eff(int64_t n) { return n < 0 ? kUnknownSize : n; }
+inline int64_t pow2ceil(int64_t v) {
+  int64_t p = 1;
+  while (p < v) p <<= 1;
+  return p;
+}
+
+int64_t prod_blocks(const Nest& n, const Choice& c) {
+  int64_t p = 1;
+  for (int l = 0; l < n.L; ++l) p *= c.blocks[l];
+  return p;
+}
+
+// G7: DOP contributed by one level
+int64_t level_dop(int64_t N, int b, int span, int64_t factor) {
+  N = eff(N);
+  switch (span) {
+    case NPP_SPAN_ONE: return N;
+    case NPP_SPAN_ALL: return b < N ? b : N;
+    case NPP_SPAN_N: return cdiv(N, factor);
+    default: {  // Split(k)
+      int64_t per = cdiv(N, factor);
+      return factor * (b < per ? b : per);
+    }
+  }
+}
+
+int64_t mapping_dop(const Nest& n, const Choice& c) {
+  int64_t d = 1;
+  for (int l = 0; l < n.L; ++l) d *= level_dop(n.N[l], c.blocks[l], c.spans[l], c.factors[l]);
+  return d;
+}
+
+// S9: indices of level l one thread block covers
+int64_t level_chunk(int64_t N, int b, int span, int64_t factor, int vec) {
+  N = eff(N);
+  switch (span) {
+    case NPP_SPAN_ONE: return int64_t(b) * vec;
+    case NPP_SPAN_N: return int64_t(b) * vec * factor;
+    case NPP_SPAN_ALL: return N > 0 ? N : 1;
+    default: {  // Split(k): contiguous chunks of ceil(N/k) (G12), rounded up to the vector width
+      int64_t ch = cdiv(N, factor);
+      return cdiv(ch, vec) * vec;
+    }
+  }
+}
+
+int acc_bytes(int pattern, int dtype) {
+  if (pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) return 8;
+  return dtype == NPP_I32 ? 4 : 8;
+}
+
+int64_t staging_bytes(const Nest& n) {
+  if (n.pattern == NPP_KMEANS_ASSIGN) return 4 * eff(n.N[1]) * eff(n.N[2]) + 4 * eff(n.N[1]);
+  return 0;
+}
+
+int64_t smem_model(const Nest& n, int dtype, const Choice& c) {
+  bool par_reduce = false;
+  for (int l = 0; l < n.L; ++l) par_reduce |= (n.sync[l] && c.blocks[l] > 1);
+  return (par_reduce ? prod_blocks(n, c) * acc_bytes(n.pattern, dtype) : 0) + staging_bytes(n);
+}
+
+bool key_greater(int64_t s1, int64_t d1, int64_t p1, int64_t s2, int64_t d2, int64_t p2) {
+  if (s1 != s2) return s1 > s2;
+  if (d1 != d2) return d1 > d2;
+  return p1 < p2;  // smaller Π b wins
+}
+
+// Alg 1 SEARCH with the S5 key. restrict_1d: b_l = 1 and Span(all) for l >= 1 (S7 1D).
+bool search(const Nest& n, int dtype, const npp_limits& lim, bool restrict_1d, Choice* best,
+            int64_t* best_score) {
+  static const int perms2[2][2] = {{0, 1}, {1, 0}};
+  static const int perms3[6][3] = {{0, 1, 2}, {0, 2, 1}, {1, 0, 2}, {1, 2, 0}, {2, 0, 1}, {2, 1, 0}};
+  const int nperm = n.L == 1 ? 1 : (n.L == 2 ? 2 : 6);
+  int64_t bs = 0, bd = 0, bp = 0;
+  bool found = false;
+  int total_sizes = 1, total_spans = 1;
+  for (int l = 0; l < n.L; ++l) {
+    total_sizes *= kSizeSetLen;
+    total_spans *= 2;
+  }
+  for (int p = 0; p < nperm; ++p) {
+    Choice c;
+    for (int l = 0; l < n.L; ++l) c.dims[l] = n.L == 1 ? 0 : (n.L == 2 ? perms2[p][l] : perms3[p][l]);
+    for (int si = 0; si < total_sizes; ++si) {  // lexicographic, level 0 most significant
+      int rem = si;
+      for (int l = n.L - 1; l >= 0; --l) {
+        c.blocks[l] = 1 << (rem % kSizeSetLen);
+        rem /= kSizeSetLen;
+      }
+      if (restrict_1d) {
+        bool ok = true;
+        for (int l = 1; l < n.L; ++l) ok &= c.blocks[l] == 1;
+        if (!ok) continue;
+      }
+      for (int sp = 0; sp < total_spans; ++sp) {  // ONE(0) < ALL(1), level 0 most significant
+        for (int l = 0; l < n.L; ++l) c.spans[l] = (sp >> (n.L - 1 - l)) & 1 ? NPP_SPAN_ALL : NPP_SPAN_ONE;
+        if (restrict_1d) {
+          bool ok = true;
+          for (int l = 1; l < n.L; ++l) ok &= c.spans[l] == NPP_SPAN_ALL;
+          if (!ok) continue;
+        }
+        for (int l = 0; l < n.L; ++l) c.factors[l] = 1;
+        if (!hard_ok(n, dtype, lim, c)) continue;
+        const int64_t s = score(n, lim, c);
+        const int64_t d = mapping_dop(n, c);
+        const int64_t pb = prod_blocks(n, c);
+        if (!found || key_greater(s, d, pb, bs, bd, bp)) {  // strict: first (lex-smallest) wins ties
+          found = true;
+          bs = s;
+          bd = d;
+          bp = pb;
+          *best = c;
+        }
+      }
+    }
+  }
+  *best_score = bs;
+  return found;
+}
+
+// S6 ControlDOP
+void control_dop(const Nest& n, const npp_limits& lim, Choice* c) {
+  const int64_t min_dop = int64_t(lim.sm_count) * lim.max_threads_per_sm;
+  const int64_t max_dop = 100 * min_dop;
+  for (int l = 0; l < n.L; ++l) c->factors[l] = 1;
+  const int64_t dop = mapping_dop(n, *c);
+  if (dop < min_dop) {  // Span(all) -> Split(k)
+    int best_l = -1;
+    int64_t best_nb = 1;
+    for (int l = 0; l < n.L; ++l) {
+      const int64_t nb = cdiv(eff(n.N[l]), c->blocks[l]);
+      if (n.sync[l] && c->spans[l] == NPP_SPAN_ALL && nb >= 2 && nb > best_nb) {
+        best_l = l;
+        best_nb = nb;
+      }
+    }
+    if (best_l >= 0) {
+      int64_t k = cdiv(min_dop, dop);
+      if (k > best_nb) k = best_nb;
+      if (k >= 2) {
+        c->spans[best_l] = NPP_SPLIT_K;
+        c->factors[best_l] = k;
+      }
+    }
+  } else if (dop > max_dop) {  // Span(1) -> Span(n)
+    for (int l = 0; l < n.L; ++l) {
+      if (c->spans[l] != NPP_SPAN_ONE) continue;
+      int64_t nn = cdiv(dop, max_dop);
+      const int64_t cap = cdiv(eff(n.N[l]), c->blocks[l]);
+      if (nn > cap) nn = cap;
+      if (nn >= 2) {
+        c->spans[l] = NPP_SPAN_N;
+        c->factors[l] = nn;
+      }
+      break;
+    }
+  }
+}
+
+int64_t slots(const npp_limits& lim, int threads_per_block) {
+  int64_t per_sm = lim.max_blocks_per_sm;
+  const int64_t by_threads = lim.max_threads_per_sm / threads_per_block;
+  const int64_t by_regs = lim.regs_per_sm / (int64_t(threads_per_block) * lim.regs_per_thread);
+  if (by_threads < per_sm) per_sm = by_threads;
+  if (by_regs < per_sm) per_sm = by_regs;
+  if (per_sm < 1) per_sm = 1;
+  return int64_t(lim.sm_count) * per_sm;
+}
+
+// S8 for the 2-level sums: keep LITERAL's dims, re-choose blocks / vec / factors / chunks.
+void r2_sums(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
+  const bool rows = n.pattern == NPP_SUM_ROWS || n.pattern == NPP_SUM_WEIGHTED_ROWS;
+  const int64_t O = n.N[0], I = n.N[1], C = n.cols;
+  const int contig_level = rows ? 1 : 0;
+  const int x_level = c->dims[0] == NPP_DIM_X ? 0 : 1;
+  const int v0 = 16 / dtype_size(dtype);
+  const int vec = (x_level == contig_level && C % v0 == 0) ? v0 : 1;
+  const int64_t S = slots(lim, kTBlock);
+  int64_t k, nn;
+  c->vec = vec;
+  if (x_level == 1) {  // class RX: inner Reduce on x
+    const int64_t bx = std::min<int64_t>(32, pow2ceil(cdiv(I, vec)));
+    const int64_t by = kTBlock / bx;
+    const int64_t g = cdiv(O, by);
+    if (g >= S) {
+      k = 1;
+      nn = cdiv(g, S);
+    } else {
+      nn = 1;
+      k = std::min<int64_t>(S / g, cdiv(I, bx * vec * kUMin));
+      if (k < 1) k = 1;
+    }
+    const int64_t chunk_i = vec * cdiv(cdiv(I, k), vec);
+    k = cdiv(I, chunk_i);
+    c->blocks[0] = int(by);
+    c->blocks[1] = int(bx);
+    c->chunks[0] = by * nn;
+    c->chunks[1] = k > 1 ? chunk_i : I;
+  } else {  // class MX: outer Map on x, inner Reduce on y
+    const int64_t bx = std::min<int64_t>(32, pow2ceil(cdiv(O, vec)));
+    const int64_t by = kTBlock / bx;
+    const int64_t g = cdiv(O, bx * vec);
+    if (g >= S) {
+      k = 1;
+      nn = cdiv(g, S);
+    } else {
+      nn = 1;
+      k = std::min<int64_t>(S / g, cdiv(I, by * kUMin));
+      if (k < 1) k = 1;
+    }
+    const int64_t chunk_i = cdiv(I, k);
+    k = cdiv(I, chunk_i);
+    c->blocks[0] = int(bx);
+    c->blocks[1] = int(by);
+    c->chunks[0] = bx * vec * nn;
+    c->chunks[1] = k > 1 ? chunk_i : I;
+  }
+  c->spans[0] = nn == 1 ? NPP_SPAN_ONE : NPP_SPAN_N;
+  c->factors[0] = nn;
+  c->spans[1] = k == 1 ? NPP_SPAN_ALL : NPP_SPLIT_K;
+  c->factors[1] = k;
+}
+
+int kernel_class_of(const Nest& n, const Choice& c) {
+  if (n.pattern == NPP_KMEANS_ASSIGN) return NPP_CLASS_KMEANS;
+  if (n.pattern == NPP_LOGREG_GRAD) return NPP_CLASS_LOGREG;
+  return c.dims[1] == NPP_DIM_X ? NPP_CLASS_RX : NPP_CLASS_MX;
+}
+
+}  // namespace
+
+thread_local std::string g_error;
+
+void set_error(const std::string& msg) { g_error = msg; }
+
+int dtype_size(int dtype) { return dtype == NPP_I64 ? 8 : 4; }
+
+bool is_sum_pattern(int p) {
+  return p == NPP_SUM_ROWS || p == NPP_SUM_COLS || p == NPP_SUM_WEIGHTED_ROWS ||
+         p == NPP_SUM_WEIGHTED_COLS;
+}
+
+int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
+  if (!shape) {
+    set_error("shape is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  Nest n;
+  n.pattern = pattern;
+  auto need = [&](int d) {
+    if (ndim != d) {
+      char buf[96];
+      std::snprintf(buf, sizeof buf, "pattern %d expects %d sizes, got %d", pattern, d, ndim);
+      set_error(buf);
+      return false;
+    }
+    return true;
+  };
+  switch (pattern) {
+    case NPP_SUM_ROWS:
+    case NPP_SUM_WEIGHTED_ROWS:
+      if (!need(2)) return NPP_ERR_INVALID_ARG;
+      n.L = 2;
+      n.N[0] = shape[0], n.sync[0] = false;  // Map rows
+      n.N[1] = shape[1], n.sync[1] = true;   // Reduce along the row (Fig 1)
+      n.acc[n.nacc++] = {0, 0x1u};           // out[r]
+      n.acc[n.nacc++] = {1, 0x3u};           // m[r,c]
+      if (pattern == NPP_SUM_WEIGHTED_ROWS) n.acc[n.nacc++] = {1, 0x3u};  // v[c]
+      n.cols = shape[1];
+      break;
+    case NPP_SUM_COLS:
+    case NPP_SUM_WEIGHTED_COLS:
+      if (!need(2)) return NPP_ERR_INVALID_ARG;
+      n.L = 2;
+      n.N[0] = shape[1], n.sync[0] = false;  // Map columns
+      n.N[1] = shape[0], n.sync[1] = true;   // Reduce down the column (Fig 1)
+      n.acc[n.nacc++] = {0, 0x1u};           // out[c]
+      n.acc[n.nacc++] = {0, 0x3u};           // m[r,c]: stride-1 index is c, i.e. level 0
+      if (pattern == NPP_SUM_WEIGHTED_COLS) n.acc[n.nacc++] = {1, 0x3u};  // v[r]
+      n.cols = shape[1];
+      break;
+    case NPP_KMEANS_ASSIGN:  // shape {N, D, K}; levels N / K / D
+      if (!need(3)) return NPP_ERR_INVALID_ARG;
+      n.L = 3;
+      n.N[0] = shape[0], n.sync[0] = false;
+      n.N[1] = shape[2], n.sync[1] = true;
+      n.N[2] = shape[1], n.sync[2] = true;
+      n.acc[n.nacc++] = {0, 0x1u};  // a[i]
+      n.acc[n.nacc++] = {2, 0x7u};  // x[i,d]
+      n.acc[n.nacc++] = {2, 0x7u};  // c[k,d]
+      n.cols = shape[1];
+      break;
+    case NPP_LOGREG_GRAD:  // shape {B, Rb, C}
+      if (!need(3)) return NPP_ERR_INVALID_ARG;
+      n.L = 3;
+      n.N[0] = shape[0], n.sync[0] = false;
+      n.N[1] = shape[1], n.sync[1] = true;
+      n.N[2] = shape[2], n.sync[2] = true;  // Map_j + Reduce_k at one level -> Span(all) (HG)
+      n.acc[n.nacc++] = {1, 0x3u};  // y[i]
+      n.acc[n.nacc++] = {2, 0x7u};  // x[i,k] (dot)
+      n.acc[n.nacc++] = {2, 0x7u};  // w[k]
+      n.acc[n.nacc++] = {2, 0x7u};  // x[i,j] (update)
+      n.acc[n.nacc++] = {2, 0x5u};  // g[b,j]
+      n.cols = shape[2];
+      break;
+    default:
+      set_error("unknown pattern");
+      return NPP_ERR_INVALID_ARG;
+  }
+  long double total = 1;
+  for (int l = 0; l < n.L; ++l) {
+    if (n.N[l] == 0 || n.N[l] < -1 || n.N[l] > (int64_t(1) << 40)) {
+      set_error("level sizes must be in [1, 2^40] or -1 (unknown)");
+      return NPP_ERR_INVALID_ARG;
+    }
+    total *= (long double)eff(n.N[l]);
+  }
+  if (total > (long double)(int64_t(1) << 50)) {
+    set_error("nest too large (product of sizes > 2^50)");
+    return NPP_ERR_INVALID_ARG;
+  }
+  *out = n;
+  return NPP_OK;
+}
+
+int check_limits(const npp_limits* lim) {
+  if (!lim) {
+    set_error("limits is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (lim->sm_count < 1 || lim->max_threads_per_sm < 1 || lim->warp_size < 1 ||
+      lim->max_blocks_per_sm < 1 || lim->regs_per_sm < 1 || lim->regs_per_thread < 1) {
+    set_error("limits: sm_count, max_threads_per_sm, warp_size, max_blocks_per_sm, regs_per_sm and "
+              "regs_per_thread must be >= 1");
+    return NPP_ERR_INVALID_ARG;
+  }
+  return NPP_OK;
+}
+
+bool hard_ok(const Nest& n, int dtype, const npp_limits& lim, const Choice& c) {
+  for (int l = 0; l < n.L; ++l) {  // H1: Reduce -> Span(all) (HL); one span per level (HG)
+    const bool all_like = c.spans[l] == NPP_SPAN_ALL || c.spans[l] == NPP_SPLIT_K;
+    if (n.sync[l] && !all_like) return false;
+  }
+  const int64_t tb = prod_blocks(n, c);
+  if (tb > lim.max_threads_per_block) return false;                       // H2
+  for (int l = 0; l < n.L; ++l) {
+    if (c.dims[l] < 0 || c.dims[l] > 2) return false;
+    if (c.blocks[l] < 1 || c.blocks[l] > lim.max_block_dim[c.dims[l]]) return false;  // H3
+  }
+  if (tb * lim.regs_per_thread > lim.regs_per_block) return false;        // H4
+  if (smem_model(n, dtype, c) > lim.smem_per_block) return false;         // H5
+  int64_t grid = 1;                                                       // H6
+  for (int l = 0; l < n.L; ++l) {
+    const int span = c.spans[l] == NPP_SPLIT_K ? NPP_SPAN_ALL
+                                               : (c.spans[l] == NPP_SPAN_N ? NPP_SPAN_ONE : c.spans[l]);
+    grid *= cdiv(eff(n.N[l]), level_chunk(n.N[l], c.blocks[l], span, 1, 1));
+    if (grid > kMaxGrid) return false;
+  }
+  return true;
+}
+
+int64_t score(const Nest& n, const npp_limits& lim, const Choice& c) {
+  int64_t total = 0;
+  for (int a = 0; a < n.nacc; ++a) {
+    const Access& ac = n.acc[a];
+    if (ac.contig < 0) continue;
+    int64_t w = kWC;
+    for (int l = 0; l < n.L; ++l)
+      if (ac.mask & (1u << l)) w *= eff(n.N[l]);
+    // SL: sequential accesses -> Dim(x) and block size a multiple of WARP_SIZE
+    if (c.dims[ac.contig] == NPP_DIM_X && c.blocks[ac.contig] % lim.warp_size == 0) total += w;
+  }
+  if (prod_blocks(n, c) >= kMinBlockSize) {  // SG: threads per block >= MIN_BLOCK_SIZE
+    int64_t w = kWB;
+    for (int l = 0; l < n.L; ++l) w *= eff(n.N[l]);
+    total += w;
+  }
+  return total;
+}
+
+int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c, int64_t score_value,
+                       npp_mapping* out) {
+  (void)lim;
+  npp_mapping m{};
+  m.nlevels = n.L;
+  m.kernel_class = kernel_class_of(n, c);
+  m.vec = c.vec;
+  int64_t grid = 1, tb = 1;
+  for (int l = 0; l < n.L; ++l) {
+    npp_level& lv = m.level[l];
+    const int v = c.dims[l] == NPP_DIM_X ? c.vec : 1;
+    lv.dim = c.dims[l];
+    lv.block = c.blocks[l];
+    lv.span = c.spans[l];
+    lv.factor = (c.spans[l] == NPP_SPAN_N || c.spans[l] == NPP_SPLIT_K) ? c.factors[l] : 1;
+    lv.chunk = c.chunks[l] > 0 ? c.chunks[l] : level_chunk(n.N[l], c.blocks[l], c.spans[l], lv.factor, v);
+    lv.grid = cdiv(eff(n.N[l]), lv.chunk);
+    grid *= lv.grid;
+    tb *= c.blocks[l];
+  }
+  m.score = score_value;
+  m.dop = mapping_dop(n, c);
+  m.grid = grid;
+  m.threads = grid * tb;
+  m.block[0] = m.block[1] = m.block[2] = 1;
+  for (int l = 0; l < n.L; ++l) m.block[c.dims[l]] = c.blocks[l];
+  m.smem_bytes = int32_t(smem_model(n, dtype, c));
+  m.workspace_bytes = 0;
+  if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
+    const int64_t part = m.level[1].grid * eff(n.N[0]) * acc_bytes(n.pattern, dtype);
+    const int64_t tick = m.level[0].grid * 4;
+    m.workspace_bytes = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256);
+  }
+  *out = m;
+  return NPP_OK;
+}
+
+int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy, npp_mapping* out) {
+  bool unknown = false;
+  for (int l = 0; l < n.L; ++l) unknown |= n.N[l] < 0;
+  Choice c;
+  int64_t sc = 0;
+  if (strategy == NPP_MAP_1D || strategy == NPP_MAP_TB_THREAD || strategy == NPP_MAP_WARP) {
+    if (n.L != 2) {
+      set_error("forced prior-work mappings (Fig 7) are defined for 2-level nests only");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    if (strategy == NPP_MAP_1D) {  // only the outermost level is parallel
+      if (!search(n, dtype, lim, true, &c, &sc)) {
+        set_error("no feasible 1D mapping");
+        return NPP_ERR_NO_FEASIBLE_MAPPING;
+      }
+    } else if (strategy == NPP_MAP_TB_THREAD) {  // Fig 7a
+      c.dims[0] = NPP_DIM_Y, c.blocks[0] = 1, c.spans[0] = NPP_SPAN_ONE;
+      c.dims[1] = NPP_DIM_X, c.spans[1] = NPP_SPAN_ALL;
+      c.blocks[1] = int(std::min<int64_t>(1024, pow2ceil(eff(n.N[1]))));
+    } else {  // Fig 7b, footnote 4 P:L621-622
+      c.dims[0] = NPP_DIM_Y, c.blocks[0] = 16, c.spans[0] = NPP_SPAN_ONE;
+      c.dims[1] = NPP_DIM_X, c.blocks[1] = 32, c.spans[1] = NPP_SPAN_ALL;
+    }
+    if (!hard_ok(n, dtype, lim, c)) {
+      set_error("forced mapping violates a hard constraint on this device");
+      return NPP_ERR_NO_FEASIBLE_MAPPING;
+    }
+    return record_from_choice(n, dtype, lim, c, score(n, lim, c), out);
+  }
+  if (strategy != NPP_MAP_AUTO && strategy != NPP_MAP_LITERAL) {
+    set_error("unknown strategy");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (!search(n, dtype, lim, false, &c, &sc)) {
+    set_error("no candidate mapping satisfies the hard constraints (Algorithm 1 CandSet is empty)");
+    return NPP_ERR_NO_FEASIBLE_MAPPING;
+  }
+  control_dop(n, lim, &c);
+  if (strategy == NPP_MAP_LITERAL) return record_from_choice(n, dtype, lim, c, sc, out);
+  if (unknown) {
+    set_error("strategy AUTO needs known sizes (use LITERAL for -1 sizes)");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  if (n.L != 2) {
+    set_error("R2 runtime step for 3-level nests is not implemented in this build");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  r2_sums(n, dtype, lim, &c);
+  return record_from_choice(n, dtype, lim, c, sc, out);
+}
+
+}  // namespace npp
+
+extern "C" int npp_select(int pattern, const int64_t* shape, int ndim, int dtype, const npp_limits* limits,
+                          int strategy, npp_mapping* out) {
+  using namespace npp;
+  if (!out) {
+    set_error("out is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (dtype < NPP_F32 || dtype > NPP_I64) {
+    set_error("unknown dtype");
+    return NPP_ERR_INVALID_ARG;
+  }
+  int st = check_limits(limits);
+  if (st) return st;
+  Nest n;
+  st = build_nest(pattern, shape, ndim, &n);
+  if (st) return st;
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) && dtype != NPP_F32) {
+    set_error("k-means and logreg are defined for f32");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  return select_mapping(n, dtype, *limits, strategy, out);
+}

@@ -1,0 +1,54 @@
+// select.hpp — internal interface of the CUDA-free mapping selector.
+#pragma once
+
+#include <cstdint>
+#include <string>
+
+#include "npp.h"
+
+namespace npp {
+
+constexpr int kMaxLevels = 3;
+constexpr int kMaxAccesses = 6;
+
+// S1: one nest = levels (size, sync) + accesses (contiguous level, execution-count mask).
+struct Access {
+  int contig;     // level whose index is stride-1 for this array (-1: none)
+  unsigned mask;  // bit l set: N_l multiplies the execution count (Fig 8)
+};
+
+struct Nest {
+  int pattern = 0;
+  int L = 0;
+  int64_t N[kMaxLevels] = {0, 0, 0};  // -1 = unknown size (G17)
+  bool sync[kMaxLevels] = {false, false, false};
+  int nacc = 0;
+  Access acc[kMaxAccesses];
+  int64_t cols = 0;  // matrix columns (sums), for the vector-width rule of R2
+};
+
+struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refinements
+  int dims[kMaxLevels] = {0, 0, 0};
+  int blocks[kMaxLevels] = {1, 1, 1};
+  int spans[kMaxLevels] = {NPP_SPAN_ONE, NPP_SPAN_ONE, NPP_SPAN_ONE};
+  int64_t factors[kMaxLevels] = {1, 1, 1};
+  int64_t chunks[kMaxLevels] = {0, 0, 0};  // 0 = derive from span/factor (S9)
+  int vec = 1;
+};
+
+// thread-local error message shared with the API layer
+void set_error(const std::string& msg);
+
+int dtype_size(int dtype);
+bool is_sum_pattern(int pattern);
+int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out);
+int check_limits(const npp_limits* lim);
+bool hard_ok(const Nest& n, int dtype, const npp_limits& lim, const Choice& c);
+int64_t score(const Nest& n, const npp_limits& lim, const Choice& c);
+// full pipeline (S2..S9) into a record
+int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy, npp_mapping* out);
+// S9 for a caller-provided choice (npp_plan_with_mapping): validates and fills the record
+int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c, int64_t score_value,
+                       npp_mapping* out);
+
+}  // namespace npp

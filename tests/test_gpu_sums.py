@@ -1,0 +1,225 @@
+"""GPU parity: the CUDA sum families (through the C-ABI) vs the fp64/int oracle, element by element.
+
+Integers: bit-exact. fp32: |gpu - oracle| <= 1e-5 * Σ|terms| per output (north_star tolerance; for the
+non-negative U[0,1) inputs this is 1e-5 relative).
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle import select as osel
+from oracle import sums
+from synth import gen
+
+pytestmark = pytest.mark.gpu
+
+STRATS = ["AUTO", "LITERAL", "1D", "TB_T", "WARP"]
+SHAPES = [(1, 1), (3, 5), (31, 33), (33, 31), (1000, 999), (1024, 1024), (4097, 300), (300, 4097),
+          (7, 70000), (70000, 7), (2, 1 << 17)]
+
+
+@pytest.fixture(scope="module")
+def npp(cuda_device):
+    from paper_conf_micro_leebsro14_b200 import npp as _npp
+    return _npp
+
+
+def _make(dtype, shape, seed, device):
+    if dtype == "f32":
+        return gen.uniform_f32(seed, shape, device=device)
+    if dtype == "i32":
+        return gen.int_uniform(seed, shape, -1000, 1000, device=device)
+    return gen.int64_wide(seed, shape, device=device)
+
+
+def _oracle(pattern, m_np):
+    return sums.sum_rows(m_np) if pattern == "SUM_ROWS" else sums.sum_cols(m_np)
+
+
+def _abs_scale(pattern, m_np):
+    return sums.sum_abs_rows(m_np) if pattern == "SUM_ROWS" else sums.sum_abs_cols(m_np)
+
+
+def check(pattern, m, got, dtype):
+    m_np = m.cpu().numpy()
+    want = _oracle(pattern, m_np)
+    g = got.cpu().numpy()
+    if dtype == "f32":
+        tol = 1e-5 * _abs_scale(pattern, m_np)
+        err = np.abs(g.astype(np.float64) - want)
+        bad = np.nonzero(err > tol)[0]
+        assert bad.size == 0, f"{pattern} first bad {bad[:5]} got {g[bad[:5]]} want {want[bad[:5]]}"
+    else:
+        assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), pattern
+
+
+@pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("strategy", STRATS)
+def test_parity_small(npp, cuda_device, pattern, dtype, strategy):
+    for i, shape in enumerate(SHAPES):
+        m = _make(dtype, shape, 100 + i, cuda_device)
+        p = npp.Plan(pattern, shape, dtype, strategy)
+        out = p.new_out()
+        p.execute([m], out)
+        torch.cuda.synchronize()
+        check(pattern, m, out, dtype)
+        # the record the plan executes is the oracle selector's record (limits from the device)
+        lim = npp.limits_query(0)
+        assert p.mapping == osel.select(pattern, shape, dtype, lim, strategy)
+
+
+@pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS"])
+def test_exact_summable_fp32_bit_exact(npp, cuda_device, pattern):
+    for shape in [(1024, 1024), (65536, 64), (64, 65536)]:
+        m = gen.exact_f32(11, shape, device=cuda_device)
+        for strategy in STRATS:
+            p = npp.Plan(pattern, shape, "f32", strategy)
+            out = p.execute([m], p.new_out())
+            torch.cuda.synchronize()
+            want = _oracle(pattern, m.cpu().numpy())
+            assert np.array_equal(out.cpu().numpy().astype(np.float64), want), (shape, strategy)
+
+
+def test_arange_int32_wrap(npp, cuda_device):
+    shape = (3000, 2500)
+    m = gen.arange_matrix(shape, torch.int32, offset=(1 << 31) - 10 ** 6, device=cuda_device)
+    for pattern in ("SUM_ROWS", "SUM_COLS"):
+        for strategy in STRATS:
+            p = npp.Plan(pattern, shape, "i32", strategy)
+            out = p.execute([m], p.new_out())
+            torch.cuda.synchronize()
+            check(pattern, m, out, "i32")
+
+
+@pytest.mark.parametrize("shape", [(65536, 1024), (8192, 8192), (1024, 65536)])
+def test_paper_shapes_full(npp, cuda_device, shape):
+    m = gen.uniform_f32(3, shape, device=cuda_device)
+    for pattern in ("SUM_ROWS", "SUM_COLS"):
+        for strategy in STRATS:
+            p = npp.Plan(pattern, shape, "f32", strategy)
+            out = p.execute([m], p.new_out())
+            out2 = p.execute([m], p.new_out())   # workspace reuse: tickets were reset
+            torch.cuda.synchronize()
+            check(pattern, m, out, "f32")
+            assert torch.equal(out, out2), "non-deterministic or stale workspace"
+
+
+def test_large_sumcols_sampled(npp, cuda_device):
+    # [1M, 4K] fp32 (16 GiB, 2^32 elements: 64-bit indexing); sampled columns recomputed by the oracle
+    R, C = 1 << 20, 4096
+    free, _ = torch.cuda.mem_get_info()
+    if free < 18 * (1 << 30):
+        pytest.skip("needs 18 GiB free")
+    m = gen.small_int_f32(4, (R, C), 0, 15, device=cuda_device)   # exact: all partial sums < 2^24
+    p = npp.Plan("SUM_COLS", (R, C), "f32", "AUTO")
+    out = p.execute([m], p.new_out())
+    pr = npp.Plan("SUM_ROWS", (R, C), "f32", "AUTO")
+    out_r = pr.execute([m], pr.new_out())
+    torch.cuda.synchronize()
+    cols = torch.tensor([0, 1, 2, 3, 127, 128, 2047, 4093, 4094, 4095], device=cuda_device)
+    sub = m.index_select(1, cols).cpu().numpy()
+    want = sums.sum_cols(sub)
+    assert np.array_equal(out.index_select(0, cols).cpu().numpy().astype(np.float64), want)
+    rows = torch.tensor([0, 1, R // 2, R - 2, R - 1], device=cuda_device)
+    want_r = sums.sum_rows(m.index_select(0, rows).cpu().numpy())
+    assert np.array_equal(out_r.index_select(0, rows).cpu().numpy().astype(np.float64), want_r)
+    # property at full size: Σ sumRows == Σ sumCols (exact for these integer-valued fp32 inputs)
+    assert float(out.double().sum()) == float(out_r.double().sum())
+    del m
+
+
+def test_empty_and_degenerate(npp, cuda_device):
+    p = npp.Plan("SUM_ROWS", (5, 0), "f32", "AUTO")
+    out = torch.full((5,), 7.0, device=cuda_device)
+    p.execute([torch.empty(0, device=cuda_device)], out)
+    torch.cuda.synchronize()
+    assert out.tolist() == [0.0] * 5
+    p = npp.Plan("SUM_COLS", (0, 3), "i32", "AUTO")
+    out = torch.full((3,), 7, dtype=torch.int32, device=cuda_device)
+    p.execute([torch.empty(0, dtype=torch.int32, device=cuda_device)], out)
+    torch.cuda.synchronize()
+    assert out.tolist() == [0, 0, 0]
+    p = npp.Plan("SUM_ROWS", (0, 3), "i32", "AUTO")
+    assert p.launches == 0
+
+
+def test_alignment_error(npp, cuda_device):
+    base = gen.uniform_f32(1, (1024 * 1024 + 1,), device=cuda_device)
+    m = base[1:].view(1024, 1024)
+    p = npp.Plan("SUM_ROWS", (1024, 1024), "f32", "AUTO")
+    assert p.mapping["vec"] == 4
+    with pytest.raises(npp.NppError) as e:
+        p.execute([m], p.new_out())
+    assert e.value.status == npp.ERR_ALIGNMENT
+    # the scalar literal mapping accepts it
+    p1 = npp.Plan("SUM_ROWS", (1024, 1024), "f32", "TB_T")
+    out = p1.execute([m], p1.new_out())
+    torch.cuda.synchronize()
+    check("SUM_ROWS", m, out, "f32")
+
+
+def test_explicit_mappings(npp, cuda_device):
+    # Fig 9's mapping (DimY 64 x DimX 32 = 2048 threads) is rejected by the hard constraints
+    fig9 = dict(levels=[dict(dim=1, block=64, span=0), dict(dim=0, block=32, span=1)], vec=1)
+    with pytest.raises(npp.NppError) as e:
+        npp.Plan("SUM_ROWS", (8192, 8192), "f32", mapping=fig9)
+    assert e.value.status == npp.ERR_NO_FEASIBLE
+    # Split on a Map level is rejected
+    bad = dict(levels=[dict(dim=1, block=8, span=3, factor=2), dict(dim=0, block=32, span=1)], vec=1)
+    with pytest.raises(npp.NppError):
+        npp.Plan("SUM_ROWS", (1000, 1000), "f32", mapping=bad)
+    # the same mapping with 16 rows per block, Split(7) on the inner level, vector loads
+    ok = dict(levels=[dict(dim=1, block=16, span=2, factor=3), dict(dim=0, block=32, span=3, factor=7)], vec=4)
+    m = gen.uniform_f32(2, (1000, 1000), device=cuda_device)
+    p = npp.Plan("SUM_ROWS", (1000, 1000), "f32", mapping=ok)
+    assert p.mapping["levels"][1]["grid"] == 7 and p.workspace_bytes > 0
+    for _ in range(3):
+        out = p.execute([m], p.new_out())
+    torch.cuda.synchronize()
+    check("SUM_ROWS", m, out, "f32")
+    # sumCols with y-outer/x-inner Split over rows (strided inner on x)
+    m2 = gen.int_uniform(5, (5000, 300), -7, 7, device=cuda_device)
+    mp = dict(levels=[dict(dim=1, block=4, span=0), dict(dim=0, block=64, span=3, factor=5)], vec=1)
+    p = npp.Plan("SUM_COLS", (5000, 300), "i32", mapping=mp)
+    out = p.execute([m2], p.new_out())
+    torch.cuda.synchronize()
+    check("SUM_COLS", m2, out, "i32")
+
+
+def test_streams_and_concurrent_plans(npp, cuda_device):
+    shapes = [(4096, 4096), (16384, 512)]
+    ms = [gen.uniform_f32(20 + i, s, device=cuda_device) for i, s in enumerate(shapes)]
+    streams = [torch.cuda.Stream() for _ in shapes]
+    outs = []
+    for m, s, st in zip(ms, shapes, streams):
+        p = npp.Plan("SUM_COLS", s, "f32", "AUTO")
+        outs.append((p, p.execute([m], p.new_out(), stream=st)))
+    torch.cuda.synchronize()
+    for m, (p, out) in zip(ms, outs):
+        check("SUM_COLS", m, out, "f32")
+
+
+def test_weighted(npp, cuda_device):
+    for dtype in ("f32", "i32"):
+        for shape in [(1000, 999), (4096, 4096), (37, 70000)]:
+            m = _make(dtype, shape, 7, cuda_device)
+            for pattern, vlen in (("SUM_WEIGHTED_ROWS", shape[1]), ("SUM_WEIGHTED_COLS", shape[0])):
+                v = _make(dtype, (vlen,), 8, cuda_device) if dtype == "i32" else \
+                    gen.uniform_f32(8, (vlen,), device=cuda_device, lo=-1.0, scale=2.0)
+                for strategy in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
+                    p = npp.Plan(pattern, shape, dtype, strategy)
+                    out = p.execute([m, v], p.new_out())
+                    torch.cuda.synchronize()
+                    mn, vn = m.cpu().numpy(), v.cpu().numpy()
+                    if pattern == "SUM_WEIGHTED_ROWS":
+                        want = sums.sum_weighted_rows(mn, vn)
+                        scale = np.abs(mn.astype(np.float64)) @ np.abs(vn.astype(np.float64))
+                    else:
+                        want = sums.sum_weighted_cols(mn, vn)
+                        scale = np.abs(vn.astype(np.float64)) @ np.abs(mn.astype(np.float64))
+                    g = out.cpu().numpy()
+                    if dtype == "f32":
+                        assert np.all(np.abs(g - want) <= 1e-5 * scale), (pattern, shape, strategy)
+                    else:
+                        assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape)
