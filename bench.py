@@ -247,6 +247,7 @@ def main():
     ap.add_argument("--no-mappings", action="store_true", help="skip the baseline-mapping table")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg")
+    ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -262,32 +263,44 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=device)
     items, reduce_bufs, _ = WORKLOADS[args.workload](npp, gen, torch, rank, world, args.strategy, device)
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream(device=device)  # all timed work is enqueued on this stream
+    use_graph = world == 1 and not args.eager
 
-    def step(evs=None):
-        for i, it in enumerate(items):
-            if evs is not None:
-                evs[i].record(stream)
+    def step():
+        for it in items:
             it.run(stream)
-        if evs is not None:
-            evs[len(items)].record(stream)
         for b in reduce_bufs:
-            dist.all_reduce(b)
+            with torch.cuda.stream(stream):
+                dist.all_reduce(b)
 
-    for _ in range(max(3, args.warmup)):
-        step()
+    # one step = the six launches; at N=1 it is captured once into a CUDA graph and replayed, so the
+    # timed region holds the kernels back to back without host launch gaps (streams and graphs are
+    # the execution model here; at N>1 the NCCL all-reduce runs eagerly between the launches)
+    graph = None
+    if use_graph:
+        step()  # warm the lazy per-kernel setup outside the capture
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(stream):
+            with torch.cuda.graph(graph, stream=stream):
+                step()
+    run_step = graph.replay if graph is not None else step
+
+    with torch.cuda.stream(stream):
+        for _ in range(max(3, args.warmup)):
+            run_step()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(items) + 1)] for _ in range(args.steps)]
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     sampler = ClockSampler(local)
     with sampler:
-        torch.cuda.synchronize()
-        t_start.record(stream)
-        for k in range(args.steps):
-            step(evs[k])
-        t_end.record(stream)
+        with torch.cuda.stream(stream):
+            torch.cuda.synchronize()
+            t_start.record(stream)
+            for _ in range(args.steps):
+                run_step()
+            t_end.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -297,18 +310,20 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_total = float(t.item())
     ms_step = ms_total / args.steps
-    per_kernel_ms = [statistics.mean(evs[k][i].elapsed_time(evs[k][i + 1]) for k in range(args.steps))
-                     for i in range(len(items))]
     step_bytes = sum(it.bytes for it in items)
     value = step_bytes * world / (ms_step * 1e-3) / 1e9
+
+    # per-kernel durations: each launch replayed back to back from a graph, alternating its input with
+    # another equal-size buffer of the step so that every launch reads cold HBM
+    per_kernel_us = [kernel_us(torch, it, items[(i + 1) % len(items)], stream) for i, it in enumerate(items)]
     peak, peak_src = measured_peaks()
-    dom = max(range(len(items)), key=lambda i: per_kernel_ms[i])
-    dom_gbs = items[dom].bytes / (per_kernel_ms[dom] * 1e-3) / 1e9
+    dom = max(range(len(items)), key=lambda i: per_kernel_us[i])
+    dom_gbs = items[dom].bytes / (per_kernel_us[dom] * 1e-6) / 1e9
     traffic = ncu_traffic().get(items[dom].name)
-    per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9, 1),
-                           "frac_of_measured": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9 / peak, 4),
-                           "frac_of_8TBs": round(it.bytes / (per_kernel_ms[i] * 1e-3) / 1e9 / 8000.0, 4),
-                           "us": round(per_kernel_ms[i] * 1e3, 2),
+    per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9, 1),
+                           "frac_of_measured": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / peak, 4),
+                           "frac_of_8TBs": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / 8000.0, 4),
+                           "us": round(per_kernel_us[i], 2),
                            "mapping": mapping_brief(it.plan.mapping)}
                  for i, it in enumerate(items)}
 
@@ -316,18 +331,20 @@ def main():
            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
            "scaling": "weak" if args.workload == "paper" else "strong", "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (counter-based U[0,1) fp32, seeded)",
-           "config": config_for(args, "libnpp.so sm_100a"),
+           "config": config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
+                                else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),
            "per_shape": per_shape,
            "roofline": {"bound": "hbm", "kernel": items[dom].name, "achieved": round(dom_gbs, 1),
                         "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": round(dom_gbs / peak, 4),
-                        "traffic": traffic, "algorithmic_bytes": items[dom].bytes},
+                        "traffic": traffic, "algorithmic_bytes": items[dom].bytes,
+                        "duration_us": round(per_kernel_us[dom], 2)},
            "clocks": sampler.summary(),
            "gpu_launches": args.steps * sum(it.plan.launches for it in items)}
 
     # e2e: same metric through the C-ABI with HOST buffers (H2D of the inputs + D2H of the result inside)
     out["e2e"] = None if args.no_e2e else e2e_host(items, torch, stream, world, dist)
     if rank == 0 and not args.no_mappings and args.workload == "paper":
-        out["mappings"] = mapping_table(npp, torch, gen, device, stream)
+        out["mappings"] = mapping_table(npp, torch, gen, device, stream, items)
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(items)
     if rank == 0:
@@ -368,28 +385,49 @@ def e2e_host(items, torch, stream, world, dist, steps=3):
             "steps": steps, "api": "npp_execute_host (pinned host buffers, blocking)"}
 
 
-def mapping_table(npp, torch, gen, device, stream, iters=5):
-    """The paper's Fig 3 comparison on B200: every strategy at every paper shape (GB/s, events)."""
+def kernel_us(torch, item, other, stream, reps=8):
+    """Average duration of one launch of item's plan: a graph of 2*reps launches alternating item's
+    input with `other`'s (same byte size, viewed with item's shape) so no launch finds its input in L2."""
+    alt = other.ins[0].view(item.ins[0].shape) if other.ins[0].numel() == item.ins[0].numel() else None
+    inputs = [item.ins[0], alt] if alt is not None else [item.ins[0]]
+    with torch.cuda.stream(stream):
+        for x in inputs:
+            item.plan.execute([x], item.out, stream=stream)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(stream):
+        with torch.cuda.graph(g, stream=stream):
+            for r in range(2 * reps):
+                item.plan.execute([inputs[r % len(inputs)]], item.out, stream=stream)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        g.replay()
+        a.record(stream)
+        g.replay()
+        b.record(stream)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) * 1e3 / (2 * reps)
+
+
+def mapping_table(npp, torch, gen, device, stream, items):
+    """The paper's Fig 3 comparison on B200: every strategy at every paper shape (GB/s, graph-timed)."""
     table = {}
+    bufs = {}
+    for it in items:
+        bufs.setdefault(tuple(it.ins[0].shape), []).append(it.ins[0])
+    flat = [it.ins[0] for it in items]
     for si, (R, C) in enumerate(PAPER_SHAPES):
-        m = gen.uniform_f32(300 + 2 * si, (R, C), device=device)
+        m = bufs[(R, C)][0]
+        other = next(x for x in flat if x.data_ptr() != m.data_ptr() and x.numel() == m.numel())
         for pattern in ("SUM_ROWS", "SUM_COLS"):
             for strat in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
                 p = npp.Plan(pattern, (R, C), "f32", strat, device=device)
-                out = p.new_out()
-                for _ in range(2):
-                    p.execute([m], out, stream=stream)
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record(stream)
-                for _ in range(iters):
-                    p.execute([m], out, stream=stream)
-                b.record(stream)
-                torch.cuda.synchronize()
-                us = a.elapsed_time(b) * 1e3 / iters
-                gbs = (R * C * 4 + out.numel() * 4) / (us * 1e-6) / 1e9
+                item = Item(pattern, p, [m], p.new_out(), R * C * 4)
+                reps = 8 if strat in ("AUTO", "LITERAL", "WARP") else 2
+                us = kernel_us(torch, item, Item("o", p, [other], None, 0), stream, reps=reps)
+                gbs = (R * C * 4 + item.out.numel() * 4) / (us * 1e-6) / 1e9
                 table[f"{pattern.lower()}{_fmt_shape((R, C))}/{strat}"] = {
                     "GB/s": round(gbs, 1), "us": round(us, 1), "mapping": mapping_brief(p.mapping)}
-        del m
     return table
 
 

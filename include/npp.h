@@ -110,7 +110,7 @@ typedef struct {
   int32_t nlevels;
   int32_t kernel_class;
   int32_t vec;
-  int32_t reserved;
+  int32_t staged;  /* 1: TMA-staged tile family (S8, §V-B prefetch); 0: direct-load family */
   npp_level level[NPP_MAX_LEVELS];
   int64_t score;
   int64_t dop;
@@ -119,6 +119,7 @@ typedef struct {
   int32_t block[3];
   int32_t smem_bytes;
   int64_t workspace_bytes;
+  int64_t claim_tiles; /* staged plans: tiles a persistent block claims at a time (dynamic Span) */
 } npp_mapping;
 
 /* Hardware limits the selector's hard constraints and ControlDOP read (L658-662, L799-803).

@@ -283,8 +283,55 @@ def slots(lim, threads_per_block: int) -> int:
     return lim["sm_count"] * max(1, per_sm)
 
 
+STAGE_ROWS = 32                                   # DESIGN.md S8 (staged): BR
+
+
+def staged_eligible(nest, dtype, dims) -> bool:
+    """DESIGN.md S8: plain sums whose row pitch is a multiple of 16 B and whose stride-1 level is on x."""
+    pattern = nest["pattern"]
+    if pattern not in ("SUM_ROWS", "SUM_COLS"):
+        return False
+    C = nest["levels"][1][0] if pattern == "SUM_ROWS" else nest["levels"][0][0]
+    contig_level = 1 if pattern == "SUM_ROWS" else 0
+    return C % (16 // DTYPE_SIZE[dtype]) == 0 and dims[contig_level] == X
+
+
+def staged_tiles(nest, dtype):
+    """DESIGN.md S8 staged: tile shape (BR rows x BC cols = 32 KB) and tiles along outer / inner."""
+    esz = DTYPE_SIZE[dtype]
+    BR, BC = STAGE_ROWS, 1024 // esz
+    O, I = nest["levels"][0][0], nest["levels"][1][0]
+    if nest["pattern"] == "SUM_ROWS":
+        return BR, BC, cdiv(O, BR), cdiv(I, BC)
+    return BR, BC, cdiv(O, BC), cdiv(I, BR)
+
+
+def r2_staged(nest, dtype, lim):
+    """DESIGN.md S8, staged family: persistent blocks (one per SM) claim 32-row x 1 KB tiles in
+    outer-major order from a global counter, CL tiles per claim; the inner level is Split(Ti)."""
+    esz = DTYPE_SIZE[dtype]
+    BR, BC, To, Ti = staged_tiles(nest, dtype)
+    I = nest["levels"][1][0]
+    P = cdiv(To * Ti, min(lim["sm_count"], To * Ti))   # tiles per block: block b streams [bP, (b+1)P)
+    G = cdiv(To * Ti, P)
+    CL = P
+    if nest["pattern"] == "SUM_ROWS":
+        blocks = (8, 32)
+        spans = (SPAN_N, ALL if Ti == 1 else SPLIT)
+        factors = (4, Ti)
+        chunks = (BR, BC if Ti > 1 else I)
+        vec = 16 // esz
+    else:
+        blocks = (BC, 256 // BC)
+        spans = (ONE, ALL if Ti == 1 else SPLIT)
+        factors = (1, Ti)
+        chunks = (BC, BR if Ti > 1 else I)
+        vec = 1
+    return blocks, spans, factors, vec, chunks, G, CL
+
+
 def r2_sums(nest, dtype, lim, dims):
-    """DESIGN.md S8 for the 2-level sums: returns (blocks, spans, factors, vec, chunks)."""
+    """DESIGN.md S8 (unstaged) for the 2-level sums: returns (blocks, spans, factors, vec, chunks)."""
     pattern = nest["pattern"]
     O, I = nest["levels"][0][0], nest["levels"][1][0]
     C = I if pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS") else O
@@ -336,7 +383,8 @@ def kernel_class(pattern, dims):
     return RX if dims[1] == X else MX
 
 
-def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chunks=None):
+def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chunks=None, staged=0,
+                persistent_grid=None, claim_tiles=0):
     L = len(blocks)
     levels = []
     for l in range(L):
@@ -346,16 +394,20 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
         levels.append(dict(dim=dims[l], block=blocks[l], span=spans[l],
                            factor=(factors[l] if spans[l] in (SPAN_N, SPLIT) else 1),
                            chunk=ch, grid=cdiv(_eff(n), ch)))
-    grid = prod(lv["grid"] for lv in levels)
+    grid = prod(lv["grid"] for lv in levels) if persistent_grid is None else persistent_grid
     block3 = [1, 1, 1]
     for l in range(L):
         block3[dims[l]] = blocks[l]
-    rec = dict(nlevels=L, kernel_class=kernel_class(nest["pattern"], dims), vec=vec, levels=levels,
-               score=score_, dop=mapping_dop(nest, blocks, spans, factors),
+    rec = dict(nlevels=L, kernel_class=kernel_class(nest["pattern"], dims), vec=vec, staged=staged,
+               levels=levels, score=score_, dop=mapping_dop(nest, blocks, spans, factors),
                threads=grid * prod(blocks), grid=grid, block=block3,
-               smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0)
+               smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0, claim_tiles=claim_tiles)
     if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
-        if levels[1]["grid"] >= 2:
+        if staged:  # counters + fp64/integer accumulators [O] (S8 staged)
+            O = _eff(nest["levels"][0][0])
+            To = staged_tiles(nest, dtype)[2]   # tickets [To] u32, then accumulators [O]
+            rec["workspace_bytes"] = 256 * cdiv(4 * To, 256) + 256 * cdiv(O * acc_bytes(nest["pattern"], dtype), 256)
+        elif levels[1]["grid"] >= 2:
             O = _eff(nest["levels"][0][0])
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
@@ -386,5 +438,9 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
         raise Unsupported("AUTO needs known sizes")
     if L != 2:
         raise Unsupported("R2 for 3-level nests")
+    if staged_eligible(nest, dtype, dims):
+        b2, s2, f2, vec, chunks, G, CL = r2_staged(nest, dtype, lim)
+        return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks, staged=1,
+                           persistent_grid=G, claim_tiles=CL)
     b2, s2, f2, vec, chunks = r2_sums(nest, dtype, lim, dims)
     return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks)

@@ -45,15 +45,18 @@ def _needs_build(force: bool) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = False) -> str:
-    if not _needs_build(force):
+def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = False, defines=(), out=None) -> str:
+    """Compile libnpp.so. `defines`/`out` produce experiment variants (e.g. -DNPP_TMA_STAGES=6)."""
+    lib_out = out or LIB
+    if out is None and not defines and not _needs_build(force):
         return LIB
     nvcc = _nvcc()
-    os.makedirs(BUILD, exist_ok=True)
-    extra = ["-Xptxas", "-v"] if ptxas_verbose else []
+    build_dir = BUILD if not defines else os.path.join(BUILD, "variant_" + "_".join(d.strip("-D").replace("=", "") for d in defines))
+    os.makedirs(build_dir, exist_ok=True)
+    extra = (["-Xptxas", "-v"] if ptxas_verbose else []) + list(defines)
 
     def compile_one(src):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = [nvcc, *ARCH, *NVCC_FLAGS, *extra, "-c", src, "-o", obj]
         if src.endswith(".cpp"):
             cmd = ["g++", "-std=c++17", "-O3", "-fPIC", "-fvisibility=hidden", "-Wall", "-I", INCLUDE, "-I", CSRC,
@@ -67,15 +70,17 @@ def build(force: bool = False, verbose: bool = False, ptxas_verbose: bool = Fals
 
     with ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
         objs = list(ex.map(compile_one, sources()))
-    tmp = LIB + ".tmp"
+    tmp = lib_out + ".tmp"
     cmd = [nvcc, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", *objs, "-o", tmp]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed: {' '.join(cmd)}\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib_out)
+    return lib_out
 
 
 if __name__ == "__main__":
+    defs = [a for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a.split("=", 1)[1] for a in sys.argv[1:] if a.startswith("--out=")]
     print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv,
-                ptxas_verbose="--ptxas" in sys.argv))
+                ptxas_verbose="--ptxas" in sys.argv, defines=defs, out=outs[0] if outs else None))

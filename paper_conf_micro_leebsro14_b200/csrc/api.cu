@@ -8,6 +8,7 @@
 
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <string>
 
 #include "kernels.hpp"
@@ -120,6 +121,25 @@ int get_limits(const npp_limits* limits, npp_limits* out) {
 }
 
 inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+void debug_print_times(const unsigned long long* dbg, int G, cudaStream_t st) {
+  static unsigned long long h[4096 * 4];
+  if (G > 4096) return;
+  cudaStreamSynchronize(st);
+  cudaMemcpy(h, dbg, size_t(G) * 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+  unsigned long long t0 = ~0ull;
+  for (int b = 0; b < G; ++b) t0 = h[b * 4] < t0 ? h[b * 4] : t0;
+  double mx[3] = {0, 0, 0}, mn[3] = {1e30, 1e30, 1e30}, sm[3] = {0, 0, 0};
+  for (int b = 0; b < G; ++b)
+    for (int i = 0; i < 3; ++i) {
+      const double v = double(h[b * 4 + i] - t0) / 1e3;
+      mx[i] = v > mx[i] ? v : mx[i];
+      mn[i] = v < mn[i] ? v : mn[i];
+      sm[i] += v;
+    }
+  std::fprintf(stderr, "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] barrier[%.2f..%.2f]\n",
+               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], mx[2]);
+}
 
 }  // namespace
 
@@ -318,10 +338,10 @@ int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, vo
     set_error("this plan needs a workspace (npp_plan_workspace_bytes)");
     return NPP_ERR_WORKSPACE;
   }
-  if (m.vec > 1) {
+  if (m.vec > 1 || m.staged) {
     for (int k = 0; k < need; ++k)
       if (!aligned16(ins[k])) {
-        set_error("vectorised plan: inputs must be 16-byte aligned");
+        set_error("vectorised / TMA-staged plan: inputs must be 16-byte aligned");
         return NPP_ERR_ALIGNMENT;
       }
   }
@@ -332,6 +352,29 @@ int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, vo
   const bool rows = plan->pattern == NPP_SUM_ROWS || plan->pattern == NPP_SUM_WEIGHTED_ROWS;
   const bool weighted = plan->pattern == NPP_SUM_WEIGHTED_ROWS || plan->pattern == NPP_SUM_WEIGHTED_COLS;
   const int64_t R = plan->shape[0], C = plan->shape[1];
+  if (m.staged) {  // TMA tile family (S8 staged)
+    const npp::StagedTiling t = npp::staged_tiling(plan->pattern, R, C, plan->dtype);
+    npp::StagedArgs s{};
+    s.out = out;
+    s.R = R;
+    s.C = C;
+    s.O = rows ? R : C;
+    s.To = t.To;
+    s.Ti = t.Ti;
+    s.per_block = m.claim_tiles;
+    s.tickets = static_cast<unsigned*>(workspace);
+    s.acc = static_cast<char*>(workspace) + ((t.To * 4 + 255) / 256) * 256;
+    // measurement knob: NPP_DEBUG_TIMES=1 prints per-phase block timestamps (synchronises the stream)
+    static unsigned long long* dbg = nullptr;
+    const bool want_times = getenv("NPP_DEBUG_TIMES") != nullptr;
+    if (want_times && !dbg && cudaMalloc(&dbg, 4096 * 4 * sizeof(unsigned long long)) != cudaSuccess) dbg = nullptr;
+    s.dbg_times = want_times ? dbg : nullptr;
+    const int G = int(m.grid);
+    cudaError_t e = npp::launch_sum_staged(plan->dtype, rows, ins[0], s, G, st);
+    if (s.dbg_times && e == cudaSuccess) debug_print_times(dbg, G, st);
+    if (e != cudaSuccess) return cuda_fail("staged kernel launch", e);
+    return NPP_OK;
+  }
   npp::SumArgs a{};
   a.m = ins[0];
   a.v = weighted ? ins[1] : nullptr;

@@ -1,0 +1,346 @@
+// kern_sum_tma.cu — the staged (TMA) kernel family for sumRows / sumCols (S8, staged).
+//
+// PAPER.md §V-B: "Multiple threads in one dimension all read a contiguous chunk of the
+// data ... and store it in shared memory" so that both nest levels see coalesced memory. On sm_100a
+// the chunk is moved by the Tensor Memory Accelerator: one elected producer thread issues 2-D
+// cp.async.bulk.tensor copies of 32-row x 1 KB tiles into a 4-deep shared-memory ring (mbarrier
+// complete_tx) and eight consumer warps reduce each tile out of shared memory; 128 KB per SM stay in
+// flight, which holds HBM3e at its copy ceiling with one persistent block per SM.
+//
+//   RX (sumRows): warp w owns rows 4w..4w+3 of every 32-row band; a lane reads 2 x 16 B of each row
+//                 (conflict-free, contiguous per warp) and accumulates per row; shuffles finish a row.
+//   MX (sumCols): thread t owns column t of every 1 KB column tile (two row halves for 8-byte types)
+//                 and walks the rows of the band; the Map level stays on x as Fig 1 / P:L596-600 need.
+// Out-of-range rows/columns of edge tiles are zero-filled by TMA, which is the identity of +.
+//
+// Work split: the To x Ti tiles are taken in outer-major order and block b streams the contiguous
+// range [b*P, (b+1)*P), P = ceil(To*Ti / G) — every block moves the same bytes (to one tile) and walks
+// memory sequentially. Partial sums stay in registers while consecutive tiles share an outer tile.
+// An outer tile that lies inside one range is written directly; an outer tile cut by range
+// boundaries is the Split(k) of P:L542-550 across the k blocks that share it: each adds its partial
+// with one fp64 / integer atomic per output and takes a ticket, and the last of the k converts the
+// accumulators to the output type and zeroes them (the combiner of P:L880-883, fused, no second
+// launch, no grid barrier). Workspace: tickets [To] + accumulators [O], zero on entry and on exit.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <type_traits>
+
+#include "kernels.hpp"
+
+#ifndef NPP_TMA_STAGES
+#define NPP_TMA_STAGES 4
+#endif
+
+namespace npp {
+
+namespace {
+
+constexpr int kStages = NPP_TMA_STAGES;
+constexpr int kTileRows = 32;
+constexpr int kTileBytes = kTileRows * 1024;
+constexpr int kConsumerWarps = 8;
+constexpr int kConsumers = kConsumerWarps * 32;
+constexpr int kThreads = kConsumers + 32;  // + one producer warp
+constexpr int kSmemHeader = 1024;          // mbarriers + per-slot tile ids; tiles start 1 KB-aligned
+constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes;
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+  return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n NPP_WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra NPP_WAIT_%=;\n}" ::"r"(smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+template <typename T> struct SOps;
+template <> struct SOps<float> {
+  using Acc = double;
+  __device__ static float finish(double a) { return float(a); }
+};
+template <> struct SOps<int32_t> {
+  using Acc = unsigned int;
+  __device__ static int32_t finish(unsigned a) { return int32_t(a); }
+};
+template <> struct SOps<int64_t> {
+  using Acc = unsigned long long;
+  __device__ static int64_t finish(unsigned long long a) { return int64_t(a); }
+};
+
+// sum of one 16-byte vector: fp32 pairwise for floats, exact unsigned for integers
+__device__ __forceinline__ float vsum(const float4& v) { return (v.x + v.y) + (v.z + v.w); }
+__device__ __forceinline__ unsigned vsum(const int4& v) {
+  return unsigned(v.x) + unsigned(v.y) + unsigned(v.z) + unsigned(v.w);
+}
+__device__ __forceinline__ unsigned long long vsum(const longlong2& v) {
+  return (unsigned long long)v.x + (unsigned long long)v.y;
+}
+template <typename T> struct V16;
+template <> struct V16<float> { using type = float4; };
+template <> struct V16<int32_t> { using type = int4; };
+template <> struct V16<int64_t> { using type = longlong2; };
+
+template <typename A>
+__device__ __forceinline__ A warp_sum(A v) {
+#pragma unroll
+  for (int off = 16; off >= 1; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+  return v;
+}
+
+// read-and-zero of one accumulator (only the last contributor of an outer tile calls this)
+__device__ __forceinline__ double take(double* p) {
+  return __longlong_as_double((long long)atomicExch(reinterpret_cast<unsigned long long*>(p), 0ull));
+}
+__device__ __forceinline__ unsigned take(unsigned* p) { return atomicExch(p, 0u); }
+__device__ __forceinline__ unsigned long long take(unsigned long long* p) { return atomicExch(p, 0ull); }
+
+}  // namespace
+
+template <typename T, bool ROWS>
+__global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_constant__ CUtensorMap map,
+                                                                  StagedArgs a) {
+  using Acc = typename SOps<T>::Acc;
+  using V = typename V16<T>::type;
+  constexpr int BC = 1024 / int(sizeof(T));            // tile columns
+  constexpr int OUT_PER_TILE = ROWS ? kTileRows : BC;  // outputs of one outer tile
+  extern __shared__ __align__(1024) unsigned char smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
+  uint64_t* empty = full + kStages;
+  long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);  // tile id, bit 62: flush after
+  unsigned* s_last = reinterpret_cast<unsigned*>(slot_tile + kStages);
+  unsigned char* tiles = smem + kSmemHeader;
+  Acc* accg = static_cast<Acc*>(a.acc);
+  constexpr long long kFlush = 1ll << 62;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long bid = blockIdx.x;
+  const long long total = a.To * a.Ti;
+  const long long P = a.per_block;
+  const long long r0 = bid * P, r1 = (total < r0 + P) ? total : r0 + P;  // my tile range
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kStages; ++i) {
+      mbar_init(full + i, 1);
+      mbar_init(empty + i, kConsumerWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (a.dbg_times) {
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      a.dbg_times[bid * 4 + 0] = gtimer();
+      a.dbg_times[bid * 4 + 3] = smid;
+    }
+  }
+  __syncthreads();
+
+  if (warp == kConsumerWarps) {
+    // ------------------------------------------------------------ producer: one elected lane
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&map) : "memory");
+      long long t = 0;
+      for (long long cur = r0; cur < r1; ++cur, ++t) {
+        const bool flush = cur + 1 >= r1 || ((cur + 1) / a.Ti) != (cur / a.Ti);
+        const int slot = int(t % kStages);
+        if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
+        slot_tile[slot] = cur | (flush ? kFlush : 0);
+        mbar_expect_tx(full + slot, kTileBytes);
+        const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
+        const int x = int(ROWS ? it * BC : ot * BC);
+        const int y = int(ROWS ? ot * kTileRows : it * kTileRows);
+        tma_load_2d(tiles + slot * kTileBytes, &map, x, y, full + slot);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ consumers
+    constexpr int kGroups = ROWS ? 1 : 256 / BC;   // MX row groups (1 for 4-byte types, 2 for 8-byte)
+    constexpr int kRowsPer = kTileRows / kGroups;  // MX rows of a tile one thread adds
+    const int col = threadIdx.x % BC;
+    const int rg = threadIdx.x / BC;
+    Acc acc[4] = {0, 0, 0, 0};  // RX: rows 4w..4w+3; MX: acc[0] = column col
+    const long long n_tiles = r1 - r0;
+    for (long long t = 0; t < n_tiles; ++t) {
+      const int slot = int(t % kStages);
+      mbar_wait(full + slot, unsigned((t / kStages) & 1));
+      const long long tag = slot_tile[slot];
+      const unsigned char* tile = tiles + slot * kTileBytes;
+      if constexpr (ROWS) {
+#pragma unroll
+        for (int rr = 0; rr < 4; ++rr) {
+          const unsigned char* row = tile + (warp * 4 + rr) * 1024;
+          const V v0 = *reinterpret_cast<const V*>(row + lane * 16);
+          const V v1 = *reinterpret_cast<const V*>(row + 512 + lane * 16);
+          acc[rr] += Acc(vsum(v0) + vsum(v1));
+        }
+      } else {
+        const T* tt = reinterpret_cast<const T*>(tile);
+        T v[kRowsPer];
+#pragma unroll
+        for (int rr = 0; rr < kRowsPer; ++rr) v[rr] = tt[(rg * kRowsPer + rr) * BC + col];
+        if constexpr (std::is_same<T, float>::value) {  // fp32: pairwise tree inside the tile
+#pragma unroll
+          for (int w = kRowsPer / 2; w >= 1; w /= 2)
+#pragma unroll
+            for (int i = 0; i < w; ++i) v[i] = v[i] + v[i + w];
+          acc[0] += Acc(v[0]);
+        } else {
+#pragma unroll
+          for (int rr = 0; rr < kRowsPer; ++rr) acc[0] += Acc(v[rr]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(empty + slot);
+      if (!(tag & kFlush)) continue;
+
+      // ---- flush the partial of outer tile ot
+      const long long ot = (tag & ~kFlush) / a.Ti;
+      const long long f0 = ot * a.Ti, f1 = (total < f0 + a.Ti) ? total : f0 + a.Ti;  // tiles of ot
+      const bool owned = f0 >= r0 && f1 <= r1;
+      long long oidx[4];
+      Acc val[4];
+      bool mine[4];
+      if constexpr (ROWS) {
+#pragma unroll
+        for (int rr = 0; rr < 4; ++rr) {
+          val[rr] = warp_sum(acc[rr]);
+          oidx[rr] = ot * kTileRows + warp * 4 + rr;
+          mine[rr] = lane == rr && oidx[rr] < a.R;
+          acc[rr] = 0;
+        }
+      } else {
+        val[0] = acc[0];
+        oidx[0] = ot * BC + col;
+        mine[0] = oidx[0] < a.C;
+        acc[0] = 0;
+      }
+      constexpr int NV = ROWS ? 4 : 1;
+      if (owned) {
+#pragma unroll
+        for (int i = 0; i < NV; ++i)
+          if (mine[i]) {
+            if (kGroups == 1) {
+              static_cast<T*>(a.out)[oidx[i]] = SOps<T>::finish(val[i]);
+            } else {
+              atomicAdd(accg + oidx[i], val[i]);  // two row halves meet in the accumulator
+            }
+          }
+        if (kGroups == 1) continue;
+      } else {
+#pragma unroll
+        for (int i = 0; i < NV; ++i)
+          if (mine[i]) atomicAdd(accg + oidx[i], val[i]);
+      }
+      // ticket: the last of the blocks (or row halves) contributing to ot converts its outputs
+      __threadfence();
+      consumers_sync();
+      if (threadIdx.x == 0) {
+        const long long b_first = f0 / P, b_last = (f1 - 1) / P;
+        const unsigned contributors = unsigned(b_last - b_first + 1);
+        const unsigned prev = atomicAdd(a.tickets + ot, 1u);
+        *s_last = (prev + 1 == contributors) ? 1u : 0u;
+        if (prev + 1 == contributors) a.tickets[ot] = 0u;
+      }
+      consumers_sync();
+      if (*s_last) {
+        __threadfence();
+        const long long o0 = ot * OUT_PER_TILE;
+        const long long oend = ROWS ? a.R : a.C;
+        for (int j = threadIdx.x; j < OUT_PER_TILE; j += kConsumers) {
+          const long long o = o0 + j;
+          if (o < oend) static_cast<T*>(a.out)[o] = SOps<T>::finish(take(accg + o));
+        }
+      }
+      consumers_sync();
+    }
+  }
+  if (a.dbg_times && threadIdx.x == 0) a.dbg_times[bid * 4 + 1] = gtimer();
+}
+
+// ====================================================================================== host side
+namespace {
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return static_cast<EncodeTiledFn>(nullptr);
+    return reinterpret_cast<EncodeTiledFn>(p);
+  }();
+  return fn;
+}
+
+template <typename T, bool ROWS>
+cudaError_t launch_typed(const CUtensorMap& map, const StagedArgs& a, int grid, cudaStream_t st) {
+  static bool attr_set = false;
+  auto kern = npp_sum_tma_kernel<T, ROWS>;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  kern<<<grid, kThreads, kSmemBytes, st>>>(map, a);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st) {
+  EncodeTiledFn encode = encode_fn();
+  if (!encode) return cudaErrorNotSupported;
+  const int esz = dtype == NPP_I64 ? 8 : 4;
+  CUtensorMap map;
+  const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
+  const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
+  const cuuint32_t box[2] = {cuuint32_t(1024 / esz), cuuint32_t(kTileRows)};
+  const cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapDataType dt = dtype == NPP_F32   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                 : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
+                                                    : CU_TENSOR_MAP_DATA_TYPE_INT64;
+  CUresult r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  switch (dtype) {
+    case NPP_F32:
+      return rows ? launch_typed<float, true>(map, a, grid, st) : launch_typed<float, false>(map, a, grid, st);
+    case NPP_I32:
+      return rows ? launch_typed<int32_t, true>(map, a, grid, st) : launch_typed<int32_t, false>(map, a, grid, st);
+    default:
+      return rows ? launch_typed<int64_t, true>(map, a, grid, st) : launch_typed<int64_t, false>(map, a, grid, st);
+  }
+}
+
+}  // namespace npp

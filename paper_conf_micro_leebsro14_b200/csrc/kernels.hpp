@@ -27,4 +27,19 @@ struct SumArgs {
 cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumArgs& a, cudaStream_t st);
 int sum_kernels_max_regs();
 
+// Arguments of one staged (TMA) sum launch (S8 staged): the matrix is [R x C]; tiles are
+// 32 rows x 1 KB, To x Ti of them in outer-major order; persistent blocks claim `claim` tiles at a time.
+struct StagedArgs {
+  void* out;
+  void* acc;           // [O] accumulators (fp64 / u32 / u64), zero on entry and on exit
+  unsigned* tickets;   // [To] contributor tickets of outer tiles cut by range boundaries, zero on entry/exit
+  int64_t O;           // outputs: R (sumRows) or C (sumCols)
+  int64_t R, C;
+  int64_t To, Ti;      // tiles along the outer / inner level
+  int64_t per_block;   // P: block b streams tiles [b*P, (b+1)*P) of the outer-major order
+  unsigned long long* dbg_times;  // measurement knob (NPP_DEBUG_TIMES): [grid x 4] globaltimer stamps
+};
+
+cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st);
+
 }  // namespace npp

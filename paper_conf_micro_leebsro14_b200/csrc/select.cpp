@@ -203,7 +203,46 @@ int64_t slots(const npp_limits& lim, int threads_per_block) {
   return int64_t(lim.sm_count) * per_sm;
 }
 
-// S8 for the 2-level sums: keep LITERAL's dims, re-choose blocks / vec / factors / chunks.
+// S8 staged family: plain sums, 16-B row pitch, stride-1 level of m on x.
+bool staged_eligible(const Nest& n, int dtype, const Choice& c) {
+  if (n.pattern != NPP_SUM_ROWS && n.pattern != NPP_SUM_COLS) return false;
+  const int contig_level = n.pattern == NPP_SUM_ROWS ? 1 : 0;
+  return n.cols % (16 / dtype_size(dtype)) == 0 && c.dims[contig_level] == NPP_DIM_X;
+}
+
+// S8 staged family: persistent blocks (one per SM) claim 32-row x 1 KB tiles in outer-major order
+// from a global counter, claim_tiles at a time; the inner level is Split(Ti).
+void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
+  const bool rows = n.pattern == NPP_SUM_ROWS;
+  const int64_t R = rows ? n.N[0] : n.N[1];
+  const StagedTiling t = staged_tiling(n.pattern, R, n.cols, dtype);
+  const int64_t tiles = t.To * t.Ti;
+  const int64_t per_block = cdiv(tiles, std::min<int64_t>(lim.sm_count, tiles));  // P
+  c->claim_tiles = per_block;
+  c->persistent_grid = cdiv(tiles, per_block);
+  c->staged = 1;
+  if (rows) {
+    c->blocks[0] = 8;
+    c->blocks[1] = 32;
+    c->spans[0] = NPP_SPAN_N;
+    c->factors[0] = 4;
+    c->chunks[0] = t.BR;
+    c->chunks[1] = t.Ti > 1 ? t.BC : n.N[1];
+    c->vec = 16 / dtype_size(dtype);
+  } else {
+    c->blocks[0] = int(t.BC);
+    c->blocks[1] = int(256 / t.BC);
+    c->spans[0] = NPP_SPAN_ONE;
+    c->factors[0] = 1;
+    c->chunks[0] = t.BC;
+    c->chunks[1] = t.Ti > 1 ? t.BR : n.N[1];
+    c->vec = 1;
+  }
+  c->spans[1] = t.Ti == 1 ? NPP_SPAN_ALL : NPP_SPLIT_K;
+  c->factors[1] = t.Ti;
+}
+
+// S8 (unstaged) for the 2-level sums: keep LITERAL's dims, re-choose blocks / vec / factors / chunks.
 void r2_sums(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const bool rows = n.pattern == NPP_SUM_ROWS || n.pattern == NPP_SUM_WEIGHTED_ROWS;
   const int64_t O = n.N[0], I = n.N[1], C = n.cols;
@@ -268,6 +307,20 @@ int kernel_class_of(const Nest& n, const Choice& c) {
 thread_local std::string g_error;
 
 void set_error(const std::string& msg) { g_error = msg; }
+
+StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
+  StagedTiling t;
+  t.BR = kStageRows;
+  t.BC = 1024 / dtype_size(dtype);
+  if (pattern == NPP_SUM_ROWS) {
+    t.To = cdiv(R, t.BR);
+    t.Ti = cdiv(C, t.BC);
+  } else {
+    t.To = cdiv(C, t.BC);
+    t.Ti = cdiv(R, t.BR);
+  }
+  return t;
+}
 
 int dtype_size(int dtype) { return dtype == NPP_I64 ? 8 : 4; }
 
@@ -437,13 +490,20 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   }
   m.score = score_value;
   m.dop = mapping_dop(n, c);
+  if (c.persistent_grid > 0) grid = c.persistent_grid;  // staged: persistent blocks, dynamic tiles
   m.grid = grid;
   m.threads = grid * tb;
   m.block[0] = m.block[1] = m.block[2] = 1;
   for (int l = 0; l < n.L; ++l) m.block[c.dims[l]] = c.blocks[l];
   m.smem_bytes = int32_t(smem_model(n, dtype, c));
   m.workspace_bytes = 0;
-  if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
+  m.staged = c.staged;
+  m.claim_tiles = c.claim_tiles;
+  if (is_sum_pattern(n.pattern) && c.staged) {
+    // counters (claim, barrier) + accumulators [O] of the accumulator type
+    const StagedTiling t = staged_tiling(n.pattern, n.pattern == NPP_SUM_ROWS ? n.N[0] : n.N[1], n.cols, dtype);
+    m.workspace_bytes = 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
+  } else if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
     const int64_t part = m.level[1].grid * eff(n.N[0]) * acc_bytes(n.pattern, dtype);
     const int64_t tick = m.level[0].grid * 4;
     m.workspace_bytes = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256);
@@ -499,7 +559,10 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
     set_error("R2 runtime step for 3-level nests is not implemented in this build");
     return NPP_ERR_UNSUPPORTED;
   }
-  r2_sums(n, dtype, lim, &c);
+  if (staged_eligible(n, dtype, c))
+    r2_staged(n, dtype, lim, &c);
+  else
+    r2_sums(n, dtype, lim, &c);
   return record_from_choice(n, dtype, lim, c, sc, out);
 }
 

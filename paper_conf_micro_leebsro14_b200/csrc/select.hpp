@@ -34,7 +34,19 @@ struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refi
   int64_t factors[kMaxLevels] = {1, 1, 1};
   int64_t chunks[kMaxLevels] = {0, 0, 0};  // 0 = derive from span/factor (S9)
   int vec = 1;
+  int staged = 0;  // 1: TMA-staged tile family (S8)
+  int64_t persistent_grid = 0;  // staged: blocks launched (0: product of the level grids)
+  int64_t claim_tiles = 0;      // staged: tiles per dynamic claim
 };
+
+constexpr int kStageRows = 32;  // BR of the staged family (S8): tiles of 32 rows x 1 KB
+
+// S8 staged-family tiling shared with the kernels: tile counts of the outer / inner level.
+struct StagedTiling {
+  int64_t BR, BC;   // tile rows, tile columns
+  int64_t To, Ti;   // tiles along the outer / inner level
+};
+StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype);
 
 // thread-local error message shared with the API layer
 void set_error(const std::string& msg);

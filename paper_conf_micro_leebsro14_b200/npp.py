@@ -12,7 +12,7 @@ import os
 import torch
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libnpp.so")
+LIB_PATH = os.environ.get("NPP_LIB_PATH") or os.path.join(_PKG, "libnpp.so")  # override: experiment builds
 
 # enums (include/npp.h)
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_ALIGNMENT, ERR_WORKSPACE, ERR_NO_FEASIBLE, ERR_CUDA = 0, -1, -2, -3, -4, -5, -6
@@ -39,10 +39,10 @@ class Level(ctypes.Structure):
 
 class Mapping(ctypes.Structure):
     _fields_ = [("nlevels", ctypes.c_int32), ("kernel_class", ctypes.c_int32), ("vec", ctypes.c_int32),
-                ("reserved", ctypes.c_int32), ("level", Level * 4), ("score", ctypes.c_int64),
+                ("staged", ctypes.c_int32), ("level", Level * 4), ("score", ctypes.c_int64),
                 ("dop", ctypes.c_int64), ("threads", ctypes.c_int64), ("grid", ctypes.c_int64),
                 ("block", ctypes.c_int32 * 3), ("smem_bytes", ctypes.c_int32),
-                ("workspace_bytes", ctypes.c_int64)]
+                ("workspace_bytes", ctypes.c_int64), ("claim_tiles", ctypes.c_int64)]
 
 
 class Limits(ctypes.Structure):
@@ -125,9 +125,10 @@ def mapping_to_dict(m: Mapping) -> dict:
     levels = [dict(dim=m.level[i].dim, block=m.level[i].block, span=m.level[i].span,
                    factor=m.level[i].factor, chunk=m.level[i].chunk, grid=m.level[i].grid)
               for i in range(m.nlevels)]
-    return dict(nlevels=m.nlevels, kernel_class=m.kernel_class, vec=m.vec, levels=levels, score=m.score,
+    return dict(nlevels=m.nlevels, kernel_class=m.kernel_class, vec=m.vec, staged=m.staged, levels=levels,
+                score=m.score,
                 dop=m.dop, threads=m.threads, grid=m.grid, block=list(m.block), smem_bytes=m.smem_bytes,
-                workspace_bytes=m.workspace_bytes)
+                workspace_bytes=m.workspace_bytes, claim_tiles=m.claim_tiles)
 
 
 def mapping_from_dict(d: dict) -> Mapping:

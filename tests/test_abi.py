@@ -32,7 +32,7 @@ def test_library_exports_every_declared_symbol():
 def test_struct_layout_matches_binding():
     from paper_conf_micro_leebsro14_b200 import npp
     assert ctypes.sizeof(npp.Level) == 40
-    assert ctypes.sizeof(npp.Mapping) == 16 + 4 * 40 + 32 + 12 + 4 + 8
+    assert ctypes.sizeof(npp.Mapping) == 16 + 4 * 40 + 32 + 12 + 4 + 8 + 8
     assert ctypes.sizeof(npp.Limits) == 4 * 12 + 8
     assert npp.lib().npp_version() == 1
     assert set(npp.EXPORTS) == set(declared_symbols())

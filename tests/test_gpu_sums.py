@@ -102,7 +102,9 @@ def test_paper_shapes_full(npp, cuda_device, shape):
             out2 = p.execute([m], p.new_out())   # workspace reuse: tickets were reset
             torch.cuda.synchronize()
             check(pattern, m, out, "f32")
-            assert torch.equal(out, out2), "non-deterministic or stale workspace"
+            # workspace reuse leaves no stale state; cut tiles add fp64 partials in arrival order, so
+            # an fp32 output may differ by one ulp near a rounding tie (S8 staged note)
+            assert torch.all((out - out2).abs() <= out.abs() * 2.0 ** -23), "stale workspace"
 
 
 def test_large_sumcols_sampled(npp, cuda_device):
