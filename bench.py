@@ -156,7 +156,28 @@ def build_sumcols_1m4k(npp, gen, torch, rank, world, strategy, device):
     return items, ([out] if world > 1 else []), "sumCols fp32 [1M,4K] row-sharded + NCCL all-reduce (strong)"
 
 
-WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k}
+def build_kmeans(npp, gen, torch, rank, world, strategy, device):
+    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids; points sharded over ranks (weak)
+    N, D, K = 1 << 22, 64, 32
+    x, c = gen.kmeans_inputs(N, D, K, row_offset=rank * N, device=device)
+    plan = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", strategy, device=device)
+    item = Item("kmeans_assign[4M,64,32]", plan, [x, c], plan.new_out(), N * D * 4 + K * D * 4 + N * 4)
+    item.flops = 2 * N * K * D  # the x·c FMAs of the expanded distance
+    return [item], [], "k-means assignment 4M x 64 x 32"
+
+
+def build_logreg(npp, gen, torch, rank, world, strategy, device):
+    # BASELINE.json config 5: [16M, 256] fp32 in B = 4096 mini-batches of 4096 rows; batches sharded
+    B, Rb, C = 4096 // world, 4096, 256
+    x, y, w = gen.logreg_inputs(B, Rb, C, seed=6, batch_offset=rank * B, device=device)
+    plan = npp.Plan("LOGREG_GRAD", (B, Rb, C), "f32", strategy, device=device)
+    item = Item(f"logreg_grad[{B * Rb // 1048576}M,256]", plan, [x, y, w], plan.new_out(),
+                B * Rb * C * 4 + B * Rb * 4 + C * 4 + B * C * 4)
+    return [item], [], "batched logistic-regression gradient [16M,256], B=4096"
+
+
+WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
+             "logreg": build_logreg}
 
 
 # ------------------------------------------------------------------------- reference arm (the oracle)
@@ -202,10 +223,11 @@ def run_reference(args):
 
 
 def config_for(args, extra):
-    if args.workload == "paper":
-        wl = "sumRows+sumCols fp32 @ [64K,1K],[8K,8K],[1K,64K] (paper shapes, BASELINE.json configs[1])"
-    else:
-        wl = "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])"
+    wl = {"paper": "sumRows+sumCols fp32 @ [64K,1K],[8K,8K],[1K,64K] (paper shapes, BASELINE.json configs[1])",
+          "sumcols_1m4k": "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])",
+          "kmeans": "k-means assignment 4M x 64 x 32 fp32, points sharded (BASELINE.json configs[3])",
+          "logreg": "batched logreg gradient [16M,256] fp32, B=4096, batches sharded (BASELINE.json configs[4])",
+          }[args.workload]
     return {"workload": wl, "strategy": args.strategy, "impl_detail": extra,
             "parallelism": f"row shards x{args.gpus}",
             "l2": "inputs larger than L2 (distinct 256 MiB buffers per launch, 1.5 GiB per step); no flush"}
@@ -214,24 +236,42 @@ def config_for(args, extra):
 # ------------------------------------------------------------------------- CPU baseline (oracle, bounded)
 
 def cpu_baseline(items, budget_s=12.0):
-    import numpy as np  # noqa: F401
+    """The oracle as it stands, on the host's cores, over a bounded sample of the same workload."""
+    import numpy as np
+    from oracle import kmeans as okm
+    from oracle import logreg as olr
     from oracle import sums
     done_bytes, t_total, n = 0, 0.0, 0
     samples = []
     for it in items:
-        m = it.ins[0].cpu().numpy()
-        samples.append((it.name, m))
+        if it.name.startswith("kmeans"):  # first 256K points (the oracle is O(N K D) in fp64)
+            samples.append((it.name, [it.ins[0][: 1 << 18].cpu().numpy(), it.ins[1].cpu().numpy()]))
+        elif it.name.startswith("logreg"):  # first 64 batches
+            Rb = it.plan.shape[1]
+            rows = 64 * Rb
+            samples.append((it.name, [it.ins[0][:rows].cpu().numpy(), it.ins[1][:rows].cpu().numpy(),
+                                      it.ins[2].cpu().numpy()]))
+        else:
+            samples.append((it.name, [it.ins[0].cpu().numpy()]))
+
+    def run(name, arrs):
+        if name.startswith("kmeans"):
+            okm.assign(*arrs)
+        elif name.startswith("logreg"):
+            olr.grad(arrs[0], arrs[1], arrs[2], 64)
+        else:
+            (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(arrs[0])
     t_end = time.perf_counter() + budget_s
     while time.perf_counter() < t_end:
-        for name, m in samples:
+        for name, arrs in samples:
             t0 = time.perf_counter()
-            (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(m)
+            run(name, arrs)
             t_total += time.perf_counter() - t0
-            done_bytes += m.size * 4
+            done_bytes += sum(x.nbytes for x in arrs)
             n += 1
     return {"value": round(done_bytes / t_total / 1e9, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} oracle sums over the step's full matrices ({len(samples)} per pass), "
-                      f"{t_total:.1f} s of single-threaded NumPy fp64"}
+            "sample": f"{n} oracle calls over the step's inputs ({len(samples)} per pass; k-means: first 256K "
+                      f"points, logreg: first 64 batches), {t_total:.1f} s of single-threaded NumPy fp64"}
 
 
 # ------------------------------------------------------------------------- main arm
@@ -320,6 +360,7 @@ def main():
     dom = max(range(len(items)), key=lambda i: per_kernel_us[i])
     dom_gbs = items[dom].bytes / (per_kernel_us[dom] * 1e-6) / 1e9
     traffic = ncu_traffic().get(items[dom].name)
+    flops = getattr(items[dom], "flops", None)
     per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9, 1),
                            "frac_of_measured": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / peak, 4),
                            "frac_of_8TBs": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / 8000.0, 4),
@@ -334,10 +375,7 @@ def main():
            "config": config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
                                 else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),
            "per_shape": per_shape,
-           "roofline": {"bound": "hbm", "kernel": items[dom].name, "achieved": round(dom_gbs, 1),
-                        "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": round(dom_gbs / peak, 4),
-                        "traffic": traffic, "algorithmic_bytes": items[dom].bytes,
-                        "duration_us": round(per_kernel_us[dom], 2)},
+           "roofline": roofline(items[dom], per_kernel_us[dom], dom_gbs, peak, peak_src, traffic, flops),
            "clocks": sampler.summary(),
            "gpu_launches": args.steps * sum(it.plan.launches for it in items)}
 
@@ -354,6 +392,20 @@ def main():
     return 0
 
 
+def roofline(item, us, gbs, peak, peak_src, traffic, flops):
+    base = {"kernel": item.name, "traffic": traffic, "algorithmic_bytes": item.bytes, "duration_us": round(us, 2),
+            "hbm_GBps": round(gbs, 1), "hbm_frac_of_measured": round(gbs / peak, 4)}
+    if flops:  # FP32 FMA-bound (k-means): peak = 148 SMs x 128 FP32 lanes x 2 flop x 1965 MHz
+        alu_peak = 148 * 128 * 2 * 1.965e9 / 1e12
+        achieved = flops / (us * 1e-6) / 1e12
+        return dict(base, bound="alu", achieved=round(achieved, 2), peak=round(alu_peak, 2), unit="TFLOP/s",
+                    frac=round(achieved / alu_peak, 4),
+                    peak_source="derived: 148 SM x 128 FP32 FMA/clk x 2 x 1965 MHz (guide unit counts)",
+                    algorithmic_flops=flops)
+    return dict(base, bound="hbm", achieved=round(gbs, 1), peak=peak, peak_source=peak_src, unit="GB/s",
+                frac=round(gbs / peak, 4))
+
+
 def mapping_brief(m):
     sp = {0: "Span(1)", 1: "Span(all)", 2: "Span(n)", 3: "Split(k)"}
     dims = "xyz"
@@ -362,14 +414,14 @@ def mapping_brief(m):
 
 
 def e2e_host(items, torch, stream, world, dist, steps=3):
-    host_ins = [it.ins[0].cpu().pin_memory() for it in items]
+    host_ins = [[x.cpu().pin_memory() for x in it.ins] for it in items]
     host_outs = [torch.empty(it.out.shape, dtype=it.out.dtype).pin_memory() for it in items]
-    h2d = sum(h.numel() * h.element_size() for h in host_ins)
+    h2d = sum(h.numel() * h.element_size() for hs in host_ins for h in hs)
     d2h = sum(h.numel() * h.element_size() for h in host_outs)
 
     def one():
         for it, hi, ho in zip(items, host_ins, host_outs):
-            it.plan.execute_host([hi], ho, it.ins, it.out, stream=stream)
+            it.plan.execute_host(hi, ho, it.ins, it.out, stream=stream)
     one()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
@@ -389,16 +441,17 @@ def kernel_us(torch, item, other, stream, reps=8):
     """Average duration of one launch of item's plan: a graph of 2*reps launches alternating item's
     input with `other`'s (same byte size, viewed with item's shape) so no launch finds its input in L2."""
     alt = other.ins[0].view(item.ins[0].shape) if other.ins[0].numel() == item.ins[0].numel() else None
-    inputs = [item.ins[0], alt] if alt is not None else [item.ins[0]]
+    firsts = [item.ins[0], alt] if alt is not None and alt.data_ptr() != item.ins[0].data_ptr() else [item.ins[0]]
+    inputs = [[f] + list(item.ins[1:]) for f in firsts]
     with torch.cuda.stream(stream):
         for x in inputs:
-            item.plan.execute([x], item.out, stream=stream)
+            item.plan.execute(x, item.out, stream=stream)
     torch.cuda.synchronize()
     g = torch.cuda.CUDAGraph()
     with torch.cuda.stream(stream):
         with torch.cuda.graph(g, stream=stream):
             for r in range(2 * reps):
-                item.plan.execute([inputs[r % len(inputs)]], item.out, stream=stream)
+                item.plan.execute(inputs[r % len(inputs)], item.out, stream=stream)
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with torch.cuda.stream(stream):
         g.replay()

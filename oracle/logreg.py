@@ -55,12 +55,12 @@ def grad(x: np.ndarray, y: np.ndarray, w: np.ndarray, B: int, chunk_batches: int
     return out
 
 
-def grad_abs_scale(x: np.ndarray, y: np.ndarray, w: np.ndarray, B: int) -> np.ndarray:
-    """Σ_i |x_ij|·(|e_i| + |Σ_k x_ik w_k|·2^-14): the scale of the fp32 tolerance."""
+def grad_scales(x: np.ndarray, y: np.ndarray, w: np.ndarray, B: int):
+    """(Σ_i |x_ij e_i|, Σ_i |x_ij|) per (b, j): the two scales of the fp32 tolerance of DESIGN.md §5
+    (relative error of the accumulated terms, and the absolute error of each fp32 residual e_i)."""
     n, C = x.shape
     Rb = n // B
     x64 = np.abs(x.astype(np.float64))
     e = np.abs(residuals(x, y, w))
-    zabs = x64 @ np.abs(w.astype(np.float64))
-    s = e + zabs * 2.0 ** -14
-    return np.add.reduce((x64 * s[:, None]).reshape(B, Rb, C), axis=1)
+    return (np.add.reduce((x64 * e[:, None]).reshape(B, Rb, C), axis=1),
+            np.add.reduce(x64.reshape(B, Rb, C), axis=1))

@@ -330,6 +330,37 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
+def r2_logreg(nest, lim, dims):
+    """DESIGN.md S8, LOGREG_GRAD staged: 32-row tiles of one batch, contiguous tile ranges."""
+    (B, _), (Rb, _), (C, _) = nest["levels"]
+    if dims[2] != X or C % 4 != 0 or C > 256:
+        raise Unsupported("LOGREG_GRAD AUTO needs C % 4 == 0, C <= 256 and L2 on x")
+    Ti = cdiv(Rb, 32)
+    tiles = B * Ti
+    P = cdiv(tiles, min(lim["sm_count"], tiles))
+    G = cdiv(tiles, P)
+    blocks = (1, 8, 32)
+    spans = (ONE, ALL if Ti == 1 else SPLIT, ALL)
+    factors = (1, Ti, 1)
+    chunks = (1, 32 if Ti > 1 else Rb, C)
+    return blocks, spans, factors, 4, chunks, G, P
+
+
+def r2_kmeans(nest, lim):
+    """DESIGN.md S8, KMEANS_ASSIGN staged: 128-point tiles, 2 points per thread, 4 centroid quarters."""
+    (N, _), (K, _), (D, _) = nest["levels"]
+    if D % 4 != 0 or D < 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384:
+        raise Unsupported("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128, K <= 256, Kpad*D <= 16384")
+    T = cdiv(N, 128)
+    P = cdiv(T, min(lim["sm_count"], T))
+    G = cdiv(T, P)
+    blocks = (64, 4, 1)
+    spans = (SPAN_N, ALL, ALL)
+    factors = (2, 1, 1)
+    chunks = (128, K, D)
+    return blocks, spans, factors, 4, chunks, G, P
+
+
 def r2_sums(nest, dtype, lim, dims):
     """DESIGN.md S8 (unstaged) for the 2-level sums: returns (blocks, spans, factors, vec, chunks)."""
     pattern = nest["pattern"]
@@ -402,6 +433,9 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
                levels=levels, score=score_, dop=mapping_dop(nest, blocks, spans, factors),
                threads=grid * prod(blocks), grid=grid, block=block3,
                smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0, claim_tiles=claim_tiles)
+    if nest["pattern"] == "LOGREG_GRAD" and staged:  # tickets [B] + fp64 accumulators [B x C]
+        B, C = _eff(nest["levels"][0][0]), _eff(nest["levels"][2][0])
+        rec["workspace_bytes"] = 256 * cdiv(4 * B, 256) + 256 * cdiv(8 * B * C, 256)
     if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
         if staged:  # counters + fp64/integer accumulators [O] (S8 staged)
             O = _eff(nest["levels"][0][0])
@@ -436,8 +470,14 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
         raise ValueError(strategy)
     if unknown:
         raise Unsupported("AUTO needs known sizes")
-    if L != 2:
-        raise Unsupported("R2 for 3-level nests")
+    if pattern == "LOGREG_GRAD":
+        b3, s3, f3, vec, chunks, G, P = r2_logreg(nest, lim, dims)
+        return make_record(nest, dtype, lim, dims, b3, s3, f3, vec, sc, chunks, staged=1,
+                           persistent_grid=G, claim_tiles=P)
+    if pattern == "KMEANS_ASSIGN":
+        b3, s3, f3, vec, chunks, G, P = r2_kmeans(nest, lim)
+        return make_record(nest, dtype, lim, dims, b3, s3, f3, vec, sc, chunks, staged=1,
+                           persistent_grid=G, claim_tiles=P)
     if staged_eligible(nest, dtype, dims):
         b2, s2, f2, vec, chunks, G, CL = r2_staged(nest, dtype, lim)
         return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks, staged=1,

@@ -204,9 +204,9 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
     delete p;
     return st;
   }
-  if (p->map.kernel_class == NPP_CLASS_KMEANS || p->map.kernel_class == NPP_CLASS_LOGREG) {
+  if ((p->map.kernel_class == NPP_CLASS_KMEANS || p->map.kernel_class == NPP_CLASS_LOGREG) && !p->map.staged) {
     delete p;
-    set_error("this build executes the 2-level sum families only");
+    set_error("3-level nests execute through their staged (AUTO) kernel families only");
     return NPP_ERR_UNSUPPORTED;
   }
   *out = p;
@@ -344,6 +344,34 @@ int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, vo
         set_error("vectorised / TMA-staged plan: inputs must be 16-byte aligned");
         return NPP_ERR_ALIGNMENT;
       }
+  }
+  if (plan->pattern == NPP_LOGREG_GRAD) {  // class LR (S8)
+    npp::LogregArgs g{};
+    g.y = static_cast<const float*>(ins[1]);
+    g.w = static_cast<const float*>(ins[2]);
+    g.g = static_cast<float*>(out);
+    g.B = plan->shape[0];
+    g.Rb = plan->shape[1];
+    g.C = plan->shape[2];
+    g.Ti = (g.Rb + 31) / 32;
+    g.per_block = m.claim_tiles;
+    g.tickets = static_cast<unsigned*>(workspace);
+    g.acc = reinterpret_cast<double*>(static_cast<char*>(workspace) + ((4 * g.B + 255) / 256) * 256);
+    cudaError_t e = npp::launch_logreg(g, static_cast<const float*>(ins[0]), int(m.grid), st);
+    if (e != cudaSuccess) return cuda_fail("logreg kernel launch", e);
+    return NPP_OK;
+  }
+  if (plan->pattern == NPP_KMEANS_ASSIGN) {  // class KM (S8)
+    npp::KmeansArgs k{};
+    k.c = static_cast<const float*>(ins[1]);
+    k.assign = static_cast<int*>(out);
+    k.N = plan->shape[0];
+    k.D = plan->shape[1];
+    k.K = plan->shape[2];
+    k.per_block = m.claim_tiles;
+    cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
+    if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);
+    return NPP_OK;
   }
   if (!npp::is_sum_pattern(plan->pattern)) {
     set_error("pattern not executable in this build");

@@ -1,0 +1,203 @@
+// kern_logreg.cu — class LR: the three-level nest of the batched logistic-regression gradient
+// (BASELINE.json config 5; G22, S8):
+//     batches map { b => rows(b) reduce { i => e_i = σ(x_i·w) − y_i ; x_i map (_ * e_i) } }
+//     g[b,j] = Σ_{i in b} x[i,j] · (σ(Σ_k x[i,k] w[k]) − y[i])
+// L0 = batches, L1 = rows of a batch (Reduce), L2 = columns (Map_j and the dot Reduce_k at one level,
+// Span(all) by the Hard Global constraint). The imperfectly nested access pattern (a dot
+// product must finish before the same row is reused) is served by shared-memory staging
+// (§V-B): each 32-row tile is loaded once by TMA and read twice from shared memory — for
+// the dot and for the update — so HBM sees every byte of x exactly once.
+//   warp w owns rows 4w..4w+3 of a tile; lane l owns columns 4l..4l+3 and 128+4l..128+4l+3 with w
+//   in registers; the dot finishes with warp shuffles; x·e accumulates per lane in fp32 over the
+//   tile and in fp64 across tiles; at a batch boundary the eight warps meet in shared memory.
+// Work split as the staged sums: block b streams tiles [bP, bP+P) of the batch-major tile order; a
+// batch cut by range boundaries adds its fp64 partial with atomics and the last contributor
+// (ticket) converts to fp32.
+#include <cstdint>
+
+#include "kernels.hpp"
+#include "tma_ring.cuh"
+
+namespace npp {
+
+namespace {
+
+constexpr int kStages = 4;
+constexpr int kTileRows = 32;
+constexpr int kMaxCols = 256;
+constexpr int kTileBytes = kTileRows * kMaxCols * 4;
+constexpr int kConsumerWarps = 8;
+constexpr int kConsumers = kConsumerWarps * 32;
+constexpr int kThreads = kConsumers + 32;
+constexpr int kSmemHeader = 1024;
+constexpr int kRedBytes = kConsumerWarps * kMaxCols * 8;
+constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes + kRedBytes;
+
+__device__ __forceinline__ float warp_sum_f(float v) {
+#pragma unroll
+  for (int off = 16; off >= 1; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+  return v;
+}
+
+}  // namespace
+
+__global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __grid_constant__ CUtensorMap map,
+                                                                     LogregArgs a) {
+  extern __shared__ __align__(1024) unsigned char smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
+  uint64_t* empty = full + kStages;
+  long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);
+  unsigned* s_last = reinterpret_cast<unsigned*>(slot_tile + kStages);
+  unsigned char* tiles = smem + kSmemHeader;
+  double* red = reinterpret_cast<double*>(smem + kSmemHeader + kStages * kTileBytes);  // [8][C]
+  constexpr long long kFlush = 1ll << 62;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long bid = blockIdx.x;
+  const long long C = a.C, Rb = a.Rb, Ti = a.Ti;
+  const long long total = a.B * Ti;
+  const long long P = a.per_block;
+  const long long r0 = bid * P, r1 = (total < r0 + P) ? total : r0 + P;
+  const unsigned tile_bytes = unsigned(kTileRows * C * 4);
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kStages; ++i) {
+      tma::mbar_init(full + i, 1);
+      tma::mbar_init(empty + i, kConsumerWarps);
+    }
+    tma::mbar_fence_init();
+  }
+  __syncthreads();
+
+  if (warp == kConsumerWarps) {
+    if (lane == 0) {  // ---------------------------------------------- producer
+      tma::prefetch_map(&map);
+      long long t = 0;
+      for (long long cur = r0; cur < r1; ++cur, ++t) {
+        const bool flush = cur + 1 >= r1 || ((cur + 1) / Ti) != (cur / Ti);
+        const int slot = int(t % kStages);
+        if (t >= kStages) tma::mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
+        slot_tile[slot] = cur | (flush ? kFlush : 0);
+        tma::mbar_expect_tx(full + slot, tile_bytes);
+        const long long b = cur / Ti, j = cur - b * Ti;
+        tma::load_2d(tiles + slot * kTileBytes, &map, 0, int(b * Rb + j * kTileRows), full + slot);
+      }
+    }
+    return;  // the producer warp takes no part in the consumer barriers below
+  }
+
+  // ------------------------------------------------------------------ consumers
+  const float* __restrict__ yv = a.y;
+  const int c0 = lane * 4, c1 = 128 + lane * 4;  // this lane's two column quads
+  const bool has0 = c0 < C, has1 = c1 < C;
+  float w0[4] = {0, 0, 0, 0}, w1[4] = {0, 0, 0, 0};
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    if (has0) w0[e] = __ldg(a.w + c0 + e);
+    if (has1) w1[e] = __ldg(a.w + c1 + e);
+  }
+  double acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const long long n_tiles = r1 - r0;
+  for (long long t = 0; t < n_tiles; ++t) {
+    const int slot = int(t % kStages);
+    const long long cur = r0 + t;  // static range: the consumers know the tile without the producer
+    const bool flush = cur + 1 >= r1 || ((cur + 1) / Ti) != (cur / Ti);
+    const long long b = cur / Ti, j = cur - b * Ti;
+    const long long row0 = b * Rb + j * kTileRows;
+    const long long rows_here = (Rb - j * kTileRows) < kTileRows ? (Rb - j * kTileRows) : kTileRows;
+    // y of the tile's rows: lane l holds y[row0 + l] (masked), broadcast by shuffles below
+    const float y_lane = lane < rows_here ? __ldg(yv + row0 + lane) : 0.f;
+    tma::mbar_wait(full + slot, unsigned((t / kStages) & 1));
+    const float* tile = reinterpret_cast<const float*>(tiles + slot * kTileBytes);
+    float p[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+      const int r = warp * 4 + rr;
+      float4 x0 = make_float4(0, 0, 0, 0), x1 = make_float4(0, 0, 0, 0);
+      if (has0) x0 = *reinterpret_cast<const float4*>(tile + r * C + c0);
+      if (has1) x1 = *reinterpret_cast<const float4*>(tile + r * C + c1);
+      float d = x0.x * w0[0];
+      d = fmaf(x0.y, w0[1], d);
+      d = fmaf(x0.z, w0[2], d);
+      d = fmaf(x0.w, w0[3], d);
+      float d1 = x1.x * w1[0];
+      d1 = fmaf(x1.y, w1[1], d1);
+      d1 = fmaf(x1.z, w1[2], d1);
+      d1 = fmaf(x1.w, w1[3], d1);
+      const float z = warp_sum_f(d + d1);
+      const float yr = __shfl_sync(0xffffffffu, y_lane, r);
+      const float e = r < rows_here ? __frcp_rn(1.f + __expf(-z)) - yr : 0.f;
+      p[0] = fmaf(x0.x, e, p[0]);
+      p[1] = fmaf(x0.y, e, p[1]);
+      p[2] = fmaf(x0.z, e, p[2]);
+      p[3] = fmaf(x0.w, e, p[3]);
+      p[4] = fmaf(x1.x, e, p[4]);
+      p[5] = fmaf(x1.y, e, p[5]);
+      p[6] = fmaf(x1.z, e, p[6]);
+      p[7] = fmaf(x1.w, e, p[7]);
+    }
+    __syncwarp();
+    if (lane == 0) tma::mbar_arrive(empty + slot);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc[e] += double(p[e]);
+    if (!flush) continue;
+
+    // ---- batch b ends in this block's range: combine the 8 warps in fixed order
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      if (has0) red[warp * C + c0 + e] = acc[e];
+      if (has1) red[warp * C + c1 + e] = acc[4 + e];
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc[e] = 0;
+    tma::bar_sync_consumers<kConsumers>();
+    const long long f0 = b * Ti, f1 = f0 + Ti;  // tiles of batch b
+    const bool owned = f0 >= r0 && f1 <= r1;
+    for (int c = threadIdx.x; c < C; c += kConsumers) {
+      double s = red[c];
+#pragma unroll
+      for (int ww = 1; ww < kConsumerWarps; ++ww) s += red[ww * C + c];
+      if (owned)
+        a.g[b * C + c] = float(s);
+      else
+        atomicAdd(a.acc + b * C + c, s);
+    }
+    if (!owned) {
+      __threadfence();
+      tma::bar_sync_consumers<kConsumers>();
+      if (threadIdx.x == 0) {
+        const unsigned contributors = unsigned((f1 - 1) / P - f0 / P + 1);
+        const unsigned prev = atomicAdd(a.tickets + b, 1u);
+        *s_last = (prev + 1 == contributors) ? 1u : 0u;
+        if (prev + 1 == contributors) a.tickets[b] = 0u;
+      }
+      tma::bar_sync_consumers<kConsumers>();
+      if (*s_last) {
+        __threadfence();
+        for (int c = threadIdx.x; c < C; c += kConsumers) {
+          unsigned long long* pa = reinterpret_cast<unsigned long long*>(a.acc + b * C + c);
+          a.g[b * C + c] = float(__longlong_as_double((long long)atomicExch(pa, 0ull)));
+        }
+      }
+    }
+    tma::bar_sync_consumers<kConsumers>();  // `red` is reused by the next flush
+  }
+}
+
+cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStream_t st) {
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(npp_logreg_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  CUtensorMap map;
+  cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.B * a.Rb, a.C, unsigned(a.C),
+                                 unsigned(kTileRows));
+  if (e != cudaSuccess) return e;
+  npp_logreg_tma_kernel<<<grid, kThreads, kSmemBytes, st>>>(map, a);
+  return cudaGetLastError();
+}
+
+}  // namespace npp

@@ -42,4 +42,26 @@ struct StagedArgs {
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st);
 
+// Batched logistic-regression gradient (class LR, S8): x [B*Rb x C] row-major fp32.
+struct LogregArgs {
+  const float* y;      // [B*Rb]
+  const float* w;      // [C]
+  float* g;            // [B x C] output
+  double* acc;         // [B x C] fp64 accumulators of batches cut by range boundaries (zero on entry/exit)
+  unsigned* tickets;   // [B] (zero on entry/exit)
+  int64_t B, Rb, C;
+  int64_t Ti;          // 32-row tiles per batch
+  int64_t per_block;   // P: block b streams tiles [b*P, (b+1)*P) of the batch-major order
+};
+cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStream_t st);
+
+// k-means assignment (class KM, S8): x [N x D], c [K x D] fp32 -> a [N] int32.
+struct KmeansArgs {
+  const float* c;      // [K x D]
+  int* assign;         // [N]
+  int64_t N, D, K;
+  int64_t per_block;   // P: block b handles 128-point tiles [b*P, (b+1)*P)
+};
+cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st);
+
 }  // namespace npp

@@ -242,6 +242,40 @@ void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   c->factors[1] = t.Ti;
 }
 
+// S8 LOGREG_GRAD staged: 32-row tiles of one batch, contiguous tile ranges (class LR).
+bool r2_logreg(const Nest& n, const npp_limits& lim, Choice* c) {
+  const int64_t B = n.N[0], Rb = n.N[1], C = n.N[2];
+  if (c->dims[2] != NPP_DIM_X || C % 4 != 0 || C > 256) return false;
+  const int64_t Ti = cdiv(Rb, 32), tiles = B * Ti;
+  const int64_t per_block = cdiv(tiles, std::min<int64_t>(lim.sm_count, tiles));
+  c->claim_tiles = per_block;
+  c->persistent_grid = cdiv(tiles, per_block);
+  c->staged = 1;
+  c->vec = 4;
+  c->blocks[0] = 1, c->blocks[1] = 8, c->blocks[2] = 32;
+  c->spans[0] = NPP_SPAN_ONE, c->factors[0] = 1, c->chunks[0] = 1;
+  c->spans[1] = Ti == 1 ? NPP_SPAN_ALL : NPP_SPLIT_K, c->factors[1] = Ti, c->chunks[1] = Ti > 1 ? 32 : Rb;
+  c->spans[2] = NPP_SPAN_ALL, c->factors[2] = 1, c->chunks[2] = C;
+  return true;
+}
+
+// S8 KMEANS_ASSIGN staged: 128-point tiles, 2 points per thread, 4 centroid quarters (class KM).
+bool r2_kmeans(const Nest& n, const npp_limits& lim, Choice* c) {
+  const int64_t N = n.N[0], K = n.N[1], D = n.N[2];
+  if (D % 4 != 0 || D < 4 || D > 128 || K > 256 || 32 * cdiv(K, 32) * D > 16384) return false;
+  const int64_t T = cdiv(N, 128);
+  const int64_t per_block = cdiv(T, std::min<int64_t>(lim.sm_count, T));
+  c->claim_tiles = per_block;
+  c->persistent_grid = cdiv(T, per_block);
+  c->staged = 1;
+  c->vec = 4;
+  c->blocks[0] = 64, c->blocks[1] = 4, c->blocks[2] = 1;
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = 2, c->chunks[0] = 128;
+  c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = K;
+  c->spans[2] = NPP_SPAN_ALL, c->factors[2] = 1, c->chunks[2] = D;
+  return true;
+}
+
 // S8 (unstaged) for the 2-level sums: keep LITERAL's dims, re-choose blocks / vec / factors / chunks.
 void r2_sums(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const bool rows = n.pattern == NPP_SUM_ROWS || n.pattern == NPP_SUM_WEIGHTED_ROWS;
@@ -499,7 +533,9 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.workspace_bytes = 0;
   m.staged = c.staged;
   m.claim_tiles = c.claim_tiles;
-  if (is_sum_pattern(n.pattern) && c.staged) {
+  if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
+    m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
+  } else if (is_sum_pattern(n.pattern) && c.staged) {
     // counters (claim, barrier) + accumulators [O] of the accumulator type
     const StagedTiling t = staged_tiling(n.pattern, n.pattern == NPP_SUM_ROWS ? n.N[0] : n.N[1], n.cols, dtype);
     m.workspace_bytes = 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
@@ -555,9 +591,19 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
     set_error("strategy AUTO needs known sizes (use LITERAL for -1 sizes)");
     return NPP_ERR_UNSUPPORTED;
   }
-  if (n.L != 2) {
-    set_error("R2 runtime step for 3-level nests is not implemented in this build");
-    return NPP_ERR_UNSUPPORTED;
+  if (n.pattern == NPP_LOGREG_GRAD) {
+    if (!r2_logreg(n, lim, &c)) {
+      set_error("LOGREG_GRAD AUTO needs C % 4 == 0, C <= 256 and the column level on x");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    return record_from_choice(n, dtype, lim, c, sc, out);
+  }
+  if (n.pattern == NPP_KMEANS_ASSIGN) {
+    if (!r2_kmeans(n, lim, &c)) {
+      set_error("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128 and K <= 256");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    return record_from_choice(n, dtype, lim, c, sc, out);
   }
   if (staged_eligible(n, dtype, c))
     r2_staged(n, dtype, lim, &c);

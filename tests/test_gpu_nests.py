@@ -1,0 +1,146 @@
+"""GPU parity for the three-level nests (k-means assignment, batched logistic-regression gradient)
+through the C-ABI against the fp64 oracle.
+
+Tolerances:
+  logreg  |g - g64| <= 1e-5 * Σ_i|x_ij e_i| + 2^-20 * Σ_i|x_ij|   (fp32 terms; fp32 residual e_i)
+  kmeans  integer-valued data: bit-exact (every fp32 distance is exact, ties -> lowest k);
+          random data: d64(x_i, c_a) - min_k d64(x_i, c_k) <= 2^-16 (|x_i|² + |c_a|² + |c_o|²)
+          (the fp32 expansion ||c||² - 2x·c can only swap near-ties within that bound)
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle import kmeans as okm
+from oracle import logreg as olr
+from oracle import select as osel
+from synth import gen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def npp(cuda_device):
+    from paper_conf_micro_leebsro14_b200 import npp as _npp
+    return _npp
+
+
+def _check_logreg(g, x, y, w, B):
+    xn, yn, wn = x.cpu().numpy(), y.cpu().numpy(), w.cpu().numpy()
+    want = olr.grad(xn, yn, wn, B)
+    s_rel, s_abs = olr.grad_scales(xn, yn, wn, B)
+    err = np.abs(g.cpu().numpy().astype(np.float64) - want)
+    tol = 1e-5 * s_rel + 2.0 ** -20 * s_abs
+    bad = np.argwhere(err > tol)
+    assert bad.size == 0, (bad[:4], err[tuple(bad[0])], tol[tuple(bad[0])])
+
+
+@pytest.mark.parametrize("B,Rb,C", [(1, 1000, 256), (3, 70, 12), (16, 4096, 256), (2, 31, 256),
+                                    (7, 33, 100), (300, 64, 256), (1, 1 << 18, 256), (64, 32, 4)])
+def test_logreg_parity(npp, cuda_device, B, Rb, C):
+    x, y, w = gen.logreg_inputs(B, Rb, C, seed=6, device=cuda_device)
+    p = npp.Plan("LOGREG_GRAD", (B, Rb, C), "f32", "AUTO")
+    assert p.mapping == osel.select("LOGREG_GRAD", (B, Rb, C), "f32", npp.limits_query(0), "AUTO")
+    for _ in range(2):  # the second run checks that the workspace came back zeroed
+        g = p.execute([x, y, w], p.new_out())
+        torch.cuda.synchronize()
+        _check_logreg(g, x, y, w, B)
+
+
+def test_logreg_y_zero_and_w_zero(npp, cuda_device):
+    B, Rb, C = 8, 512, 256
+    x, y, w = gen.logreg_inputs(B, Rb, C, seed=7, device=cuda_device, y_zero=True)
+    p = npp.Plan("LOGREG_GRAD", (B, Rb, C), "f32", "AUTO")
+    g = p.execute([x, y, w], p.new_out())
+    torch.cuda.synchronize()
+    _check_logreg(g, x, y, w, B)
+    w0 = torch.zeros_like(w)
+    g0 = p.execute([x, y, w0], p.new_out())
+    torch.cuda.synchronize()
+    want = (x.double() * 0.5).view(B, Rb, C).sum(1)  # closed form: e = 1/2 - 0
+    assert torch.allclose(g0.double(), want, rtol=1e-6, atol=0)
+
+
+def test_logreg_full_size_sampled(npp, cuda_device):
+    # BASELINE.json config 5: [16M, 256] fp32 (16 GiB), B = 4096 batches of 4096 rows
+    B, Rb, C = 4096, 4096, 256
+    free, _ = torch.cuda.mem_get_info()
+    if free < 24 * (1 << 30):
+        pytest.skip("needs 24 GiB free")
+    x, y, w = gen.logreg_inputs(B, Rb, C, seed=6, device=cuda_device)
+    p = npp.Plan("LOGREG_GRAD", (B, Rb, C), "f32", "AUTO")
+    g = p.execute([x, y, w], p.new_out())
+    torch.cuda.synchronize()
+    for b in (0, 1, 1777, 4094, 4095):
+        rows = slice(b * Rb, (b + 1) * Rb)
+        _check_logreg(g[b:b + 1], x[rows], y[rows], w, 1)
+    del x
+
+
+def _check_kmeans_valid(a, x, c):
+    xn, cn = x.cpu().numpy(), c.cpu().numpy()
+    d = okm.distances(xn, cn)
+    best = d.min(axis=1)
+    a = a.cpu().numpy().astype(np.int64)
+    chosen = d[np.arange(len(a)), a]
+    o = okm.assign(xn, cn).astype(np.int64)
+    scale = (xn.astype(np.float64) ** 2).sum(1) + (cn.astype(np.float64) ** 2).sum(1)[a] + \
+        (cn.astype(np.float64) ** 2).sum(1)[o]
+    assert np.all(chosen - best <= 2.0 ** -16 * scale)
+    return float(np.mean(a == o))
+
+
+@pytest.mark.parametrize("N,D,K", [(10000, 64, 32), (1000, 12, 5), (4099, 128, 96), (127, 4, 1),
+                                   (20000, 64, 256), (129, 32, 33)])
+def test_kmeans_integer_data_exact(npp, cuda_device, N, D, K):
+    x, c = gen.kmeans_inputs(N, D, K, integer=True, device=cuda_device)
+    p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
+    assert p.mapping == osel.select("KMEANS_ASSIGN", (N, D, K), "f32", npp.limits_query(0), "AUTO")
+    a = p.execute([x, c], p.new_out())
+    torch.cuda.synchronize()
+    assert a.cpu().numpy().tolist() == okm.assign(x.cpu().numpy(), c.cpu().numpy()).tolist()
+
+
+@pytest.mark.parametrize("N,D,K", [(50000, 64, 32), (3000, 16, 7)])
+def test_kmeans_random_data(npp, cuda_device, N, D, K):
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
+    p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
+    a = p.execute([x, c], p.new_out())
+    torch.cuda.synchronize()
+    agree = _check_kmeans_valid(a, x, c)
+    assert agree > 0.999
+
+
+def test_kmeans_full_size_sampled(npp, cuda_device):
+    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids
+    N, D, K = 1 << 22, 64, 32
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
+    p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
+    a = p.execute([x, c], p.new_out())
+    torch.cuda.synchronize()
+    idx = torch.cat([torch.arange(0, 4096), torch.arange(N - 4096, N),
+                     torch.randint(0, N, (12000,), generator=torch.Generator().manual_seed(3))]).to(cuda_device)
+    agree = _check_kmeans_valid(a.index_select(0, idx), x.index_select(0, idx), c)
+    assert agree > 0.999
+
+
+def test_kmeans_points_on_centroids(npp, cuda_device):
+    _, c = gen.kmeans_inputs(4, 64, 32, device=cuda_device)
+    perm = torch.randint(0, 32, (5000,), generator=torch.Generator().manual_seed(1)).to(cuda_device)
+    x = c.index_select(0, perm).contiguous()
+    p = npp.Plan("KMEANS_ASSIGN", (5000, 64, 32), "f32", "AUTO")
+    a = p.execute([x, c], p.new_out())
+    torch.cuda.synchronize()
+    assert torch.equal(a.long(), perm)
+
+
+def test_unsupported_shapes(npp, cuda_device):
+    with pytest.raises(npp.NppError) as e:
+        npp.Plan("LOGREG_GRAD", (4, 64, 512), "f32", "AUTO")
+    assert e.value.status == npp.ERR_UNSUPPORTED
+    with pytest.raises(npp.NppError) as e:
+        npp.Plan("KMEANS_ASSIGN", (100, 6, 3), "f32", "AUTO")
+    assert e.value.status == npp.ERR_UNSUPPORTED
+    with pytest.raises(npp.NppError) as e:
+        npp.Plan("KMEANS_ASSIGN", (100, 64, 3), "f32", "LITERAL")
+    assert e.value.status == npp.ERR_UNSUPPORTED

@@ -49,10 +49,14 @@ def test_sums_exhaustive(profile, pattern):
 @pytest.mark.parametrize("profile", list(PROFILES))
 def test_three_level_literal(profile):
     lim = PROFILES[profile]
-    for shape in [(1 << 22, 64, 32), (1000, 3, 5), (17, 256, 1), (64, 1, 64), (4096 * 4096, 64, 32)]:
-        _cmp("KMEANS_ASSIGN", shape, "f32", lim, "LITERAL")
-    for shape in [(4096, 4096, 256), (1, 1 << 24, 256), (3, 7, 5), (512, 4096, 256)]:
-        _cmp("LOGREG_GRAD", shape, "f32", lim, "LITERAL")
+    for shape in [(1 << 22, 64, 32), (1000, 3, 5), (17, 256, 1), (64, 1, 64), (4096 * 4096, 64, 32),
+                  (4099, 128, 96), (20000, 64, 256), (10, 128, 256)]:
+        for strat in ("LITERAL", "AUTO"):
+            _cmp("KMEANS_ASSIGN", shape, "f32", lim, strat)
+    for shape in [(4096, 4096, 256), (1, 1 << 24, 256), (3, 7, 5), (512, 4096, 256), (7, 33, 100),
+                  (2, 5, 512), (64, 32, 4)]:
+        for strat in ("LITERAL", "AUTO"):
+            _cmp("LOGREG_GRAD", shape, "f32", lim, strat)
     for strat in ("1D", "TB_T", "WARP"):
         _cmp("KMEANS_ASSIGN", (1000, 64, 32), "f32", lim, strat)
 
