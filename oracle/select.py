@@ -351,13 +351,14 @@ def r2_kmeans(nest, lim):
     (N, _), (K, _), (D, _) = nest["levels"]
     if D % 4 != 0 or D < 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384:
         raise Unsupported("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128, K <= 256, Kpad*D <= 16384")
-    T = cdiv(N, 128)
+    TP = 256 if D <= 64 else 128                 # points per tile: 4 (or 2) per thread
+    T = cdiv(N, TP)
     P = cdiv(T, min(lim["sm_count"], T))
     G = cdiv(T, P)
     blocks = (64, 4, 1)
     spans = (SPAN_N, ALL, ALL)
-    factors = (2, 1, 1)
-    chunks = (128, K, D)
+    factors = (TP // 64, 1, 1)
+    chunks = (TP, K, D)
     return blocks, spans, factors, 4, chunks, G, P
 
 

@@ -31,7 +31,9 @@ constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;
 constexpr int kSmemHeader = 1024;
 constexpr int kRedBytes = kConsumerWarps * kMaxCols * 8;
-constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes + kRedBytes;
+constexpr int kYBox = kTileRows + 4;  // y box starts 16-B aligned (row0 rounded down to 4): 36 floats
+constexpr int kYSlot = 256;           // bytes per ring slot of y (TMA destinations are 128-B aligned)
+constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes + kRedBytes + kStages * kYSlot;
 
 __device__ __forceinline__ float warp_sum_f(float v) {
 #pragma unroll
@@ -42,8 +44,11 @@ __device__ __forceinline__ float warp_sum_f(float v) {
 }  // namespace
 
 __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __grid_constant__ CUtensorMap map,
+                                                                     const __grid_constant__ CUtensorMap ymap,
                                                                      LogregArgs a) {
   extern __shared__ __align__(1024) unsigned char smem[];
+  // y of each staged tile (1-D TMA box of 36 floats from row0 & ~3), one 256-B slot per stage
+  unsigned char* y_ring = smem + kSmemHeader + kStages * kTileBytes + kRedBytes;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + kStages;
   long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);
@@ -78,16 +83,17 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
         const int slot = int(t % kStages);
         if (t >= kStages) tma::mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
         slot_tile[slot] = cur | (flush ? kFlush : 0);
-        tma::mbar_expect_tx(full + slot, tile_bytes);
+        tma::mbar_expect_tx(full + slot, tile_bytes + kYBox * 4);
         const long long b = cur / Ti, j = cur - b * Ti;
-        tma::load_2d(tiles + slot * kTileBytes, &map, 0, int(b * Rb + j * kTileRows), full + slot);
+        const long long row0 = b * Rb + j * kTileRows;
+        tma::load_2d(tiles + slot * kTileBytes, &map, 0, int(row0), full + slot);
+        tma::load_1d(y_ring + slot * kYSlot, &ymap, int(row0 & ~3ll), full + slot);
       }
     }
     return;  // the producer warp takes no part in the consumer barriers below
   }
 
   // ------------------------------------------------------------------ consumers
-  const float* __restrict__ yv = a.y;
   const int c0 = lane * 4, c1 = 128 + lane * 4;  // this lane's two column quads
   const bool has0 = c0 < C, has1 = c1 < C;
   float w0[4] = {0, 0, 0, 0}, w1[4] = {0, 0, 0, 0};
@@ -103,38 +109,56 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
     const long long cur = r0 + t;  // static range: the consumers know the tile without the producer
     const bool flush = cur + 1 >= r1 || ((cur + 1) / Ti) != (cur / Ti);
     const long long b = cur / Ti, j = cur - b * Ti;
-    const long long row0 = b * Rb + j * kTileRows;
     const long long rows_here = (Rb - j * kTileRows) < kTileRows ? (Rb - j * kTileRows) : kTileRows;
     // y of the tile's rows: lane l holds y[row0 + l] (masked), broadcast by shuffles below
-    const float y_lane = lane < rows_here ? __ldg(yv + row0 + lane) : 0.f;
     tma::mbar_wait(full + slot, unsigned((t / kStages) & 1));
+    const int yoff = int((b * Rb + j * kTileRows) & 3);
+    const float y_lane = lane < rows_here ? reinterpret_cast<const float*>(y_ring + slot * kYSlot)[yoff + lane] : 0.f;
     const float* tile = reinterpret_cast<const float*>(tiles + slot * kTileBytes);
-    float p[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    // dot products of the warp's 4 rows: per-lane partials over the lane's 8 columns ...
+    float4 x0[4], x1[4];
+    float dp[4];
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {
       const int r = warp * 4 + rr;
-      float4 x0 = make_float4(0, 0, 0, 0), x1 = make_float4(0, 0, 0, 0);
-      if (has0) x0 = *reinterpret_cast<const float4*>(tile + r * C + c0);
-      if (has1) x1 = *reinterpret_cast<const float4*>(tile + r * C + c1);
-      float d = x0.x * w0[0];
-      d = fmaf(x0.y, w0[1], d);
-      d = fmaf(x0.z, w0[2], d);
-      d = fmaf(x0.w, w0[3], d);
-      float d1 = x1.x * w1[0];
-      d1 = fmaf(x1.y, w1[1], d1);
-      d1 = fmaf(x1.z, w1[2], d1);
-      d1 = fmaf(x1.w, w1[3], d1);
-      const float z = warp_sum_f(d + d1);
-      const float yr = __shfl_sync(0xffffffffu, y_lane, r);
-      const float e = r < rows_here ? __frcp_rn(1.f + __expf(-z)) - yr : 0.f;
-      p[0] = fmaf(x0.x, e, p[0]);
-      p[1] = fmaf(x0.y, e, p[1]);
-      p[2] = fmaf(x0.z, e, p[2]);
-      p[3] = fmaf(x0.w, e, p[3]);
-      p[4] = fmaf(x1.x, e, p[4]);
-      p[5] = fmaf(x1.y, e, p[5]);
-      p[6] = fmaf(x1.z, e, p[6]);
-      p[7] = fmaf(x1.w, e, p[7]);
+      x0[rr] = has0 ? *reinterpret_cast<const float4*>(tile + r * C + c0) : make_float4(0, 0, 0, 0);
+      x1[rr] = has1 ? *reinterpret_cast<const float4*>(tile + r * C + c1) : make_float4(0, 0, 0, 0);
+      float d = x0[rr].x * w0[0];
+      d = fmaf(x0[rr].y, w0[1], d);
+      d = fmaf(x0[rr].z, w0[2], d);
+      d = fmaf(x0[rr].w, w0[3], d);
+      d = fmaf(x1[rr].x, w1[0], d);
+      d = fmaf(x1[rr].y, w1[1], d);
+      d = fmaf(x1[rr].z, w1[2], d);
+      dp[rr] = fmaf(x1[rr].w, w1[3], d);
+    }
+    // ... finished by a transposing butterfly: 6 shuffles leave lane l with the whole dot of row
+    // m(l) = 2*bit4(l) + bit3(l), so each lane evaluates one sigmoid, then 4 shuffles share them.
+    const bool h16 = (lane & 16) != 0, h8 = (lane & 8) != 0;
+    float a0 = h16 ? dp[2] : dp[0], a1 = h16 ? dp[3] : dp[1];
+    a0 += __shfl_xor_sync(0xffffffffu, h16 ? dp[0] : dp[2], 16);
+    a1 += __shfl_xor_sync(0xffffffffu, h16 ? dp[1] : dp[3], 16);
+    float z = h8 ? a1 : a0;
+    z += __shfl_xor_sync(0xffffffffu, h8 ? a0 : a1, 8);
+    z += __shfl_xor_sync(0xffffffffu, z, 4);
+    z += __shfl_xor_sync(0xffffffffu, z, 2);
+    z += __shfl_xor_sync(0xffffffffu, z, 1);
+    const int my_row = warp * 4 + (h16 ? 2 : 0) + (h8 ? 1 : 0);
+    const float yr = __shfl_sync(0xffffffffu, y_lane, my_row);
+    const float zc = fminf(fmaxf(z, -80.f), 80.f);
+    const float e_mine = my_row < rows_here ? __fdividef(1.f, 1.f + __expf(-zc)) - yr : 0.f;
+    float p[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+      const float e = __shfl_sync(0xffffffffu, e_mine, ((rr >> 1) << 4) | ((rr & 1) << 3));
+      p[0] = fmaf(x0[rr].x, e, p[0]);
+      p[1] = fmaf(x0[rr].y, e, p[1]);
+      p[2] = fmaf(x0[rr].z, e, p[2]);
+      p[3] = fmaf(x0[rr].w, e, p[3]);
+      p[4] = fmaf(x1[rr].x, e, p[4]);
+      p[5] = fmaf(x1[rr].y, e, p[5]);
+      p[6] = fmaf(x1[rr].z, e, p[6]);
+      p[7] = fmaf(x1[rr].w, e, p[7]);
     }
     __syncwarp();
     if (lane == 0) tma::mbar_arrive(empty + slot);
@@ -196,8 +220,13 @@ cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStr
   cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.B * a.Rb, a.C, unsigned(a.C),
                                  unsigned(kTileRows));
   if (e != cudaSuccess) return e;
-  npp_logreg_tma_kernel<<<grid, kThreads, kSmemBytes, st>>>(map, a);
-  return cudaGetLastError();
+  CUtensorMap ymap;
+  e = tma::encode_1d(&ymap, a.y, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, a.B * a.Rb, unsigned(kYBox));
+  if (e != cudaSuccess) return e;
+  npp_logreg_tma_kernel<<<grid, kThreads, kSmemBytes, st>>>(map, ymap, a);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) std::fprintf(stderr, "npp: logreg launch grid=%d smem=%d: %s\n", grid, kSmemBytes, cudaGetErrorString(e));
+  return e;
 }
 
 }  // namespace npp

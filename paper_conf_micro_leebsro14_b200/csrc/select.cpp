@@ -263,14 +263,15 @@ bool r2_logreg(const Nest& n, const npp_limits& lim, Choice* c) {
 bool r2_kmeans(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], K = n.N[1], D = n.N[2];
   if (D % 4 != 0 || D < 4 || D > 128 || K > 256 || 32 * cdiv(K, 32) * D > 16384) return false;
-  const int64_t T = cdiv(N, 128);
+  const int64_t TP = D <= 64 ? 256 : 128;  // points per tile: 4 (or 2) per thread
+  const int64_t T = cdiv(N, TP);
   const int64_t per_block = cdiv(T, std::min<int64_t>(lim.sm_count, T));
   c->claim_tiles = per_block;
   c->persistent_grid = cdiv(T, per_block);
   c->staged = 1;
   c->vec = 4;
   c->blocks[0] = 64, c->blocks[1] = 4, c->blocks[2] = 1;
-  c->spans[0] = NPP_SPAN_N, c->factors[0] = 2, c->chunks[0] = 128;
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = TP / 64, c->chunks[0] = TP;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = K;
   c->spans[2] = NPP_SPAN_ALL, c->factors[2] = 1, c->chunks[2] = D;
   return true;

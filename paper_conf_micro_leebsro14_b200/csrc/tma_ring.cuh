@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdio>
 
 namespace npp {
 namespace tma {
@@ -38,6 +39,13 @@ __device__ __forceinline__ void load_2d(void* dst, const CUtensorMap* map, int x
       "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
           smem_u32(dst)),
       "l"(map), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void load_1d(void* dst, const CUtensorMap* map, int x, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(x), "r"(smem_u32(bar))
       : "memory");
 }
 __device__ __forceinline__ void prefetch_map(const CUtensorMap* map) {
@@ -79,6 +87,20 @@ inline cudaError_t encode_2d(CUtensorMap* map, const void* base, CUtensorMapData
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = encode(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                       swizzle, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+// 1-D map over a contiguous vector of `n` elements, box of `box` elements (zero-filled past the end).
+inline cudaError_t encode_1d(CUtensorMap* map, const void* base, CUtensorMapDataType dt, int64_t n, unsigned box) {
+  EncodeTiledFn encode = encoder();
+  if (!encode) return cudaErrorNotSupported;
+  const cuuint64_t dims[1] = {cuuint64_t(n)};
+  const cuuint64_t strides[1] = {cuuint64_t(n) * 4};  // unused for rank 1 (rank-1 entries are read)
+  const cuuint32_t boxd[1] = {box};
+  const cuuint32_t estr[1] = {1};
+  CUresult r = encode(map, dt, 1, const_cast<void*>(base), dims, strides, boxd, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) std::fprintf(stderr, "npp: cuTensorMapEncodeTiled(1d) failed: %d\n", int(r));
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 

@@ -198,7 +198,7 @@ class Plan:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and _lib is not None:  # _lib is None during interpreter shutdown
             _lib.npp_plan_destroy(h)
             self._h = None
 
