@@ -1,0 +1,76 @@
+"""Multi-GPU partitioning of the nested patterns over torch.distributed (one process per GPU).
+
+SURVEY.md §8e / DESIGN.md §8. The outer (storage-row) dimension of every input is split into contiguous
+shards, one per rank. Where the rows are the Map level (sumRows, k-means points, logreg mini-batches)
+the shards are independent problems and no collective runs. Where the rows are the level being
+reduced (sumCols, the full-batch logreg gradient) the shard results are a cross-device Split(P) of that
+Reduce and NCCL adds them — the only data-path collective.
+
+Every rank plans and executes its shard through libnpp.so (``compute=None``). The ``compute`` hook
+exists so the host-side sharding and reduction logic can be tested on CPU with the gloo backend;
+the product path never runs on the CPU.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def shard_range(n: int, world: int, rank: int):
+    """Contiguous, balanced shard [lo, hi) of n outer indices for `rank` (sizes differ by <= 1)."""
+    base, extra = divmod(n, world)
+    lo = rank * base + min(rank, extra)
+    return lo, lo + base + (1 if rank < extra else 0)
+
+
+def _world(group):
+    return dist.get_world_size(group), dist.get_rank(group)
+
+
+def _npp():
+    from . import npp  # raises if libnpp.so is missing: no CPU fallback
+    return npp
+
+
+def sum_rows(local: torch.Tensor, group=None, gather: bool = False, compute=None):
+    """Row sums of this rank's row shard; rows are independent, so no collective unless `gather`."""
+    out = compute(local) if compute is not None else _npp().sum_rows(local)
+    if not gather:
+        return out
+    world, _ = _world(group)
+    sizes = [torch.zeros(1, dtype=torch.int64, device=out.device) for _ in range(world)]
+    dist.all_gather(sizes, torch.tensor([out.numel()], dtype=torch.int64, device=out.device), group=group)
+    mx = int(max(int(s.item()) for s in sizes))
+    buf = torch.zeros(mx, dtype=out.dtype, device=out.device)
+    buf[: out.numel()] = out
+    parts = [torch.empty_like(buf) for _ in range(world)]
+    dist.all_gather(parts, buf, group=group)
+    return torch.cat([p[: int(s.item())] for p, s in zip(parts, sizes)])
+
+
+def sum_cols(local: torch.Tensor, group=None, op: str = "all_reduce", dst: int = 0, compute=None):
+    """Column sums of a row-sharded matrix: local column sums, then one NCCL reduction of [C]."""
+    out = compute(local) if compute is not None else _npp().sum_cols(local)
+    if op == "all_reduce":
+        dist.all_reduce(out, op=dist.ReduceOp.SUM, group=group)
+    elif op == "reduce":
+        dist.reduce(out, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    else:
+        raise ValueError(op)
+    return out
+
+
+def kmeans_assign(local_x: torch.Tensor, centroids: torch.Tensor, group=None, compute=None):
+    """Assignments of this rank's points (centroids replicated); points are independent."""
+    return compute(local_x, centroids) if compute is not None else _npp().kmeans_assign(local_x, centroids)
+
+
+def logreg_grad(local_x: torch.Tensor, local_y: torch.Tensor, w: torch.Tensor, batches: int, group=None,
+                full_batch: bool = False, compute=None):
+    """Per-mini-batch gradients of this rank's batches (independent), or with ``full_batch`` the
+    gradient over all ranks' rows (local [1 x C] partial, then an all-reduce of C floats)."""
+    fn = compute if compute is not None else _npp().logreg_grad
+    g = fn(local_x, local_y, w, 1 if full_batch else batches)
+    if full_batch:
+        dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
+    return g
