@@ -2,16 +2,23 @@
 //     points mapRows { x_i => (0 until K) argmin { k => Σ_d (x_id − c_kd)² } }     ties -> lowest k
 // L0 = points (Map), L1 = centroids (argmin Reduce), L2 = dims (Reduce). The mapping keeps L2 on x
 // for coalescing, which the staged access satisfies (§V-B): TP-point tiles of x arrive
-// by TMA with the 128-byte swizzle, so the per-point reads of a warp are bank-conflict free, and the
-// centroids stay resident in shared memory for the whole launch (reused N/TP times per block).
-//   thread t owns points pq + 64i (i < PPT = TP/64) of a tile and centroid quarter q = t / 64 (warp-
-//   uniform, so centroid reads are shared-memory broadcasts); it ranks its centroids by
-//   s_k = ||c_k||² − 2 x·c_k (the x-independent expansion of the squared distance: same argmin),
-//   keeping the first minimum in increasing k; the four quarters meet in shared memory in order.
-//   x·c runs on the packed FP32 pipe (Blackwell FFMA2, fma.rn.f32x2): even and odd dims accumulate
-//   in the two halves of a float2, which halves the FMA instruction count.
-// The path is FP32-FMA-bound: 2·N·K·D flops against 1 KB of x per 4 points.
+// by TMA with the 128-byte swizzle (conflict-free per-point reads), while the centroids — read by
+// every point — sit in the constant bank for the whole launch.
+//   Why the constant bank: every thread of a warp reads the same centroid element at the same time,
+//   which is exactly what the constant cache serves; ptxas loads it into uniform registers (LDCU)
+//   and the packed FMA takes the uniform register as an operand, so the centroid stream never
+//   touches the shared-memory pipe. (With centroids in shared memory the LSU wavefronts, not the
+//   FMA pipe, set the pace: profiles/r01/SUMMARY.md.) The S8 limit 32·⌈K/32⌉·D ≤ 16384 floats is
+//   the 64 KB constant bank.
+//   Thread t of centroid group g (warp-uniform, G = 32/CPT groups) owns points lt + (256/G)·i
+//   (i < PPT) of a tile and centroids kc + g·CPT + m (m < CPT) of each 32-centroid chunk kc; it
+//   ranks them by s_k = ||c_k||² − 2 x·c_k (same argmin as the squared distance), keeping the first
+//   minimum in increasing k; with G = 2 the two groups meet in shared memory (lower k on ties).
+//   x·c runs on the packed FP32 pipe (FFMA2, fma.rn.f32x2): even and odd dims accumulate in the two
+//   halves of a float2.
+// The path is FP32-FMA-bound: 2·N·K·D flops against 4·D bytes of x per point.
 #include <cstdint>
+#include <mutex>
 
 #include "kernels.hpp"
 #include "tma_ring.cuh"
@@ -20,19 +27,49 @@ namespace npp {
 
 namespace {
 
-constexpr int kStages = 2;
+constexpr int kMaxStages = 3;
 constexpr int kBoxCols = 32;  // 128 B of floats: the 128-B swizzle span
-constexpr int kConsumerWarps = 8;
-constexpr int kConsumers = kConsumerWarps * 32;
-constexpr int kThreads = kConsumers + 32;
+// ping-pong: kSets sets of 8 warps take alternate tiles, so one set's per-tile epilogue (argmin,
+// group combine, set barrier) overlaps the other set's FMA stream
+#ifndef NPP_KM_SETS
+#define NPP_KM_SETS 1
+#endif
+constexpr int kSets = NPP_KM_SETS;
+constexpr int kConsumerWarps = 8;                 // per set
+constexpr int kConsumers = kConsumerWarps * 32;   // per set
+constexpr int kThreads = kSets * kConsumers;      // no producer warp: see the refill below
 constexpr int kSmemHeader = 1024;
 constexpr int kMaxStageBytes = 64 * 1024;
+constexpr int kSmemLimit = 227 * 1024;
+constexpr int kConstFloats = 16384;  // DESIGN.md S8: 32·⌈K/32⌉·D ≤ 16384
+
+// D <= 64: PPT points x CPT centroids per thread (G = 32/CPT groups, 256-point tiles)
+#ifndef NPP_KM_PPT
+#define NPP_KM_PPT 4
+#endif
+constexpr int kPptSmallD = NPP_KM_PPT;
+constexpr int kCptSmallD = 32 / NPP_KM_PPT;  // so that TP = PPT·256·CPT/32 = 256
+// register cap: low enough that ptxas keeps the centroid reads on the uniform datapath (LDCU);
+// with a generous budget it prefers per-thread LDC, which the constant cache serves ~5x slower
+// (tools/micro_const.cu). tests/test_sass.py checks the built kernel.
+#ifndef NPP_KM_MAXNREG
+#define NPP_KM_MAXNREG 120
+#endif
+#define NPP_KM_BOUNDS __maxnreg__(NPP_KM_MAXNREG)
+
+__constant__ float km_centroids[kConstFloats];  // [K][D] as given (padded rows: stale, see cn)
 
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
-inline size_t km_smem_bytes(int64_t D, int64_t K, int tp) {
-  return size_t(1024) /* alignment pad */ + size_t(kSmemHeader) + size_t(kStages) * kMaxStageBytes +
-         size_t(km_kpad(K)) * size_t(D) * 4 + size_t(km_kpad(K)) * 4 + size_t(4) * tp * 8;
+__host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
+  return 1024 /* alignment pad */ + kSmemHeader + km_kpad(K) * 4 + kSets * 2 * 3 * int64_t(tp) * 8;
+}
+// ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
+__host__ __device__ inline int km_stages(int64_t K, int tp) {
+  return km_rest_bytes(K, tp) + 3 * int64_t(kMaxStageBytes) <= kSmemLimit ? 3 : 2;
+}
+inline size_t km_smem_bytes(int64_t K, int tp) {
+  return size_t(km_rest_bytes(K, tp) + int64_t(km_stages(K, tp)) * kMaxStageBytes);
 }
 
 // x·c with even/odd dims in the two halves of an f32x2 accumulator
@@ -44,158 +81,224 @@ __device__ __forceinline__ void ffma2(float2& acc, const float2 a, const float2 
   acc = *reinterpret_cast<float2*>(&C);
 }
 
-template <int TP>
-__device__ __forceinline__ float4 ld_point(const unsigned char* tile, int p, int d4) {
-  // 128-byte swizzle: 16-byte chunk j of row p lives at chunk j ^ (p & 7)
-  const int box = d4 >> 3, j = d4 & 7;
-  return *reinterpret_cast<const float4*>(tile + box * (TP * 128) + p * 128 + ((j ^ (p & 7)) << 4));
-}
-
 }  // namespace
 
-template <int PPT>
-__global__ void __launch_bounds__(kThreads, 1) npp_kmeans_tma_kernel(const __grid_constant__ CUtensorMap map,
+// PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
+// groups; a tile is TP = PPT·256/G points.
+template <int PPT, int CPT>
+__global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUtensorMap map,
                                                                      KmeansArgs a) {
-  constexpr int TP = 64 * PPT;  // points per tile
+  constexpr int G = 32 / CPT;
+  constexpr int LP = kConsumers / G;  // threads (and point lanes) per centroid group
+  constexpr int TP = PPT * LP;        // points per tile
   extern __shared__ __align__(1024) unsigned char smem[];
   const int nb = km_boxes(a.D);
   const int stage_bytes = nb * TP * 128;
+  const int kStages = km_stages(a.K, TP);  // ring depth (2 or 3)
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
-  uint64_t* empty = full + kStages;
+  uint64_t* empty = full + kMaxStages;
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
   unsigned char* ring = smem + pad + kSmemHeader;
-  const int64_t D = a.D, K = a.K, Kp = km_kpad(K);
-  float* cs = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp][D]
-  float* cn = cs + Kp * D;                                                // [Kp]
-  float* sb_s = cn + Kp;                                                  // [4][TP]
-  int* sb_k = reinterpret_cast<int*>(sb_s + 4 * TP);                      // [4][TP]
+  const int D = int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
+  float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp]
+  // minima of groups 1..G-1 handed to group 0: [set][2 (tile parity)][G-1 <= 3][TP]
+  float* xs_s = cn + Kp;
+  int* xs_k = reinterpret_cast<int*>(xs_s + kSets * 2 * 3 * TP);
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // warp index broadcast from lane 0: ptxas then knows the producer/consumer split is warp-
+  // uniform and may use the uniform datapath (LDCU) for the centroid reads after it
+  const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
   const long long bid = blockIdx.x;
   const long long T = (a.N + TP - 1) / TP;
   const long long P = a.per_block;
   const long long r0 = bid * P, r1 = (T < r0 + P) ? T : r0 + P;
 
+  unsigned* released = reinterpret_cast<unsigned*>(empty);  // [kStages] warps done with the slot
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       tma::mbar_init(full + i, 1);
-      tma::mbar_init(empty + i, kConsumerWarps);
+      released[i] = 0;
     }
     tma::mbar_fence_init();
   }
-  // centroids -> shared memory (padded rows are zero, padded norms +inf: never selected)
-  for (int64_t i = threadIdx.x; i < Kp * D; i += kThreads) cs[i] = i < K * D ? __ldg(a.c + i) : 0.f;
-  __syncthreads();
-  for (int64_t k = threadIdx.x; k < Kp; k += kThreads) {
+  // ||c_k||² (fp32 FMA chain over d); padded rows get +inf and are never selected (their
+  // constant-bank rows are stale: inf − 2·finite = inf, inf − inf = NaN, both lose)
+  for (int k = threadIdx.x; k < Kp; k += kThreads) {
     float s = 0.f;
-    for (int64_t d = 0; d < D; ++d) s = fmaf(cs[k * D + d], cs[k * D + d], s);
+    if (k < K)
+      for (int d = 0; d < D; ++d) s = fmaf(__ldg(a.c + k * D + d), __ldg(a.c + k * D + d), s);
     cn[k] = k < K ? s : __int_as_float(0x7f800000);
   }
   __syncthreads();
 
-  if (warp == kConsumerWarps) {
-    if (lane == 0) {  // ---------------------------------------------- producer
-      tma::prefetch_map(&map);
-      long long t = 0;
-      for (long long cur = r0; cur < r1; ++cur, ++t) {
-        const int slot = int(t % kStages);
-        if (t >= kStages) tma::mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-        tma::mbar_expect_tx(full + slot, unsigned(stage_bytes));
-        for (int bx = 0; bx < nb; ++bx)
-          tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int(cur * TP),
-                       full + slot);
-      }
-    }
-    return;
+  const long long n_tiles = r1 - r0;
+  auto issue = [&](long long t) {  // tile t of the block's range into slot t % kStages
+    const int slot = int(t % kStages);
+    tma::mbar_expect_tx(full + slot, unsigned(stage_bytes));
+    for (int bx = 0; bx < nb; ++bx)
+      tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
+                   full + slot);
+  };
+  if (threadIdx.x == 0) {
+    tma::prefetch_map(&map);
+    for (long long t = 0; t < kStages && t < n_tiles; ++t) issue(t);
   }
 
   // ------------------------------------------------------------------ consumers
-  const int pq = threadIdx.x & 63;
-  const int q = threadIdx.x >> 6;  // centroid quarter (warp-uniform)
-  const int nd4 = int(D / 4);
-  const long long n_tiles = r1 - r0;
-  for (long long t = 0; t < n_tiles; ++t) {
+  // centroid group; redux.sync lands in a uniform register, so ptxas treats g as warp-uniform and
+  // keeps the centroid reads on the uniform datapath (LDCU)
+  const int set = int(__reduce_min_sync(0xffffffffu, unsigned(warp / kConsumerWarps)));
+  const int g = int(__reduce_min_sync(0xffffffffu, unsigned((warp % kConsumerWarps) / (kConsumerWarps / G))));
+  const int lt = threadIdx.x % LP;  // point lane: points lt + LP·i
+  // 128-byte swizzle: 16-byte chunk j of tile row p lives at chunk j ^ (p & 7); LP is a multiple
+  // of 8, so every point of the thread has the key lt & 7
+  const unsigned key = unsigned(lt & 7);
+  const int nd4 = D / 4;
+  for (long long t = set; t < n_tiles; t += kSets) {
     const int slot = int(t % kStages);
-    tma::mbar_wait(full + slot, unsigned((t / kStages) & 1));
-    const unsigned char* tile = ring + slot * kMaxStageBytes;
+    tma::mbar_wait_warp(full + slot, unsigned((t / kStages) & 1));
+    const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
     float bs[PPT];
     int bk[PPT];
 #pragma unroll
     for (int i = 0; i < PPT; ++i) bs[i] = __int_as_float(0x7f800000), bk[i] = 0x7fffffff;
-    for (int64_t kc = 0; kc < Kp; kc += 32) {
-      float2 acc[PPT][8];
+    for (int kc = 0; kc < Kp; kc += 32) {
+      const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
+      float2 acc[PPT][CPT];
 #pragma unroll
       for (int i = 0; i < PPT; ++i)
 #pragma unroll
-        for (int c = 0; c < 8; ++c) acc[i][c] = make_float2(0.f, 0.f);
-      const float* cq = cs + (kc + q * 8) * D;
+        for (int m = 0; m < CPT; ++m) acc[i][m] = make_float2(0.f, 0.f);
+      const float* cq = km_centroids + k0 * D;
 #pragma unroll 2
       for (int d4 = 0; d4 < nd4; ++d4) {
+        const unsigned char* xb = tile + (d4 >> 3) * (TP * 128) + ((unsigned(d4 & 7) ^ key) << 4);
         float4 xv[PPT];
 #pragma unroll
-        for (int i = 0; i < PPT; ++i) xv[i] = ld_point<TP>(tile, pq + 64 * i, d4);
+        for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-          const float4 cv = *reinterpret_cast<const float4*>(cq + c * D + d4 * 4);
+        for (int m = 0; m < CPT; ++m) {
+          const float4 cv = *reinterpret_cast<const float4*>(cq + m * D + 4 * d4);  // warp-uniform
 #pragma unroll
           for (int i = 0; i < PPT; ++i) {
-            ffma2(acc[i][c], make_float2(xv[i].x, xv[i].y), make_float2(cv.x, cv.y));
-            ffma2(acc[i][c], make_float2(xv[i].z, xv[i].w), make_float2(cv.z, cv.w));
+            ffma2(acc[i][m], make_float2(xv[i].x, xv[i].y), make_float2(cv.x, cv.y));
+            ffma2(acc[i][m], make_float2(xv[i].z, xv[i].w), make_float2(cv.z, cv.w));
           }
         }
       }
 #pragma unroll
-      for (int c = 0; c < 8; ++c) {  // increasing k within the quarter: strict < keeps the first
-        const int k = int(kc) + q * 8 + c;
+      for (int m = 0; m < CPT; ++m) {  // increasing k within the thread: strict < keeps the first
+        const int k = k0 + m;
+        const float nk = cn[k];
 #pragma unroll
         for (int i = 0; i < PPT; ++i) {
-          const float s = fmaf(-2.f, acc[i][c].x + acc[i][c].y, cn[k]);
+          const float s = fmaf(-2.f, acc[i][m].x + acc[i][m].y, nk);
           if (s < bs[i]) bs[i] = s, bk[i] = k;
         }
       }
     }
-    __syncwarp();
-    if (lane == 0) tma::mbar_arrive(empty + slot);  // the tile is no longer read
+    const long long base = (r0 + t) * TP;
+    if (G == 1) {
 #pragma unroll
-    for (int i = 0; i < PPT; ++i) {
-      sb_s[q * TP + pq + 64 * i] = bs[i];
-      sb_k[q * TP + pq + 64 * i] = bk[i];
-    }
-    tma::bar_sync_consumers<kConsumers>();
-    for (int p = threadIdx.x; p < TP; p += kConsumers) {
-      float s = sb_s[p];
-      int k = sb_k[p];
-#pragma unroll
-      for (int qq = 1; qq < 4; ++qq) {
-        const float s2 = sb_s[qq * TP + p];
-        const int k2 = sb_k[qq * TP + p];
-        if (s2 < s || (s2 == s && k2 < k)) s = s2, k = k2;
+      for (int i = 0; i < PPT; ++i) {
+        const long long gi = base + lt + LP * i;
+        if (gi < a.N) a.assign[gi] = bk[i];
       }
-      const long long i = (r0 + t) * TP + p;
-      if (i < a.N) a.assign[i] = k;
+    } else {  // groups 1.. hand their minima to group 0 (double-buffered by tile parity)
+      float* ss = xs_s + (set * 2 + int((t / kSets) & 1)) * 3 * TP;
+      int* sk = xs_k + (set * 2 + int((t / kSets) & 1)) * 3 * TP;
+      if (g > 0) {
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) ss[(g - 1) * TP + lt + LP * i] = bs[i], sk[(g - 1) * TP + lt + LP * i] = bk[i];
+      }
+      asm volatile("bar.sync %0, %1;" ::"r"(1 + set), "n"(kConsumers) : "memory");  // this set only
+      if (g == 0) {
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+          float s = bs[i];
+          int k = bk[i];
+#pragma unroll
+          for (int h = 1; h < G; ++h) {
+            const float s2 = ss[(h - 1) * TP + lt + LP * i];
+            const int k2 = sk[(h - 1) * TP + lt + LP * i];
+            if (s2 < s || (s2 == s && k2 < k)) s = s2, k = k2;
+          }
+          const long long gi = base + lt + LP * i;
+          if (gi < a.N) a.assign[gi] = k;
+        }
+      }
     }
-    tma::bar_sync_consumers<kConsumers>();
+    // release the slot: the last of the 8 warps to finish with it refills it with tile t+kStages
+    // (nobody waits on an "empty" barrier). Every x value the warp read is already consumed, the
+    // fences order those reads and the counter before the TMA (async proxy) overwrites the slot.
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence_block();
+      if (atomicAdd(released + slot, 1u) == kConsumerWarps - 1) {
+        __threadfence_block();
+        released[slot] = 0;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        if (t + kStages < n_tiles) issue(t + kStages);
+      }
+    }
   }
 }
 
+namespace {
+
+// The constant bank is one per device and module: KMEANS_ASSIGN launches on different streams are
+// ordered by an event so one launch's centroids are never overwritten while another still runs.
+// (Inside a stream capture the ordering is the graph's: captured KMEANS_ASSIGN work must not run
+// concurrently with other KMEANS_ASSIGN work.)
+std::mutex g_km_mutex;
+cudaEvent_t g_km_done[64] = {};
+
+template <int PPT, int CPT>
+cudaError_t launch_tp(const CUtensorMap& map, const KmeansArgs& a, int grid, size_t smem, cudaStream_t st) {
+  cudaError_t e =
+      cudaFuncSetAttribute(npp_kmeans_tma_kernel<PPT, CPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (e != cudaSuccess) return e;
+  npp_kmeans_tma_kernel<PPT, CPT><<<grid, kThreads, smem, st>>>(map, a);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st) {
-  const int tp = a.D <= 64 ? 256 : 128;  // DESIGN.md S8 (KMEANS_ASSIGN)
-  const size_t smem = km_smem_bytes(a.D, a.K, tp);
+  // tile: 256 points when D <= 64 (PPT points x 256/G lanes), else 128 (one point, two groups)
+  const bool small = a.D <= 64;
+  const int ppt = small ? kPptSmallD : 1;
+  const int cpt = small ? kCptSmallD : 16;
+  const int tp = ppt * kConsumers / (32 / cpt);
+  const size_t smem = km_smem_bytes(a.K, tp);
+  if (km_kpad(a.K) * a.D > kConstFloats) return cudaErrorInvalidValue;  // S8 bound (constant bank)
+  // a.per_block counts the record's tiles (256 points when D <= 64, else 128: DESIGN.md S8)
+  KmeansArgs b = a;
+  b.per_block = a.per_block * (small ? 256 : 128) / tp;
   CUtensorMap map;
   cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(kBoxCols),
                                  unsigned(tp), CU_TENSOR_MAP_SWIZZLE_128B);
   if (e != cudaSuccess) return e;
-  if (tp == 256) {
-    e = cudaFuncSetAttribute(npp_kmeans_tma_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    if (e != cudaSuccess) return e;
-    npp_kmeans_tma_kernel<4><<<grid, kThreads, smem, st>>>(map, a);
-  } else {
-    e = cudaFuncSetAttribute(npp_kmeans_tma_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    if (e != cudaSuccess) return e;
-    npp_kmeans_tma_kernel<2><<<grid, kThreads, smem, st>>>(map, a);
-  }
-  return cudaGetLastError();
+  int dev = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if ((e = cudaStreamIsCapturing(st, &cap)) != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lock(g_km_mutex);
+  if (!g_km_done[dev] && (e = cudaEventCreateWithFlags(&g_km_done[dev], cudaEventDisableTiming)) != cudaSuccess)
+    return e;
+  if (cap == cudaStreamCaptureStatusNone && (e = cudaStreamWaitEvent(st, g_km_done[dev], 0)) != cudaSuccess)
+    return e;
+  e = cudaMemcpyToSymbolAsync(km_centroids, a.c, size_t(a.K * a.D) * 4, 0, cudaMemcpyDeviceToDevice, st);
+  if (e != cudaSuccess) return e;
+  if (small)
+    e = launch_tp<kPptSmallD, kCptSmallD>(map, b, grid, smem, st);
+  else
+    e = launch_tp<1, 16>(map, b, grid, smem, st);
+  if (e != cudaSuccess) return e;
+  if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);
+  return e;
 }
 
 }  // namespace npp

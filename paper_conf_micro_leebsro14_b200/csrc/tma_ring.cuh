@@ -34,6 +34,21 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
       "r"(parity)
       : "memory");
 }
+__device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
+  unsigned ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// whole-warp wait whose exit is a vote: the compiler sees the warp converged after it (the phase
+// cannot flip back while these threads still hold the buffer), so uniform-datapath code may follow
+__device__ __forceinline__ void mbar_wait_warp(uint64_t* b, unsigned parity) {
+  while (!__all_sync(0xffffffffu, mbar_try(b, parity))) {
+  }
+}
 __device__ __forceinline__ void load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(

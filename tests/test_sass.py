@@ -1,0 +1,72 @@
+"""The built sm_100a code uses the instructions the design depends on (checked here, without a GPU,
+from `cuobjdump -sass` of the in-tree library): a compiler heuristic that silently picks a slower
+instruction form would otherwise only show up as a lower bench number.
+
+- staged sums / logreg / k-means move their tiles with TMA (UTMALDG) — DESIGN.md §6;
+- k-means reads centroids on the uniform datapath (LDCU into uniform registers feeding FFMA2), not
+  per-thread LDC, which measured ~5x slower in tools/micro_const.cu;
+- the ALU-bound x·c products run on the packed FP32 pipe (FFMA2).
+"""
+import collections
+import os
+import re
+import shutil
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIB = os.path.join(ROOT, "paper_conf_micro_leebsro14_b200", "libnpp.so")
+CUOBJDUMP = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+
+pytestmark = pytest.mark.skipif(not os.path.exists(CUOBJDUMP), reason="cuobjdump not available")
+
+
+@pytest.fixture(scope="module")
+def sass():
+    assert os.path.exists(LIB), "run python -m paper_conf_micro_leebsro14_b200.build"
+    out = subprocess.run([CUOBJDUMP, "-sass", LIB], capture_output=True, text=True, check=True).stdout
+    funcs, name = collections.defaultdict(collections.Counter), None
+    for line in out.splitlines():
+        m = re.search(r"Function : (\S+)", line)
+        if m:
+            name = m.group(1)
+            continue
+        m = re.match(r"\s+/\*[0-9a-f]+\*/\s+(?:@!?U?P\w+\s+)?([A-Z][A-Z0-9_.]*)", line)
+        if m and name:
+            funcs[name][m.group(1)] += 1
+    return funcs
+
+
+def _find(sass, *parts):
+    names = [n for n in sass if all(p in n for p in parts)]
+    assert names, parts
+    return names
+
+
+def test_all_kernels_built_for_sm100a():
+    out = subprocess.run([CUOBJDUMP, "-lelf", LIB], capture_output=True, text=True, check=True).stdout
+    archs = set(re.findall(r"sm_\d+a?", out))
+    assert archs == {"sm_100a"}, archs
+
+
+def test_staged_kernels_use_tma(sass):
+    for parts in (("npp_sum_tma_kernel",), ("npp_logreg_tma_kernel",), ("npp_kmeans_tma_kernel",)):
+        for n in _find(sass, *parts):
+            assert sass[n]["UTMALDG.2D"] + sass[n]["UBLKCP.S.G"] + sass[n]["UTMALDG.1D"] > 0, n
+
+
+def test_kmeans_centroids_on_uniform_datapath(sass):
+    for n in _find(sass, "npp_kmeans_tma_kernel"):
+        c = sass[n]
+        ffma2 = c["FFMA2"]
+        assert ffma2 >= 64, (n, ffma2)
+        # every centroid operand pair comes from a uniform register: ~one LDCU.64 per 2·PPT FFMA2,
+        # and no per-thread constant loads in the inner loop
+        assert c["LDCU.64"] + 2 * c["LDCU.128"] >= ffma2 // 8, (n, dict(c))
+        assert c["LDC.64"] <= 16, (n, c["LDC.64"])
+
+
+def test_packed_fma_in_kmeans(sass):
+    for n in _find(sass, "npp_kmeans_tma_kernel"):
+        assert sass[n]["FFMA2"] >= 2 * sass[n]["FFMA"], (n, sass[n]["FFMA2"], sass[n]["FFMA"])
