@@ -177,11 +177,16 @@ NPP_API int npp_plan_mapping(npp_plan_t plan, npp_mapping* out);
  * use with a plan; every successful execute leaves it zero-filled again (Split tickets reset). */
 NPP_API int64_t npp_plan_workspace_bytes(npp_plan_t plan);
 
-/* Enqueue the plan's kernel(s) on `stream` (async; no host sync; one kernel launch for every pattern,
- * Split combine fused). `ins` holds `n_in` device pointers in the order of the pattern table above;
+/* Enqueue the plan's kernel(s) on `stream` (async; no host sync; one kernel launch for every sum and
+ * logreg pattern, Split combine fused; KMEANS_ASSIGN adds a small centroid-pack kernel). `ins` holds `n_in` device pointers in the order of the pattern table above;
  * `out` is the device output. Vector plans (mapping.vec > 1) need 16-byte aligned pointers.
  * Errors: INVALID_ARG, ALIGNMENT, WORKSPACE, CUDA (launch error; async faults surface at the
- * caller's next synchronisation). Concurrent executes of one plan need distinct workspaces. */
+ * caller's next synchronisation). Concurrent executes of one plan need distinct workspaces.
+ * KMEANS_ASSIGN first packs the centroids as pairs (a 64 KB module buffer) and copies them
+ * device-to-device into the library's constant bank (one per device) before its kernel; executes of KMEANS_ASSIGN plans on
+ * different streams are ordered by an internal event so they never overwrite each other's
+ * centroids. Inside a stream capture that ordering is the caller's: captured KMEANS_ASSIGN work
+ * must not run concurrently with other KMEANS_ASSIGN work on the same device. */
 NPP_API int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace,
                 void* stream);
 

@@ -300,7 +300,7 @@ int64_t npp_plan_workspace_bytes(npp_plan_t plan) { return plan ? plan->map.work
 int npp_plan_launches(npp_plan_t plan) {
   if (!plan) return 0;
   if (plan->empty) return output_bytes(plan) > 0 ? 1 : 0;
-  return 1;
+  return plan->pattern == NPP_KMEANS_ASSIGN ? 2 : 1;  // k-means: centroid pack + assignment
 }
 
 void npp_plan_destroy(npp_plan_t plan) { delete plan; }

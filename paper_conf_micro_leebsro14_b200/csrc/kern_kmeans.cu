@@ -43,21 +43,21 @@ constexpr int kMaxStageBytes = 64 * 1024;
 constexpr int kSmemLimit = 227 * 1024;
 constexpr int kConstFloats = 16384;  // DESIGN.md S8: 32·⌈K/32⌉·D ≤ 16384
 
-// D <= 64: PPT points x CPT centroids per thread (G = 32/CPT groups, 256-point tiles)
-#ifndef NPP_KM_PPT
-#define NPP_KM_PPT 4
-#endif
-constexpr int kPptSmallD = NPP_KM_PPT;
-constexpr int kCptSmallD = 32 / NPP_KM_PPT;  // so that TP = PPT·256·CPT/32 = 256
-// register cap: low enough that ptxas keeps the centroid reads on the uniform datapath (LDCU);
-// with a generous budget it prefers per-thread LDC, which the constant cache serves ~5x slower
-// (tools/micro_const.cu). tests/test_sass.py checks the built kernel.
-#ifndef NPP_KM_MAXNREG
-#define NPP_KM_MAXNREG 120
-#endif
-#define NPP_KM_BOUNDS __maxnreg__(NPP_KM_MAXNREG)
 
-__constant__ float km_centroids[kConstFloats];  // [K][D] as given (padded rows: stale, see cn)
+// centroids as pairs: km_pairs[(k/2)·D + d] = (c[k & ~1][d], c[k | 1][d]), padded rows zero. One
+// packed FFMA2 then advances the dot products of two centroids with one (broadcast) x element, so
+// each accumulator half ends as a whole dot product (no final add of even/odd halves).
+__constant__ float2 km_pairs[kConstFloats / 2];
+__device__ float2 km_pack_buf[kConstFloats / 2];  // staging for the copy into the constant bank
+
+__global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int Kp, int D) {
+  const int n = Kp / 2 * D;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int k2 = i / D, d = i - k2 * D;
+    const int k = 2 * k2;
+    km_pack_buf[i] = make_float2(k < K ? c[k * D + d] : 0.f, k + 1 < K ? c[(k + 1) * D + d] : 0.f);
+  }
+}
 
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
@@ -86,8 +86,8 @@ __device__ __forceinline__ void ffma2(float2& acc, const float2 a, const float2 
 // PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
 // groups; a tile is TP = PPT·256/G points.
 template <int PPT, int CPT>
-__global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUtensorMap map,
-                                                                     KmeansArgs a) {
+__device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const KmeansArgs& a) {
+  const CUtensorMap& map = *mapp;
   constexpr int G = 32 / CPT;
   constexpr int LP = kConsumers / G;  // threads (and point lanes) per centroid group
   constexpr int TP = PPT * LP;        // points per tile
@@ -122,8 +122,7 @@ __global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUte
     }
     tma::mbar_fence_init();
   }
-  // ||c_k||² (fp32 FMA chain over d); padded rows get +inf and are never selected (their
-  // constant-bank rows are stale: inf − 2·finite = inf, inf − inf = NaN, both lose)
+  // ||c_k||² (fp32 FMA chain over d); padded rows (zero) get +inf and are never selected
   for (int k = threadIdx.x; k < Kp; k += kThreads) {
     float s = 0.f;
     if (k < K)
@@ -165,12 +164,12 @@ __global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUte
     for (int i = 0; i < PPT; ++i) bs[i] = __int_as_float(0x7f800000), bk[i] = 0x7fffffff;
     for (int kc = 0; kc < Kp; kc += 32) {
       const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
-      float2 acc[PPT][CPT];
+      float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1
 #pragma unroll
       for (int i = 0; i < PPT; ++i)
 #pragma unroll
-        for (int m = 0; m < CPT; ++m) acc[i][m] = make_float2(0.f, 0.f);
-      const float* cq = km_centroids + k0 * D;
+        for (int p = 0; p < CPT / 2; ++p) acc[i][p] = make_float2(0.f, 0.f);
+      const float2* cq = km_pairs + (k0 >> 1) * D;
 #pragma unroll 2
       for (int d4 = 0; d4 < nd4; ++d4) {
         const unsigned char* xb = tile + (d4 >> 3) * (TP * 128) + ((unsigned(d4 & 7) ^ key) << 4);
@@ -178,23 +177,29 @@ __global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUte
 #pragma unroll
         for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
 #pragma unroll
-        for (int m = 0; m < CPT; ++m) {
-          const float4 cv = *reinterpret_cast<const float4*>(cq + m * D + 4 * d4);  // warp-uniform
+        for (int p = 0; p < CPT / 2; ++p) {
 #pragma unroll
-          for (int i = 0; i < PPT; ++i) {
-            ffma2(acc[i][m], make_float2(xv[i].x, xv[i].y), make_float2(cv.x, cv.y));
-            ffma2(acc[i][m], make_float2(xv[i].z, xv[i].w), make_float2(cv.z, cv.w));
+          for (int q = 0; q < 4; ++q) {
+            const float2 cv = cq[p * D + 4 * d4 + q];  // warp-uniform
+#pragma unroll
+            for (int i = 0; i < PPT; ++i) {
+              const float xs = q == 0 ? xv[i].x : q == 1 ? xv[i].y : q == 2 ? xv[i].z : xv[i].w;
+              ffma2(acc[i][p], make_float2(xs, xs), cv);
+            }
           }
         }
       }
 #pragma unroll
-      for (int m = 0; m < CPT; ++m) {  // increasing k within the thread: strict < keeps the first
-        const int k = k0 + m;
-        const float nk = cn[k];
+      for (int p = 0; p < CPT / 2; ++p) {  // increasing k within the thread: strict < keeps the first
 #pragma unroll
-        for (int i = 0; i < PPT; ++i) {
-          const float s = fmaf(-2.f, acc[i][m].x + acc[i][m].y, nk);
-          if (s < bs[i]) bs[i] = s, bk[i] = k;
+        for (int h = 0; h < 2; ++h) {
+          const int k = k0 + 2 * p + h;
+          const float nk = cn[k];
+#pragma unroll
+          for (int i = 0; i < PPT; ++i) {
+            const float s = fmaf(-2.f, h ? acc[i][p].y : acc[i][p].x, nk);
+            if (s < bs[i]) bs[i] = s, bk[i] = k;
+          }
         }
       }
     }
@@ -245,6 +250,24 @@ __global__ void NPP_KM_BOUNDS npp_kmeans_tma_kernel(const __grid_constant__ CUte
   }
 }
 
+// One wrapper per tile shape, each with its own register cap: the cap is what keeps ptxas on the
+// uniform datapath (LDCU) for the centroid operands, and the value that does so differs per shape
+// (tests/test_sass.py checks the result).
+#ifndef NPP_KM_MAXNREG_D64
+#define NPP_KM_MAXNREG_D64 80
+#endif
+#ifndef NPP_KM_MAXNREG_D128
+#define NPP_KM_MAXNREG_D128 48
+#endif
+__global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
+                                                                         KmeansArgs a) {
+  kmeans_body<4, 8>(&map, a);  // D <= 64: 256-point tiles
+}
+__global__ void __maxnreg__(NPP_KM_MAXNREG_D128) npp_kmeans_tma_kernel_d128(
+    const __grid_constant__ CUtensorMap map, KmeansArgs a) {
+  kmeans_body<2, 8>(&map, a);  // 64 < D <= 128: 128-point tiles
+}
+
 namespace {
 
 // The constant bank is one per device and module: KMEANS_ASSIGN launches on different streams are
@@ -254,28 +277,23 @@ namespace {
 std::mutex g_km_mutex;
 cudaEvent_t g_km_done[64] = {};
 
-template <int PPT, int CPT>
-cudaError_t launch_tp(const CUtensorMap& map, const KmeansArgs& a, int grid, size_t smem, cudaStream_t st) {
-  cudaError_t e =
-      cudaFuncSetAttribute(npp_kmeans_tma_kernel<PPT, CPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+cudaError_t launch_tp(void (*kern)(const CUtensorMap, KmeansArgs), const CUtensorMap& map, const KmeansArgs& a,
+                      int grid, size_t smem, cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
-  npp_kmeans_tma_kernel<PPT, CPT><<<grid, kThreads, smem, st>>>(map, a);
+  kern<<<grid, kThreads, smem, st>>>(map, a);
   return cudaGetLastError();
 }
 
 }  // namespace
 
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st) {
-  // tile: 256 points when D <= 64 (PPT points x 256/G lanes), else 128 (one point, two groups)
+  // tile: 256 points when D <= 64 (4 points x 64 lanes), else 128 (2 points x 64 lanes); both
+  // with 4 centroid groups of 8 (S8)
   const bool small = a.D <= 64;
-  const int ppt = small ? kPptSmallD : 1;
-  const int cpt = small ? kCptSmallD : 16;
-  const int tp = ppt * kConsumers / (32 / cpt);
+  const int tp = small ? 256 : 128;
   const size_t smem = km_smem_bytes(a.K, tp);
   if (km_kpad(a.K) * a.D > kConstFloats) return cudaErrorInvalidValue;  // S8 bound (constant bank)
-  // a.per_block counts the record's tiles (256 points when D <= 64, else 128: DESIGN.md S8)
-  KmeansArgs b = a;
-  b.per_block = a.per_block * (small ? 256 : 128) / tp;
   CUtensorMap map;
   cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(kBoxCols),
                                  unsigned(tp), CU_TENSOR_MAP_SWIZZLE_128B);
@@ -290,12 +308,14 @@ cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStr
     return e;
   if (cap == cudaStreamCaptureStatusNone && (e = cudaStreamWaitEvent(st, g_km_done[dev], 0)) != cudaSuccess)
     return e;
-  e = cudaMemcpyToSymbolAsync(km_centroids, a.c, size_t(a.K * a.D) * 4, 0, cudaMemcpyDeviceToDevice, st);
+  const int Kp = int(km_kpad(a.K)), D = int(a.D);
+  npp_kmeans_pack_kernel<<<8, 256, 0, st>>>(a.c, int(a.K), Kp, D);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  void* pack = nullptr;
+  if ((e = cudaGetSymbolAddress(&pack, km_pack_buf)) != cudaSuccess) return e;
+  e = cudaMemcpyToSymbolAsync(km_pairs, pack, size_t(Kp) * D * 4, 0, cudaMemcpyDeviceToDevice, st);
   if (e != cudaSuccess) return e;
-  if (small)
-    e = launch_tp<kPptSmallD, kCptSmallD>(map, b, grid, smem, st);
-  else
-    e = launch_tp<1, 16>(map, b, grid, smem, st);
+  e = launch_tp(small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128, map, a, grid, smem, st);
   if (e != cudaSuccess) return e;
   if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);
   return e;

@@ -91,7 +91,7 @@ def _check_kmeans_valid(a, x, c):
 
 
 @pytest.mark.parametrize("N,D,K", [(10000, 64, 32), (1000, 12, 5), (4099, 128, 96), (127, 4, 1),
-                                   (20000, 64, 256), (129, 32, 33)])
+                                   (20000, 64, 256), (129, 32, 33), (5000, 128, 128), (3000, 8, 256)])
 def test_kmeans_integer_data_exact(npp, cuda_device, N, D, K):
     x, c = gen.kmeans_inputs(N, D, K, integer=True, device=cuda_device)
     p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
@@ -122,6 +122,32 @@ def test_kmeans_full_size_sampled(npp, cuda_device):
                      torch.randint(0, N, (12000,), generator=torch.Generator().manual_seed(3))]).to(cuda_device)
     agree = _check_kmeans_valid(a.index_select(0, idx), x.index_select(0, idx), c)
     assert agree > 0.999
+
+
+def test_kmeans_two_streams_distinct_centroids(npp, cuda_device):
+    """The centroids live in one constant bank per device: interleaved executes of two plans on two
+    streams, with different centroids and no host sync in between, must each see their own."""
+    N = 1 << 16
+    xa, ca = gen.kmeans_inputs(N, 64, 32, seed=21, integer=True, device=cuda_device)
+    xb, cb = gen.kmeans_inputs(N, 32, 7, seed=22, integer=True, device=cuda_device)
+    pa = npp.Plan("KMEANS_ASSIGN", (N, 64, 32), "f32", "AUTO")
+    pb = npp.Plan("KMEANS_ASSIGN", (N, 32, 7), "f32", "AUTO")
+    sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    outs = []
+    for _ in range(8):
+        oa, ob = pa.new_out(), pb.new_out()
+        with torch.cuda.stream(sa):
+            pa.execute([xa, ca], oa, stream=sa)
+        with torch.cuda.stream(sb):
+            pb.execute([xb, cb], ob, stream=sb)
+        outs.append((oa, ob))
+    torch.cuda.synchronize()
+    wa = okm.assign(xa.cpu().numpy(), ca.cpu().numpy()).tolist()
+    wb = okm.assign(xb.cpu().numpy(), cb.cpu().numpy()).tolist()
+    for oa, ob in outs:
+        assert oa.cpu().numpy().tolist() == wa
+        assert ob.cpu().numpy().tolist() == wb
 
 
 def test_kmeans_points_on_centroids(npp, cuda_device):
