@@ -118,8 +118,8 @@ class Item:
     def __init__(self, name, plan, ins, out, algo_bytes):
         self.name, self.plan, self.ins, self.out, self.bytes = name, plan, ins, out, algo_bytes
 
-    def run(self, stream):
-        self.plan.execute(self.ins, self.out, stream=stream)
+    def run(self, stream, overlap=False):
+        self.plan.execute(self.ins, self.out, stream=stream, overlap=overlap)
 
 
 def build_paper(npp, gen, torch, rank, world, strategy, device):
@@ -288,6 +288,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
+    ap.add_argument("--no-overlap", action="store_true",
+                    help="serialise the step's launches (no NPP_EXEC_OVERLAP programmatic dependent launch)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -306,9 +308,13 @@ def main():
     stream = torch.cuda.Stream(device=device)  # all timed work is enqueued on this stream
     use_graph = world == 1 and not args.eager
 
+    # the step's inputs are resident before it starts, so each launch may overlap the previous one's
+    # drain (npp_execute_ex NPP_EXEC_OVERLAP); outputs still wait for the previous kernel
+    overlap = not args.no_overlap
+
     def step():
         for it in items:
-            it.run(stream)
+            it.run(stream, overlap)
         for b in reduce_bufs:
             with torch.cuda.stream(stream):
                 dist.all_reduce(b)
@@ -356,6 +362,8 @@ def main():
     # per-kernel durations: each launch replayed back to back from a graph, alternating its input with
     # another equal-size buffer of the step so that every launch reads cold HBM
     per_kernel_us = [kernel_us(torch, it, items[(i + 1) % len(items)], stream) for i, it in enumerate(items)]
+    per_kernel_ov = [kernel_us(torch, it, items[(i + 1) % len(items)], stream, overlap=True)
+                     for i, it in enumerate(items)]
     peak, peak_src = measured_peaks()
     dom = max(range(len(items)), key=lambda i: per_kernel_us[i])
     dom_gbs = items[dom].bytes / (per_kernel_us[dom] * 1e-6) / 1e9
@@ -365,6 +373,8 @@ def main():
                            "frac_of_measured": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / peak, 4),
                            "frac_of_8TBs": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / 8000.0, 4),
                            "us": round(per_kernel_us[i], 2),
+                           "us_overlapped": round(per_kernel_ov[i], 2),
+                           "GB/s_overlapped": round(it.bytes / (per_kernel_ov[i] * 1e-6) / 1e9, 1),
                            "mapping": mapping_brief(it.plan.mapping)}
                  for i, it in enumerate(items)}
 
@@ -372,8 +382,10 @@ def main():
            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
            "scaling": "weak" if args.workload == "paper" else "strong", "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (counter-based U[0,1) fp32, seeded)",
-           "config": config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
-                                else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),
+           "config": dict(config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
+                                     else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),
+                          launches="programmatic dependent launch (NPP_EXEC_OVERLAP)" if overlap
+                          else "serialised"),
            "per_shape": per_shape,
            "roofline": roofline(items[dom], per_kernel_us[dom], dom_gbs, peak, peak_src, traffic, flops),
            "clocks": sampler.summary(),
@@ -437,9 +449,11 @@ def e2e_host(items, torch, stream, world, dist, steps=3):
             "steps": steps, "api": "npp_execute_host (pinned host buffers, blocking)"}
 
 
-def kernel_us(torch, item, other, stream, reps=8):
+def kernel_us(torch, item, other, stream, reps=8, overlap=False):
     """Average duration of one launch of item's plan: a graph of 2*reps launches alternating item's
-    input with `other`'s (same byte size, viewed with item's shape) so no launch finds its input in L2."""
+    input with `other`'s (same byte size, viewed with item's shape) so no launch finds its input in L2.
+    overlap=False: serialised launches (the per-kernel duration the roofline uses); True: launch-to-launch
+    interval with NPP_EXEC_OVERLAP."""
     alt = other.ins[0].view(item.ins[0].shape) if other.ins[0].numel() == item.ins[0].numel() else None
     firsts = [item.ins[0], alt] if alt is not None and alt.data_ptr() != item.ins[0].data_ptr() else [item.ins[0]]
     inputs = [[f] + list(item.ins[1:]) for f in firsts]
@@ -451,7 +465,7 @@ def kernel_us(torch, item, other, stream, reps=8):
     with torch.cuda.stream(stream):
         with torch.cuda.graph(g, stream=stream):
             for r in range(2 * reps):
-                item.plan.execute(inputs[r % len(inputs)], item.out, stream=stream)
+                item.plan.execute(inputs[r % len(inputs)], item.out, stream=stream, overlap=overlap)
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with torch.cuda.stream(stream):
         g.replay()

@@ -190,6 +190,17 @@ NPP_API int64_t npp_plan_workspace_bytes(npp_plan_t plan);
 NPP_API int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace,
                 void* stream);
 
+/* Execution flags of npp_execute_ex. */
+#define NPP_EXEC_OVERLAP 1u
+/* npp_execute with flags. NPP_EXEC_OVERLAP: the caller asserts that no work enqueued earlier on
+ * `stream` writes this call's inputs (e.g. inputs resident before the preceding kernel started); the
+ * staged (TMA) kernels are then launched as programmatic dependent launches (sm_90+ PDL): their blocks
+ * start streaming the inputs while the previous kernel on the stream drains, and they write `out` and
+ * the workspace only after that kernel has completed (griddepcontrol.wait). Other plans ignore the
+ * flag. Unknown flag bits: NPP_ERR_INVALID_ARG. Otherwise identical to npp_execute. */
+NPP_API int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace,
+                           void* stream, unsigned flags);
+
 /* End-to-end call with HOST buffers: copies `host_ins` (pinned or pageable host memory, same order
  * and sizes as npp_execute) into the caller's device buffers `dev_ins`, executes, copies the result
  * into `host_out` and synchronises `stream` before returning. */

@@ -306,15 +306,29 @@ def staged_tiles(nest, dtype):
     return BR, BC, cdiv(O, BC), cdiv(I, BR)
 
 
+POOL_DIV = 8                                      # DESIGN.md S8 balance rule
+POOL_UNIT = 4
+WHOLE_UNIT_MAX = 8
+
+
+def balance(To, Ti, lim):
+    """DESIGN.md S8 balance rule over T = To*Ti tiles: G = min(SMs, T) persistent blocks; pool claim
+    unit U = Ti if Ti <= 8 else 4; Ts = U*floor((T - floor(T/8))/U) tiles split statically (block b
+    streams [b*Ts/G, (b+1)*Ts/G)); the units of [Ts, T) are claimed in order by whichever block is
+    free. Returns (G, U, Ts)."""
+    T = To * Ti
+    G = min(lim["sm_count"], T)
+    U = Ti if Ti <= WHOLE_UNIT_MAX else POOL_UNIT
+    return G, U, U * ((T - T // POOL_DIV) // U)
+
+
 def r2_staged(nest, dtype, lim):
-    """DESIGN.md S8, staged family: persistent blocks (one per SM) claim 32-row x 1 KB tiles in
-    outer-major order from a global counter, CL tiles per claim; the inner level is Split(Ti)."""
+    """DESIGN.md S8, staged family: persistent blocks (one per SM) stream 32-row x 1 KB tiles in
+    outer-major order (static range + pool, balance()); the inner level is Split(Ti)."""
     esz = DTYPE_SIZE[dtype]
     BR, BC, To, Ti = staged_tiles(nest, dtype)
     I = nest["levels"][1][0]
-    P = cdiv(To * Ti, min(lim["sm_count"], To * Ti))   # tiles per block: block b streams [bP, (b+1)P)
-    G = cdiv(To * Ti, P)
-    CL = P
+    G, CL, _ = balance(To, Ti, lim)
     if nest["pattern"] == "SUM_ROWS":
         blocks = (8, 32)
         spans = (SPAN_N, ALL if Ti == 1 else SPLIT)
@@ -438,10 +452,11 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
         B, C = _eff(nest["levels"][0][0]), _eff(nest["levels"][2][0])
         rec["workspace_bytes"] = 256 * cdiv(4 * B, 256) + 256 * cdiv(8 * B * C, 256)
     if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
-        if staged:  # counters + fp64/integer accumulators [O] (S8 staged)
+        if staged:  # pool counters (256 B) + tickets [To] + accumulators [O] (S8 staged)
             O = _eff(nest["levels"][0][0])
             To = staged_tiles(nest, dtype)[2]   # tickets [To] u32, then accumulators [O]
-            rec["workspace_bytes"] = 256 * cdiv(4 * To, 256) + 256 * cdiv(O * acc_bytes(nest["pattern"], dtype), 256)
+            rec["workspace_bytes"] = (256 + 256 * cdiv(4 * To, 256)
+                                      + 256 * cdiv(O * acc_bytes(nest["pattern"], dtype), 256))
         elif levels[1]["grid"] >= 2:
             O = _eff(nest["levels"][0][0])
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)

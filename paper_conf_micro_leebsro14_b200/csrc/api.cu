@@ -137,8 +137,8 @@ void debug_print_times(const unsigned long long* dbg, int G, cudaStream_t st) {
       mn[i] = v < mn[i] ? v : mn[i];
       sm[i] += v;
     }
-  std::fprintf(stderr, "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] barrier[%.2f..%.2f]\n",
-               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], mx[2]);
+  std::fprintf(stderr, "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] combiner_end[%.2f avg %.2f max %.2f]\n",
+               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], sm[2] / G, mx[2]);
 }
 
 }  // namespace
@@ -306,6 +306,16 @@ int npp_plan_launches(npp_plan_t plan) {
 void npp_plan_destroy(npp_plan_t plan) { delete plan; }
 
 int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream) {
+  return npp_execute_ex(plan, ins, n_in, out, workspace, stream, 0u);
+}
+
+int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream,
+                   unsigned flags) {
+  if (flags & ~NPP_EXEC_OVERLAP) {
+    set_error("unknown npp_execute_ex flag bits");
+    return NPP_ERR_INVALID_ARG;
+  }
+  const bool overlap = (flags & NPP_EXEC_OVERLAP) != 0;
   if (!plan) {
     set_error("plan is NULL");
     return NPP_ERR_INVALID_ARG;
@@ -389,9 +399,13 @@ int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, vo
     s.O = rows ? R : C;
     s.To = t.To;
     s.Ti = t.Ti;
-    s.per_block = m.claim_tiles;
-    s.tickets = static_cast<unsigned*>(workspace);
-    s.acc = static_cast<char*>(workspace) + ((t.To * 4 + 255) / 256) * 256;
+    const npp::StagedBalance bal = npp::staged_balance(t.To, t.Ti, plan->lim.sm_count);
+    s.static_tiles = bal.Ts;
+    s.unit = bal.U;
+    s.early_reads = overlap ? 1 : 0;
+    s.pool = static_cast<unsigned*>(workspace);  // S9 staged workspace: [256 B pool][tickets][acc]
+    s.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + 256);
+    s.acc = static_cast<char*>(workspace) + 256 + ((t.To * 4 + 255) / 256) * 256;
     // measurement knob: NPP_DEBUG_TIMES=1 prints per-phase block timestamps (synchronises the stream)
     static unsigned long long* dbg = nullptr;
     const bool want_times = getenv("NPP_DEBUG_TIMES") != nullptr;

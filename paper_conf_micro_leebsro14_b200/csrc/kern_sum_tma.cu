@@ -43,7 +43,10 @@ constexpr int kTileRows = 32;
 constexpr int kTileBytes = kTileRows * 1024;
 constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
-constexpr int kThreads = kConsumers + 32;  // + one producer warp
+constexpr int kProducerWarp = kConsumerWarps;      // warp 8: TMA producer (one elected lane)
+constexpr int kCombinerWarp = kConsumerWarps + 1;  // warp 9: tickets + conversion of cut outer tiles
+constexpr int kThreads = kConsumers + 64;
+constexpr int kFlushRing = 8;  // flushes of cut outer tiles in flight between consumers and the combiner
 constexpr int kSmemHeader = 1024;          // mbarriers + per-slot tile ids; tiles start 1 KB-aligned
 constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes;
 
@@ -73,6 +76,15 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, i
           smem_u32(dst)),
       "l"(map), "r"(x), "r"(y), "r"(smem_u32(bar))
       : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
+  unsigned ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
 }
 __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -115,12 +127,6 @@ __device__ __forceinline__ A warp_sum(A v) {
   return v;
 }
 
-// read-and-zero of one accumulator (only the last contributor of an outer tile calls this)
-__device__ __forceinline__ double take(double* p) {
-  return __longlong_as_double((long long)atomicExch(reinterpret_cast<unsigned long long*>(p), 0ull));
-}
-__device__ __forceinline__ unsigned take(unsigned* p) { return atomicExch(p, 0u); }
-__device__ __forceinline__ unsigned long long take(unsigned long long* p) { return atomicExch(p, 0ull); }
 
 }  // namespace
 
@@ -134,22 +140,33 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   extern __shared__ __align__(1024) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + kStages;
-  long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);  // tile id, bit 62: flush after
-  unsigned* s_last = reinterpret_cast<unsigned*>(slot_tile + kStages);
+  uint64_t* fl_full = empty + kStages;        // [kFlushRing] consumer warps -> combiner
+  uint64_t* fl_free = fl_full + kFlushRing;   // [kFlushRing] combiner -> consumers
+  long long* slot_tile = reinterpret_cast<long long*>(fl_free + kFlushRing);  // tile | kFlush, -1 = end
+  long long* fl_ot = slot_tile + kStages;     // [kFlushRing] outer tile of a flush, -1 = end
+  unsigned* fl_cnt = reinterpret_cast<unsigned*>(fl_ot + kFlushRing);  // tiles it contributes
   unsigned char* tiles = smem + kSmemHeader;
   Acc* accg = static_cast<Acc*>(a.acc);
   constexpr long long kFlush = 1ll << 62;
 
+  // PDL: let the next launch in the stream become resident as SMs free up (its griddepcontrol.wait
+  // still orders it after this grid's completion).
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long bid = blockIdx.x;
+  const long long bid = blockIdx.x, G = gridDim.x;
   const long long total = a.To * a.Ti;
-  const long long P = a.per_block;
-  const long long r0 = bid * P, r1 = (total < r0 + P) ? total : r0 + P;  // my tile range
+  const long long s0 = bid * a.static_tiles / G, s1 = (bid + 1) * a.static_tiles / G;  // static range
+  const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(full + i, 1);
       mbar_init(empty + i, kConsumerWarps);
+    }
+    for (int i = 0; i < kFlushRing; ++i) {
+      mbar_init(fl_full + i, kConsumerWarps);
+      mbar_init(fl_free + i, 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     if (a.dbg_times) {
@@ -161,13 +178,41 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   }
   __syncthreads();
 
-  if (warp == kConsumerWarps) {
+  if (warp == kProducerWarp) {
     // ------------------------------------------------------------ producer: one elected lane
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(&map) : "memory");
+      long long sn = s0, u_cur = 0, u_end = 0;
+      // Every launch is a programmatic dependent launch: this block may already be resident while the
+      // previous kernel in the stream drains. Unless the caller asserted NPP_EXEC_OVERLAP (inputs not
+      // written by earlier stream work), the first read waits for that kernel to complete.
+      bool waited = !a.early_reads;
+      if (waited) asm volatile("griddepcontrol.wait;" ::: "memory");
+      // static range, then pool units in claim order (S8 balance rule)
+      auto next_tile = [&]() -> long long {
+        if (sn < s1) return sn++;
+        if (u_cur < u_end) return u_cur++;
+        if (!waited) {  // the pool counter is workspace: touch it only after the previous grid is done
+          asm volatile("griddepcontrol.wait;" ::: "memory");
+          waited = true;
+        }
+        const unsigned k = atomicAdd(a.pool, 1u);
+        const long long c = a.static_tiles + (long long)k * U;
+        if (c >= total) {
+          // every producer makes exactly one failing claim, so the counter ends at units + G: the
+          // block taking the last value re-arms it for the next launch
+          if ((long long)k + 1 == (total - a.static_tiles + U - 1) / U + G) a.pool[0] = 0u;
+          return -1;
+        }
+        u_cur = c;
+        u_end = (c + U < total) ? c + U : total;
+        return u_cur++;
+      };
+      long long cur = next_tile();
       long long t = 0;
-      for (long long cur = r0; cur < r1; ++cur, ++t) {
-        const bool flush = cur + 1 >= r1 || ((cur + 1) / a.Ti) != (cur / a.Ti);
+      for (; cur >= 0; ++t) {
+        const long long nxt = next_tile();  // claimed one ahead: its latency hides behind the slot wait
+        const bool flush = nxt < 0 || (nxt / a.Ti) != (cur / a.Ti);
         const int slot = int(t % kStages);
         if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
         slot_tile[slot] = cur | (flush ? kFlush : 0);
@@ -176,8 +221,68 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         const int x = int(ROWS ? it * BC : ot * BC);
         const int y = int(ROWS ? ot * kTileRows : it * kTileRows);
         tma_load_2d(tiles + slot * kTileBytes, &map, x, y, full + slot);
+        cur = nxt;
       }
+      const int slot = int(t % kStages);  // end marker: an arrival without bytes
+      if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
+      slot_tile[slot] = -1;
+      mbar_arrive(full + slot);
     }
+  } else if (warp == kCombinerWarp) {
+    // ------------------------------------------------------------ combiner: the fused Split combine
+    // of outer tiles this block only partly covered. Consumers RED their partials into
+    // the accumulators and hand the flush over through fl_full (CTA-scope release/acquire); here one
+    // gpu-scope fence publishes them (the barrier-then-release pattern), the ticket counts tiles, and
+    // whoever completes the Ti tiles of ot converts its outputs — off the consumers' critical path.
+    // Flushes are taken in batches: lane j owns the j-th ready entry, so the fences and ticket round
+    // trips of up to kFlushRing flushes overlap.
+    for (long long k = 0;;) {
+      mbar_wait(fl_full + int(k % kFlushRing), unsigned((k / kFlushRing) & 1));
+      int nb = 1;
+      while (nb < kFlushRing &&
+             mbar_try(fl_full + int((k + nb) % kFlushRing), unsigned(((k + nb) / kFlushRing) & 1)))
+        ++nb;
+      const int i = int((k + lane) % kFlushRing);
+      const long long ot = lane < nb ? fl_ot[i] : -1;
+      const unsigned cnt = lane < nb ? fl_cnt[i] : 0u;
+      const unsigned ends = __ballot_sync(0xffffffffu, lane < nb && ot < 0);
+      const int n = ends ? __ffs(ends) - 1 : nb;  // entries before the end marker
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      bool last = false;
+      if (lane < n) {
+        const unsigned prev = atomicAdd(a.tickets + ot, cnt);
+        last = prev + cnt == unsigned(a.Ti);
+        if (last) a.tickets[ot] = 0u;
+      }
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      unsigned lasts = __ballot_sync(0xffffffffu, last);
+      while (lasts) {  // every contribution to these outer tiles is in: read (L2), convert, re-zero
+        const int j = __ffs(lasts) - 1;
+        lasts &= lasts - 1;
+        const long long o0 = __shfl_sync(0xffffffffu, ot, j) * OUT_PER_TILE;
+        const long long oend = ROWS ? a.R : a.C;
+        constexpr int J = OUT_PER_TILE / 32;
+        Acc v[J];
+#pragma unroll
+        for (int q = 0; q < J; ++q) {
+          const long long o = o0 + lane + 32 * q;
+          v[q] = o < oend ? __ldcg(accg + o) : Acc(0);
+        }
+#pragma unroll
+        for (int q = 0; q < J; ++q) {
+          const long long o = o0 + lane + 32 * q;
+          if (o < oend) {
+            __stcg(accg + o, Acc(0));
+            static_cast<T*>(a.out)[o] = SOps<T>::finish(v[q]);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane < n) mbar_arrive(fl_free + i);
+      k += n;
+      if (ends) break;
+    }
+    if (a.dbg_times && lane == 0) a.dbg_times[bid * 4 + 2] = gtimer();
   } else {
     // ------------------------------------------------------------ consumers
     constexpr int kGroups = ROWS ? 1 : 256 / BC;   // MX row groups (1 for 4-byte types, 2 for 8-byte)
@@ -185,11 +290,14 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     const int col = threadIdx.x % BC;
     const int rg = threadIdx.x / BC;
     Acc acc[4] = {0, 0, 0, 0};  // RX: rows 4w..4w+3; MX: acc[0] = column col
-    const long long n_tiles = r1 - r0;
-    for (long long t = 0; t < n_tiles; ++t) {
+    unsigned n_acc = 0;         // tiles of the current outer tile accumulated since the last flush
+    long long nfl = 0;          // flushes handed to the combiner
+    bool waited = false;
+    for (long long t = 0;; ++t) {
       const int slot = int(t % kStages);
       mbar_wait(full + slot, unsigned((t / kStages) & 1));
       const long long tag = slot_tile[slot];
+      if (tag < 0) break;
       const unsigned char* tile = tiles + slot * kTileBytes;
       if constexpr (ROWS) {
 #pragma unroll
@@ -215,14 +323,18 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
           for (int rr = 0; rr < kRowsPer; ++rr) acc[0] += Acc(v[rr]);
         }
       }
+      ++n_acc;
       __syncwarp();
       if (lane == 0) mbar_arrive(empty + slot);
       if (!(tag & kFlush)) continue;
 
-      // ---- flush the partial of outer tile ot
+      // ---- flush the partial of outer tile ot (n_acc of its Ti tiles)
+      if (!waited) {  // out / accumulators: only after the previous grid in the stream is done
+        asm volatile("griddepcontrol.wait;" ::: "memory");
+        waited = true;
+      }
       const long long ot = (tag & ~kFlush) / a.Ti;
-      const long long f0 = ot * a.Ti, f1 = (total < f0 + a.Ti) ? total : f0 + a.Ti;  // tiles of ot
-      const bool owned = f0 >= r0 && f1 <= r1;
+      const bool whole = n_acc == unsigned(a.Ti);  // this block added every tile of ot
       long long oidx[4];
       Acc val[4];
       bool mine[4];
@@ -241,43 +353,36 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         acc[0] = 0;
       }
       constexpr int NV = ROWS ? 4 : 1;
-      if (owned) {
+      const unsigned contributed = n_acc;
+      n_acc = 0;
+      if (whole && kGroups == 1) {
 #pragma unroll
         for (int i = 0; i < NV; ++i)
-          if (mine[i]) {
-            if (kGroups == 1) {
-              static_cast<T*>(a.out)[oidx[i]] = SOps<T>::finish(val[i]);
-            } else {
-              atomicAdd(accg + oidx[i], val[i]);  // two row halves meet in the accumulator
-            }
-          }
-        if (kGroups == 1) continue;
-      } else {
+          if (mine[i]) static_cast<T*>(a.out)[oidx[i]] = SOps<T>::finish(val[i]);
+        continue;
+      }
+      const int fi = int(nfl % kFlushRing);
+      if (nfl >= kFlushRing) mbar_wait(fl_free + fi, unsigned(((nfl / kFlushRing) - 1) & 1));
 #pragma unroll
-        for (int i = 0; i < NV; ++i)
-          if (mine[i]) atomicAdd(accg + oidx[i], val[i]);
-      }
-      // ticket: the last of the blocks (or row halves) contributing to ot converts its outputs
-      __threadfence();
-      consumers_sync();
-      if (threadIdx.x == 0) {
-        const long long b_first = f0 / P, b_last = (f1 - 1) / P;
-        const unsigned contributors = unsigned(b_last - b_first + 1);
-        const unsigned prev = atomicAdd(a.tickets + ot, 1u);
-        *s_last = (prev + 1 == contributors) ? 1u : 0u;
-        if (prev + 1 == contributors) a.tickets[ot] = 0u;
-      }
-      consumers_sync();
-      if (*s_last) {
-        __threadfence();
-        const long long o0 = ot * OUT_PER_TILE;
-        const long long oend = ROWS ? a.R : a.C;
-        for (int j = threadIdx.x; j < OUT_PER_TILE; j += kConsumers) {
-          const long long o = o0 + j;
-          if (o < oend) static_cast<T*>(a.out)[o] = SOps<T>::finish(take(accg + o));
+      for (int i = 0; i < NV; ++i)
+        if (mine[i]) atomicAdd(accg + oidx[i], val[i]);
+      __syncwarp();
+      if (lane == 0) {
+        if (warp == 0) {
+          fl_ot[fi] = ot;
+          fl_cnt[fi] = contributed;
         }
+        mbar_arrive(fl_full + fi);
       }
-      consumers_sync();
+      ++nfl;
+    }
+    // end marker for the combiner
+    const int fi = int(nfl % kFlushRing);
+    if (nfl >= kFlushRing) mbar_wait(fl_free + fi, unsigned(((nfl / kFlushRing) - 1) & 1));
+    __syncwarp();
+    if (lane == 0) {
+      if (warp == 0) fl_ot[fi] = -1;
+      mbar_arrive(fl_full + fi);
     }
   }
   if (a.dbg_times && threadIdx.x == 0) a.dbg_times[bid * 4 + 1] = gtimer();
@@ -311,8 +416,7 @@ cudaError_t launch_typed(const CUtensorMap& map, const StagedArgs& a, int grid, 
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  kern<<<grid, kThreads, kSmemBytes, st>>>(map, a);
-  return cudaGetLastError();
+  return launch_pdl(kern, grid, kThreads, kSmemBytes, st, true, map, a);
 }
 
 }  // namespace

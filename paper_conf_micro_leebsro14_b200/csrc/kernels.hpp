@@ -4,10 +4,30 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <utility>
 
 #include "npp.h"
 
 namespace npp {
+
+// Launch `kern` on `st`; with `overlap` as a programmatic dependent launch (PDL): its blocks may become
+// resident while the previous kernel in the stream drains; the kernel orders itself after that kernel
+// with `griddepcontrol.wait` (before its first read, or — NPP_EXEC_OVERLAP — before its first write).
+template <typename... Params, typename... Args>
+cudaError_t launch_pdl(void (*kern)(Params...), int grid, int threads, int smem, cudaStream_t st, bool overlap,
+                       Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(unsigned(grid));
+  cfg.blockDim = dim3(unsigned(threads));
+  cfg.dynamicSmemBytes = size_t(smem);
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = overlap ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 // Arguments of one 2-level sum launch (S9). Element (o, i) of the nest lives at
 // m[o*so + i*si]; level o is split into go blocks of co indices, level i into gi blocks of ci.
@@ -28,15 +48,19 @@ cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumA
 int sum_kernels_max_regs();
 
 // Arguments of one staged (TMA) sum launch (S8 staged): the matrix is [R x C]; tiles are
-// 32 rows x 1 KB, To x Ti of them in outer-major order; persistent blocks claim `claim` tiles at a time.
+// 32 rows x 1 KB, To x Ti of them in outer-major order. Block b of G streams the static range
+// [b*Ts/G, (b+1)*Ts/G), then claims units of `unit` tiles of the pool [Ts, To*Ti) (S8).
 struct StagedArgs {
   void* out;
   void* acc;           // [O] accumulators (fp64 / u32 / u64), zero on entry and on exit
-  unsigned* tickets;   // [To] contributor tickets of outer tiles cut by range boundaries, zero on entry/exit
+  unsigned* pool;      // [2]: pool claim counter, blocks-done ticket (zero on entry and on exit)
+  unsigned* tickets;   // [To] tiles contributed per outer tile (partial contributors), zero on entry/exit
   int64_t O;           // outputs: R (sumRows) or C (sumCols)
   int64_t R, C;
   int64_t To, Ti;      // tiles along the outer / inner level
-  int64_t per_block;   // P: block b streams tiles [b*P, (b+1)*P) of the outer-major order
+  int64_t static_tiles; // Ts
+  int64_t unit;         // U: pool claim unit (tiles)
+  int early_reads;      // NPP_EXEC_OVERLAP: stream the inputs before the previous kernel completes
   unsigned long long* dbg_times;  // measurement knob (NPP_DEBUG_TIMES): [grid x 4] globaltimer stamps
 };
 

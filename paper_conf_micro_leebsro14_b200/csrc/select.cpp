@@ -16,6 +16,7 @@
 
 #include <algorithm>
 #include <climits>
+#include <cstdlib>
 #include <cstdio>
 
 namespace npp {
@@ -210,16 +211,15 @@ bool staged_eligible(const Nest& n, int dtype, const Choice& c) {
   return n.cols % (16 / dtype_size(dtype)) == 0 && c.dims[contig_level] == NPP_DIM_X;
 }
 
-// S8 staged family: persistent blocks (one per SM) claim 32-row x 1 KB tiles in outer-major order
-// from a global counter, claim_tiles at a time; the inner level is Split(Ti).
+// S8 staged family: persistent blocks (one per SM) stream 32-row x 1 KB tiles in outer-major order
+// (static range + pool); the inner level is Split(Ti).
 void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const bool rows = n.pattern == NPP_SUM_ROWS;
   const int64_t R = rows ? n.N[0] : n.N[1];
   const StagedTiling t = staged_tiling(n.pattern, R, n.cols, dtype);
-  const int64_t tiles = t.To * t.Ti;
-  const int64_t per_block = cdiv(tiles, std::min<int64_t>(lim.sm_count, tiles));  // P
-  c->claim_tiles = per_block;
-  c->persistent_grid = cdiv(tiles, per_block);
+  const StagedBalance bal = staged_balance(t.To, t.Ti, lim.sm_count);
+  c->claim_tiles = bal.U;
+  c->persistent_grid = bal.G;
   c->staged = 1;
   if (rows) {
     c->blocks[0] = 8;
@@ -342,6 +342,29 @@ int kernel_class_of(const Nest& n, const Choice& c) {
 thread_local std::string g_error;
 
 void set_error(const std::string& msg) { g_error = msg; }
+
+// S8 balance rule (S8): G = min(SMs, T) persistent blocks over T tiles in order. The pool
+// unit is U = Ti when an outer tile has at most kWholeUnitMax tiles (a claim then covers whole outer
+// tiles), else kPoolUnit. Ts = U * floor((T - floor(T / kPoolDiv)) / U) tiles are split statically:
+// block b streams [b*Ts/G, (b+1)*Ts/G); the units of [Ts, T) are claimed in order from a counter by
+// whichever block is free, which absorbs the per-SM bandwidth differences of a static split.
+// (NPP_POOL_DIV / NPP_POOL_UNIT override the constants for measurements; tests never set them.)
+StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count) {
+  static const int64_t div = [] {
+    const char* e = getenv("NPP_POOL_DIV");
+    return e ? std::max<int64_t>(1, atoll(e)) : kPoolDiv;
+  }();
+  static const int64_t unit = [] {
+    const char* e = getenv("NPP_POOL_UNIT");
+    return e ? std::max<int64_t>(1, atoll(e)) : kPoolUnit;
+  }();
+  StagedBalance b;
+  const int64_t T = To * Ti;
+  b.G = std::min<int64_t>(sm_count, T);
+  b.U = Ti <= kWholeUnitMax ? Ti : unit;
+  b.Ts = b.U * ((T - T / div) / b.U);
+  return b;
+}
 
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   StagedTiling t;
@@ -537,9 +560,10 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
   } else if (is_sum_pattern(n.pattern) && c.staged) {
-    // counters (claim, barrier) + accumulators [O] of the accumulator type
+    // pool counters (256 B) + tickets [To] + accumulators [O] of the accumulator type
     const StagedTiling t = staged_tiling(n.pattern, n.pattern == NPP_SUM_ROWS ? n.N[0] : n.N[1], n.cols, dtype);
-    m.workspace_bytes = 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
+    m.workspace_bytes =
+        256 + 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
   } else if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
     const int64_t part = m.level[1].grid * eff(n.N[0]) * acc_bytes(n.pattern, dtype);
     const int64_t tick = m.level[0].grid * 4;

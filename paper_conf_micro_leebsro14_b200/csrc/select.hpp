@@ -40,6 +40,9 @@ struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refi
 };
 
 constexpr int kStageRows = 32;  // BR of the staged family (S8): tiles of 32 rows x 1 KB
+constexpr int64_t kPoolDiv = 8;       // S8 balance rule: about 1/kPoolDiv of the tiles form the shared pool
+constexpr int64_t kPoolUnit = 4;      // S8 balance rule: pool claim unit when outer tiles are long
+constexpr int64_t kWholeUnitMax = 8;  // S8 balance rule: outer tiles of <= 8 tiles are claimed whole
 
 // S8 staged-family tiling shared with the kernels: tile counts of the outer / inner level.
 struct StagedTiling {
@@ -47,6 +50,10 @@ struct StagedTiling {
   int64_t To, Ti;   // tiles along the outer / inner level
 };
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype);
+struct StagedBalance {
+  int64_t G, U, Ts;  // persistent blocks, pool claim unit, statically split tiles
+};
+StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count);
 
 // thread-local error message shared with the API layer
 void set_error(const std::string& msg);

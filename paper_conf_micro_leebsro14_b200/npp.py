@@ -54,9 +54,11 @@ class Limits(ctypes.Structure):
                 ("smem_per_block", ctypes.c_int64)]
 
 
+EXEC_OVERLAP = 1  # npp.h NPP_EXEC_OVERLAP
+
 EXPORTS = ("npp_version", "npp_last_error", "npp_limits_query", "npp_select", "npp_plan",
            "npp_plan_with_mapping", "npp_plan_mapping", "npp_plan_workspace_bytes", "npp_execute",
-           "npp_execute_host", "npp_plan_launches", "npp_plan_destroy")
+           "npp_execute_ex", "npp_execute_host", "npp_plan_launches", "npp_plan_destroy")
 
 
 def _load():
@@ -78,6 +80,7 @@ def _load():
     lib.npp_plan_workspace_bytes.argtypes = [P]
     lib.npp_plan_workspace_bytes.restype = ctypes.c_int64
     lib.npp_execute.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, P, P]
+    lib.npp_execute_ex.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, P, P, ctypes.c_uint]
     lib.npp_execute_host.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, ctypes.POINTER(P), P, P, P]
     lib.npp_plan_launches.argtypes = [P]
     lib.npp_plan_destroy.argtypes = [P]
@@ -220,14 +223,17 @@ class Plan:
     def new_out(self):
         return torch.empty(self.out_shape(), dtype=self.out_dtype(), device=self.device)
 
-    def execute(self, ins, out, stream=None, workspace=None):
-        """Enqueue on `stream` (default: torch's current stream). Inputs must be contiguous device tensors."""
+    def execute(self, ins, out, stream=None, workspace=None, overlap=False):
+        """Enqueue on `stream` (default: torch's current stream). Inputs must be contiguous device tensors.
+        overlap=True is npp_execute_ex(NPP_EXEC_OVERLAP): the caller asserts no earlier work on the
+        stream writes `ins` (the staged kernels then start while the previous kernel drains)."""
         for t in ins:
             if not t.is_contiguous():
                 raise ValueError("inputs must be contiguous")
         arr = (ctypes.c_void_p * len(ins))(*[t.data_ptr() for t in ins])
         ws = workspace if workspace is not None else self.workspace
-        _check(_lib.npp_execute(self._h, arr, len(ins), _ptr(out), _ptr(ws), _stream_handle(stream)))
+        _check(_lib.npp_execute_ex(self._h, arr, len(ins), _ptr(out), _ptr(ws), _stream_handle(stream),
+                                   EXEC_OVERLAP if overlap else 0))
         return out
 
     def execute_host(self, host_ins, host_out, dev_ins, dev_out, stream=None):

@@ -107,6 +107,31 @@ def test_paper_shapes_full(npp, cuda_device, shape):
             assert torch.all((out - out2).abs() <= out.abs() * 2.0 ** -23), "stale workspace"
 
 
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+def test_overlap_back_to_back(npp, cuda_device, dtype):
+    # npp_execute_ex(NPP_EXEC_OVERLAP): programmatic dependent launches back to back on one stream —
+    # the same plan (shared workspace: pool counter, tickets, accumulators) and different plans.
+    # Results equal the oracle's and every workspace ends zero (S8 balance rule).
+    shapes = [(65536, 1024), (1024, 65536), (4097, 300), (300, 4100), (33, 1 << 16)]
+    if dtype == "i64":
+        shapes = [(s[0], s[1] // 2) if s[1] % 2 == 0 else s for s in shapes]
+    plans = []
+    for i, s in enumerate(shapes):
+        m = _make(dtype, s, 40 + i, cuda_device)
+        for pat in ("SUM_ROWS", "SUM_COLS"):
+            plans.append((npp.Plan(pat, s, dtype, "AUTO"), m))
+    outs = []
+    for rep in range(3):
+        for p, m in plans:
+            outs.append((p, m, p.execute([m], p.new_out(), overlap=True)))
+    torch.cuda.synchronize()
+    for p, m, o in outs:
+        check(p.pattern, m, o, dtype)
+    for p, _ in plans:
+        assert p.mapping["staged"] == 1
+        assert int(p.workspace.count_nonzero()) == 0, p.shape
+
+
 def test_large_sumcols_sampled(npp, cuda_device):
     # [1M, 4K] fp32 (16 GiB, 2^32 elements: 64-bit indexing); sampled columns recomputed by the oracle
     R, C = 1 << 20, 4096
