@@ -297,13 +297,18 @@ def staged_eligible(nest, dtype, dims) -> bool:
 
 
 def staged_tiles(nest, dtype):
-    """DESIGN.md S8 staged: tile shape (BR rows x BC cols = 32 KB) and tiles along outer / inner."""
+    """DESIGN.md S8 staged: tile = BR rows x W columns (32 KB) of 1 KB chunks (BC elements each).
+    Narrow tiles: 32 rows x 1 KB. Wide tiles (SUM_ROWS, row pitch a multiple of 4 KB): 8 rows x 4 KB. Outer tiles:
+    BR-row bands (SUM_ROWS) or W-column strips (SUM_COLS). Returns (BR, BC, W, To, Ti)."""
     esz = DTYPE_SIZE[dtype]
-    BR, BC = STAGE_ROWS, 1024 // esz
+    BC = 1024 // esz
     O, I = nest["levels"][0][0], nest["levels"][1][0]
+    C = I if nest["pattern"] == "SUM_ROWS" else O
+    wide = nest["pattern"] == "SUM_ROWS" and (C * esz) % 4096 == 0
+    BR, W = (8, 4 * BC) if wide else (STAGE_ROWS, BC)
     if nest["pattern"] == "SUM_ROWS":
-        return BR, BC, cdiv(O, BR), cdiv(I, BC)
-    return BR, BC, cdiv(O, BC), cdiv(I, BR)
+        return BR, BC, W, cdiv(O, BR), cdiv(I, W)
+    return BR, BC, W, cdiv(O, W), cdiv(I, BR)
 
 
 POOL_DIV = 8                                      # DESIGN.md S8 balance rule
@@ -323,23 +328,24 @@ def balance(To, Ti, lim):
 
 
 def r2_staged(nest, dtype, lim):
-    """DESIGN.md S8, staged family: persistent blocks (one per SM) stream 32-row x 1 KB tiles in
-    outer-major order (static range + pool, balance()); the inner level is Split(Ti)."""
+    """DESIGN.md S8, staged family: persistent blocks (one per SM) stream BR x W tiles in outer-major
+    order (static range + pool, balance()); the inner level is Split(Ti)."""
     esz = DTYPE_SIZE[dtype]
-    BR, BC, To, Ti = staged_tiles(nest, dtype)
+    BR, BC, W, To, Ti = staged_tiles(nest, dtype)
+    wide = W > BC
     I = nest["levels"][1][0]
     G, CL, _ = balance(To, Ti, lim)
-    if nest["pattern"] == "SUM_ROWS":
+    if nest["pattern"] == "SUM_ROWS":     # 8 warps; narrow: 4 rows per warp, wide: 1 row per warp
         blocks = (8, 32)
-        spans = (SPAN_N, ALL if Ti == 1 else SPLIT)
-        factors = (4, Ti)
-        chunks = (BR, BC if Ti > 1 else I)
+        spans = (ONE if wide else SPAN_N, ALL if Ti == 1 else SPLIT)
+        factors = (1 if wide else 4, Ti)
+        chunks = (BR, W if Ti > 1 else I)
         vec = 16 // esz
-    else:
+    else:                                 # one thread per column of each 1 KB chunk (W/BC chunks)
         blocks = (BC, 256 // BC)
-        spans = (ONE, ALL if Ti == 1 else SPLIT)
-        factors = (1, Ti)
-        chunks = (BC, BR if Ti > 1 else I)
+        spans = (SPAN_N if wide else ONE, ALL if Ti == 1 else SPLIT)
+        factors = (W // BC, Ti)
+        chunks = (W, BR if Ti > 1 else I)
         vec = 1
     return blocks, spans, factors, vec, chunks, G, CL
 
@@ -454,7 +460,7 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
     if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
         if staged:  # pool counters (256 B) + tickets [To] + accumulators [O] (S8 staged)
             O = _eff(nest["levels"][0][0])
-            To = staged_tiles(nest, dtype)[2]   # tickets [To] u32, then accumulators [O]
+            To = staged_tiles(nest, dtype)[3]   # tickets [To] u32, then accumulators [O]
             rec["workspace_bytes"] = (256 + 256 * cdiv(4 * To, 256)
                                       + 256 * cdiv(O * acc_bytes(nest["pattern"], dtype), 256))
         elif levels[1]["grid"] >= 2:

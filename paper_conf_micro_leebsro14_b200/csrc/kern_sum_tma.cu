@@ -86,6 +86,13 @@ __device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
       : "memory");
   return ok != 0;
 }
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int x, int y, int z, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
+      : "memory");
+}
 __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -130,13 +137,16 @@ __device__ __forceinline__ A warp_sum(A v) {
 
 }  // namespace
 
-template <typename T, bool ROWS>
+template <typename T, bool ROWS, bool WIDE>
 __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_constant__ CUtensorMap map,
                                                                   StagedArgs a) {
   using Acc = typename SOps<T>::Acc;
   using V = typename V16<T>::type;
-  constexpr int BC = 1024 / int(sizeof(T));            // tile columns
-  constexpr int OUT_PER_TILE = ROWS ? kTileRows : BC;  // outputs of one outer tile
+  constexpr int BC = 1024 / int(sizeof(T));     // columns of one 1 KB chunk
+  constexpr int NCH = WIDE ? 4 : 1;             // chunks per tile row: tile = RT rows x NCH KB
+  constexpr int RT = kTileRows / NCH;           // tile rows (narrow 32, wide 8)
+  constexpr int W = NCH * BC;                   // tile columns
+  constexpr int OUT_PER_TILE = ROWS ? RT : W;   // outputs of one outer tile (band / strip)
   extern __shared__ __align__(1024) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + kStages;
@@ -218,9 +228,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         slot_tile[slot] = cur | (flush ? kFlush : 0);
         mbar_expect_tx(full + slot, kTileBytes);
         const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
-        const int x = int(ROWS ? it * BC : ot * BC);
-        const int y = int(ROWS ? ot * kTileRows : it * kTileRows);
-        tma_load_2d(tiles + slot * kTileBytes, &map, x, y, full + slot);
+        const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
+        const int y = int(ROWS ? ot * RT : it * RT);     // first row
+        if constexpr (WIDE)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
+          tma_load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
+        else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
+          tma_load_2d(tiles + slot * kTileBytes, &map, ch * BC, y, full + slot);
         cur = nxt;
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
@@ -261,19 +274,21 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         lasts &= lasts - 1;
         const long long o0 = __shfl_sync(0xffffffffu, ot, j) * OUT_PER_TILE;
         const long long oend = ROWS ? a.R : a.C;
-        constexpr int J = OUT_PER_TILE / 32;
-        Acc v[J];
+        constexpr int J = OUT_PER_TILE >= 256 ? 8 : (OUT_PER_TILE + 31) / 32;  // loads in flight per lane
+        for (int base = 0; base < OUT_PER_TILE; base += 32 * J) {
+          Acc v[J];
 #pragma unroll
-        for (int q = 0; q < J; ++q) {
-          const long long o = o0 + lane + 32 * q;
-          v[q] = o < oend ? __ldcg(accg + o) : Acc(0);
-        }
+          for (int q = 0; q < J; ++q) {
+            const long long o = o0 + base + lane + 32 * q;
+            v[q] = (base + lane + 32 * q < OUT_PER_TILE && o < oend) ? __ldcg(accg + o) : Acc(0);
+          }
 #pragma unroll
-        for (int q = 0; q < J; ++q) {
-          const long long o = o0 + lane + 32 * q;
-          if (o < oend) {
-            __stcg(accg + o, Acc(0));
-            static_cast<T*>(a.out)[o] = SOps<T>::finish(v[q]);
+          for (int q = 0; q < J; ++q) {
+            const long long o = o0 + base + lane + 32 * q;
+            if (base + lane + 32 * q < OUT_PER_TILE && o < oend) {
+              __stcg(accg + o, Acc(0));
+              static_cast<T*>(a.out)[o] = SOps<T>::finish(v[q]);
+            }
           }
         }
       }
@@ -285,11 +300,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     if (a.dbg_times && lane == 0) a.dbg_times[bid * 4 + 2] = gtimer();
   } else {
     // ------------------------------------------------------------ consumers
-    constexpr int kGroups = ROWS ? 1 : 256 / BC;   // MX row groups (1 for 4-byte types, 2 for 8-byte)
-    constexpr int kRowsPer = kTileRows / kGroups;  // MX rows of a tile one thread adds
+    constexpr int kGroups = ROWS ? 1 : 256 / BC;  // MX row groups (1 for 4-byte types, 2 for 8-byte)
+    constexpr int kRowsPer = RT / kGroups;        // MX rows of a tile one thread adds
     const int col = threadIdx.x % BC;
     const int rg = threadIdx.x / BC;
-    Acc acc[4] = {0, 0, 0, 0};  // RX: rows 4w..4w+3; MX: acc[0] = column col
+    // RX narrow: rows 4w..4w+3; RX wide: acc[0] = row w; MX: acc[k] = column col of chunk k
+    Acc acc[4] = {0, 0, 0, 0};
     unsigned n_acc = 0;         // tiles of the current outer tile accumulated since the last flush
     long long nfl = 0;          // flushes handed to the combiner
     bool waited = false;
@@ -299,7 +315,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       const long long tag = slot_tile[slot];
       if (tag < 0) break;
       const unsigned char* tile = tiles + slot * kTileBytes;
-      if constexpr (ROWS) {
+      if constexpr (ROWS && !WIDE) {
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr) {
           const unsigned char* row = tile + (warp * 4 + rr) * 1024;
@@ -307,20 +323,33 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
           const V v1 = *reinterpret_cast<const V*>(row + 512 + lane * 16);
           acc[rr] += Acc(vsum(v0) + vsum(v1));
         }
+      } else if constexpr (ROWS) {  // wide: warp w adds the 4 KB of row w, 8 x 16 B per lane
+        const unsigned char* row = tile + warp * 4096;
+        decltype(vsum(V{})) p[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) p[k] = vsum(*reinterpret_cast<const V*>(row + k * 512 + lane * 16));
+#pragma unroll
+        for (int w = 4; w >= 1; w /= 2)
+#pragma unroll
+          for (int i = 0; i < w; ++i) p[i] = p[i] + p[i + w];
+        acc[0] += Acc(p[0]);
       } else {
         const T* tt = reinterpret_cast<const T*>(tile);
-        T v[kRowsPer];
 #pragma unroll
-        for (int rr = 0; rr < kRowsPer; ++rr) v[rr] = tt[(rg * kRowsPer + rr) * BC + col];
-        if constexpr (std::is_same<T, float>::value) {  // fp32: pairwise tree inside the tile
+        for (int k = 0; k < NCH; ++k) {
+          T v[kRowsPer];
 #pragma unroll
-          for (int w = kRowsPer / 2; w >= 1; w /= 2)
+          for (int rr = 0; rr < kRowsPer; ++rr) v[rr] = tt[(rg * kRowsPer + rr) * W + k * BC + col];
+          if constexpr (std::is_same<T, float>::value) {  // fp32: pairwise tree inside the tile
 #pragma unroll
-            for (int i = 0; i < w; ++i) v[i] = v[i] + v[i + w];
-          acc[0] += Acc(v[0]);
-        } else {
+            for (int w = kRowsPer / 2; w >= 1; w /= 2)
 #pragma unroll
-          for (int rr = 0; rr < kRowsPer; ++rr) acc[0] += Acc(v[rr]);
+              for (int i = 0; i < w; ++i) v[i] = v[i] + v[i + w];
+            acc[k] += Acc(v[0]);
+          } else {
+#pragma unroll
+            for (int rr = 0; rr < kRowsPer; ++rr) acc[k] += Acc(v[rr]);
+          }
         }
       }
       ++n_acc;
@@ -338,21 +367,29 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       long long oidx[4];
       Acc val[4];
       bool mine[4];
-      if constexpr (ROWS) {
+      if constexpr (ROWS && !WIDE) {
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr) {
           val[rr] = warp_sum(acc[rr]);
-          oidx[rr] = ot * kTileRows + warp * 4 + rr;
+          oidx[rr] = ot * RT + warp * 4 + rr;
           mine[rr] = lane == rr && oidx[rr] < a.R;
           acc[rr] = 0;
         }
-      } else {
-        val[0] = acc[0];
-        oidx[0] = ot * BC + col;
-        mine[0] = oidx[0] < a.C;
+      } else if constexpr (ROWS) {
+        val[0] = warp_sum(acc[0]);
+        oidx[0] = ot * RT + warp;
+        mine[0] = lane == 0 && oidx[0] < a.R;
         acc[0] = 0;
+      } else {
+#pragma unroll
+        for (int k = 0; k < NCH; ++k) {
+          val[k] = acc[k];
+          oidx[k] = ot * W + k * BC + col;
+          mine[k] = oidx[k] < a.C;
+          acc[k] = 0;
+        }
       }
-      constexpr int NV = ROWS ? 4 : 1;
+      constexpr int NV = ROWS ? (WIDE ? 1 : 4) : NCH;
       const unsigned contributed = n_acc;
       n_acc = 0;
       if (whole && kGroups == 1) {
@@ -407,10 +444,10 @@ EncodeTiledFn encode_fn() {
   return fn;
 }
 
-template <typename T, bool ROWS>
+template <typename T, bool ROWS, bool WIDE>
 cudaError_t launch_typed(const CUtensorMap& map, const StagedArgs& a, int grid, cudaStream_t st) {
   static bool attr_set = false;
-  auto kern = npp_sum_tma_kernel<T, ROWS>;
+  auto kern = npp_sum_tma_kernel<T, ROWS, WIDE>;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
     if (e != cudaSuccess) return e;
@@ -419,31 +456,46 @@ cudaError_t launch_typed(const CUtensorMap& map, const StagedArgs& a, int grid, 
   return launch_pdl(kern, grid, kThreads, kSmemBytes, st, true, map, a);
 }
 
+template <typename T>
+cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const StagedArgs& a, int grid, cudaStream_t st) {
+  // wide tiles are selected for sumRows only (S8); the MX-wide path of the kernel template (4 KB
+  // column strips) measured slower than 1 KB strips because of the larger combine per cut strip
+  if (rows) return a.wide ? launch_typed<T, true, true>(map, a, grid, st) : launch_typed<T, true, false>(map, a, grid, st);
+  return launch_typed<T, false, false>(map, a, grid, st);
+}
+
 }  // namespace
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st) {
   EncodeTiledFn encode = encode_fn();
   if (!encode) return cudaErrorNotSupported;
   const int esz = dtype == NPP_I64 ? 8 : 4;
+  const cuuint64_t bc = cuuint64_t(1024 / esz);
   CUtensorMap map;
-  const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
-  const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
-  const cuuint32_t box[2] = {cuuint32_t(1024 / esz), cuuint32_t(kTileRows)};
-  const cuuint32_t estr[2] = {1, 1};
   const CUtensorMapDataType dt = dtype == NPP_F32   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                  : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
                                                     : CU_TENSOR_MAP_DATA_TYPE_INT64;
-  CUresult r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                      CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUresult r;
+  if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (row pitch is a multiple of 4 KB)
+    const cuuint64_t dims[3] = {bc, cuuint64_t(a.C) / bc, cuuint64_t(a.R)};
+    const cuuint64_t strides[2] = {1024, cuuint64_t(a.C) * esz};
+    const cuuint32_t box[3] = {cuuint32_t(bc), 4, cuuint32_t(kTileRows / 4)};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    r = encode(&map, dt, 3, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  } else {  // {C, R}; box 32 rows x 1 KB
+    const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
+    const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
+    const cuuint32_t box[2] = {cuuint32_t(bc), cuuint32_t(kTileRows)};
+    const cuuint32_t estr[2] = {1, 1};
+    r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  }
   if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
   switch (dtype) {
-    case NPP_F32:
-      return rows ? launch_typed<float, true>(map, a, grid, st) : launch_typed<float, false>(map, a, grid, st);
-    case NPP_I32:
-      return rows ? launch_typed<int32_t, true>(map, a, grid, st) : launch_typed<int32_t, false>(map, a, grid, st);
-    default:
-      return rows ? launch_typed<int64_t, true>(map, a, grid, st) : launch_typed<int64_t, false>(map, a, grid, st);
+    case NPP_F32: return launch_dtype<float>(rows, map, a, grid, st);
+    case NPP_I32: return launch_dtype<int32_t>(rows, map, a, grid, st);
+    default: return launch_dtype<int64_t>(rows, map, a, grid, st);
   }
 }
 

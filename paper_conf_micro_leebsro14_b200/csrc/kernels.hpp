@@ -48,7 +48,7 @@ cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumA
 int sum_kernels_max_regs();
 
 // Arguments of one staged (TMA) sum launch (S8 staged): the matrix is [R x C]; tiles are
-// 32 rows x 1 KB, To x Ti of them in outer-major order. Block b of G streams the static range
+// 32 rows x 1 KB (or 8 rows x 4 KB, `wide`), To x Ti of them in outer-major order. Block b of G streams the static range
 // [b*Ts/G, (b+1)*Ts/G), then claims units of `unit` tiles of the pool [Ts, To*Ti) (S8).
 struct StagedArgs {
   void* out;
@@ -61,6 +61,7 @@ struct StagedArgs {
   int64_t static_tiles; // Ts
   int64_t unit;         // U: pool claim unit (tiles)
   int early_reads;      // NPP_EXEC_OVERLAP: stream the inputs before the previous kernel completes
+  int wide;             // tiles of 8 rows x 4 KB (row pitch a multiple of 4 KB), else 32 rows x 1 KB
   unsigned long long* dbg_times;  // measurement knob (NPP_DEBUG_TIMES): [grid x 4] globaltimer stamps
 };
 

@@ -211,7 +211,7 @@ bool staged_eligible(const Nest& n, int dtype, const Choice& c) {
   return n.cols % (16 / dtype_size(dtype)) == 0 && c.dims[contig_level] == NPP_DIM_X;
 }
 
-// S8 staged family: persistent blocks (one per SM) stream 32-row x 1 KB tiles in outer-major order
+// S8 staged family: persistent blocks (one per SM) stream BR x W tiles in outer-major order
 // (static range + pool); the inner level is Split(Ti).
 void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const bool rows = n.pattern == NPP_SUM_ROWS;
@@ -221,20 +221,20 @@ void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   c->claim_tiles = bal.U;
   c->persistent_grid = bal.G;
   c->staged = 1;
-  if (rows) {
+  if (rows) {  // 8 warps; narrow: 4 rows per warp, wide: 1 row per warp
     c->blocks[0] = 8;
     c->blocks[1] = 32;
-    c->spans[0] = NPP_SPAN_N;
-    c->factors[0] = 4;
+    c->spans[0] = t.wide ? NPP_SPAN_ONE : NPP_SPAN_N;
+    c->factors[0] = t.wide ? 1 : 4;
     c->chunks[0] = t.BR;
-    c->chunks[1] = t.Ti > 1 ? t.BC : n.N[1];
+    c->chunks[1] = t.Ti > 1 ? t.W : n.N[1];
     c->vec = 16 / dtype_size(dtype);
-  } else {
+  } else {  // one thread per column of each 1 KB chunk (W / BC chunks per tile row)
     c->blocks[0] = int(t.BC);
     c->blocks[1] = int(256 / t.BC);
-    c->spans[0] = NPP_SPAN_ONE;
-    c->factors[0] = 1;
-    c->chunks[0] = t.BC;
+    c->spans[0] = t.wide ? NPP_SPAN_N : NPP_SPAN_ONE;
+    c->factors[0] = t.W / t.BC;
+    c->chunks[0] = t.W;
     c->chunks[1] = t.Ti > 1 ? t.BR : n.N[1];
     c->vec = 1;
   }
@@ -368,13 +368,16 @@ StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count) {
 
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   StagedTiling t;
-  t.BR = kStageRows;
-  t.BC = 1024 / dtype_size(dtype);
+  const int64_t esz = dtype_size(dtype);
+  t.BC = 1024 / esz;
+  t.wide = pattern == NPP_SUM_ROWS && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
+  t.BR = t.wide ? 8 : kStageRows;
+  t.W = t.wide ? 4 * t.BC : t.BC;
   if (pattern == NPP_SUM_ROWS) {
     t.To = cdiv(R, t.BR);
-    t.Ti = cdiv(C, t.BC);
+    t.Ti = cdiv(C, t.W);
   } else {
-    t.To = cdiv(C, t.BC);
+    t.To = cdiv(C, t.W);
     t.Ti = cdiv(R, t.BR);
   }
   return t;

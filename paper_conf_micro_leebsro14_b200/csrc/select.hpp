@@ -44,10 +44,13 @@ constexpr int64_t kPoolDiv = 8;       // S8 balance rule: about 1/kPoolDiv of th
 constexpr int64_t kPoolUnit = 4;      // S8 balance rule: pool claim unit when outer tiles are long
 constexpr int64_t kWholeUnitMax = 8;  // S8 balance rule: outer tiles of <= 8 tiles are claimed whole
 
-// S8 staged-family tiling shared with the kernels: tile counts of the outer / inner level.
+// S8 staged-family tiling shared with the kernels: a tile is BR rows x W columns (32 KB) made of
+// 1 KB chunks of BC elements. Narrow: 32 rows x 1 KB; wide (SUM_ROWS with a row pitch that is a
+// multiple of 4 KB): 8 rows x 4 KB.
 struct StagedTiling {
-  int64_t BR, BC;   // tile rows, tile columns
-  int64_t To, Ti;   // tiles along the outer / inner level
+  int64_t BR, BC, W;  // tile rows, chunk columns, tile columns
+  int64_t To, Ti;     // tiles along the outer / inner level
+  bool wide;
 };
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype);
 struct StagedBalance {

@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 
 STRATS = ["AUTO", "LITERAL", "1D", "TB_T", "WARP"]
 SHAPES = [(1, 1), (3, 5), (31, 33), (33, 31), (1000, 999), (1024, 1024), (4097, 300), (300, 4097),
-          (7, 70000), (70000, 7), (2, 1 << 17)]
+          (7, 70000), (70000, 7), (2, 1 << 17), (1001, 1024), (9, 3072)]
 
 
 @pytest.fixture(scope="module")

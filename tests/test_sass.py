@@ -53,7 +53,7 @@ def test_all_kernels_built_for_sm100a():
 def test_staged_kernels_use_tma(sass):
     for parts in (("npp_sum_tma_kernel",), ("npp_logreg_tma_kernel",), ("npp_kmeans_tma_kernel",)):
         for n in _find(sass, *parts):
-            assert sass[n]["UTMALDG.2D"] + sass[n]["UBLKCP.S.G"] + sass[n]["UTMALDG.1D"] > 0, n
+            assert sum(sass[n][f"UTMALDG.{d}D"] for d in (1, 2, 3)) + sass[n]["UBLKCP.S.G"] > 0, n
 
 
 def test_kmeans_centroids_on_uniform_datapath(sass):
