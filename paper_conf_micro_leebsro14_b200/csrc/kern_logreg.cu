@@ -51,8 +51,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
   unsigned char* y_ring = smem + kSmemHeader + kStages * kTileBytes + kRedBytes;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + kStages;
-  long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);
-  unsigned* s_last = reinterpret_cast<unsigned*>(slot_tile + kStages);
+  long long* slot_tile = reinterpret_cast<long long*>(empty + kStages);  // batch b | kFlush
+  int* slot_rows = reinterpret_cast<int*>(slot_tile + kStages);            // rows of the tile in batch b
+  int* slot_yoff = slot_rows + kStages;                                     // y offset in its y slot
+  unsigned* s_last = reinterpret_cast<unsigned*>(slot_yoff + kStages);
   unsigned char* tiles = smem + kSmemHeader;
   double* red = reinterpret_cast<double*>(smem + kSmemHeader + kStages * kTileBytes);  // [8][C]
   constexpr long long kFlush = 1ll << 62;
@@ -77,17 +79,21 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
   if (warp == kConsumerWarps) {
     if (lane == 0) {  // ---------------------------------------------- producer
       tma::prefetch_map(&map);
-      long long t = 0;
-      for (long long cur = r0; cur < r1; ++cur, ++t) {
-        const bool flush = cur + 1 >= r1 || ((cur + 1) / Ti) != (cur / Ti);
-        const int slot = int(t % kStages);
-        if (t >= kStages) tma::mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-        slot_tile[slot] = cur | (flush ? kFlush : 0);
-        tma::mbar_expect_tx(full + slot, tile_bytes + kYBox * 4);
-        const long long b = cur / Ti, j = cur - b * Ti;
+      long long b = r0 / Ti, j = r0 - (r0 / Ti) * Ti;  // batch and row tile, advanced incrementally
+      int slot = 0;
+      unsigned ph = 0;
+      for (long long cur = r0, t = 0; cur < r1; ++cur, ++t) {
+        const bool flush = cur + 1 >= r1 || j + 1 == Ti;
+        if (t >= kStages) tma::mbar_wait(empty + slot, ph ^ 1u);
         const long long row0 = b * Rb + j * kTileRows;
+        slot_tile[slot] = b | (flush ? kFlush : 0);
+        slot_rows[slot] = int((Rb - j * kTileRows) < kTileRows ? (Rb - j * kTileRows) : kTileRows);
+        slot_yoff[slot] = int(row0 & 3);
+        tma::mbar_expect_tx(full + slot, tile_bytes + kYBox * 4);
         tma::load_2d(tiles + slot * kTileBytes, &map, 0, int(row0), full + slot);
         tma::load_1d(y_ring + slot * kYSlot, &ymap, int(row0 & ~3ll), full + slot);
+        if (++j == Ti) j = 0, ++b;
+        if (++slot == kStages) slot = 0, ph ^= 1u;
       }
     }
     return;  // the producer warp takes no part in the consumer barriers below
@@ -95,7 +101,8 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
 
   // ------------------------------------------------------------------ consumers
   const int c0 = lane * 4, c1 = 128 + lane * 4;  // this lane's two column quads
-  const bool has0 = c0 < C, has1 = c1 < C;
+  const int Ci = int(C);
+  const bool has0 = c0 < Ci, has1 = c1 < Ci;
   float w0[4] = {0, 0, 0, 0}, w1[4] = {0, 0, 0, 0};
 #pragma unroll
   for (int e = 0; e < 4; ++e) {
@@ -104,15 +111,16 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
   }
   double acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   const long long n_tiles = r1 - r0;
+  int slot = 0;
+  unsigned ph = 0;
   for (long long t = 0; t < n_tiles; ++t) {
-    const int slot = int(t % kStages);
-    const long long cur = r0 + t;  // static range: the consumers know the tile without the producer
-    const bool flush = cur + 1 >= r1 || ((cur + 1) / Ti) != (cur / Ti);
-    const long long b = cur / Ti, j = cur - b * Ti;
-    const long long rows_here = (Rb - j * kTileRows) < kTileRows ? (Rb - j * kTileRows) : kTileRows;
     // y of the tile's rows: lane l holds y[row0 + l] (masked), broadcast by shuffles below
-    tma::mbar_wait(full + slot, unsigned((t / kStages) & 1));
-    const int yoff = int((b * Rb + j * kTileRows) & 3);
+    tma::mbar_wait(full + slot, ph);
+    const long long tag = slot_tile[slot];
+    const bool flush = (tag & kFlush) != 0;
+    const long long b = tag & ~kFlush;
+    const int rows_here = slot_rows[slot];
+    const int yoff = slot_yoff[slot];
     const float y_lane = lane < rows_here ? reinterpret_cast<const float*>(y_ring + slot * kYSlot)[yoff + lane] : 0.f;
     const float* tile = reinterpret_cast<const float*>(tiles + slot * kTileBytes);
     // dot products of the warp's 4 rows: per-lane partials over the lane's 8 columns ...
@@ -121,8 +129,8 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {
       const int r = warp * 4 + rr;
-      x0[rr] = has0 ? *reinterpret_cast<const float4*>(tile + r * C + c0) : make_float4(0, 0, 0, 0);
-      x1[rr] = has1 ? *reinterpret_cast<const float4*>(tile + r * C + c1) : make_float4(0, 0, 0, 0);
+      x0[rr] = has0 ? *reinterpret_cast<const float4*>(tile + r * Ci + c0) : make_float4(0, 0, 0, 0);
+      x1[rr] = has1 ? *reinterpret_cast<const float4*>(tile + r * Ci + c1) : make_float4(0, 0, 0, 0);
       float d = x0[rr].x * w0[0];
       d = fmaf(x0[rr].y, w0[1], d);
       d = fmaf(x0[rr].z, w0[2], d);
@@ -162,6 +170,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
     }
     __syncwarp();
     if (lane == 0) tma::mbar_arrive(empty + slot);
+    if (++slot == kStages) slot = 0, ph ^= 1u;
 #pragma unroll
     for (int e = 0; e < 8; ++e) acc[e] += double(p[e]);
     if (!flush) continue;
