@@ -367,7 +367,8 @@ def r2_logreg(nest, lim, dims):
 
 
 def r2_kmeans(nest, lim):
-    """DESIGN.md S8, KMEANS_ASSIGN staged: 128-point tiles, 2 points per thread, 4 centroid quarters."""
+    """DESIGN.md S8, KMEANS_ASSIGN staged: TP-point tiles, TP/64 points per thread, 4 centroid groups,
+    two warp sets taking alternate tiles."""
     (N, _), (K, _), (D, _) = nest["levels"]
     if D % 4 != 0 or D < 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384:
         raise Unsupported("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128, K <= 256, Kpad*D <= 16384")
@@ -375,10 +376,10 @@ def r2_kmeans(nest, lim):
     T = cdiv(N, TP)
     P = cdiv(T, min(lim["sm_count"], T))
     G = cdiv(T, P)
-    blocks = (64, 4, 1)
+    blocks = (128, 4, 1)                         # two sets of 64 x 4 threads take alternate tiles
     spans = (SPAN_N, ALL, ALL)
     factors = (TP // 64, 1, 1)
-    chunks = (TP, K, D)
+    chunks = (2 * TP, K, D)
     return blocks, spans, factors, 4, chunks, G, P
 
 

@@ -32,7 +32,7 @@ constexpr int kBoxCols = 32;  // 128 B of floats: the 128-B swizzle span
 // ping-pong: kSets sets of 8 warps take alternate tiles, so one set's per-tile epilogue (argmin,
 // group combine, set barrier) overlaps the other set's FMA stream
 #ifndef NPP_KM_SETS
-#define NPP_KM_SETS 1
+#define NPP_KM_SETS 2
 #endif
 constexpr int kSets = NPP_KM_SETS;
 constexpr int kConsumerWarps = 8;                 // per set
@@ -132,8 +132,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   __syncthreads();
 
   const long long n_tiles = r1 - r0;
-  auto issue = [&](long long t) {  // tile t of the block's range into slot t % kStages
-    const int slot = int(t % kStages);
+  auto issue = [&](long long t, int slot) {  // tile t of the block's range into slot t % kStages
     tma::mbar_expect_tx(full + slot, unsigned(stage_bytes));
     for (int bx = 0; bx < nb; ++bx)
       tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
@@ -141,7 +140,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   };
   if (threadIdx.x == 0) {
     tma::prefetch_map(&map);
-    for (long long t = 0; t < kStages && t < n_tiles; ++t) issue(t);
+    for (int t = 0; t < kStages && t < n_tiles; ++t) issue(t, t);
   }
 
   // ------------------------------------------------------------------ consumers
@@ -154,9 +153,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // of 8, so every point of the thread has the key lt & 7
   const unsigned key = unsigned(lt & 7);
   const int nd4 = D / 4;
+  // slot = t % kStages and round = t / kStages advance incrementally (no 64-bit division per tile)
+  int slot = set % kStages;
+  unsigned round = unsigned(set / kStages);
   for (long long t = set; t < n_tiles; t += kSets) {
-    const int slot = int(t % kStages);
-    tma::mbar_wait_warp(full + slot, unsigned((t / kStages) & 1));
+    tma::mbar_wait_warp(full + slot, round & 1u);
     const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
     float bs[PPT];
     int bk[PPT];
@@ -211,8 +212,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         if (gi < a.N) a.assign[gi] = bk[i];
       }
     } else {  // groups 1.. hand their minima to group 0 (double-buffered by tile parity)
-      float* ss = xs_s + (set * 2 + int((t / kSets) & 1)) * 3 * TP;
-      int* sk = xs_k + (set * 2 + int((t / kSets) & 1)) * 3 * TP;
+      const int par = int(((t - set) / kSets) & 1);  // kSets is a compile-time constant
+      float* ss = xs_s + (set * 2 + par) * 3 * TP;
+      int* sk = xs_k + (set * 2 + par) * 3 * TP;
       if (g > 0) {
 #pragma unroll
         for (int i = 0; i < PPT; ++i) ss[(g - 1) * TP + lt + LP * i] = bs[i], sk[(g - 1) * TP + lt + LP * i] = bk[i];
@@ -244,9 +246,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         __threadfence_block();
         released[slot] = 0;
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        if (t + kStages < n_tiles) issue(t + kStages);
+        if (t + kStages < n_tiles) issue(t + kStages, slot);
       }
     }
+    for (slot += kSets; slot >= kStages; slot -= kStages) ++round;
   }
 }
 

@@ -259,7 +259,7 @@ bool r2_logreg(const Nest& n, const npp_limits& lim, Choice* c) {
   return true;
 }
 
-// S8 KMEANS_ASSIGN staged: 128-point tiles, 2 points per thread, 4 centroid quarters (class KM).
+// S8 KMEANS_ASSIGN staged: TP-point tiles, TP/64 points per thread, 4 centroid groups, 2 warp sets (class KM).
 bool r2_kmeans(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], K = n.N[1], D = n.N[2];
   if (D % 4 != 0 || D < 4 || D > 128 || K > 256 || 32 * cdiv(K, 32) * D > 16384) return false;
@@ -270,8 +270,9 @@ bool r2_kmeans(const Nest& n, const npp_limits& lim, Choice* c) {
   c->persistent_grid = cdiv(T, per_block);
   c->staged = 1;
   c->vec = 4;
-  c->blocks[0] = 64, c->blocks[1] = 4, c->blocks[2] = 1;
-  c->spans[0] = NPP_SPAN_N, c->factors[0] = TP / 64, c->chunks[0] = TP;
+  // two sets of 64 x 4 threads take alternate tiles (ping-pong): y = 128, a block covers 2 tiles at once
+  c->blocks[0] = 128, c->blocks[1] = 4, c->blocks[2] = 1;
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = TP / 64, c->chunks[0] = 2 * TP;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = K;
   c->spans[2] = NPP_SPAN_ALL, c->factors[2] = 1, c->chunks[2] = D;
   return true;
