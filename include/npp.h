@@ -158,6 +158,16 @@ NPP_API int npp_limits_query(int device, npp_limits* out);
 NPP_API int npp_select(int pattern, const int64_t* shape, int ndim, int dtype, const npp_limits* limits,
                int strategy, npp_mapping* out);
 
+/* Algorithm 1's search space (S2, Alg 1): every candidate that passes the hard
+ * constraints (S3), in enumeration order (dims permutations lexicographic, then block sizes with
+ * level 0 most significant, then spans ONE < ALL), each with ControlDOP (S6) applied and recorded as
+ * strategy LITERAL records it (S9; score = its S4 soft score). Pure and CUDA-free like npp_select.
+ * Writes the first min(cap, count) records to `out` (caller-owned array; NULL allowed with cap 0)
+ * and returns count (>= 0), or a negative npp_status. Used for the score-vs-performance sweep of
+ * P:L1358-1415 (Fig 17); every record is executable through npp_plan_with_mapping (2-level sums). */
+NPP_API int64_t npp_enumerate(int pattern, const int64_t* shape, int ndim, int dtype, const npp_limits* limits,
+                              npp_mapping* out, int64_t cap);
+
 /* Build an immutable plan for (pattern, shape, dtype, strategy). limits == NULL queries the current
  * device. Sizes may be 0 (the plan then zero-fills the output). The plan is a host object owned by
  * the caller (npp_plan_destroy). Errors: as npp_select, plus NPP_ERR_CUDA from the limits query. */

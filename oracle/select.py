@@ -474,6 +474,23 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
 
 # ------------------------------------------------------------------ entry point
 
+def enumerate_mappings(pattern: str, shape, dtype: str, lim: dict) -> list:
+    """DESIGN.md S2/S3/S6/S9: every hard-feasible candidate of Algorithm 1's CandSet (L772-777), in
+    enumeration order, each with ControlDOP applied and recorded as LITERAL records it (its S4 score)."""
+    nest = build_nest(pattern, shape)
+    L = len(nest["levels"])
+    out = []
+    for dims in itertools.permutations(range(L)):
+        for blocks in itertools.product(SIZE_SET, repeat=L):
+            for spans in itertools.product((ONE, ALL), repeat=L):
+                if not hard_ok(nest, dtype, lim, dims, blocks, spans):
+                    continue
+                sc = score(nest, lim, dims, blocks)
+                sp, factors = control_dop(nest, lim, blocks, spans)
+                out.append(make_record(nest, dtype, lim, dims, blocks, sp, factors, 1, sc))
+    return out
+
+
 def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -> dict:
     """The mapping record for (pattern, shape, dtype, limits, strategy) per DESIGN.md §3."""
     nest = build_nest(pattern, shape)

@@ -103,13 +103,14 @@ bool key_greater(int64_t s1, int64_t d1, int64_t p1, int64_t s2, int64_t d2, int
 }
 
 // Alg 1 SEARCH with the S5 key. restrict_1d: b_l = 1 and Span(all) for l >= 1 (S7 1D).
-bool search(const Nest& n, int dtype, const npp_limits& lim, bool restrict_1d, Choice* best,
-            int64_t* best_score) {
+// S2: every candidate of Algorithm 1's CandSet (L772-777) in enumeration order — dims permutations
+// lexicographic, then block sizes (level 0 most significant), then spans (ONE < ALL) — that passes the
+// hard constraints (S3). `visit(c)` sees each one.
+template <typename Visit>
+void for_each_candidate(const Nest& n, int dtype, const npp_limits& lim, bool restrict_1d, Visit visit) {
   static const int perms2[2][2] = {{0, 1}, {1, 0}};
   static const int perms3[6][3] = {{0, 1, 2}, {0, 2, 1}, {1, 0, 2}, {1, 2, 0}, {2, 0, 1}, {2, 1, 0}};
   const int nperm = n.L == 1 ? 1 : (n.L == 2 ? 2 : 6);
-  int64_t bs = 0, bd = 0, bp = 0;
-  bool found = false;
   int total_sizes = 1, total_spans = 1;
   for (int l = 0; l < n.L; ++l) {
     total_sizes *= kSizeSetLen;
@@ -138,19 +139,28 @@ bool search(const Nest& n, int dtype, const npp_limits& lim, bool restrict_1d, C
         }
         for (int l = 0; l < n.L; ++l) c.factors[l] = 1;
         if (!hard_ok(n, dtype, lim, c)) continue;
-        const int64_t s = score(n, lim, c);
-        const int64_t d = mapping_dop(n, c);
-        const int64_t pb = prod_blocks(n, c);
-        if (!found || key_greater(s, d, pb, bs, bd, bp)) {  // strict: first (lex-smallest) wins ties
-          found = true;
-          bs = s;
-          bd = d;
-          bp = pb;
-          *best = c;
-        }
+        visit(c);
       }
     }
   }
+}
+
+bool search(const Nest& n, int dtype, const npp_limits& lim, bool restrict_1d, Choice* best,
+            int64_t* best_score) {
+  int64_t bs = 0, bd = 0, bp = 0;
+  bool found = false;
+  for_each_candidate(n, dtype, lim, restrict_1d, [&](const Choice& c) {
+    const int64_t s = score(n, lim, c);
+    const int64_t d = mapping_dop(n, c);
+    const int64_t pb = prod_blocks(n, c);
+    if (!found || key_greater(s, d, pb, bs, bd, bp)) {  // strict: first (lex-smallest) wins ties
+      found = true;
+      bs = s;
+      bd = d;
+      bp = pb;
+      *best = c;
+    }
+  });
   *best_score = bs;
   return found;
 }
@@ -664,4 +674,33 @@ extern "C" int npp_select(int pattern, const int64_t* shape, int ndim, int dtype
     return NPP_ERR_UNSUPPORTED;
   }
   return select_mapping(n, dtype, *limits, strategy, out);
+}
+
+extern "C" int64_t npp_enumerate(int pattern, const int64_t* shape, int ndim, int dtype, const npp_limits* limits,
+                                 npp_mapping* out, int64_t cap) {
+  using namespace npp;
+  if (cap < 0 || (cap > 0 && !out)) {
+    set_error("out is NULL or cap < 0");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (dtype < NPP_F32 || dtype > NPP_I64) {
+    set_error("unknown dtype");
+    return NPP_ERR_INVALID_ARG;
+  }
+  int st = check_limits(limits);
+  if (st) return st;
+  Nest n;
+  st = build_nest(pattern, shape, ndim, &n);
+  if (st) return st;
+  int64_t count = 0;
+  for_each_candidate(n, dtype, *limits, false, [&](const Choice& c0) {
+    if (count < cap) {
+      Choice c = c0;
+      const int64_t s = score(n, *limits, c);
+      control_dop(n, *limits, &c);
+      record_from_choice(n, dtype, *limits, c, s, out + count);
+    }
+    ++count;
+  });
+  return count;
 }

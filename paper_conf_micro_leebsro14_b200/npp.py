@@ -58,7 +58,7 @@ EXEC_OVERLAP = 1  # npp.h NPP_EXEC_OVERLAP
 
 EXPORTS = ("npp_version", "npp_last_error", "npp_limits_query", "npp_select", "npp_plan",
            "npp_plan_with_mapping", "npp_plan_mapping", "npp_plan_workspace_bytes", "npp_execute",
-           "npp_execute_ex", "npp_execute_host", "npp_plan_launches", "npp_plan_destroy")
+           "npp_execute_ex", "npp_execute_host", "npp_enumerate", "npp_plan_launches", "npp_plan_destroy")
 
 
 def _load():
@@ -83,6 +83,9 @@ def _load():
     lib.npp_execute_ex.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, P, P, ctypes.c_uint]
     lib.npp_execute_host.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, ctypes.POINTER(P), P, P, P]
     lib.npp_plan_launches.argtypes = [P]
+    lib.npp_enumerate.argtypes = [ctypes.c_int, I64P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(Limits),
+                                  ctypes.c_void_p, ctypes.c_int64]
+    lib.npp_enumerate.restype = ctypes.c_int64
     lib.npp_plan_destroy.argtypes = [P]
     lib.npp_plan_destroy.restype = None
     return lib
@@ -159,6 +162,22 @@ def select(pattern: str, shape, dtype: str, limits: dict, strategy: str = "AUTO"
     _check(_lib.npp_select(PATTERNS[pattern], _shape_arr(shape), len(shape), DTYPES[dtype], ctypes.byref(l),
                            STRATEGIES[strategy], ctypes.byref(m)))
     return mapping_to_dict(m)
+
+
+def enumerate_mappings(pattern: str, shape, dtype: str, limits: dict) -> list:
+    """npp_enumerate: every hard-feasible Algorithm 1 candidate with ControlDOP applied, as LITERAL
+    records (S2-S6, S9), in enumeration order."""
+    l = limits_from_dict(limits)
+    n = _lib.npp_enumerate(PATTERNS[pattern], _shape_arr(shape), len(shape), DTYPES[dtype], ctypes.byref(l),
+                           None, 0)
+    if n < 0:
+        _check(int(n))
+    arr = (Mapping * max(1, n))()
+    got = _lib.npp_enumerate(PATTERNS[pattern], _shape_arr(shape), len(shape), DTYPES[dtype], ctypes.byref(l),
+                             arr, n)
+    if got < 0:
+        _check(int(got))
+    return [mapping_to_dict(arr[i]) for i in range(n)]
 
 
 def _ptr(t) -> ctypes.c_void_p:

@@ -80,3 +80,27 @@ def test_invalid_arguments():
     with pytest.raises(npp.NppError) as e:
         npp.select("KMEANS_ASSIGN", (4, 4, 4), "i32", S.B200, "LITERAL")
     assert e.value.status == npp.ERR_UNSUPPORTED
+
+
+@pytest.mark.parametrize("profile", ["b200", "k20c", "tiny"])
+def test_enumerate_parity(profile):
+    # npp_enumerate (Fig 17 sweep space) == oracle enumeration, record by record and in order
+    lim = PROFILES[profile]
+    for pattern in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_COLS"):
+        for shape in [(65536, 1024), (1024, 65536), (50, 20000), (3, 5)]:
+            for dtype in ("f32", "i64"):
+                want = S.enumerate_mappings(pattern, shape, dtype, lim)
+                got = npp.enumerate_mappings(pattern, shape, dtype, lim)
+                assert got == want, (pattern, shape, dtype)
+    for pattern, shape in [("KMEANS_ASSIGN", (1000, 8, 4)), ("LOGREG_GRAD", (4, 64, 8))]:
+        assert npp.enumerate_mappings(pattern, shape, "f32", lim) == S.enumerate_mappings(pattern, shape, "f32", lim)
+
+
+def test_enumerate_contains_the_selection():
+    # the LITERAL selection is the S5-best member of the enumerated space (same record)
+    for pattern, shape in [("SUM_ROWS", (8192, 8192)), ("SUM_COLS", (65536, 1024)), ("SUM_COLS", (1024, 65536))]:
+        space = npp.enumerate_mappings(pattern, shape, "f32", S.B200)
+        lit = npp.select(pattern, shape, "f32", S.B200, "LITERAL")
+        assert lit in space
+        assert lit["score"] == max(r["score"] for r in space)
+    assert npp.enumerate_mappings("SUM_ROWS", (3, 5), "f32", S.B200)  # never empty for feasible nests

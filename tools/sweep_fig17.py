@@ -1,0 +1,170 @@
+"""Score-vs-performance sweep over the mapping space (§VI-G, Fig 17) on B200.
+
+For sumRows and sumCols at the paper's three shapes, every hard-feasible Algorithm 1 candidate
+(npp_enumerate: S2-S6, ControlDOP applied, recorded as LITERAL) is executed through
+npp_plan_with_mapping on the direct-load kernel family and timed; AUTO (R2 + staged TMA family),
+LITERAL (the selector's pick), TB/T, warp-based and 1D are timed as markers.
+
+    python tools/sweep_fig17.py [--out gpurun_out/fig17.json] [--shapes 65536x1024,...]
+    python tools/sweep_fig17.py --summarize gpurun_out/fig17.json    # markdown summary (no GPU)
+
+Timing: CUDA events around a graph of launches alternating two distinct 256 MiB inputs (L2-cold),
+median of 3 replays; algorithmic bytes = R*C*4 + outputs*4.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+SHAPES = [(65536, 1024), (8192, 8192), (1024, 65536)]
+SPAN = {0: "1", 1: "all", 2: "n", 3: "split"}
+
+
+def brief(m):
+    out = []
+    for l in m["levels"]:
+        sp = SPAN[l["span"]]
+        if sp in ("n", "split"):
+            sp = f"{sp}({l['factor']})"
+        out.append(f"{'xyz'[l['dim']]}{l['block']}/{sp}")
+    return " ".join(out)
+
+
+def time_plan(torch, plan, ins_a, ins_b, out, stream, budget_ms=400.0):
+    """Median per-launch microseconds of a graph alternating two inputs."""
+    with torch.cuda.stream(stream):
+        plan.execute(ins_a, out, stream=stream)
+        plan.execute(ins_b, out, stream=stream)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    with torch.cuda.stream(stream):
+        plan.execute(ins_a, out, stream=stream)
+    torch.cuda.synchronize()
+    one_ms = (time.perf_counter() - t0) * 1e3
+    n = int(max(2, min(16, budget_ms / max(one_ms, 1e-3) / 3)))
+    n += n % 2
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(stream):
+        with torch.cuda.graph(g, stream=stream):
+            for r in range(n):
+                plan.execute(ins_a if r % 2 == 0 else ins_b, out, stream=stream)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for _ in range(3):
+        with torch.cuda.stream(stream):
+            a.record(stream)
+            g.replay()
+            b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b) * 1e3 / n)
+    return statistics.median(ts)
+
+
+def run(args):
+    import torch
+    from paper_conf_micro_leebsro14_b200 import npp
+    from synth import gen
+
+    dev = torch.device("cuda:0")
+    torch.cuda.set_device(dev)
+    lim = npp.limits_query(0)
+    stream = torch.cuda.Stream(device=dev)
+    shapes = SHAPES if not args.shapes else [tuple(int(v) for v in s.split("x")) for s in args.shapes.split(",")]
+    result = {"device": torch.cuda.get_device_name(0), "limits": lim, "rows": []}
+    for (R, C) in shapes:
+        ma = gen.uniform_f32(3, (R, C), device=dev)
+        mb = gen.uniform_f32(4, (R, C), device=dev)
+        for pattern in ("SUM_ROWS", "SUM_COLS"):
+            nbytes = R * C * 4 + (R if pattern == "SUM_ROWS" else C) * 4
+            cands = npp.enumerate_mappings(pattern, (R, C), "f32", lim)
+            entries = [("candidate", c) for c in cands]
+            for strat in ("AUTO", "LITERAL", "TB_T", "WARP", "1D"):
+                entries.append((strat, None))
+            t_shape = time.perf_counter()
+            for kind, rec in entries:
+                if rec is None:
+                    plan = npp.Plan(pattern, (R, C), "f32", kind, device=dev)
+                else:
+                    plan = npp.Plan(pattern, (R, C), "f32", mapping=rec, device=dev)
+                out = plan.new_out()
+                us = time_plan(torch, plan, [ma], [mb], out, stream)
+                m = plan.mapping
+                result["rows"].append({
+                    "pattern": pattern, "shape": [R, C], "kind": kind, "score": m["score"], "dop": m["dop"],
+                    "grid": m["grid"], "block": m["block"], "mapping": brief(m), "staged": m["staged"],
+                    "us": round(us, 2), "GB/s": round(nbytes / (us * 1e-6) / 1e9, 1)})
+                del plan, out
+            print(f"{pattern} {R}x{C}: {len(entries)} mappings in {time.perf_counter() - t_shape:.1f} s",
+                  flush=True)
+        del ma, mb
+        torch.cuda.empty_cache()
+    os.makedirs(os.path.dirname(os.path.abspath(args.out)), exist_ok=True)
+    with open(args.out, "w") as f:
+        json.dump(result, f)
+    print(summarize(result))
+
+
+def _spearman(xs, ys):
+    def ranks(v):
+        order = sorted(range(len(v)), key=lambda i: v[i])
+        r = [0.0] * len(v)
+        i = 0
+        while i < len(v):
+            j = i
+            while j + 1 < len(v) and v[order[j + 1]] == v[order[i]]:
+                j += 1
+            for k in range(i, j + 1):
+                r[order[k]] = (i + j) / 2.0
+            i = j + 1
+        return r
+    rx, ry = ranks(xs), ranks(ys)
+    mx, my = statistics.fmean(rx), statistics.fmean(ry)
+    num = sum((a - mx) * (b - my) for a, b in zip(rx, ry))
+    den = (sum((a - mx) ** 2 for a in rx) * sum((b - my) ** 2 for b in ry)) ** 0.5
+    return num / den if den else 0.0
+
+
+def summarize(result):
+    rows = result["rows"]
+    keys = []
+    for r in rows:
+        k = (r["pattern"], tuple(r["shape"]))
+        if k not in keys:
+            keys.append(k)
+    lines = ["| nest | candidates | best candidate GB/s (score, mapping) | LITERAL GB/s (score) | LITERAL rank | "
+             "AUTO GB/s | TB/T | warp | 1D | Spearman(score, GB/s) | false negatives (C) |",
+             "|---|---|---|---|---|---|---|---|---|---|---|"]
+    for pattern, shape in keys:
+        sel = [r for r in rows if r["pattern"] == pattern and tuple(r["shape"]) == shape]
+        cand = [r for r in sel if r["kind"] == "candidate"]
+        mk = {r["kind"]: r for r in sel if r["kind"] != "candidate"}
+        best = max(cand, key=lambda r: r["GB/s"])
+        top_score = max(r["score"] for r in cand)
+        lit = mk["LITERAL"]
+        rank = 1 + sum(1 for r in cand if r["GB/s"] > lit["GB/s"])
+        rho = _spearman([r["score"] for r in cand], [r["GB/s"] for r in cand])
+        fneg = sum(1 for r in cand if r["score"] < top_score // 2 and r["GB/s"] >= 0.9 * best["GB/s"])
+        lines.append(
+            f"| {pattern.lower()}[{shape[0]}x{shape[1]}] | {len(cand)} | {best['GB/s']} ({best['score']}, "
+            f"{best['mapping']}) | {lit['GB/s']} ({lit['score']}) | {rank}/{len(cand)} | {mk['AUTO']['GB/s']} | "
+            f"{mk['TB_T']['GB/s']} | {mk['WARP']['GB/s']} | {mk['1D']['GB/s']} | {rho:.2f} | {fneg} |")
+    return "\n".join(lines)
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default="gpurun_out/fig17.json")
+    ap.add_argument("--shapes", default="")
+    ap.add_argument("--summarize", default="")
+    a = ap.parse_args()
+    if a.summarize:
+        print(summarize(json.load(open(a.summarize))))
+    else:
+        run(a)
