@@ -176,6 +176,8 @@ def build_logreg(npp, gen, torch, rank, world, strategy, device):
     return [item], [], "batched logistic-regression gradient [16M,256], B=4096"
 
 
+# per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
+SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
              "logreg": build_logreg}
 
@@ -380,7 +382,7 @@ def main():
 
     out = {"metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
-           "scaling": "weak" if args.workload == "paper" else "strong", "vs_baseline": None, "dtype": "f32",
+           "scaling": SCALING[args.workload], "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (counter-based U[0,1) fp32, seeded)",
            "config": dict(config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
                                      else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),

@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define NPP_VERSION 1
+#define NPP_VERSION 2
 
 #if defined(__GNUC__)
 #define NPP_API __attribute__((visibility("default")))
@@ -81,6 +81,13 @@ typedef enum {
 
 typedef enum { NPP_SPAN_ONE = 0, NPP_SPAN_ALL = 1, NPP_SPAN_N = 2, NPP_SPLIT_K = 3 } npp_span;
 typedef enum { NPP_DIM_X = 0, NPP_DIM_Y = 1, NPP_DIM_Z = 2 } npp_dim;
+/* Where the inner zipWith of the weighted sums (Fig 15) keeps its per-outer-iteration
+ * result (§V-A, Fig 16): NONE = not materialised (the product is reduced in registers;
+ * AUTO); MALLOC = a device malloc per outer iteration (the unoptimised code of Fig 16);
+ * PREALLOC = one [outer x inner] buffer in the plan's workspace, addressed
+ * o*temp_stride[0] + i*temp_stride[1] — (inner, 1) is Fig 11a (offset m*N, stride 1), (1, outer) is
+ * Fig 11b (offset m, stride M). */
+typedef enum { NPP_TEMP_NONE = 0, NPP_TEMP_MALLOC = 1, NPP_TEMP_PREALLOC = 2 } npp_temp;
 typedef enum {
   NPP_CLASS_RX = 0,      /* inner Reduce on x (sumRows family; TB/T and warp baselines)   */
   NPP_CLASS_MX = 1,      /* outer Map on x, inner Reduce on y (sumCols family; 1D)        */
@@ -120,6 +127,9 @@ typedef struct {
   int32_t smem_bytes;
   int64_t workspace_bytes;
   int64_t claim_tiles; /* staged plans: tiles a persistent block claims at a time (dynamic Span) */
+  int32_t temp;           /* npp_temp: the weighted sums' inner allocation (S10) */
+  int32_t reserved2;
+  int64_t temp_stride[2]; /* PREALLOC: element strides of the temp buffer along (outer, inner) */
 } npp_mapping;
 
 /* Hardware limits the selector's hard constraints and ControlDOP read (L658-662, L799-803).
@@ -184,7 +194,10 @@ NPP_API int npp_plan_with_mapping(int pattern, const int64_t* shape, int ndim, i
 NPP_API int npp_plan_mapping(npp_plan_t plan, npp_mapping* out);
 
 /* Workspace bytes npp_execute needs (0 if none). The workspace must be zero-filled before its first
- * use with a plan; every successful execute leaves it zero-filled again (Split tickets reset). */
+ * use with a plan; every successful execute leaves its counters, tickets and accumulators zero-filled
+ * again (Split tickets reset). The S10 temp region of a PREALLOC weighted plan (the last
+ * outer*inner*sizeof(dtype) bytes rounded up to 256) is scratch: written before it is read, left
+ * holding the zipWith products. */
 NPP_API int64_t npp_plan_workspace_bytes(npp_plan_t plan);
 
 /* Enqueue the plan's kernel(s) on `stream` (async; no host sync; one kernel launch for every sum and

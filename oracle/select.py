@@ -287,12 +287,14 @@ STAGE_ROWS = 32                                   # DESIGN.md S8 (staged): BR
 
 
 def staged_eligible(nest, dtype, dims) -> bool:
-    """DESIGN.md S8: plain sums whose row pitch is a multiple of 16 B and whose stride-1 level is on x."""
+    """DESIGN.md S8: (weighted) sums whose row pitch is a multiple of 16 B and whose stride-1 level of m
+    is on x."""
     pattern = nest["pattern"]
-    if pattern not in ("SUM_ROWS", "SUM_COLS"):
+    if pattern not in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
         return False
-    C = nest["levels"][1][0] if pattern == "SUM_ROWS" else nest["levels"][0][0]
-    contig_level = 1 if pattern == "SUM_ROWS" else 0
+    rows = pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS")
+    C = nest["levels"][1][0] if rows else nest["levels"][0][0]
+    contig_level = 1 if rows else 0
     return C % (16 // DTYPE_SIZE[dtype]) == 0 and dims[contig_level] == X
 
 
@@ -303,10 +305,11 @@ def staged_tiles(nest, dtype):
     esz = DTYPE_SIZE[dtype]
     BC = 1024 // esz
     O, I = nest["levels"][0][0], nest["levels"][1][0]
-    C = I if nest["pattern"] == "SUM_ROWS" else O
-    wide = nest["pattern"] == "SUM_ROWS" and (C * esz) % 4096 == 0
+    rows = nest["pattern"] in ("SUM_ROWS", "SUM_WEIGHTED_ROWS")
+    C = I if rows else O
+    wide = rows and (C * esz) % 4096 == 0
     BR, W = (8, 4 * BC) if wide else (STAGE_ROWS, BC)
-    if nest["pattern"] == "SUM_ROWS":
+    if rows:
         return BR, BC, W, cdiv(O, BR), cdiv(I, W)
     return BR, BC, W, cdiv(O, W), cdiv(I, BR)
 
@@ -335,7 +338,7 @@ def r2_staged(nest, dtype, lim):
     wide = W > BC
     I = nest["levels"][1][0]
     G, CL, _ = balance(To, Ti, lim)
-    if nest["pattern"] == "SUM_ROWS":     # 8 warps; narrow: 4 rows per warp, wide: 1 row per warp
+    if nest["pattern"] in ("SUM_ROWS", "SUM_WEIGHTED_ROWS"):  # 8 warps; narrow: 4 rows/warp, wide: 1
         blocks = (8, 32)
         spans = (ONE if wide else SPAN_N, ALL if Ti == 1 else SPLIT)
         factors = (1 if wide else 4, Ti)
@@ -436,8 +439,21 @@ def kernel_class(pattern, dims):
     return RX if dims[1] == X else MX
 
 
+TEMP_NONE, TEMP_MALLOC, TEMP_PREALLOC = 0, 1, 2     # DESIGN.md S10
+
+
+def temp_layout(nest, dims):
+    """DESIGN.md S10 (§V-A, Fig 11): a weighted sum's inner zipWith result goes to one
+    preallocated [outer x inner] buffer laid out for the mapping: outer level on x -> offset m, stride
+    M (Fig 11b); otherwise offset m*N, stride 1 (Fig 11a). Returns (temp, (outer stride, inner stride))."""
+    if nest["pattern"] not in ("SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
+        return TEMP_NONE, (0, 0)
+    M, N = _eff(nest["levels"][0][0]), _eff(nest["levels"][1][0])
+    return TEMP_PREALLOC, ((1, M) if dims[0] == X else (N, 1))
+
+
 def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chunks=None, staged=0,
-                persistent_grid=None, claim_tiles=0):
+                persistent_grid=None, claim_tiles=0, temp=(TEMP_NONE, (0, 0))):
     L = len(blocks)
     levels = []
     for l in range(L):
@@ -454,7 +470,8 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
     rec = dict(nlevels=L, kernel_class=kernel_class(nest["pattern"], dims), vec=vec, staged=staged,
                levels=levels, score=score_, dop=mapping_dop(nest, blocks, spans, factors),
                threads=grid * prod(blocks), grid=grid, block=block3,
-               smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0, claim_tiles=claim_tiles)
+               smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0, claim_tiles=claim_tiles,
+               temp=temp[0], temp_stride=[temp[1][0], temp[1][1]])
     if nest["pattern"] == "LOGREG_GRAD" and staged:  # tickets [B] + fp64 accumulators [B x C]
         B, C = _eff(nest["levels"][0][0]), _eff(nest["levels"][2][0])
         rec["workspace_bytes"] = 256 * cdiv(4 * B, 256) + 256 * cdiv(8 * B * C, 256)
@@ -469,6 +486,11 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
+    if temp[0] == TEMP_PREALLOC:   # S10: the [outer x inner] buffer after partials and tickets
+        M, N = _eff(nest["levels"][0][0]), _eff(nest["levels"][1][0])
+        rec["workspace_bytes"] += 256 * cdiv(M * N * DTYPE_SIZE[dtype], 256)
+    elif temp[0] == TEMP_MALLOC:   # S10: an error flag
+        rec["workspace_bytes"] += 256
     return rec
 
 
@@ -487,7 +509,8 @@ def enumerate_mappings(pattern: str, shape, dtype: str, lim: dict) -> list:
                     continue
                 sc = score(nest, lim, dims, blocks)
                 sp, factors = control_dop(nest, lim, blocks, spans)
-                out.append(make_record(nest, dtype, lim, dims, blocks, sp, factors, 1, sc))
+                out.append(make_record(nest, dtype, lim, dims, blocks, sp, factors, 1, sc,
+                                       temp=temp_layout(nest, dims)))
     return out
 
 
@@ -501,11 +524,11 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
     if strategy in ("1D", "TB_T", "WARP"):
         dims, blocks, spans = forced(nest, dtype, lim, strategy)
         return make_record(nest, dtype, lim, dims, blocks, spans, [1] * L, 1,
-                           score(nest, lim, dims, blocks))
+                           score(nest, lim, dims, blocks), temp=temp_layout(nest, dims))
     dims, blocks, spans, sc = search(nest, dtype, lim)
     spans, factors = control_dop(nest, lim, blocks, spans)
     if strategy == "LITERAL":
-        return make_record(nest, dtype, lim, dims, blocks, spans, factors, 1, sc)
+        return make_record(nest, dtype, lim, dims, blocks, spans, factors, 1, sc, temp=temp_layout(nest, dims))
     if strategy != "AUTO":
         raise ValueError(strategy)
     if unknown:

@@ -123,22 +123,36 @@ int get_limits(const npp_limits* limits, npp_limits* out) {
 inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 void debug_print_times(const unsigned long long* dbg, int G, cudaStream_t st) {
-  static unsigned long long h[4096 * 4];
+  static unsigned long long h[4096 * 8];
   if (G > 4096) return;
   cudaStreamSynchronize(st);
-  cudaMemcpy(h, dbg, size_t(G) * 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+  cudaMemcpy(h, dbg, size_t(G) * 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+  cudaMemset(const_cast<unsigned long long*>(dbg), 0, size_t(G) * 8 * sizeof(unsigned long long));
   unsigned long long t0 = ~0ull;
-  for (int b = 0; b < G; ++b) t0 = h[b * 4] < t0 ? h[b * 4] : t0;
+  for (int b = 0; b < G; ++b) t0 = h[b * 8] < t0 ? h[b * 8] : t0;
   double mx[3] = {0, 0, 0}, mn[3] = {1e30, 1e30, 1e30}, sm[3] = {0, 0, 0};
-  for (int b = 0; b < G; ++b)
+  double fence_ticket = 0, convert = 0, flushes = 0, last_n = 0;
+  int nb = 0;
+  for (int b = 0; b < G; ++b) {
     for (int i = 0; i < 3; ++i) {
-      const double v = double(h[b * 4 + i] - t0) / 1e3;
+      const double v = double(h[b * 8 + i] - t0) / 1e3;
       mx[i] = v > mx[i] ? v : mx[i];
       mn[i] = v < mn[i] ? v : mn[i];
       sm[i] += v;
     }
-  std::fprintf(stderr, "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] combiner_end[%.2f avg %.2f max %.2f]\n",
-               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], sm[2] / G, mx[2]);
+    if (h[b * 8 + 4]) {
+      fence_ticket += double(h[b * 8 + 5] - h[b * 8 + 4]) / 1e3;
+      convert += double(h[b * 8 + 2] - h[b * 8 + 5]) / 1e3;
+      last_n += double(h[b * 8 + 7]);
+      ++nb;
+    }
+    flushes += double(h[b * 8 + 6]);
+  }
+  std::fprintf(stderr,
+               "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] combiner_end[%.2f avg %.2f "
+               "max %.2f] last batch: fence+ticket %.2f, convert+exit %.2f, size %.2f; flushes/block %.2f\n",
+               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], sm[2] / G, mx[2], nb ? fence_ticket / nb : 0.0,
+               nb ? convert / nb : 0.0, nb ? last_n / nb : 0.0, flushes / G);
 }
 
 }  // namespace
@@ -274,6 +288,41 @@ int npp_plan_with_mapping(int pattern, const int64_t* shape, int ndim, int dtype
     set_error("vec must be 1, or 16/sizeof(dtype) on the stride-1 x level with C % vec == 0");
     return NPP_ERR_UNSUPPORTED;
   }
+  // S10: the inner allocation of a weighted sum (NONE, MALLOC, or PREALLOC with a Fig 11 layout)
+  const bool weighted_pat = pattern == NPP_SUM_WEIGHTED_ROWS || pattern == NPP_SUM_WEIGHTED_COLS;
+  c.temp = forced->temp;
+  if (c.temp != NPP_TEMP_NONE) {
+    const int64_t M = nest.N[0], N = nest.N[1];
+    if (!weighted_pat || c.vec != 1 || (c.temp != NPP_TEMP_MALLOC && c.temp != NPP_TEMP_PREALLOC)) {
+      set_error("temp (S10) applies to the weighted sums with vec = 1 (NONE, MALLOC or PREALLOC)");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    if (c.temp == NPP_TEMP_PREALLOC) {
+      const int64_t so = forced->temp_stride[0], si = forced->temp_stride[1];
+      if (!((so == N && si == 1) || (so == 1 && si == M))) {
+        set_error("PREALLOC temp strides must be (inner, 1) (Fig 11a) or (1, outer) (Fig 11b)");
+        return NPP_ERR_INVALID_ARG;
+      }
+      c.temp_stride[0] = so;
+      c.temp_stride[1] = si;
+    } else {
+      c.temp_stride[0] = 0;
+      c.temp_stride[1] = 1;
+      // device-side malloc draws from the context's heap; it can only be sized before the first
+      // kernel that uses it, so the first MALLOC plan reserves max(1 GiB, 1.25 x the nest's bytes)
+      const size_t need = size_t(double(M) * double(N) * npp::dtype_size(dtype) * 1.25) + (64u << 20);
+      size_t cur = 0;
+      if (cudaDeviceGetLimit(&cur, cudaLimitMallocHeapSize) != cudaSuccess) cur = 0;
+      if (cur < need) {
+        const size_t want = need > (size_t(1) << 30) ? need : (size_t(1) << 30);
+        if (cudaDeviceSetLimit(cudaLimitMallocHeapSize, want) != cudaSuccess) {
+          cudaGetLastError();
+          set_error("MALLOC temp: the device malloc heap is already fixed below this nest's size");
+          return NPP_ERR_UNSUPPORTED;
+        }
+      }
+    }
+  }
   npp_plan_s* p = new npp_plan_s();
   p->pattern = pattern;
   p->dtype = dtype;
@@ -394,6 +443,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     const npp::StagedTiling t = npp::staged_tiling(plan->pattern, R, C, plan->dtype);
     npp::StagedArgs s{};
     s.out = out;
+    s.v = weighted ? ins[1] : nullptr;
     s.R = R;
     s.C = C;
     s.O = rows ? R : C;
@@ -410,7 +460,10 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     // measurement knob: NPP_DEBUG_TIMES=1 prints per-phase block timestamps (synchronises the stream)
     static unsigned long long* dbg = nullptr;
     const bool want_times = getenv("NPP_DEBUG_TIMES") != nullptr;
-    if (want_times && !dbg && cudaMalloc(&dbg, 4096 * 4 * sizeof(unsigned long long)) != cudaSuccess) dbg = nullptr;
+    if (want_times && !dbg) {
+      if (cudaMalloc(&dbg, 4096 * 8 * sizeof(unsigned long long)) != cudaSuccess) dbg = nullptr;
+      else cudaMemset(dbg, 0, 4096 * 8 * sizeof(unsigned long long));
+    }
     s.dbg_times = want_times ? dbg : nullptr;
     const int G = int(m.grid);
     cudaError_t e = npp::launch_sum_staged(plan->dtype, rows, ins[0], s, G, st);
@@ -434,11 +487,25 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
   a.ci = li.chunk;
   a.go = lo.grid;
   a.gi = li.grid;
+  int64_t ws_used = 0;  // S9 workspace: [partials][tickets] (Split), then the S10 temp region
   if (a.gi > 1) {
     const int acc = plan->dtype == NPP_I32 ? 4 : 8;
     const int64_t part = ((a.gi * a.O * acc + 255) / 256) * 256;
     a.partials = workspace;
     a.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + part);
+    ws_used = part + ((a.go * 4 + 255) / 256) * 256;
+  }
+  if (m.temp != NPP_TEMP_NONE) {  // S10: the weighted sum with its zipWith materialised
+    if (m.temp == NPP_TEMP_PREALLOC) {
+      a.temp = static_cast<char*>(workspace) + ws_used;
+      a.ts_o = m.temp_stride[0];
+      a.ts_i = m.temp_stride[1];
+    } else {
+      a.err = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + ws_used);
+    }
+    cudaError_t e = npp::launch_sum_temp(plan->dtype, m.kernel_class, m.temp == NPP_TEMP_MALLOC, a, st);
+    if (e != cudaSuccess) return cuda_fail("temp kernel launch", e);
+    return NPP_OK;
   }
   cudaError_t e = npp::launch_sum(plan->dtype, m.kernel_class, m.vec, weighted, a, st);
   if (e != cudaSuccess) return cuda_fail("kernel launch", e);

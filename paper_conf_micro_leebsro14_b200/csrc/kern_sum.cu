@@ -367,6 +367,114 @@ cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumA
   }
 }
 
+// ====================================================================================== S10 temp family
+// The weighted sums with their inner zipWith materialised (Fig 15; §V-A):
+// phase A writes t(o, i) = m[o, i]·v[i] into the inner allocation, phase B reduces it — the code the
+// paper's compiler generates, kept to reproduce Fig 16. MALLOC: one device malloc per outer iteration
+// (per block chunk), by the thread with inner index 0, shared through shared memory and freed after
+// the reduce; PREALLOC: one [O x I] buffer of the workspace at o*ts_o + i*ts_i (Fig 11a / 11b). The
+// block is the record's (RXC: x = inner; else x = outer), scalar accesses (vec = 1), the inner threads
+// meet in a shared-memory tree, Split(k) partials combine as in the other families.
+template <typename T, bool RXC, bool MALLOC>
+__global__ void __launch_bounds__(1024) npp_sum_temp_kernel(SumArgs a) {
+  using O_ = Ops<T>;
+  using Acc = typename O_::Acc;
+  extern __shared__ unsigned char smem_raw[];
+  const int to = RXC ? threadIdx.y : threadIdx.x;  // outer-thread index
+  const int ti = RXC ? threadIdx.x : threadIdx.y;  // inner-thread index
+  const int nbo = a.bo, nbi = a.bi;
+  Acc* red = reinterpret_cast<Acc*>(smem_raw);                       // [nbo][nbi]
+  T** ptrs = reinterpret_cast<T**>(red + size_t(nbo) * nbi);         // [nbo] (MALLOC)
+  const int64_t bid = blockIdx.x;
+  const int64_t g_outer = bid % a.go, s = bid / a.go;
+  const int64_t o_begin = g_outer * a.co;
+  const int64_t o_end = min(a.O, o_begin + a.co);
+  const int64_t i_begin = s * a.ci;
+  const int64_t i_end = min(a.I, i_begin + a.ci);
+  const T* __restrict__ m = static_cast<const T*>(a.m);
+  const T* __restrict__ wv = static_cast<const T*>(a.v);
+  T* temp = static_cast<T*>(a.temp);
+  const int nrep = int((a.co + nbo - 1) / nbo);
+  int wtop = 1;
+  while (wtop < nbi) wtop <<= 1;
+  for (int j = 0; j < nrep; ++j) {
+    const int64_t o = o_begin + to + int64_t(j) * nbo;
+    const bool valid = o < o_end;
+    T* buf = nullptr;
+    if constexpr (MALLOC) {
+      if (ti == 0) {
+        T* p = nullptr;
+        if (valid && i_end > i_begin) {
+          p = static_cast<T*>(malloc(size_t(i_end - i_begin) * sizeof(T)));
+          if (!p) atomicExch(a.err, 1u);
+        }
+        ptrs[to] = p;
+      }
+      __syncthreads();
+      buf = ptrs[to];
+    }
+    const bool work = valid && (!MALLOC || buf != nullptr);
+    if (work)  // phase A: temp = c zipWith v (the inner Map's allocation)
+      for (int64_t i = i_begin + ti; i < i_end; i += nbi) {
+        const T x = T(O_::mul(m[o * a.so + i * a.si], __ldg(wv + i)));
+        if constexpr (MALLOC)
+          buf[i - i_begin] = x;
+        else
+          temp[o * a.ts_o + i * a.ts_i] = x;
+      }
+    __syncthreads();
+    Acc acc = 0;
+    if (work)  // phase B: temp reduce +
+      for (int64_t i = i_begin + ti; i < i_end; i += nbi) {
+        T x;
+        if constexpr (MALLOC)
+          x = buf[i - i_begin];
+        else
+          x = temp[o * a.ts_o + i * a.ts_i];
+        acc += O_::widen(O_::from(x));
+      }
+    red[to * nbi + ti] = acc;
+    __syncthreads();
+    for (int w = wtop >> 1; w >= 1; w >>= 1) {
+      if (ti < w && ti + w < nbi) red[to * nbi + ti] += red[to * nbi + ti + w];
+      __syncthreads();
+    }
+    if (ti == 0 && valid) emit<T>(a, s, o, red[to * nbi]);
+    __syncthreads();
+    if constexpr (MALLOC) {
+      if (ti == 0 && buf) free(buf);
+    }
+  }
+  if (a.gi > 1) split_combine<T>(a, g_outer, o_begin, o_end);
+}
+
+template <typename T>
+static cudaError_t launch_temp_t(int kclass, bool malloc_mode, const SumArgs& a, dim3 grid, dim3 block, size_t smem,
+                                 cudaStream_t st) {
+  const bool rx = kclass == NPP_CLASS_RX;
+  if (rx && malloc_mode)
+    npp_sum_temp_kernel<T, true, true><<<grid, block, smem, st>>>(a);
+  else if (rx)
+    npp_sum_temp_kernel<T, true, false><<<grid, block, smem, st>>>(a);
+  else if (malloc_mode)
+    npp_sum_temp_kernel<T, false, true><<<grid, block, smem, st>>>(a);
+  else
+    npp_sum_temp_kernel<T, false, false><<<grid, block, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sum_temp(int dtype, int kclass, bool malloc_mode, const SumArgs& a, cudaStream_t st) {
+  const int acc = dtype == NPP_I32 ? 4 : 8;
+  dim3 grid(unsigned(a.go * a.gi));
+  dim3 block = kclass == NPP_CLASS_RX ? dim3(unsigned(a.bi), unsigned(a.bo)) : dim3(unsigned(a.bo), unsigned(a.bi));
+  const size_t smem = size_t(a.bo) * a.bi * acc + size_t(a.bo) * sizeof(void*);
+  switch (dtype) {
+    case NPP_F32: return launch_temp_t<float>(kclass, malloc_mode, a, grid, block, smem, st);
+    case NPP_I32: return launch_temp_t<int32_t>(kclass, malloc_mode, a, grid, block, smem, st);
+    default: return launch_temp_t<int64_t>(kclass, malloc_mode, a, grid, block, smem, st);
+  }
+}
+
 template <typename T, int V, bool W>
 static void add_attr(int* regs) {
   cudaFuncAttributes fa;

@@ -26,6 +26,7 @@
 
 #include <cstdint>
 #include <cstdlib>
+#include <cstring>
 #include <type_traits>
 
 #include "kernels.hpp"
@@ -49,6 +50,8 @@ constexpr int kThreads = kConsumers + 64;
 constexpr int kFlushRing = 8;  // flushes of cut outer tiles in flight between consumers and the combiner
 constexpr int kSmemHeader = 1024;          // mbarriers + per-slot tile ids; tiles start 1 KB-aligned
 constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes;
+constexpr int kVSlot = 4096;  // weighted sums: the tile's slice of v (<= 4 KB) per ring slot
+constexpr int kSmemBytesW = kSmemBytes + kStages * kVSlot;
 
 __device__ __forceinline__ unsigned smem_u32(const void* p) {
   return static_cast<unsigned>(__cvta_generic_to_shared(p));
@@ -86,6 +89,13 @@ __device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
       : "memory");
   return ok != 0;
 }
+__device__ __forceinline__ void tma_load_1d(void* dst, const CUtensorMap* map, int x, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(x), "r"(smem_u32(bar))
+      : "memory");
+}
 __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int x, int y, int z, uint64_t* bar) {
   asm volatile(
       "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
@@ -122,6 +132,22 @@ __device__ __forceinline__ unsigned vsum(const int4& v) {
 __device__ __forceinline__ unsigned long long vsum(const longlong2& v) {
   return (unsigned long long)v.x + (unsigned long long)v.y;
 }
+// weighted: Σ of the 16-byte vector's products with the weights (fp32 pairwise; integers wrap)
+__device__ __forceinline__ float vdot(const float4& x, const float4& w) {
+  return (x.x * w.x + x.y * w.y) + (x.z * w.z + x.w * w.w);
+}
+__device__ __forceinline__ unsigned vdot(const int4& x, const int4& w) {
+  return unsigned(x.x) * unsigned(w.x) + unsigned(x.y) * unsigned(w.y) + unsigned(x.z) * unsigned(w.z) +
+         unsigned(x.w) * unsigned(w.w);
+}
+__device__ __forceinline__ unsigned long long vdot(const longlong2& x, const longlong2& w) {
+  return (unsigned long long)x.x * (unsigned long long)w.x + (unsigned long long)x.y * (unsigned long long)w.y;
+}
+__device__ __forceinline__ float vmul(float x, float w) { return x * w; }
+__device__ __forceinline__ int32_t vmul(int32_t x, int32_t w) { return int32_t(unsigned(x) * unsigned(w)); }
+__device__ __forceinline__ int64_t vmul(int64_t x, int64_t w) {
+  return int64_t((unsigned long long)x * (unsigned long long)w);
+}
 template <typename T> struct V16;
 template <> struct V16<float> { using type = float4; };
 template <> struct V16<int32_t> { using type = int4; };
@@ -137,8 +163,12 @@ __device__ __forceinline__ A warp_sum(A v) {
 
 }  // namespace
 
-template <typename T, bool ROWS, bool WIDE>
+// WT: weighted sums (sumWeightedRows / sumWeightedCols, Fig 15) fused: the zipWith
+// product m·v is formed in registers from the staged tile and the tile's slice of v (staged by a 1-D
+// TMA box on the same mbarrier), so no inner allocation exists at all (§V-A taken to its limit).
+template <typename T, bool ROWS, bool WIDE, bool WT>
 __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_constant__ CUtensorMap map,
+                                                                  const __grid_constant__ CUtensorMap vmap,
                                                                   StagedArgs a) {
   using Acc = typename SOps<T>::Acc;
   using V = typename V16<T>::type;
@@ -156,6 +186,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   long long* fl_ot = slot_tile + kStages;     // [kFlushRing] outer tile of a flush, -1 = end
   unsigned* fl_cnt = reinterpret_cast<unsigned*>(fl_ot + kFlushRing);  // tiles it contributes
   unsigned char* tiles = smem + kSmemHeader;
+  unsigned char* vslots = tiles + kStages * kTileBytes;  // WT only: [kStages][kVSlot]
   Acc* accg = static_cast<Acc*>(a.acc);
   constexpr long long kFlush = 1ll << 62;
 
@@ -182,8 +213,8 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     if (a.dbg_times) {
       unsigned smid;
       asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-      a.dbg_times[bid * 4 + 0] = gtimer();
-      a.dbg_times[bid * 4 + 3] = smid;
+      a.dbg_times[bid * 8 + 0] = gtimer();
+      a.dbg_times[bid * 8 + 3] = smid;
     }
   }
   __syncthreads();
@@ -192,6 +223,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     // ------------------------------------------------------------ producer: one elected lane
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(&map) : "memory");
+      if constexpr (WT) asm volatile("prefetch.tensormap [%0];" ::"l"(&vmap) : "memory");
       long long sn = s0, u_cur = 0, u_end = 0;
       // Every launch is a programmatic dependent launch: this block may already be resident while the
       // previous kernel in the stream drains. Unless the caller asserted NPP_EXEC_OVERLAP (inputs not
@@ -226,10 +258,20 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         const int slot = int(t % kStages);
         if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
         slot_tile[slot] = cur | (flush ? kFlush : 0);
-        mbar_expect_tx(full + slot, kTileBytes);
+        constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
+        mbar_expect_tx(full + slot, kTileBytes + kVBytes);
         const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
         const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
         const int y = int(ROWS ? ot * RT : it * RT);     // first row
+        if constexpr (WT) {  // v over the tile's columns (RX) or rows (MX); zero-filled past the end
+          if constexpr (ROWS) {
+#pragma unroll
+            for (int q = 0; q < NCH; ++q)
+              tma_load_1d(vslots + slot * kVSlot + q * 1024, &vmap, (ch + q) * BC, full + slot);
+          } else {
+            tma_load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
+          }
+        }
         if constexpr (WIDE)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
           tma_load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
         else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
@@ -260,6 +302,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       const unsigned cnt = lane < nb ? fl_cnt[i] : 0u;
       const unsigned ends = __ballot_sync(0xffffffffu, lane < nb && ot < 0);
       const int n = ends ? __ffs(ends) - 1 : nb;  // entries before the end marker
+      const unsigned long long t_b0 = a.dbg_times ? gtimer() : 0ull;
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
       bool last = false;
       if (lane < n) {
@@ -268,6 +311,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         if (last) a.tickets[ot] = 0u;
       }
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      if (a.dbg_times && lane == 0 && n > 0) {  // measurement knob: the last batch's phases
+        a.dbg_times[bid * 8 + 4] = t_b0;
+        a.dbg_times[bid * 8 + 5] = gtimer();
+        a.dbg_times[bid * 8 + 6] += n;
+        a.dbg_times[bid * 8 + 7] = n;
+      }
       unsigned lasts = __ballot_sync(0xffffffffu, last);
       while (lasts) {  // every contribution to these outer tiles is in: read (L2), convert, re-zero
         const int j = __ffs(lasts) - 1;
@@ -297,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       k += n;
       if (ends) break;
     }
-    if (a.dbg_times && lane == 0) a.dbg_times[bid * 4 + 2] = gtimer();
+    if (a.dbg_times && lane == 0) a.dbg_times[bid * 8 + 2] = gtimer();
   } else {
     // ------------------------------------------------------------ consumers
     constexpr int kGroups = ROWS ? 1 : 256 / BC;  // MX row groups (1 for 4-byte types, 2 for 8-byte)
@@ -315,19 +364,34 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       const long long tag = slot_tile[slot];
       if (tag < 0) break;
       const unsigned char* tile = tiles + slot * kTileBytes;
+      const unsigned char* vs = vslots + slot * kVSlot;
       if constexpr (ROWS && !WIDE) {
+        V w0{}, w1{};
+        if constexpr (WT) {
+          w0 = *reinterpret_cast<const V*>(vs + lane * 16);
+          w1 = *reinterpret_cast<const V*>(vs + 512 + lane * 16);
+        }
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr) {
           const unsigned char* row = tile + (warp * 4 + rr) * 1024;
           const V v0 = *reinterpret_cast<const V*>(row + lane * 16);
           const V v1 = *reinterpret_cast<const V*>(row + 512 + lane * 16);
-          acc[rr] += Acc(vsum(v0) + vsum(v1));
+          if constexpr (WT)
+            acc[rr] += Acc(vdot(v0, w0) + vdot(v1, w1));
+          else
+            acc[rr] += Acc(vsum(v0) + vsum(v1));
         }
       } else if constexpr (ROWS) {  // wide: warp w adds the 4 KB of row w, 8 x 16 B per lane
         const unsigned char* row = tile + warp * 4096;
         decltype(vsum(V{})) p[8];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) p[k] = vsum(*reinterpret_cast<const V*>(row + k * 512 + lane * 16));
+        for (int k = 0; k < 8; ++k) {
+          const V x = *reinterpret_cast<const V*>(row + k * 512 + lane * 16);
+          if constexpr (WT)
+            p[k] = vdot(x, *reinterpret_cast<const V*>(vs + k * 512 + lane * 16));
+          else
+            p[k] = vsum(x);
+        }
 #pragma unroll
         for (int w = 4; w >= 1; w /= 2)
 #pragma unroll
@@ -339,7 +403,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         for (int k = 0; k < NCH; ++k) {
           T v[kRowsPer];
 #pragma unroll
-          for (int rr = 0; rr < kRowsPer; ++rr) v[rr] = tt[(rg * kRowsPer + rr) * W + k * BC + col];
+          for (int rr = 0; rr < kRowsPer; ++rr) {
+            v[rr] = tt[(rg * kRowsPer + rr) * W + k * BC + col];
+            if constexpr (WT) v[rr] = vmul(v[rr], reinterpret_cast<const T*>(vs)[rg * kRowsPer + rr]);
+          }
           if constexpr (std::is_same<T, float>::value) {  // fp32: pairwise tree inside the tile
 #pragma unroll
             for (int w = kRowsPer / 2; w >= 1; w /= 2)
@@ -422,7 +489,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       mbar_arrive(fl_full + fi);
     }
   }
-  if (a.dbg_times && threadIdx.x == 0) a.dbg_times[bid * 4 + 1] = gtimer();
+  if (a.dbg_times && threadIdx.x == 0) a.dbg_times[bid * 8 + 1] = gtimer();
 }
 
 // ====================================================================================== host side
@@ -444,24 +511,35 @@ EncodeTiledFn encode_fn() {
   return fn;
 }
 
-template <typename T, bool ROWS, bool WIDE>
-cudaError_t launch_typed(const CUtensorMap& map, const StagedArgs& a, int grid, cudaStream_t st) {
+template <typename T, bool ROWS, bool WIDE, bool WT>
+cudaError_t launch_typed(const CUtensorMap& map, const CUtensorMap& vmap, const StagedArgs& a, int grid,
+                         cudaStream_t st) {
   static bool attr_set = false;
-  auto kern = npp_sum_tma_kernel<T, ROWS, WIDE>;
+  auto kern = npp_sum_tma_kernel<T, ROWS, WIDE, WT>;
+  const int smem = WT ? kSmemBytesW : kSmemBytes;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  return launch_pdl(kern, grid, kThreads, kSmemBytes, st, true, map, a);
+  return launch_pdl(kern, grid, kThreads, smem, st, true, map, vmap, a);
+}
+
+template <typename T, bool WT>
+cudaError_t launch_w(bool rows, const CUtensorMap& map, const CUtensorMap& vmap, const StagedArgs& a, int grid,
+                     cudaStream_t st) {
+  // wide tiles are selected for sumRows only (S8); the MX-wide path of the kernel template (4 KB
+  // column strips) measured slower than 1 KB strips because of the larger combine per cut strip
+  if (rows)
+    return a.wide ? launch_typed<T, true, true, WT>(map, vmap, a, grid, st)
+                  : launch_typed<T, true, false, WT>(map, vmap, a, grid, st);
+  return launch_typed<T, false, false, WT>(map, vmap, a, grid, st);
 }
 
 template <typename T>
-cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const StagedArgs& a, int grid, cudaStream_t st) {
-  // wide tiles are selected for sumRows only (S8); the MX-wide path of the kernel template (4 KB
-  // column strips) measured slower than 1 KB strips because of the larger combine per cut strip
-  if (rows) return a.wide ? launch_typed<T, true, true>(map, a, grid, st) : launch_typed<T, true, false>(map, a, grid, st);
-  return launch_typed<T, false, false>(map, a, grid, st);
+cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const CUtensorMap& vmap, const StagedArgs& a, int grid,
+                         cudaStream_t st) {
+  return a.v ? launch_w<T, true>(rows, map, vmap, a, grid, st) : launch_w<T, false>(rows, map, vmap, a, grid, st);
 }
 
 }  // namespace
@@ -492,10 +570,21 @@ cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedA
                CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   }
   if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  CUtensorMap vmap;  // weighted: 1-D map over v (C elements for sumRows, R for sumCols)
+  std::memset(&vmap, 0, sizeof vmap);
+  if (a.v) {
+    const cuuint64_t vd[1] = {cuuint64_t(rows ? a.C : a.R)};
+    const cuuint64_t vs[1] = {vd[0] * esz};
+    const cuuint32_t vb[1] = {cuuint32_t(rows ? bc : kTileRows)};
+    const cuuint32_t ve[1] = {1};
+    r = encode(&vmap, dt, 1, const_cast<void*>(a.v), vd, vs, vb, ve, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  }
   switch (dtype) {
-    case NPP_F32: return launch_dtype<float>(rows, map, a, grid, st);
-    case NPP_I32: return launch_dtype<int32_t>(rows, map, a, grid, st);
-    default: return launch_dtype<int64_t>(rows, map, a, grid, st);
+    case NPP_F32: return launch_dtype<float>(rows, map, vmap, a, grid, st);
+    case NPP_I32: return launch_dtype<int32_t>(rows, map, vmap, a, grid, st);
+    default: return launch_dtype<int64_t>(rows, map, vmap, a, grid, st);
   }
 }
 

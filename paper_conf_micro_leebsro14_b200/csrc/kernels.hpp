@@ -42,9 +42,14 @@ struct SumArgs {
   int bo, bi;          // threads along the outer / inner level
   int64_t co, ci;      // chunk (indices per block) of the outer / inner level
   int64_t go, gi;      // blocks along the outer / inner level
+  void* temp;          // S10 PREALLOC: the [O x I] zipWith buffer (weighted sums), else NULL
+  int64_t ts_o, ts_i;  // its element strides along the outer / inner index (Fig 11)
+  unsigned* err;       // S10 MALLOC: set to 1 when a device malloc returns NULL
 };
 
 cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumArgs& a, cudaStream_t st);
+// S10: weighted sums with the inner allocation materialised (MALLOC or PREALLOC), vec = 1
+cudaError_t launch_sum_temp(int dtype, int kclass, bool malloc_mode, const SumArgs& a, cudaStream_t st);
 int sum_kernels_max_regs();
 
 // Arguments of one staged (TMA) sum launch (S8 staged): the matrix is [R x C]; tiles are
@@ -52,6 +57,7 @@ int sum_kernels_max_regs();
 // [b*Ts/G, (b+1)*Ts/G), then claims units of `unit` tiles of the pool [Ts, To*Ti) (S8).
 struct StagedArgs {
   void* out;
+  const void* v;        // weighted sums: v [C] (sumWeightedRows) or [R] (sumWeightedCols), else NULL
   void* acc;           // [O] accumulators (fp64 / u32 / u64), zero on entry and on exit
   unsigned* pool;      // [2]: pool claim counter, blocks-done ticket (zero on entry and on exit)
   unsigned* tickets;   // [To] tiles contributed per outer tile (partial contributors), zero on entry/exit

@@ -216,15 +216,15 @@ int64_t slots(const npp_limits& lim, int threads_per_block) {
 
 // S8 staged family: plain sums, 16-B row pitch, stride-1 level of m on x.
 bool staged_eligible(const Nest& n, int dtype, const Choice& c) {
-  if (n.pattern != NPP_SUM_ROWS && n.pattern != NPP_SUM_COLS) return false;
-  const int contig_level = n.pattern == NPP_SUM_ROWS ? 1 : 0;
+  if (!is_sum_pattern(n.pattern)) return false;
+  const int contig_level = is_rows_pattern(n.pattern) ? 1 : 0;
   return n.cols % (16 / dtype_size(dtype)) == 0 && c.dims[contig_level] == NPP_DIM_X;
 }
 
 // S8 staged family: persistent blocks (one per SM) stream BR x W tiles in outer-major order
 // (static range + pool); the inner level is Split(Ti).
 void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
-  const bool rows = n.pattern == NPP_SUM_ROWS;
+  const bool rows = is_rows_pattern(n.pattern);
   const int64_t R = rows ? n.N[0] : n.N[1];
   const StagedTiling t = staged_tiling(n.pattern, R, n.cols, dtype);
   const StagedBalance bal = staged_balance(t.To, t.Ti, lim.sm_count);
@@ -381,10 +381,10 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   StagedTiling t;
   const int64_t esz = dtype_size(dtype);
   t.BC = 1024 / esz;
-  t.wide = pattern == NPP_SUM_ROWS && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
+  t.wide = is_rows_pattern(pattern) && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
   t.BR = t.wide ? 8 : kStageRows;
   t.W = t.wide ? 4 * t.BC : t.BC;
-  if (pattern == NPP_SUM_ROWS) {
+  if (is_rows_pattern(pattern)) {
     t.To = cdiv(R, t.BR);
     t.Ti = cdiv(C, t.W);
   } else {
@@ -395,6 +395,8 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
 }
 
 int dtype_size(int dtype) { return dtype == NPP_I64 ? 8 : 4; }
+
+bool is_rows_pattern(int p) { return p == NPP_SUM_ROWS || p == NPP_SUM_WEIGHTED_ROWS; }
 
 bool is_sum_pattern(int p) {
   return p == NPP_SUM_ROWS || p == NPP_SUM_COLS || p == NPP_SUM_WEIGHTED_ROWS ||
@@ -571,11 +573,14 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.workspace_bytes = 0;
   m.staged = c.staged;
   m.claim_tiles = c.claim_tiles;
+  m.temp = c.temp;
+  m.temp_stride[0] = c.temp_stride[0];
+  m.temp_stride[1] = c.temp_stride[1];
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
   } else if (is_sum_pattern(n.pattern) && c.staged) {
     // pool counters (256 B) + tickets [To] + accumulators [O] of the accumulator type
-    const StagedTiling t = staged_tiling(n.pattern, n.pattern == NPP_SUM_ROWS ? n.N[0] : n.N[1], n.cols, dtype);
+    const StagedTiling t = staged_tiling(n.pattern, is_rows_pattern(n.pattern) ? n.N[0] : n.N[1], n.cols, dtype);
     m.workspace_bytes =
         256 + 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
   } else if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
@@ -583,8 +588,24 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
     const int64_t tick = m.level[0].grid * 4;
     m.workspace_bytes = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256);
   }
+  if (c.temp == NPP_TEMP_PREALLOC)  // S10: the [outer x inner] buffer after partials and tickets
+    m.workspace_bytes += 256 * cdiv(eff(n.N[0]) * eff(n.N[1]) * dtype_size(dtype), 256);
+  else if (c.temp == NPP_TEMP_MALLOC)  // S10: one error flag (a device malloc that returned NULL)
+    m.workspace_bytes += 256;
   *out = m;
   return NPP_OK;
+}
+
+void temp_layout(const Nest& n, Choice* c) {
+  if (n.pattern != NPP_SUM_WEIGHTED_ROWS && n.pattern != NPP_SUM_WEIGHTED_COLS) return;
+  c->temp = NPP_TEMP_PREALLOC;
+  if (c->dims[0] == NPP_DIM_X) {  // Fig 11b
+    c->temp_stride[0] = 1;
+    c->temp_stride[1] = eff(n.N[0]);
+  } else {  // Fig 11a
+    c->temp_stride[0] = eff(n.N[1]);
+    c->temp_stride[1] = 1;
+  }
 }
 
 int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy, npp_mapping* out) {
@@ -614,6 +635,7 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
       set_error("forced mapping violates a hard constraint on this device");
       return NPP_ERR_NO_FEASIBLE_MAPPING;
     }
+    temp_layout(n, &c);  // the paper's generated code preallocates with the mapping's layout (S10)
     return record_from_choice(n, dtype, lim, c, score(n, lim, c), out);
   }
   if (strategy != NPP_MAP_AUTO && strategy != NPP_MAP_LITERAL) {
@@ -625,7 +647,10 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
     return NPP_ERR_NO_FEASIBLE_MAPPING;
   }
   control_dop(n, lim, &c);
-  if (strategy == NPP_MAP_LITERAL) return record_from_choice(n, dtype, lim, c, sc, out);
+  if (strategy == NPP_MAP_LITERAL) {
+    temp_layout(n, &c);
+    return record_from_choice(n, dtype, lim, c, sc, out);
+  }
   if (unknown) {
     set_error("strategy AUTO needs known sizes (use LITERAL for -1 sizes)");
     return NPP_ERR_UNSUPPORTED;
@@ -698,6 +723,7 @@ extern "C" int64_t npp_enumerate(int pattern, const int64_t* shape, int ndim, in
       Choice c = c0;
       const int64_t s = score(n, *limits, c);
       control_dop(n, *limits, &c);
+      temp_layout(n, &c);
       record_from_choice(n, dtype, *limits, c, s, out + count);
     }
     ++count;

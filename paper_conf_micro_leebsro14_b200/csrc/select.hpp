@@ -37,7 +37,13 @@ struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refi
   int staged = 0;  // 1: TMA-staged tile family (S8)
   int64_t persistent_grid = 0;  // staged: blocks launched (0: product of the level grids)
   int64_t claim_tiles = 0;      // staged: tiles per dynamic claim
+  int temp = NPP_TEMP_NONE;     // weighted sums: inner allocation (S10)
+  int64_t temp_stride[2] = {0, 0};
 };
+
+// S10 (§V-A, Fig 11): the preallocated [outer x inner] buffer of a weighted sum is laid out
+// for the mapping — outer level on x: offset m, stride M (Fig 11b); otherwise offset m*N, stride 1.
+void temp_layout(const struct Nest& n, Choice* c);
 
 constexpr int kStageRows = 32;  // BR of the staged family (S8): tiles of 32 rows x 1 KB
 constexpr int64_t kPoolDiv = 8;       // S8 balance rule: about 1/kPoolDiv of the tiles form the shared pool
@@ -63,6 +69,7 @@ void set_error(const std::string& msg);
 
 int dtype_size(int dtype);
 bool is_sum_pattern(int pattern);
+bool is_rows_pattern(int pattern);  // SUM_ROWS / SUM_WEIGHTED_ROWS
 int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out);
 int check_limits(const npp_limits* lim);
 bool hard_ok(const Nest& n, int dtype, const npp_limits& lim, const Choice& c);

@@ -42,7 +42,8 @@ class Mapping(ctypes.Structure):
                 ("staged", ctypes.c_int32), ("level", Level * 4), ("score", ctypes.c_int64),
                 ("dop", ctypes.c_int64), ("threads", ctypes.c_int64), ("grid", ctypes.c_int64),
                 ("block", ctypes.c_int32 * 3), ("smem_bytes", ctypes.c_int32),
-                ("workspace_bytes", ctypes.c_int64), ("claim_tiles", ctypes.c_int64)]
+                ("workspace_bytes", ctypes.c_int64), ("claim_tiles", ctypes.c_int64),
+                ("temp", ctypes.c_int32), ("reserved2", ctypes.c_int32), ("temp_stride", ctypes.c_int64 * 2)]
 
 
 class Limits(ctypes.Structure):
@@ -55,6 +56,7 @@ class Limits(ctypes.Structure):
 
 
 EXEC_OVERLAP = 1  # npp.h NPP_EXEC_OVERLAP
+TEMP_NONE, TEMP_MALLOC, TEMP_PREALLOC = 0, 1, 2  # npp.h npp_temp
 
 EXPORTS = ("npp_version", "npp_last_error", "npp_limits_query", "npp_select", "npp_plan",
            "npp_plan_with_mapping", "npp_plan_mapping", "npp_plan_workspace_bytes", "npp_execute",
@@ -134,7 +136,8 @@ def mapping_to_dict(m: Mapping) -> dict:
     return dict(nlevels=m.nlevels, kernel_class=m.kernel_class, vec=m.vec, staged=m.staged, levels=levels,
                 score=m.score,
                 dop=m.dop, threads=m.threads, grid=m.grid, block=list(m.block), smem_bytes=m.smem_bytes,
-                workspace_bytes=m.workspace_bytes, claim_tiles=m.claim_tiles)
+                workspace_bytes=m.workspace_bytes, claim_tiles=m.claim_tiles, temp=m.temp,
+                temp_stride=[m.temp_stride[0], m.temp_stride[1]])
 
 
 def mapping_from_dict(d: dict) -> Mapping:
@@ -146,6 +149,9 @@ def mapping_from_dict(d: dict) -> Mapping:
         m.level[i].block = int(lv["block"])
         m.level[i].span = int(lv["span"])
         m.level[i].factor = int(lv.get("factor", 1))
+    m.temp = int(d.get("temp", 0))
+    ts = d.get("temp_stride", (0, 0))
+    m.temp_stride[0], m.temp_stride[1] = int(ts[0]), int(ts[1])
     return m
 
 

@@ -2,6 +2,8 @@
 import ctypes
 import os
 import re
+import shutil
+import subprocess
 
 import pytest
 
@@ -29,12 +31,28 @@ def test_library_exports_every_declared_symbol():
         assert hasattr(lib, s), s
 
 
-def test_struct_layout_matches_binding():
+def _c_layout(tmp_path, struct, fields):
+    """sizeof/offsetof of a struct of include/npp.h as the C compiler lays it out."""
+    src = tmp_path / "layout.c"
+    body = "".join(f'  printf("%zu\\n", offsetof({struct}, {f}));\n' for f in fields)
+    src.write_text(f'#include <stddef.h>\n#include <stdio.h>\n#include "npp.h"\n'
+                   f'int main(void) {{\n  printf("%zu\\n", sizeof({struct}));\n{body}  return 0;\n}}\n')
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    vals = [int(v) for v in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
+    return vals[0], vals[1:]
+
+
+@pytest.mark.skipif(shutil.which("gcc") is None, reason="gcc not available")
+def test_struct_layout_matches_binding(tmp_path):
+    # the ctypes mirrors of npp_level / npp_mapping / npp_limits have the C compiler's layout
     from paper_conf_micro_leebsro14_b200 import npp
-    assert ctypes.sizeof(npp.Level) == 40
-    assert ctypes.sizeof(npp.Mapping) == 16 + 4 * 40 + 32 + 12 + 4 + 8 + 8
-    assert ctypes.sizeof(npp.Limits) == 4 * 12 + 8
-    assert npp.lib().npp_version() == 1
+    for struct, cls in (("npp_level", npp.Level), ("npp_mapping", npp.Mapping), ("npp_limits", npp.Limits)):
+        names = [f[0] for f in cls._fields_]
+        size, offs = _c_layout(tmp_path, struct, names)
+        assert ctypes.sizeof(cls) == size, struct
+        assert [getattr(cls, n).offset for n in names] == offs, struct
+    assert npp.lib().npp_version() == 2
     assert set(npp.EXPORTS) == set(declared_symbols())
 
 

@@ -227,26 +227,83 @@ def test_streams_and_concurrent_plans(npp, cuda_device):
         check("SUM_COLS", m, out, "f32")
 
 
-def test_weighted(npp, cuda_device):
-    for dtype in ("f32", "i32"):
-        for shape in [(1000, 999), (4096, 4096), (37, 70000)]:
-            m = _make(dtype, shape, 7, cuda_device)
-            for pattern, vlen in (("SUM_WEIGHTED_ROWS", shape[1]), ("SUM_WEIGHTED_COLS", shape[0])):
-                v = _make(dtype, (vlen,), 8, cuda_device) if dtype == "i32" else \
-                    gen.uniform_f32(8, (vlen,), device=cuda_device, lo=-1.0, scale=2.0)
-                for strategy in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
-                    p = npp.Plan(pattern, shape, dtype, strategy)
-                    out = p.execute([m, v], p.new_out())
-                    torch.cuda.synchronize()
-                    mn, vn = m.cpu().numpy(), v.cpu().numpy()
-                    if pattern == "SUM_WEIGHTED_ROWS":
-                        want = sums.sum_weighted_rows(mn, vn)
-                        scale = np.abs(mn.astype(np.float64)) @ np.abs(vn.astype(np.float64))
-                    else:
-                        want = sums.sum_weighted_cols(mn, vn)
-                        scale = np.abs(vn.astype(np.float64)) @ np.abs(mn.astype(np.float64))
-                    g = out.cpu().numpy()
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+def test_weighted(npp, cuda_device, dtype):
+    # sumWeightedRows / sumWeightedCols (Fig 15): AUTO runs the staged TMA family with v staged per
+    # tile (narrow and wide tiles, ragged edges), the literal / prior-work mappings the direct family
+    shapes = [(1000, 999), (4096, 4096), (37, 70000), (1001, 1024), (9, 3072), (70000, 36)]
+    for shape in shapes:
+        m = _make(dtype, shape, 7, cuda_device)
+        for pattern, vlen in (("SUM_WEIGHTED_ROWS", shape[1]), ("SUM_WEIGHTED_COLS", shape[0])):
+            v = _make(dtype, (vlen,), 8, cuda_device) if dtype != "f32" else \
+                gen.uniform_f32(8, (vlen,), device=cuda_device, lo=-1.0, scale=2.0)
+            mn, vn = m.cpu().numpy(), v.cpu().numpy()
+            if pattern == "SUM_WEIGHTED_ROWS":
+                want = sums.sum_weighted_rows(mn, vn)
+                scale = np.abs(mn.astype(np.float64)) @ np.abs(vn.astype(np.float64))
+            else:
+                want = sums.sum_weighted_cols(mn, vn)
+                scale = np.abs(vn.astype(np.float64)) @ np.abs(mn.astype(np.float64))
+            for strategy in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
+                p = npp.Plan(pattern, shape, dtype, strategy)
+                if strategy == "AUTO":
+                    assert p.mapping["staged"] == int(shape[1] % (16 // np.dtype(mn.dtype).itemsize) == 0)
+                out = p.execute([m, v], p.new_out())
+                out2 = p.execute([m, v], p.new_out(), overlap=True)  # PDL back to back, same workspace
+                torch.cuda.synchronize()
+                for o in (out, out2):
+                    g = o.cpu().numpy()
                     if dtype == "f32":
                         assert np.all(np.abs(g - want) <= 1e-5 * scale), (pattern, shape, strategy)
                     else:
-                        assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape)
+                        assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape, strategy)
+                if p.workspace is not None and p.mapping["temp"] == 0:  # S10 temp regions are scratch
+                    assert int(p.workspace.count_nonzero()) == 0
+
+
+@pytest.mark.parametrize("dtype", ["f32", "i32"])
+def test_weighted_temp_modes(npp, cuda_device, dtype):
+    # S10 (§V-A, Fig 16): the LITERAL weighted sums materialise their zipWith in a preallocated
+    # [outer x inner] buffer laid out for the mapping (Fig 11); the same mapping also runs with the
+    # row-major buffer ("prealloc w/o layout opt") and with a device malloc per outer iteration
+    for shape in [(1000, 999), (300, 4097), (4097, 300), (64, 65)]:
+        m = _make(dtype, shape, 17, cuda_device)
+        for pattern, vlen in (("SUM_WEIGHTED_ROWS", shape[1]), ("SUM_WEIGHTED_COLS", shape[0])):
+            v = _make(dtype, (vlen,), 18, cuda_device) if dtype != "f32" else \
+                gen.uniform_f32(18, (vlen,), device=cuda_device, lo=-1.0, scale=2.0)
+            mn, vn = m.cpu().numpy(), v.cpu().numpy()
+            rows = pattern == "SUM_WEIGHTED_ROWS"
+            want = sums.sum_weighted_rows(mn, vn) if rows else sums.sum_weighted_cols(mn, vn)
+            scale = (np.abs(mn.astype(np.float64)) @ np.abs(vn.astype(np.float64)) if rows
+                     else np.abs(vn.astype(np.float64)) @ np.abs(mn.astype(np.float64)))
+            lit = npp.Plan(pattern, shape, dtype, "LITERAL").mapping
+            M, N = (shape[0], shape[1]) if rows else (shape[1], shape[0])   # outer, inner sizes
+            outer_on_x = lit["levels"][0]["dim"] == 0
+            assert lit["temp"] == npp.TEMP_PREALLOC
+            assert lit["temp_stride"] == ([1, M] if outer_on_x else [N, 1])   # Fig 11b / 11a
+            variants = [("layout", dict(lit)), ("rowmajor", dict(lit, temp_stride=[N, 1])),
+                        ("malloc", dict(lit, temp=npp.TEMP_MALLOC, temp_stride=[0, 1]))]
+            for name, rec in variants:
+                p = npp.Plan(pattern, shape, dtype, mapping=rec)
+                out = p.execute([m, v], p.new_out())
+                torch.cuda.synchronize()
+                g = out.cpu().numpy()
+                if dtype == "f32":
+                    assert np.all(np.abs(g - want) <= 1e-5 * scale), (pattern, shape, name)
+                else:
+                    assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape, name)
+                ws = p.workspace
+                if name == "malloc":
+                    assert int(ws[-256:].count_nonzero()) == 0, "a device malloc returned NULL"
+                elif p.mapping["levels"][1]["grid"] == 1:
+                    # white box: the buffer holds t(o, i) = m·v at o*ts_o + i*ts_i (Fig 11)
+                    tdt = {"f32": torch.float32, "i32": torch.int32}[dtype]
+                    t = ws[:M * N * 4].view(tdt).cpu().numpy()
+                    so, si = rec["temp_stride"]
+                    for (o, i) in [(0, 0), (M - 1, N - 1), (M // 2, N // 3), (1 % M, 2 % N)]:
+                        r, c = (o, i) if rows else (i, o)
+                        if dtype == "f32":
+                            prod = np.float32(mn[r, c]) * np.float32(vn[i])
+                        else:
+                            prod = np.int32((int(mn[r, c]) * int(vn[i]) + (1 << 31)) % (1 << 32) - (1 << 31))
+                        assert t[o * so + i * si] == prod, (pattern, shape, name, o, i)

@@ -1,0 +1,58 @@
+"""One small invocation of every kernel family of libnpp.so, for compute-sanitizer
+(memcheck / racecheck / synccheck):
+
+    compute-sanitizer --tool memcheck --error-exitcode 1 python tools/sanitize_run.py
+
+Covers: staged sums (narrow/wide tiles, RX/MX, f32/i32/i64, ragged edges, pool + combiner, PDL
+overlap), weighted staged sums, the direct-load family under every strategy (Split(k) combine), the
+S10 temp family (PREALLOC layouts and MALLOC), k-means assignment, logreg gradient.
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from paper_conf_micro_leebsro14_b200 import npp  # noqa: E402
+from synth import gen  # noqa: E402
+
+
+def main():
+    dev = torch.device("cuda:0")
+    n = 0
+    for dtype in ("f32", "i32", "i64"):
+        for shape in [(300, 1024), (67, 520), (1000, 36), (5, 3)]:
+            m = (gen.uniform_f32(1, shape, device=dev) if dtype == "f32" else
+                 gen.int_uniform(2, shape, -50, 50, device=dev) if dtype == "i32" else
+                 gen.int64_wide(3, shape, device=dev))
+            for pattern in ("SUM_ROWS", "SUM_COLS"):
+                for strat in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
+                    p = npp.Plan(pattern, shape, dtype, strat)
+                    p.execute([m], p.new_out())
+                    p.execute([m], p.new_out(), overlap=True)
+                    n += 2
+            for pattern, vlen in (("SUM_WEIGHTED_ROWS", shape[1]), ("SUM_WEIGHTED_COLS", shape[0])):
+                v = m[0, :vlen].contiguous() if pattern == "SUM_WEIGHTED_ROWS" else m[:vlen, 0].contiguous()
+                for strat in ("AUTO", "LITERAL"):
+                    p = npp.Plan(pattern, shape, dtype, strat)
+                    p.execute([m, v], p.new_out())
+                    n += 1
+                if dtype != "i64":
+                    lit = npp.Plan(pattern, shape, dtype, "LITERAL").mapping
+                    M, N = (shape[0], shape[1]) if pattern == "SUM_WEIGHTED_ROWS" else (shape[1], shape[0])
+                    for rec in (dict(lit, temp_stride=[N, 1]), dict(lit, temp=npp.TEMP_MALLOC, temp_stride=[0, 1])):
+                        p = npp.Plan(pattern, shape, dtype, mapping=rec)
+                        p.execute([m, v], p.new_out())
+                        n += 1
+    x, c = gen.kmeans_inputs(5000, 64, 32, device=dev)
+    npp.Plan("KMEANS_ASSIGN", (5000, 64, 32)).execute([x, c], torch.empty(5000, dtype=torch.int32, device=dev))
+    x, c = gen.kmeans_inputs(700, 96, 40, device=dev)
+    npp.Plan("KMEANS_ASSIGN", (700, 96, 40)).execute([x, c], torch.empty(700, dtype=torch.int32, device=dev))
+    lx, ly, lw = gen.logreg_inputs(5, 100, 256, device=dev)
+    npp.Plan("LOGREG_GRAD", (5, 100, 256)).execute([lx, ly, lw], torch.empty(5, 256, device=dev))
+    torch.cuda.synchronize()
+    print(f"sanitize_run ok: {n + 3} executes")
+
+
+if __name__ == "__main__":
+    main()
