@@ -2,7 +2,7 @@
 """Benchmark of the nested-pattern hot path (BASELINE.json metric: achieved HBM GB/s for sumRows /
 sumCols per shape, 1/2/4/8 GPU).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload paper|sumcols_1m4k]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload paper|sumcols_1m4k|kmeans|logreg|rowscols]
                     [--strategy AUTO|LITERAL|1D|TB_T|WARP] [--impl reference] [--no-mappings]
 
 A step (workload `paper`, the default) = sumRows and sumCols, AUTO mapping, at the paper's three shapes
@@ -176,10 +176,23 @@ def build_logreg(npp, gen, torch, rank, world, strategy, device):
     return [item], [], "batched logistic-regression gradient [16M,256], B=4096"
 
 
+def build_rowscols(npp, gen, torch, rank, world, strategy, device):
+    # the Naive Bayes counts (§VI-E): row AND column sums of each paper-shape matrix from
+    # one pass (SUM_ROWS_COLS, S8 RC); rank r owns a row shard, the column sums are all-reduced
+    items, col_views = [], []
+    for si, (R, C) in enumerate(PAPER_SHAPES):
+        m = gen.uniform_f32(300 + 2 * si, (R, C), offset=rank * R * C, device=device)
+        plan = npp.Plan("SUM_ROWS_COLS", (R, C), "f32", "AUTO", device=device)
+        out = plan.new_out()
+        col_views.append(out[R:])
+        items.append(Item(f"sum_rows_cols{_fmt_shape((R, C))}", plan, [m], out, R * C * 4 + (R + C) * 4))
+    return items, (col_views if world > 1 else []), "sumRows and sumCols in one pass (Naive Bayes counts)"
+
+
 # per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
-SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong"}
+SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
-             "logreg": build_logreg}
+             "logreg": build_logreg, "rowscols": build_rowscols}
 
 
 # ------------------------------------------------------------------------- reference arm (the oracle)
@@ -229,6 +242,8 @@ def config_for(args, extra):
           "sumcols_1m4k": "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])",
           "kmeans": "k-means assignment 4M x 64 x 32 fp32, points sharded (BASELINE.json configs[3])",
           "logreg": "batched logreg gradient [16M,256] fp32, B=4096, batches sharded (BASELINE.json configs[4])",
+          "rowscols": "sumRows+sumCols in ONE pass (SUM_ROWS_COLS) fp32 @ [64K,1K],[8K,8K],[1K,64K] "
+                      "(Naive Bayes counts, SURVEY §8f NEXT 2)",
           }[args.workload]
     return {"workload": wl, "strategy": args.strategy, "impl_detail": extra,
             "parallelism": f"row shards x{args.gpus}",
@@ -261,6 +276,8 @@ def cpu_baseline(items, budget_s=12.0):
             okm.assign(*arrs)
         elif name.startswith("logreg"):
             olr.grad(arrs[0], arrs[1], arrs[2], 64)
+        elif name.startswith("sum_rows_cols"):
+            sums.sum_rows_cols(arrs[0])
         else:
             (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(arrs[0])
     t_end = time.perf_counter() + budget_s
@@ -397,6 +414,7 @@ def main():
     out["e2e"] = None if args.no_e2e else e2e_host(items, torch, stream, world, dist)
     if rank == 0 and not args.no_mappings and args.workload == "paper":
         out["mappings"] = mapping_table(npp, torch, gen, device, stream, items)
+        out["fused_rows_cols"] = fused_table(npp, torch, device, stream, items, per_shape)
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(items)
     if rank == 0:
@@ -476,6 +494,24 @@ def kernel_us(torch, item, other, stream, reps=8, overlap=False):
         b.record(stream)
     torch.cuda.synchronize()
     return a.elapsed_time(b) * 1e3 / (2 * reps)
+
+
+def fused_table(npp, torch, device, stream, items, per_shape):
+    """Both sums of one matrix: the one-pass SUM_ROWS_COLS launch vs the sumRows + sumCols launches
+    (graph-timed, L2-cold like per_shape). GB/s counts the one algorithmic read + both outputs."""
+    table = {}
+    flat = [it.ins[0] for it in items]
+    for R, C in PAPER_SHAPES:
+        m = next(x for x in flat if tuple(x.shape) == (R, C))
+        other = next(x for x in flat if x.data_ptr() != m.data_ptr() and x.numel() == m.numel())
+        p = npp.Plan("SUM_ROWS_COLS", (R, C), "f32", "AUTO", device=device)
+        item = Item("rc", p, [m], p.new_out(), R * C * 4 + (R + C) * 4)
+        us = kernel_us(torch, item, Item("o", p, [other], None, 0), stream)
+        two = per_shape[f"sum_rows{_fmt_shape((R, C))}"]["us"] + per_shape[f"sum_cols{_fmt_shape((R, C))}"]["us"]
+        table[f"sum_rows_cols{_fmt_shape((R, C))}"] = {
+            "GB/s": round(item.bytes / (us * 1e-6) / 1e9, 1), "us": round(us, 2), "two_pass_us": round(two, 2),
+            "speedup_vs_two_pass": round(two / us, 3), "mapping": mapping_brief(p.mapping)}
+    return table
 
 
 def mapping_table(npp, torch, gen, device, stream, items):

@@ -58,14 +58,19 @@ typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2 } npp_dtype;
  *   LOGREG_GRAD        {B,Rb,C} ins={x[B*Rb*C] f32, y[B*Rb] f32, w[C] f32}
  *                                                            out[B*C] f32 = Σ_{i in batch b} x_ij(σ(x_i·w)-y_i)
  *   SUM_WEIGHTED_ROWS  {R,C}   ins={m[R*C], v[C]}            out[R]  = Σ_c m[r,c]·v[c]
- *   SUM_WEIGHTED_COLS  {R,C}   ins={m[R*C], v[R]}            out[C]  = Σ_r m[r,c]·v[r]          */
+ *   SUM_WEIGHTED_COLS  {R,C}   ins={m[R*C], v[R]}            out[C]  = Σ_r m[r,c]·v[r]
+ *   SUM_ROWS_COLS      {R,C}   ins={m[R*C]}                  out[R+C] = [Σ_c m[r,c] (r<R) | Σ_r m[r,c] (c<C)]
+ *                      both outputs of the Naive Bayes counts (§VI-E) from ONE read of m;
+ *                      executable with strategy AUTO (npp_select/npp_enumerate give every strategy's
+ *                      record for analysis; the paper's two-kernel schedule = a SUM_ROWS and a SUM_COLS plan) */
 typedef enum {
   NPP_SUM_ROWS = 0,
   NPP_SUM_COLS = 1,
   NPP_KMEANS_ASSIGN = 2,
   NPP_LOGREG_GRAD = 3,
   NPP_SUM_WEIGHTED_ROWS = 4,
-  NPP_SUM_WEIGHTED_COLS = 5
+  NPP_SUM_WEIGHTED_COLS = 5,
+  NPP_SUM_ROWS_COLS = 6
 } npp_pattern;
 
 /* AUTO     = Algorithm 1 + ControlDOP + the runtime step R2 (L810-817; S8)
@@ -93,7 +98,8 @@ typedef enum {
   NPP_CLASS_MX = 1,      /* outer Map on x, inner Reduce on y (sumCols family; 1D)        */
   NPP_CLASS_KMEANS = 2,  /* 3-level: Map points / argmin centroids / Reduce dims          */
   NPP_CLASS_LOGREG = 3,  /* 3-level: Map batches / Reduce rows / Map+Reduce columns       */
-  NPP_CLASS_EMPTY = 4    /* a zero-sized level: output zero-filled (or nothing to do)     */
+  NPP_CLASS_EMPTY = 4,   /* a zero-sized level: output zero-filled (or nothing to do)     */
+  NPP_CLASS_RC = 5       /* 2-level, both levels Reduce: row and column sums in one pass  */
 } npp_kernel_class;
 
 /* One nest level of a mapping (§IV-A). dim: npp_dim; span: npp_span; factor: n of Span(n) or k of

@@ -22,7 +22,7 @@ X, Y, Z = 0, 1, 2
 # span codes (S9 / record)
 ONE, ALL, SPAN_N, SPLIT = 0, 1, 2, 3
 # kernel classes (S9)
-RX, MX, KM, LR = 0, 1, 2, 3
+RX, MX, KM, LR, EMPTY, RC = 0, 1, 2, 3, 4, 5
 
 SIZE_SET = [1 << i for i in range(11)]          # {1,2,4,...,1024}  Alg 1
 W_C, W_B = 8, 1                                  # DESIGN.md G3
@@ -32,7 +32,7 @@ T_BLOCK, U_MIN = 256, 8                          # DESIGN.md S8
 MAX_GRID = (1 << 31) - 1                         # DESIGN.md S3 H6
 
 PATTERNS = ("SUM_ROWS", "SUM_COLS", "KMEANS_ASSIGN", "LOGREG_GRAD",
-            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS")
+            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS")
 DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8}
 
 B200 = dict(sm_count=148, max_threads_per_sm=2048, max_threads_per_block=1024,
@@ -88,6 +88,10 @@ def build_nest(pattern: str, shape) -> dict:
         acc = [(0, (0,)), (0, (0, 1))]              # out[c], m[r,c] (stride-1 index is c = L0)
         if pattern == "SUM_WEIGHTED_COLS":
             acc.append((1, (0, 1)))                 # v[r]
+    elif pattern == "SUM_ROWS_COLS":                 # Naive Bayes counts, §VI-E
+        R, C = shape
+        levels = [(R, True), (C, True)]             # rows Reduce (column sums), cols Reduce (row sums)
+        acc = [(0, (0,)), (1, (1,)), (1, (0, 1))]   # out_rows[r], out_cols[c], m[r,c]
     elif pattern == "KMEANS_ASSIGN":
         N, D, K = shape
         levels = [(N, False), (K, True), (D, True)]
@@ -353,6 +357,51 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
+RC_COL_TILES_MAX = 32                             # DESIGN.md S8 RC: column tiles of one region
+
+
+def rc_tiling(R, C, dtype, lim):
+    """DESIGN.md S8 RC region rule. The ceil(R/32) x ceil(C/BC) tile grid is cut into regions of cr row
+    bands x cc column tiles (cc <= 32). Written as the plain double loop over gc and gr:
+    for gc in [ceil(Tc/32), max(that, min(Tc, S))], gr in [1, min(Tr, S // gc')], with cc = ceil(Tc/gc),
+    gc' = ceil(Tc/cc), cr = ceil(Tr/gr), gr' = ceil(Tr/cr), nreg = gr'*gc', G = min(S, nreg):
+    minimise (ceil(nreg/G)*cr*cc, nreg, gc'), the first minimum winning.
+    Returns dict(BC, Tr, Tc, cr, cc, gr, gc, nreg, G)."""
+    S = lim["sm_count"]
+    BC = 1024 // DTYPE_SIZE[dtype]
+    Tr, Tc = cdiv(R, STAGE_ROWS), cdiv(C, BC)
+    gc_lo = cdiv(Tc, RC_COL_TILES_MAX)
+    best, best_key = None, None
+    for gc in range(gc_lo, max(gc_lo, min(Tc, S)) + 1):
+        cc = cdiv(Tc, gc)
+        gce = cdiv(Tc, cc)
+        for gr in range(1, min(Tr, max(1, S // gce)) + 1):
+            cr = cdiv(Tr, gr)
+            gre = cdiv(Tr, cr)
+            nreg = gre * gce
+            G = min(S, nreg)
+            key = (cdiv(nreg, G) * cr * cc, nreg, gce)
+            if best_key is None or key < best_key:
+                best_key = key
+                best = dict(BC=BC, Tr=Tr, Tc=Tc, cr=cr, cc=cc, gr=gre, gc=gce, nreg=nreg, G=G)
+    return best
+
+
+def r2_rowscols(nest, dtype, lim):
+    """DESIGN.md S8 RC: columns on x, one thread per column of a 1 KB tile (256/BC row halves), the
+    regions of rc_tiling as Split levels. Returns (dims, blocks, spans, factors, vec, chunks, staged, G,
+    claim)."""
+    (R, _), (C, _) = nest["levels"]
+    t = rc_tiling(R, C, dtype, lim)
+    dims = (Y, X)
+    blocks = (256 // t["BC"], t["BC"])
+    spans = (SPLIT if t["gr"] > 1 else ALL, SPLIT if t["gc"] > 1 else ALL)
+    factors = (t["gr"], t["gc"])
+    chunks = (STAGE_ROWS * t["cr"] if t["gr"] > 1 else R, t["BC"] * t["cc"] if t["gc"] > 1 else C)
+    staged = 1 if C % (16 // DTYPE_SIZE[dtype]) == 0 else 0
+    return dims, blocks, spans, factors, 1, chunks, staged, t["G"], t["cr"] * t["cc"]
+
+
 def r2_logreg(nest, lim, dims):
     """DESIGN.md S8, LOGREG_GRAD staged: 32-row tiles of one batch, contiguous tile ranges."""
     (B, _), (Rb, _), (C, _) = nest["levels"]
@@ -436,6 +485,8 @@ def kernel_class(pattern, dims):
         return KM
     if pattern == "LOGREG_GRAD":
         return LR
+    if pattern == "SUM_ROWS_COLS":
+        return RC
     return RX if dims[1] == X else MX
 
 
@@ -486,6 +537,13 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
+    if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:
+        # S9 RC: tickets [Tr] + tickets [gc] (u32), accumulators [R] + [C] of the accumulator type
+        R, C = nest["levels"][0][0], nest["levels"][1][0]
+        t = rc_tiling(R, C, dtype, lim)
+        ab = acc_bytes(nest["pattern"], dtype)
+        rec["workspace_bytes"] = (256 * cdiv(4 * t["Tr"], 256) + 256 * cdiv(4 * t["gc"], 256)
+                                  + 256 * cdiv(R * ab, 256) + 256 * cdiv(C * ab, 256))
     if temp[0] == TEMP_PREALLOC:   # S10: the [outer x inner] buffer after partials and tickets
         M, N = _eff(nest["levels"][0][0]), _eff(nest["levels"][1][0])
         rec["workspace_bytes"] += 256 * cdiv(M * N * DTYPE_SIZE[dtype], 256)
@@ -541,6 +599,10 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
         b3, s3, f3, vec, chunks, G, P = r2_kmeans(nest, lim)
         return make_record(nest, dtype, lim, dims, b3, s3, f3, vec, sc, chunks, staged=1,
                            persistent_grid=G, claim_tiles=P)
+    if pattern == "SUM_ROWS_COLS":
+        d2, b2, s2, f2, vec, chunks, staged, G, CL = r2_rowscols(nest, dtype, lim)
+        return make_record(nest, dtype, lim, d2, b2, s2, f2, vec, sc, chunks, staged=staged,
+                           persistent_grid=G, claim_tiles=CL)
     if staged_eligible(nest, dtype, dims):
         b2, s2, f2, vec, chunks, G, CL = r2_staged(nest, dtype, lim)
         return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks, staged=1,

@@ -7,6 +7,9 @@ Definitions (plain, no blocking or reordering beyond the definition):
                                               PAPER.md §IV-A, Fig 6c; G12
   sumWeightedRows/Cols: the inner pattern is zipWith(v)(*) then reduce(+)
                                               PAPER.md Fig 15; G9
+  sumRowsCols: both counts of the Naive Bayes classifier ("the number of words per document and the
+  number of documents for each ... word") over one matrix, out = [sumRows | sumCols]
+                                              PAPER.md §VI-E; S8 RC
 Floating point: fp64 (``math.fsum`` = the correctly rounded exact sum in the literal evaluator).
 Integers: exact Python / unsigned NumPy arithmetic, wrapped to the element width (G19).
 """
@@ -111,6 +114,15 @@ def sum_cols(m: np.ndarray) -> np.ndarray:
     if acc is None:
         acc = _acc_reduce(m, axis=0)
     return _finish(acc, m)
+
+
+def sum_rows_cols(m: np.ndarray) -> np.ndarray:
+    """[sumRows(m) | sumCols(m)] — the two Naive Bayes counts (§VI-E), concatenated."""
+    return np.concatenate([sum_rows(m), sum_cols(m)])
+
+
+def sum_rows_cols_literal(m: np.ndarray) -> list:
+    return sum_rows_literal(m) + sum_cols_literal(m)
 
 
 def sum_weighted_rows(m: np.ndarray, v: np.ndarray) -> np.ndarray:

@@ -43,7 +43,8 @@ int cuda_fail(const char* what, cudaError_t e) {
 int n_inputs(int pattern) {
   switch (pattern) {
     case NPP_SUM_ROWS:
-    case NPP_SUM_COLS: return 1;
+    case NPP_SUM_COLS:
+    case NPP_SUM_ROWS_COLS: return 1;
     case NPP_SUM_WEIGHTED_ROWS:
     case NPP_SUM_WEIGHTED_COLS:
     case NPP_KMEANS_ASSIGN: return 2;
@@ -58,7 +59,8 @@ int64_t input_bytes(const npp_plan_s* p, int k) {
   const int64_t* s = p->shape;
   switch (p->pattern) {
     case NPP_SUM_ROWS:
-    case NPP_SUM_COLS: return s[0] * s[1] * es;
+    case NPP_SUM_COLS:
+    case NPP_SUM_ROWS_COLS: return s[0] * s[1] * es;
     case NPP_SUM_WEIGHTED_ROWS: return k == 0 ? s[0] * s[1] * es : s[1] * es;
     case NPP_SUM_WEIGHTED_COLS: return k == 0 ? s[0] * s[1] * es : s[0] * es;
     case NPP_KMEANS_ASSIGN: return k == 0 ? s[0] * s[1] * 4 : s[2] * s[1] * 4;
@@ -75,6 +77,7 @@ int64_t output_bytes(const npp_plan_s* p) {
     case NPP_SUM_WEIGHTED_ROWS: return s[0] * es;
     case NPP_SUM_COLS:
     case NPP_SUM_WEIGHTED_COLS: return s[1] * es;
+    case NPP_SUM_ROWS_COLS: return (s[0] + s[1]) * es;
     case NPP_KMEANS_ASSIGN: return s[0] * 4;
     case NPP_LOGREG_GRAD: return s[0] * s[2] * 4;
     default: return 0;
@@ -221,6 +224,12 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
   if ((p->map.kernel_class == NPP_CLASS_KMEANS || p->map.kernel_class == NPP_CLASS_LOGREG) && !p->map.staged) {
     delete p;
     set_error("3-level nests execute through their staged (AUTO) kernel families only");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  if (pattern == NPP_SUM_ROWS_COLS && strategy != NPP_MAP_AUTO) {
+    delete p;
+    set_error("SUM_ROWS_COLS executes with strategy AUTO only (the one-pass family); the paper's two-kernel "
+              "schedule is a SUM_ROWS plan plus a SUM_COLS plan");
     return NPP_ERR_UNSUPPORTED;
   }
   *out = p;
@@ -430,6 +439,28 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     k.per_block = m.claim_tiles;
     cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);
+    return NPP_OK;
+  }
+  if (plan->pattern == NPP_SUM_ROWS_COLS) {  // class RC (S8 RC): one pass, both outputs
+    const npp::RcTiling t = npp::rc_tiling(plan->shape[0], plan->shape[1], plan->dtype, plan->lim.sm_count);
+    const int64_t ab = plan->dtype == NPP_I32 ? 4 : 8;
+    char* ws = static_cast<char*>(workspace);
+    npp::RowsColsArgs r{};
+    r.m = ins[0];
+    r.out = out;
+    r.R = plan->shape[0];
+    r.C = plan->shape[1];
+    r.Tr = t.Tr, r.Tc = t.Tc, r.cr = t.cr, r.cc = t.cc, r.gr = t.gr, r.gc = t.gc, r.nreg = t.nreg;
+    const int64_t o_tc = ((4 * t.Tr + 255) / 256) * 256;
+    const int64_t o_ar = o_tc + ((4 * t.gc + 255) / 256) * 256;
+    const int64_t o_ac = o_ar + ((r.R * ab + 255) / 256) * 256;
+    r.tick_r = reinterpret_cast<unsigned*>(ws);
+    r.tick_c = reinterpret_cast<unsigned*>(ws + o_tc);
+    r.accR = ws + o_ar;
+    r.accC = ws + o_ac;
+    r.early_reads = overlap ? 1 : 0;
+    cudaError_t e = npp::launch_rowscols(plan->dtype, m.staged != 0, r, int(m.grid), st);
+    if (e != cudaSuccess) return cuda_fail("rows+cols kernel launch", e);
     return NPP_OK;
   }
   if (!npp::is_sum_pattern(plan->pattern)) {

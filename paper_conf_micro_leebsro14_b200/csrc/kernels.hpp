@@ -95,4 +95,23 @@ struct KmeansArgs {
 };
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st);
 
+// sumRows + sumCols of one matrix in one pass (class RC, S8 RC): the ceil(R/32) x ceil(C/BC)
+// tile grid is cut into regions of cr row bands x cc column tiles, gr x gc of them in row-region-major
+// order; block b of G takes regions [b*nreg/G, (b+1)*nreg/G). out = [R row sums | C column sums].
+struct RowsColsArgs {
+  const void* m;       // [R x C]
+  void* out;           // [R + C]
+  void* accR;          // [R] accumulators (fp64 / u32 / u64) of row bands cut by column regions
+  void* accC;          // [C] accumulators of columns cut by row regions
+  unsigned* tick_r;    // [Tr] column regions done per row band (zero on entry and on exit)
+  unsigned* tick_c;    // [gc] row regions done per column group (zero on entry and on exit)
+  int64_t R, C;
+  int64_t Tr, Tc;      // 32-row bands, BC-column tiles
+  int64_t cr, cc;      // bands / column tiles per region
+  int64_t gr, gc;      // regions along rows / columns
+  int64_t nreg;        // gr * gc
+  int early_reads;     // NPP_EXEC_OVERLAP
+};
+cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int grid, cudaStream_t st);
+
 }  // namespace npp

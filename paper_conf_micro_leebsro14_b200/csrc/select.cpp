@@ -342,9 +342,27 @@ void r2_sums(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   c->factors[1] = k;
 }
 
+// S8 RC: both outputs from one pass; columns on x (the stride-1 level of m and of the column output),
+// one thread per column of a 1 KB tile (two row halves for 8-byte types), regions from rc_tiling.
+void r2_rowscols(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
+  const int64_t R = n.N[0], C = n.N[1];
+  const RcTiling t = rc_tiling(R, C, dtype, lim.sm_count);
+  c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
+  c->blocks[0] = int(256 / t.BC), c->blocks[1] = int(t.BC);
+  c->spans[0] = t.gr > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[0] = t.gr;
+  c->chunks[0] = t.gr > 1 ? kStageRows * t.cr : R;
+  c->spans[1] = t.gc > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[1] = t.gc;
+  c->chunks[1] = t.gc > 1 ? t.BC * t.cc : C;
+  c->vec = 1;
+  c->staged = C % (16 / dtype_size(dtype)) == 0 ? 1 : 0;  // TMA needs a 16-B row pitch
+  c->persistent_grid = t.G;
+  c->claim_tiles = t.cr * t.cc;
+}
+
 int kernel_class_of(const Nest& n, const Choice& c) {
   if (n.pattern == NPP_KMEANS_ASSIGN) return NPP_CLASS_KMEANS;
   if (n.pattern == NPP_LOGREG_GRAD) return NPP_CLASS_LOGREG;
+  if (n.pattern == NPP_SUM_ROWS_COLS) return NPP_CLASS_RC;
   return c.dims[1] == NPP_DIM_X ? NPP_CLASS_RX : NPP_CLASS_MX;
 }
 
@@ -394,6 +412,34 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   return t;
 }
 
+// S8 RC region rule: over gc in [ceil(Tc/32), max(that, min(Tc, S))] and gr in [1, min(Tr, S/gc')]
+// (gc', gr' the region counts after rounding the region sizes cc = ceil(Tc/gc), cr = ceil(Tr/gr)),
+// minimise (ceil(nreg/G) * cr * cc = tiles of the busiest block, nreg, gc'); first minimum wins.
+RcTiling rc_tiling(int64_t R, int64_t C, int dtype, int sm_count) {
+  RcTiling best{};
+  const int64_t S = sm_count;
+  best.BC = 1024 / dtype_size(dtype);
+  best.Tr = cdiv(R, kStageRows);
+  best.Tc = cdiv(C, best.BC);
+  const int64_t gc_lo = cdiv(best.Tc, kRcColTilesMax);
+  const int64_t gc_hi = std::max(gc_lo, std::min(best.Tc, S));
+  int64_t kc = -1, kn = 0, kg = 0;
+  for (int64_t gc = gc_lo; gc <= gc_hi; ++gc) {
+    const int64_t cc = cdiv(best.Tc, gc), gce = cdiv(best.Tc, cc);
+    const int64_t gr_hi = std::min(best.Tr, std::max<int64_t>(1, S / gce));
+    for (int64_t gr = 1; gr <= gr_hi; ++gr) {
+      const int64_t cr = cdiv(best.Tr, gr), gre = cdiv(best.Tr, cr);
+      const int64_t nreg = gre * gce, G = std::min(S, nreg);
+      const int64_t cost = cdiv(nreg, G) * cr * cc;
+      if (kc < 0 || cost < kc || (cost == kc && (nreg < kn || (nreg == kn && gce < kg)))) {
+        kc = cost, kn = nreg, kg = gce;
+        best.cr = cr, best.cc = cc, best.gr = gre, best.gc = gce, best.nreg = nreg, best.G = G;
+      }
+    }
+  }
+  return best;
+}
+
 int dtype_size(int dtype) { return dtype == NPP_I64 ? 8 : 4; }
 
 bool is_rows_pattern(int p) { return p == NPP_SUM_ROWS || p == NPP_SUM_WEIGHTED_ROWS; }
@@ -440,6 +486,16 @@ int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
       n.acc[n.nacc++] = {0, 0x1u};           // out[c]
       n.acc[n.nacc++] = {0, 0x3u};           // m[r,c]: stride-1 index is c, i.e. level 0
       if (pattern == NPP_SUM_WEIGHTED_COLS) n.acc[n.nacc++] = {1, 0x3u};  // v[r]
+      n.cols = shape[1];
+      break;
+    case NPP_SUM_ROWS_COLS:  // both levels Reduce: rows for the column sums, columns for the row sums
+      if (!need(2)) return NPP_ERR_INVALID_ARG;
+      n.L = 2;
+      n.N[0] = shape[0], n.sync[0] = true;
+      n.N[1] = shape[1], n.sync[1] = true;
+      n.acc[n.nacc++] = {0, 0x1u};  // out_rows[r]
+      n.acc[n.nacc++] = {1, 0x2u};  // out_cols[c]
+      n.acc[n.nacc++] = {1, 0x3u};  // m[r,c]
       n.cols = shape[1];
       break;
     case NPP_KMEANS_ASSIGN:  // shape {N, D, K}; levels N / K / D
@@ -544,7 +600,6 @@ int64_t score(const Nest& n, const npp_limits& lim, const Choice& c) {
 
 int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c, int64_t score_value,
                        npp_mapping* out) {
-  (void)lim;
   npp_mapping m{};
   m.nlevels = n.L;
   m.kernel_class = kernel_class_of(n, c);
@@ -578,6 +633,12 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.temp_stride[1] = c.temp_stride[1];
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
+  } else if (n.pattern == NPP_SUM_ROWS_COLS && c.persistent_grid > 0) {
+    // S9 RC: tickets [Tr] + tickets [gc] (u32) + accumulators [R] + [C] of the accumulator type
+    const RcTiling t = rc_tiling(n.N[0], n.N[1], dtype, lim.sm_count);
+    const int64_t ab = acc_bytes(n.pattern, dtype);
+    m.workspace_bytes = 256 * cdiv(4 * t.Tr, 256) + 256 * cdiv(4 * t.gc, 256) + 256 * cdiv(n.N[0] * ab, 256) +
+                        256 * cdiv(n.N[1] * ab, 256);
   } else if (is_sum_pattern(n.pattern) && c.staged) {
     // pool counters (256 B) + tickets [To] + accumulators [O] of the accumulator type
     const StagedTiling t = staged_tiling(n.pattern, is_rows_pattern(n.pattern) ? n.N[0] : n.N[1], n.cols, dtype);
@@ -667,6 +728,10 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
       set_error("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128 and K <= 256");
       return NPP_ERR_UNSUPPORTED;
     }
+    return record_from_choice(n, dtype, lim, c, sc, out);
+  }
+  if (n.pattern == NPP_SUM_ROWS_COLS) {
+    r2_rowscols(n, dtype, lim, &c);
     return record_from_choice(n, dtype, lim, c, sc, out);
   }
   if (staged_eligible(n, dtype, c))

@@ -19,10 +19,10 @@ OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_ALIGNMENT, ERR_WORKSPACE, ERR_NO_FEASI
 DTYPES = {"f32": 0, "i32": 1, "i64": 2}
 TORCH_DTYPES = {"f32": torch.float32, "i32": torch.int32, "i64": torch.int64}
 PATTERNS = {"SUM_ROWS": 0, "SUM_COLS": 1, "KMEANS_ASSIGN": 2, "LOGREG_GRAD": 3,
-            "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5}
+            "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5, "SUM_ROWS_COLS": 6}
 STRATEGIES = {"AUTO": 0, "LITERAL": 1, "1D": 2, "TB_T": 3, "WARP": 4}
 SPAN_ONE, SPAN_ALL, SPAN_N, SPLIT_K = 0, 1, 2, 3
-CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY = 0, 1, 2, 3, 4
+CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY, CLASS_RC = 0, 1, 2, 3, 4, 5
 
 
 class NppError(RuntimeError):
@@ -236,6 +236,8 @@ class Plan:
             return (s[0],)
         if p in ("SUM_COLS", "SUM_WEIGHTED_COLS"):
             return (s[1],)
+        if p == "SUM_ROWS_COLS":
+            return (s[0] + s[1],)
         if p == "KMEANS_ASSIGN":
             return (s[0],)
         return (s[0], s[2])
@@ -301,6 +303,15 @@ def sum_cols(m: torch.Tensor, strategy: str = "AUTO", out=None, stream=None) -> 
     """m mapCols { c => c reduce + } (Fig 1)."""
     p = _cached_plan("SUM_COLS", m.shape, _dtype_name(m), strategy, m.device)
     return p.execute([m], out if out is not None else p.new_out(), stream)
+
+
+def sum_rows_cols(m: torch.Tensor, out=None, stream=None):
+    """Both Naive Bayes counts (§VI-E) in one pass over m: returns (row sums, column
+    sums), views of one [R + C] output (SUM_ROWS_COLS, strategy AUTO)."""
+    R = m.shape[0]
+    p = _cached_plan("SUM_ROWS_COLS", m.shape, _dtype_name(m), "AUTO", m.device)
+    o = p.execute([m], out if out is not None else p.new_out(), stream)
+    return o[:R], o[R:]
 
 
 def sum_weighted_rows(m, v, strategy="AUTO", out=None, stream=None):

@@ -227,6 +227,18 @@ def test_streams_and_concurrent_plans(npp, cuda_device):
         check("SUM_COLS", m, out, "f32")
 
 
+def _counters(p):
+    """The part of a plan's workspace every execute must leave zero (S9): all of a staged
+    plan's (pool counters, tickets, accumulators); the tickets of a direct-load Split plan (its
+    partials [G_1 x O] are written before they are read and keep their values)."""
+    ws, m = p.workspace, p.mapping
+    if m["staged"]:
+        return ws
+    acc = 4 if p.dtype == "i32" else 8
+    part = -(-m["levels"][1]["grid"] * p.out_shape()[0] * acc // 256) * 256
+    return ws[part:part + -(-4 * m["levels"][0]["grid"] // 256) * 256]
+
+
 @pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
 def test_weighted(npp, cuda_device, dtype):
     # sumWeightedRows / sumWeightedCols (Fig 15): AUTO runs the staged TMA family with v staged per
@@ -258,7 +270,7 @@ def test_weighted(npp, cuda_device, dtype):
                     else:
                         assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape, strategy)
                 if p.workspace is not None and p.mapping["temp"] == 0:  # S10 temp regions are scratch
-                    assert int(p.workspace.count_nonzero()) == 0
+                    assert int(_counters(p).count_nonzero()) == 0
 
 
 @pytest.mark.parametrize("dtype", ["f32", "i32"])
@@ -307,3 +319,77 @@ def test_weighted_temp_modes(npp, cuda_device, dtype):
                         else:
                             prod = np.int32((int(mn[r, c]) * int(vn[i]) + (1 << 31)) % (1 << 32) - (1 << 31))
                         assert t[o * so + i * si] == prod, (pattern, shape, name, o, i)
+
+
+RC_SHAPES = [(1, 1), (3, 5), (31, 33), (33, 31), (1000, 999), (1024, 1024), (4097, 300), (300, 4097),
+             (7, 70000), (70000, 7), (2, 1 << 17), (1001, 1024), (9, 3072), (5000, 8192), (100000, 36)]
+
+
+def _check_rc(m, got, dtype):
+    """SUM_ROWS_COLS output = [sumRows | sumCols] (S8 RC), each half to the sums' bar."""
+    R = m.shape[0]
+    check("SUM_ROWS", m, got[:R], dtype)
+    check("SUM_COLS", m, got[R:], dtype)
+
+
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+def test_rows_cols_parity(npp, cuda_device, dtype):
+    # one pass, both outputs: staged (16-B row pitch) and direct (ragged pitch) variants, regions cut
+    # along rows only, columns only and both (tickets), ragged edge tiles; back-to-back executes
+    # (plain and PDL-overlapped) on one workspace leave it zero
+    lim = npp.limits_query(0)
+    for i, shape in enumerate(RC_SHAPES):
+        m = _make(dtype, shape, 300 + i, cuda_device)
+        p = npp.Plan("SUM_ROWS_COLS", shape, dtype, "AUTO")
+        assert p.mapping == osel.select("SUM_ROWS_COLS", shape, dtype, lim, "AUTO")
+        assert p.mapping["kernel_class"] == npp.CLASS_RC
+        assert p.mapping["staged"] == int(shape[1] % (16 // np.dtype(m.cpu().numpy().dtype).itemsize) == 0)
+        outs = [p.execute([m], p.new_out()), p.execute([m], p.new_out(), overlap=True),
+                p.execute([m], p.new_out())]
+        torch.cuda.synchronize()
+        for o in outs:
+            _check_rc(m, o, dtype)
+        assert int(p.workspace.count_nonzero()) == 0, shape
+
+
+def test_rows_cols_exact_and_wrap(npp, cuda_device):
+    # exact-summable fp32 makes both halves bit-exact; int32 arange wraps mod 2^32 in both directions
+    for shape in [(1024, 1024), (65536, 64), (64, 65536)]:
+        m = gen.exact_f32(11, shape, device=cuda_device)
+        o = npp.Plan("SUM_ROWS_COLS", shape, "f32").execute([m], torch.empty(sum(shape), device=cuda_device))
+        torch.cuda.synchronize()
+        assert np.array_equal(o.cpu().numpy().astype(np.float64), sums.sum_rows_cols(m.cpu().numpy())), shape
+    shape = (3000, 2500)
+    m = gen.arange_matrix(shape, torch.int32, offset=(1 << 31) - 10 ** 6, device=cuda_device)
+    o = npp.Plan("SUM_ROWS_COLS", shape, "i32").execute(
+        [m], torch.empty(sum(shape), dtype=torch.int32, device=cuda_device))
+    torch.cuda.synchronize()
+    _check_rc(m, o, "i32")
+
+
+@pytest.mark.parametrize("shape", [(65536, 1024), (8192, 8192), (1024, 65536)])
+def test_rows_cols_paper_shapes(npp, cuda_device, shape):
+    m = gen.uniform_f32(3, shape, device=cuda_device)
+    rows, cols = npp.sum_rows_cols(m)
+    torch.cuda.synchronize()
+    check("SUM_ROWS", m, rows, "f32")
+    check("SUM_COLS", m, cols, "f32")
+    # the fused pass agrees with the two single-pattern plans
+    r2, c2 = npp.sum_rows(m), npp.sum_cols(m)
+    torch.cuda.synchronize()
+    assert torch.all((rows - r2).abs() <= r2.abs() * 2.0 ** -22)
+    assert torch.all((cols - c2).abs() <= c2.abs() * 2.0 ** -22)
+
+
+def test_rows_cols_plan_rules(npp, cuda_device):
+    # the one-pass family is AUTO only; the empty nest zero-fills both halves
+    for strategy in ("LITERAL", "1D", "TB_T", "WARP"):
+        with pytest.raises(npp.NppError) as e:
+            npp.Plan("SUM_ROWS_COLS", (64, 64), "f32", strategy)
+        assert e.value.status == npp.ERR_UNSUPPORTED
+    for shape in [(0, 5), (7, 0)]:
+        p = npp.Plan("SUM_ROWS_COLS", shape, "i32")
+        o = p.execute([torch.empty(shape, dtype=torch.int32, device=cuda_device)],
+                      torch.full((sum(shape),), 7, dtype=torch.int32, device=cuda_device))
+        torch.cuda.synchronize()
+        assert int(o.abs().sum()) == 0

@@ -137,3 +137,18 @@ def test_weighted_closed_forms():
     assert sums.sum_weighted_rows(mi, vi).tolist() == sums.sum_weighted_rows_literal(mi, vi)
     vri = gen.int_uniform(10, (R,), -9, 9).numpy()
     assert sums.sum_weighted_cols(mi, vri).tolist() == sums.sum_weighted_cols_literal(mi, vri)
+
+
+@pytest.mark.parametrize("R,C", [(1, 1), (3, 5), (33, 31), (100, 64)])
+def test_rows_cols_closed_forms(R, C):
+    # sumRowsCols (Naive Bayes counts, §VI-E) = [sumRows | sumCols]: ones give C per row and
+    # R per column; arange m[r,c] = r*C + c gives r*C^2 + C(C-1)/2 and C*R(R-1)/2 + R*c; both halves
+    # total RC(RC-1)/2; the literal nested loops agree
+    ones = np.ones((R, C), dtype=np.int32)
+    assert sums.sum_rows_cols(ones).tolist() == [C] * R + [R] * C
+    a = np.arange(R * C, dtype=np.int64).reshape(R, C)
+    want = [r * C * C + C * (C - 1) // 2 for r in range(R)] + [C * R * (R - 1) // 2 + R * c for c in range(C)]
+    got = sums.sum_rows_cols(a)
+    assert got.tolist() == want
+    assert int(got[:R].sum()) == int(got[R:].sum()) == R * C * (R * C - 1) // 2
+    assert sums.sum_rows_cols_literal(a) == want

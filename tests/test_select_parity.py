@@ -35,7 +35,8 @@ def _cmp(pattern, shape, dtype, lim, strat):
 
 
 @pytest.mark.parametrize("profile", list(PROFILES))
-@pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"])
+@pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS",
+                                     "SUM_ROWS_COLS"])
 def test_sums_exhaustive(profile, pattern):
     lim = PROFILES[profile]
     for R, C in itertools.product(SIZES, SIZES):
@@ -86,7 +87,7 @@ def test_invalid_arguments():
 def test_enumerate_parity(profile):
     # npp_enumerate (Fig 17 sweep space) == oracle enumeration, record by record and in order
     lim = PROFILES[profile]
-    for pattern in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_COLS"):
+    for pattern in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS"):
         for shape in [(65536, 1024), (1024, 65536), (50, 20000), (3, 5)]:
             for dtype in ("f32", "i64"):
                 want = S.enumerate_mappings(pattern, shape, dtype, lim)

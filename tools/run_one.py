@@ -1,4 +1,4 @@
-"""Run one plan a few times (for ncu captures): python tools/run_one.py logreg|kmeans|sumrows|sumcols [args]"""
+"""Run one plan a few times (for ncu captures): python tools/run_one.py logreg|kmeans|sumrows|sumcols|rowscols [args]"""
 import sys
 sys.path.insert(0, '/root/repo')
 import torch
@@ -17,7 +17,8 @@ elif what == 'kmeans':
 else:
     R, C = (int(v) for v in sys.argv[2].split('x'))
     m = gen.uniform_f32(1, (R, C), device=dev)
-    p = npp.Plan('SUM_ROWS' if what == 'sumrows' else 'SUM_COLS', (R, C), 'f32', 'AUTO'); ins = [m]
+    pat = {'sumrows': 'SUM_ROWS', 'sumcols': 'SUM_COLS', 'rowscols': 'SUM_ROWS_COLS'}[what]
+    p = npp.Plan(pat, (R, C), 'f32', 'AUTO'); ins = [m]
 out = p.new_out()
 for _ in range(4):
     p.execute(ins, out)
