@@ -538,11 +538,11 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
     if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:
-        # S9 RC: tickets [Tr] + tickets [gc] (u32), accumulators [R] + [C] of the accumulator type
+        # S9 RC: tickets [gr] + tickets [gc] (u32), accumulators [R] + [C] of the accumulator type
         R, C = nest["levels"][0][0], nest["levels"][1][0]
         t = rc_tiling(R, C, dtype, lim)
         ab = acc_bytes(nest["pattern"], dtype)
-        rec["workspace_bytes"] = (256 * cdiv(4 * t["Tr"], 256) + 256 * cdiv(4 * t["gc"], 256)
+        rec["workspace_bytes"] = (256 * cdiv(4 * t["gr"], 256) + 256 * cdiv(4 * t["gc"], 256)
                                   + 256 * cdiv(R * ab, 256) + 256 * cdiv(C * ab, 256))
     if temp[0] == TEMP_PREALLOC:   # S10: the [outer x inner] buffer after partials and tickets
         M, N = _eff(nest["levels"][0][0]), _eff(nest["levels"][1][0])

@@ -215,6 +215,12 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
     *out = p;
     return NPP_OK;
   }
+  if (pattern == NPP_SUM_ROWS_COLS && strategy != NPP_MAP_AUTO) {
+    delete p;
+    set_error("SUM_ROWS_COLS executes with strategy AUTO only (the one-pass family); the paper's two-kernel "
+              "schedule is a SUM_ROWS plan plus a SUM_COLS plan");
+    return NPP_ERR_UNSUPPORTED;
+  }
   st = get_limits(limits, &p->lim);
   if (!st) st = npp_select(pattern, shape, ndim, dtype, &p->lim, strategy, &p->map);
   if (st) {
@@ -226,7 +232,7 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
     set_error("3-level nests execute through their staged (AUTO) kernel families only");
     return NPP_ERR_UNSUPPORTED;
   }
-  if (pattern == NPP_SUM_ROWS_COLS && strategy != NPP_MAP_AUTO) {
+  if (pattern == NPP_SUM_ROWS_COLS && strategy != NPP_MAP_AUTO) {  // (also checked before selection)
     delete p;
     set_error("SUM_ROWS_COLS executes with strategy AUTO only (the one-pass family); the paper's two-kernel "
               "schedule is a SUM_ROWS plan plus a SUM_COLS plan");
@@ -451,7 +457,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     r.R = plan->shape[0];
     r.C = plan->shape[1];
     r.Tr = t.Tr, r.Tc = t.Tc, r.cr = t.cr, r.cc = t.cc, r.gr = t.gr, r.gc = t.gc, r.nreg = t.nreg;
-    const int64_t o_tc = ((4 * t.Tr + 255) / 256) * 256;
+    const int64_t o_tc = ((4 * t.gr + 255) / 256) * 256;
     const int64_t o_ar = o_tc + ((4 * t.gc + 255) / 256) * 256;
     const int64_t o_ac = o_ar + ((r.R * ab + 255) / 256) * 256;
     r.tick_r = reinterpret_cast<unsigned*>(ws);

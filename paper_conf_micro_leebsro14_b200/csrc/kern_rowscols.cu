@@ -17,8 +17,8 @@
 //            butterfly (lane l ends with row l), keeps them in a register across the band's column
 //            tiles, and the eight warps meet in shared memory once per band.
 // A row band (column region) covered by several regions is the Split of P:L542-550: contributions meet
-// through fp64 / integer atomics and a ticket per band (per column group); the last contributor
-// converts and re-zeroes (the combiner of P:L880-883, fused). gc == 1 rows and gr == 1 columns are
+// through fp64 / integer atomics and one ticket per row region (column group), taken once at region
+// end; the last contributor converts and re-zeroes (the combiner of P:L880-883, fused). gc == 1 rows and gr == 1 columns are
 // written directly. Without 16-B row pitch (no tensor map) the same consumers load the tile straight
 // from global memory (STAGED = false; the producer warp idles).
 #include <cuda.h>
@@ -212,25 +212,11 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
         for (int j = 0; j < WPG; ++j) s += rsum[(rb * kConsumerWarps + g * WPG + j) * 32 + li];
         const long long row = br * kTileRows + lane;
-        if (a.gc == 1) {
-          if (row < a.R) out[row] = RcOps<T>::finish(s);
-        } else {
-          if (row < a.R) atomicAdd(accR + row, s);
-          __threadfence();
-          __syncwarp();
-          unsigned last = 0;
-          if (lane == 0) {
-            last = atomicAdd(a.tick_r + br, 1u) + 1u == unsigned(a.gc);
-            if (last) a.tick_r[br] = 0u;
-          }
-          if (__shfl_sync(0xffffffffu, last, 0)) {
-            __threadfence();
-            if (row < a.R) {
-              const Acc val = __ldcg(accR + row);
-              __stcg(accR + row, Acc(0));
-              out[row] = RcOps<T>::finish(val);
-            }
-          }
+        if (row < a.R) {
+          if (a.gc == 1)
+            out[row] = RcOps<T>::finish(s);
+          else
+            atomicAdd(accR + row, s);  // completed by the row-region ticket at region end
         }
       }
       rb ^= 1;
@@ -253,17 +239,37 @@ __global__ void __launch_bounds__(kThreads, 1)
           atomicAdd(accC + cg, s);
       }
     }
-    if (a.gr > 1) {
+    // Split combine (fused): one fence and one ticket per region and direction. The gc
+    // column regions of row region ri add their row partials (band ends above), the gr row regions of
+    // column group cj their column partials; the last of each converts and re-zeroes.
+    if (a.gr > 1 || a.gc > 1) {
       __threadfence();
       consumers_sync();
       if (threadIdx.x == 0) {
-        const bool last = atomicAdd(a.tick_c + cj, 1u) + 1u == unsigned(a.gr);
-        if (last) a.tick_c[cj] = 0u;
-        *flag = last ? 1 : 0;
+        bool last_r = false, last_c = false;
+        if (a.gc > 1) {
+          last_r = atomicAdd(a.tick_r + ri, 1u) + 1u == unsigned(a.gc);
+          if (last_r) a.tick_r[ri] = 0u;
+        }
+        if (a.gr > 1) {
+          last_c = atomicAdd(a.tick_c + cj, 1u) + 1u == unsigned(a.gr);
+          if (last_c) a.tick_c[cj] = 0u;
+        }
+        flag[0] = last_r ? 1 : 0;
+        flag[1] = last_c ? 1 : 0;
       }
       consumers_sync();
-      if (*flag) {
-        __threadfence();
+      const bool last_r = flag[0] != 0, last_c = flag[1] != 0;
+      if (last_r || last_c) __threadfence();
+      if (last_r) {
+        const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
+        for (long long row = rlo + threadIdx.x; row < rhi; row += kConsumers) {
+          const Acc val = __ldcg(accR + row);
+          __stcg(accR + row, Acc(0));
+          out[row] = RcOps<T>::finish(val);
+        }
+      }
+      if (last_c) {
         for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
           const long long cg = c0 * BC + c;
           if (cg < a.C) {
@@ -274,7 +280,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
-    consumers_sync();  // accumulators re-zeroed and the flag read before the next region
+    consumers_sync();  // accumulators re-zeroed and the flags read before the next region
   }
 }
 

@@ -103,7 +103,7 @@ struct RowsColsArgs {
   void* out;           // [R + C]
   void* accR;          // [R] accumulators (fp64 / u32 / u64) of row bands cut by column regions
   void* accC;          // [C] accumulators of columns cut by row regions
-  unsigned* tick_r;    // [Tr] column regions done per row band (zero on entry and on exit)
+  unsigned* tick_r;    // [gr] column regions done per row region (zero on entry and on exit)
   unsigned* tick_c;    // [gc] row regions done per column group (zero on entry and on exit)
   int64_t R, C;
   int64_t Tr, Tc;      // 32-row bands, BC-column tiles

@@ -634,10 +634,10 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
   } else if (n.pattern == NPP_SUM_ROWS_COLS && c.persistent_grid > 0) {
-    // S9 RC: tickets [Tr] + tickets [gc] (u32) + accumulators [R] + [C] of the accumulator type
+    // S9 RC: tickets [gr] + tickets [gc] (u32) + accumulators [R] + [C] of the accumulator type
     const RcTiling t = rc_tiling(n.N[0], n.N[1], dtype, lim.sm_count);
     const int64_t ab = acc_bytes(n.pattern, dtype);
-    m.workspace_bytes = 256 * cdiv(4 * t.Tr, 256) + 256 * cdiv(4 * t.gc, 256) + 256 * cdiv(n.N[0] * ab, 256) +
+    m.workspace_bytes = 256 * cdiv(4 * t.gr, 256) + 256 * cdiv(4 * t.gc, 256) + 256 * cdiv(n.N[0] * ab, 256) +
                         256 * cdiv(n.N[1] * ab, 256);
   } else if (is_sum_pattern(n.pattern) && c.staged) {
     // pool counters (256 B) + tickets [To] + accumulators [O] of the accumulator type
