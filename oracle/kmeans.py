@@ -6,6 +6,12 @@ MSMBuilder clustering case study L1256-1271):
 i.e.  a[i] = min{ k : Σ_d (x[i,d] − c[k,d])² is minimal }   — ties go to the lowest k (G20).
 fp64: the difference of two fp32 values and its square are exact in fp64, so the literal evaluator's
 ``math.fsum`` distance is the correctly rounded exact distance.
+
+The centroid update that follows an assignment is Table I's groupBy (L292) followed
+by a Reduce per group:
+    points groupBy { i => a_i }  map { g => ((g map x) reduce +, g.size) }
+i.e. for k in [0, K):  U[k, d] = Σ_{i : a_i = k} x[i, d]  (d < D),  U[k, D] = |{i : a_i = k}|.
+Points whose a_i lies outside [0, K) belong to no group (reading G23). fp64 sums, exact counts.
 """
 from __future__ import annotations
 
@@ -44,3 +50,33 @@ def assign(x: np.ndarray, c: np.ndarray, chunk: int = 4096) -> np.ndarray:
     for s in range(0, x.shape[0], chunk):
         out[s:s + chunk] = np.argmin(distances(x[s:s + chunk], c), axis=1)
     return out
+
+
+def update_literal(x: np.ndarray, a: np.ndarray, K: int) -> list:
+    """Pure-Python groupBy then Reduce: rows [Σ_{a_i = k} x_i (math.fsum per dim) ..., count_k]."""
+    xs, aa = x.tolist(), [int(v) for v in a.tolist()]
+    D = x.shape[1]
+    groups = {k: [] for k in range(K)}
+    for xi, k in zip(xs, aa):
+        if 0 <= k < K:
+            groups[k].append(xi)
+    return [[math.fsum(float(p[d]) for p in groups[k]) for d in range(D)] + [float(len(groups[k]))]
+            for k in range(K)]
+
+
+def update(x: np.ndarray, a: np.ndarray, K: int) -> np.ndarray:
+    """Vectorised: U[k] = (np.add.reduce over the rows with a_i = k in fp64, count) -> [K, D+1] fp64."""
+    N, D = x.shape
+    out = np.zeros((K, D + 1), dtype=np.float64)
+    x64 = x.astype(np.float64)
+    a = np.asarray(a).astype(np.int64)
+    for k in range(K):
+        mask = a == k
+        out[k, :D] = np.add.reduce(x64[mask], axis=0) if mask.any() else 0.0
+        out[k, D] = float(mask.sum())
+    return out
+
+
+def update_scale(x: np.ndarray, a: np.ndarray, K: int) -> np.ndarray:
+    """Σ_{a_i = k} |x[i, d]| — the scale of the fp32 tolerance bound for signed data."""
+    return update(np.abs(x.astype(np.float64)), a, K)[:, :-1]

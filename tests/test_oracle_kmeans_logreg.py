@@ -118,3 +118,51 @@ def test_finite_differences():
         e[j] = h
         fd = (loss(w64 + e) - loss(w64 - e)) / (2 * h)
         assert math.isclose(fd, g[j], rel_tol=1e-6, abs_tol=1e-9)
+
+
+# ---------------------------------------------------------------- k-means update (groupBy + Reduce)
+
+def test_update_closed_forms():
+    from oracle import sums
+    rng = np.random.default_rng(7)
+    x = rng.integers(-50, 50, size=(300, 12)).astype(np.float32)
+    # one group holding every point: the sums are sumCols (independently pinned), the count is N
+    u = kmeans.update(x, np.zeros(300, dtype=np.int32), 1)
+    assert np.array_equal(u[0, :12], sums.sum_cols(x)) and u[0, 12] == 300
+    # a_i = i mod K on arange data: closed form Σ_{i ≡ k} (i*D + d)
+    N, D, K = 100, 3, 7
+    xa = np.arange(N * D, dtype=np.float32).reshape(N, D)
+    ua = kmeans.update(xa, np.arange(N) % K, K)
+    for k in range(K):
+        ids = list(range(k, N, K))
+        assert ua[k, D] == len(ids)
+        for d in range(D):
+            assert ua[k, d] == sum(i * D + d for i in ids)
+    # invalid keys belong to no group; counts of valid keys sum to their number; groups partition
+    a = rng.integers(-2, 9, size=300)
+    u = kmeans.update(x, a, 7)
+    valid = (a >= 0) & (a < 7)
+    assert u[:, 12].sum() == valid.sum()
+    assert np.array_equal(u[:, :12].sum(axis=0), sums.sum_cols(x[valid]))
+
+
+def test_update_literal_matches_vectorised():
+    rng = np.random.default_rng(3)
+    x = rng.standard_normal((57, 5)).astype(np.float32)
+    a = rng.integers(-1, 4, size=57)
+    lit = np.array(kmeans.update_literal(x, a, 4))
+    vec = kmeans.update(x, a, 4)
+    assert np.allclose(lit, vec, rtol=1e-14, atol=1e-12)
+    assert np.array_equal(lit[:, -1], vec[:, -1])
+
+
+def test_update_after_assign_is_a_lloyd_step():
+    # Lloyd: the new centroids U[:, :D] / U[:, D] never increase the assignment's total squared distance
+    x, c = gen.kmeans_inputs(2000, 8, 5, seed=21)
+    x, c = x.numpy(), c.numpy()
+    a = kmeans.assign(x, c)
+    u = kmeans.update(x, a, 5)
+    newc = np.where(u[:, -1:] > 0, u[:, :-1] / np.maximum(u[:, -1:], 1), c.astype(np.float64))
+    before = ((x.astype(np.float64) - c.astype(np.float64)[a]) ** 2).sum()
+    after = ((x.astype(np.float64) - newc[a]) ** 2).sum()
+    assert after <= before + 1e-9
