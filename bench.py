@@ -166,6 +166,18 @@ def build_kmeans(npp, gen, torch, rank, world, strategy, device):
     return [item], [], "k-means assignment 4M x 64 x 32"
 
 
+def build_kmeans_update(npp, gen, torch, rank, world, strategy, device):
+    # the centroid update after the config-4 assignment: 4M points x 64 dims into
+    # 32 groups; keys = the assignment of the same points (computed once, outside the timed region)
+    N, D, K = 1 << 22, 64, 32
+    x, c = gen.kmeans_inputs(N, D, K, row_offset=rank * N, device=device)
+    a = npp.kmeans_assign(x, c)
+    plan = npp.Plan("KMEANS_UPDATE", (N, D, K), "f32", "AUTO", device=device)
+    out = plan.new_out()
+    item = Item("kmeans_update[4M,64,32]", plan, [x, a], out, N * D * 4 + N * 4 + K * (D + 1) * 4)
+    return [item], ([out] if world > 1 else []), "k-means centroid update 4M x 64 -> 32 groups"
+
+
 def build_logreg(npp, gen, torch, rank, world, strategy, device):
     # BASELINE.json config 5: [16M, 256] fp32 in B = 4096 mini-batches of 4096 rows; batches sharded
     B, Rb, C = 4096 // world, 4096, 256
@@ -190,9 +202,10 @@ def build_rowscols(npp, gen, torch, rank, world, strategy, device):
 
 
 # per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
-SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak"}
+SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak",
+           "kmeans_update": "weak"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
-             "logreg": build_logreg, "rowscols": build_rowscols}
+             "logreg": build_logreg, "rowscols": build_rowscols, "kmeans_update": build_kmeans_update}
 
 
 # ------------------------------------------------------------------------- reference arm (the oracle)
@@ -242,6 +255,8 @@ def config_for(args, extra):
           "sumcols_1m4k": "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])",
           "kmeans": "k-means assignment 4M x 64 x 32 fp32, points sharded (BASELINE.json configs[3])",
           "logreg": "batched logreg gradient [16M,256] fp32, B=4096, batches sharded (BASELINE.json configs[4])",
+          "kmeans_update": "k-means centroid update 4M x 64 -> 32 groups fp32, points sharded + all-reduce "
+                           "of [32, 65] (SURVEY §8f NEXT 4)",
           "rowscols": "sumRows+sumCols in ONE pass (SUM_ROWS_COLS) fp32 @ [64K,1K],[8K,8K],[1K,64K] "
                       "(Naive Bayes counts, SURVEY §8f NEXT 2)",
           }[args.workload]
@@ -261,7 +276,9 @@ def cpu_baseline(items, budget_s=12.0):
     done_bytes, t_total, n = 0, 0.0, 0
     samples = []
     for it in items:
-        if it.name.startswith("kmeans"):  # first 256K points (the oracle is O(N K D) in fp64)
+        if it.name.startswith("kmeans_update"):  # first 1M points
+            samples.append((it.name, [it.ins[0][: 1 << 20].cpu().numpy(), it.ins[1][: 1 << 20].cpu().numpy()]))
+        elif it.name.startswith("kmeans"):  # first 256K points (the oracle is O(N K D) in fp64)
             samples.append((it.name, [it.ins[0][: 1 << 18].cpu().numpy(), it.ins[1].cpu().numpy()]))
         elif it.name.startswith("logreg"):  # first 64 batches
             Rb = it.plan.shape[1]
@@ -272,7 +289,9 @@ def cpu_baseline(items, budget_s=12.0):
             samples.append((it.name, [it.ins[0].cpu().numpy()]))
 
     def run(name, arrs):
-        if name.startswith("kmeans"):
+        if name.startswith("kmeans_update"):
+            okm.update(arrs[0], arrs[1], it_k)
+        elif name.startswith("kmeans"):
             okm.assign(*arrs)
         elif name.startswith("logreg"):
             olr.grad(arrs[0], arrs[1], arrs[2], 64)
@@ -280,6 +299,7 @@ def cpu_baseline(items, budget_s=12.0):
             sums.sum_rows_cols(arrs[0])
         else:
             (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(arrs[0])
+    it_k = items[0].plan.shape[2] if items and items[0].plan.pattern == "KMEANS_UPDATE" else 0
     t_end = time.perf_counter() + budget_s
     while time.perf_counter() < t_end:
         for name, arrs in samples:

@@ -70,7 +70,8 @@ typedef enum {
   NPP_LOGREG_GRAD = 3,
   NPP_SUM_WEIGHTED_ROWS = 4,
   NPP_SUM_WEIGHTED_COLS = 5,
-  NPP_SUM_ROWS_COLS = 6
+  NPP_SUM_ROWS_COLS = 6,
+  NPP_KMEANS_UPDATE = 7
 } npp_pattern;
 
 /* AUTO     = Algorithm 1 + ControlDOP + the runtime step R2 (L810-817; S8)
@@ -99,7 +100,8 @@ typedef enum {
   NPP_CLASS_KMEANS = 2,  /* 3-level: Map points / argmin centroids / Reduce dims          */
   NPP_CLASS_LOGREG = 3,  /* 3-level: Map batches / Reduce rows / Map+Reduce columns       */
   NPP_CLASS_EMPTY = 4,   /* a zero-sized level: output zero-filled (or nothing to do)     */
-  NPP_CLASS_RC = 5       /* 2-level, both levels Reduce: row and column sums in one pass  */
+  NPP_CLASS_RC = 5,      /* 2-level, both levels Reduce: row and column sums in one pass  */
+  NPP_CLASS_KMUPDATE = 6 /* groupBy + Reduce: per-centroid sums and counts                */
 } npp_kernel_class;
 
 /* One nest level of a mapping (§IV-A). dim: npp_dim; span: npp_span; factor: n of Span(n) or k of

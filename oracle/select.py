@@ -22,7 +22,7 @@ X, Y, Z = 0, 1, 2
 # span codes (S9 / record)
 ONE, ALL, SPAN_N, SPLIT = 0, 1, 2, 3
 # kernel classes (S9)
-RX, MX, KM, LR, EMPTY, RC = 0, 1, 2, 3, 4, 5
+RX, MX, KM, LR, EMPTY, RC, KU = 0, 1, 2, 3, 4, 5, 6
 
 SIZE_SET = [1 << i for i in range(11)]          # {1,2,4,...,1024}  Alg 1
 W_C, W_B = 8, 1                                  # DESIGN.md G3
@@ -32,7 +32,7 @@ T_BLOCK, U_MIN = 256, 8                          # DESIGN.md S8
 MAX_GRID = (1 << 31) - 1                         # DESIGN.md S3 H6
 
 PATTERNS = ("SUM_ROWS", "SUM_COLS", "KMEANS_ASSIGN", "LOGREG_GRAD",
-            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS")
+            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS", "KMEANS_UPDATE")
 DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8}
 
 B200 = dict(sm_count=148, max_threads_per_sm=2048, max_threads_per_block=1024,
@@ -92,6 +92,13 @@ def build_nest(pattern: str, shape) -> dict:
         R, C = shape
         levels = [(R, True), (C, True)]             # rows Reduce (column sums), cols Reduce (row sums)
         acc = [(0, (0,)), (1, (1,)), (1, (0, 1))]   # out_rows[r], out_cols[c], m[r,c]
+    elif pattern == "KMEANS_UPDATE":                 # groupBy (Table I) + Reduce per group
+        N, D, K = shape
+        if K < 1:
+            raise ValueError("KMEANS_UPDATE needs K >= 1")
+        levels = [(N, True), (D, False)]            # points: Reduce into K groups; dims: Map
+        acc = [(1, (0, 1)), (0, (0,)), (1, (1,))]   # x[i,d], a[i], U[k,d]
+        return {"pattern": pattern, "levels": levels, "accesses": acc, "K": K}
     elif pattern == "KMEANS_ASSIGN":
         N, D, K = shape
         levels = [(N, False), (K, True), (D, True)]
@@ -146,7 +153,7 @@ def level_chunk(n: int, b: int, span: int, factor: int, vec: int = 1) -> int:
 # ------------------------------------------------------------------ S3 hard constraints
 
 def acc_bytes(pattern: str, dtype: str) -> int:
-    if pattern in ("KMEANS_ASSIGN", "LOGREG_GRAD"):
+    if pattern in ("KMEANS_ASSIGN", "LOGREG_GRAD", "KMEANS_UPDATE"):
         return 8
     return 4 if dtype == "i32" else 8
 
@@ -402,6 +409,21 @@ def r2_rowscols(nest, dtype, lim):
     return dims, blocks, spans, factors, 1, chunks, staged, t["G"], t["cr"] * t["cc"]
 
 
+def r2_kmupdate(nest, lim):
+    """DESIGN.md S8 KU: 128-point tiles, contiguous ranges of P tiles, 8 warps x 32 lanes (2 dims per lane).
+    Returns (dims, blocks, spans, factors, vec, chunks, G, P)."""
+    (N, _), (D, _) = nest["levels"]
+    K = nest["K"]
+    if D % 4 != 0 or D < 4 or D > 64 or K < 1 or K > 256 or K * D > 2048:
+        raise Unsupported("KMEANS_UPDATE AUTO needs D % 4 == 0, 4 <= D <= 64, 1 <= K <= 256, K*D <= 2048")
+    T = cdiv(N, 128)
+    P = cdiv(T, min(lim["sm_count"], T))
+    G = cdiv(T, P)
+    spans = (SPLIT if G > 1 else ALL, ALL)
+    chunks = (128 * P if G > 1 else N, D)
+    return (Y, X), (8, 32), spans, (G, 1), 2, chunks, G, P
+
+
 def r2_logreg(nest, lim, dims):
     """DESIGN.md S8, LOGREG_GRAD staged: 32-row tiles of one batch, contiguous tile ranges."""
     (B, _), (Rb, _), (C, _) = nest["levels"]
@@ -487,6 +509,8 @@ def kernel_class(pattern, dims):
         return LR
     if pattern == "SUM_ROWS_COLS":
         return RC
+    if pattern == "KMEANS_UPDATE":
+        return KU
     return RX if dims[1] == X else MX
 
 
@@ -537,6 +561,8 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
+    if nest["pattern"] == "KMEANS_UPDATE" and staged:  # ticket (256 B) + fp64 accumulators [K x (D+1)]
+        rec["workspace_bytes"] = 256 + 256 * cdiv(8 * nest["K"] * (_eff(nest["levels"][1][0]) + 1), 256)
     if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:
         # S9 RC: tickets [gr] + tickets [gc] (u32), accumulators [R] + [C] of the accumulator type
         R, C = nest["levels"][0][0], nest["levels"][1][0]
@@ -598,6 +624,10 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
     if pattern == "KMEANS_ASSIGN":
         b3, s3, f3, vec, chunks, G, P = r2_kmeans(nest, lim)
         return make_record(nest, dtype, lim, dims, b3, s3, f3, vec, sc, chunks, staged=1,
+                           persistent_grid=G, claim_tiles=P)
+    if pattern == "KMEANS_UPDATE":
+        d2, b2, s2, f2, vec, chunks, G, P = r2_kmupdate(nest, lim)
+        return make_record(nest, dtype, lim, d2, b2, s2, f2, vec, sc, chunks, staged=1,
                            persistent_grid=G, claim_tiles=P)
     if pattern == "SUM_ROWS_COLS":
         d2, b2, s2, f2, vec, chunks, staged, G, CL = r2_rowscols(nest, dtype, lim)

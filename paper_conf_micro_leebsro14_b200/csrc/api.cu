@@ -47,7 +47,8 @@ int n_inputs(int pattern) {
     case NPP_SUM_ROWS_COLS: return 1;
     case NPP_SUM_WEIGHTED_ROWS:
     case NPP_SUM_WEIGHTED_COLS:
-    case NPP_KMEANS_ASSIGN: return 2;
+    case NPP_KMEANS_ASSIGN:
+    case NPP_KMEANS_UPDATE: return 2;
     case NPP_LOGREG_GRAD: return 3;
     default: return -1;
   }
@@ -64,6 +65,7 @@ int64_t input_bytes(const npp_plan_s* p, int k) {
     case NPP_SUM_WEIGHTED_ROWS: return k == 0 ? s[0] * s[1] * es : s[1] * es;
     case NPP_SUM_WEIGHTED_COLS: return k == 0 ? s[0] * s[1] * es : s[0] * es;
     case NPP_KMEANS_ASSIGN: return k == 0 ? s[0] * s[1] * 4 : s[2] * s[1] * 4;
+    case NPP_KMEANS_UPDATE: return k == 0 ? s[0] * s[1] * 4 : s[0] * 4;
     case NPP_LOGREG_GRAD: return k == 0 ? s[0] * s[1] * s[2] * 4 : (k == 1 ? s[0] * s[1] * 4 : s[2] * 4);
     default: return 0;
   }
@@ -79,6 +81,7 @@ int64_t output_bytes(const npp_plan_s* p) {
     case NPP_SUM_WEIGHTED_COLS: return s[1] * es;
     case NPP_SUM_ROWS_COLS: return (s[0] + s[1]) * es;
     case NPP_KMEANS_ASSIGN: return s[0] * 4;
+    case NPP_KMEANS_UPDATE: return s[2] * (s[1] + 1) * 4;
     case NPP_LOGREG_GRAD: return s[0] * s[2] * 4;
     default: return 0;
   }
@@ -97,7 +100,8 @@ int validate_request(int pattern, const int64_t* shape, int ndim, int dtype, boo
     set_error("unknown pattern");
     return NPP_ERR_INVALID_ARG;
   }
-  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) && dtype != NPP_F32) {
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) &&
+      dtype != NPP_F32) {
     set_error("k-means and logreg are defined for f32");
     return NPP_ERR_UNSUPPORTED;
   }
@@ -219,6 +223,11 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
     delete p;
     set_error("SUM_ROWS_COLS executes with strategy AUTO only (the one-pass family); the paper's two-kernel "
               "schedule is a SUM_ROWS plan plus a SUM_COLS plan");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  if (pattern == NPP_KMEANS_UPDATE && strategy != NPP_MAP_AUTO) {
+    delete p;
+    set_error("KMEANS_UPDATE executes with strategy AUTO only (class KU)");
     return NPP_ERR_UNSUPPORTED;
   }
   st = get_limits(limits, &p->lim);
@@ -445,6 +454,21 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     k.per_block = m.claim_tiles;
     cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);
+    return NPP_OK;
+  }
+  if (plan->pattern == NPP_KMEANS_UPDATE) {  // class KU (S8 KU)
+    npp::KmUpdateArgs u{};
+    u.out = static_cast<float*>(out);
+    u.ticket = static_cast<unsigned*>(workspace);
+    u.acc = reinterpret_cast<double*>(static_cast<char*>(workspace) + 256);
+    u.N = plan->shape[0];
+    u.D = plan->shape[1];
+    u.K = plan->shape[2];
+    u.per_block = m.claim_tiles;
+    u.early_reads = overlap ? 1 : 0;
+    cudaError_t e = npp::launch_kmupdate(u, static_cast<const float*>(ins[0]), static_cast<const int*>(ins[1]),
+                                         int(m.grid), st);
+    if (e != cudaSuccess) return cuda_fail("k-means update kernel launch", e);
     return NPP_OK;
   }
   if (plan->pattern == NPP_SUM_ROWS_COLS) {  // class RC (S8 RC): one pass, both outputs

@@ -1,0 +1,201 @@
+// kern_kmupdate.cu — class KU: the k-means centroid update that follows an assignment (SURVEY §8f
+// NEXT 4), Table I's groupBy followed by a Reduce per group:
+//     points groupBy { i => a_i } map { g => ((g map x) reduce +, g.size) }
+//     U[k, d] = Σ_{i: a_i = k} x[i, d],  U[k, D] = |{i : a_i = k}|     (a_i outside [0, K): no group)
+// The path is HBM-bound (4·D + 4 bytes per point, D adds): tiles of 128 points (x: 2-D TMA box of
+// 128 rows x D floats; a: 1-D box of 128 ints) stream through a 4-deep mbarrier ring, one block per
+// SM, contiguous tile ranges. The data-dependent key is why this is not a sum family: the reduction
+// target of a point is only known when its a_i arrives.
+//   Consumer warp w adds points w, w+8, ... of each tile: lane l owns dims 2l, 2l+1 (float2), so a
+//   point is one conflict-free 8-byte read of the tile plus a read-modify-write of the warp's OWN
+//   fp32 accumulator row k in shared memory (no atomics: one warp, one point at a time; shared-memory
+//   float atomics are CAS loops on sm_100a). Every 8 tiles (<= 128 points per warp accumulator, so the
+//   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
+//   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
+//   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
+//   fused).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.hpp"
+#include "tma_ring.cuh"
+
+namespace npp {
+
+namespace {
+
+using namespace tma;
+
+constexpr int kStages = 4;
+constexpr int kTP = 128;                  // points per tile
+constexpr int kXSlot = 32 * 1024;         // kTP * D * 4 <= 32 KB (D <= 64)
+constexpr int kASlot = kTP * 4;           // 512 B of keys
+constexpr int kConsumerWarps = 8;
+constexpr int kConsumers = kConsumerWarps * 32;
+constexpr int kThreads = kConsumers + 32;  // + producer warp
+constexpr int kHeader = 1024;
+constexpr int kMaxKD = 2048;               // DESIGN.md S8 KU: K*D <= 2048, K <= 256
+constexpr int kMaxK = 256;
+constexpr int kFlushTiles = 8;
+constexpr int kSmemBytes = kHeader + kStages * (kXSlot + kASlot) + kConsumerWarps * kMaxKD * 4 +
+                           kConsumerWarps * kMaxK * 4 + (kMaxKD + kMaxK) * 8;
+
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
+
+}  // namespace
+
+__global__ void __launch_bounds__(kThreads, 1)
+    npp_kmupdate_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap amap,
+                        const KmUpdateArgs a) {
+  extern __shared__ __align__(1024) unsigned char smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
+  uint64_t* empty = full + kStages;
+  volatile int* flag = reinterpret_cast<volatile int*>(empty + kStages);
+  unsigned char* xring = smem + kHeader;
+  unsigned char* aring = xring + kStages * kXSlot;
+  float* accw = reinterpret_cast<float*>(aring + kStages * kASlot);           // [8][K*D]
+  unsigned* cntw = reinterpret_cast<unsigned*>(accw + kConsumerWarps * kMaxKD);  // [8][K]
+  double* bacc = reinterpret_cast<double*>(cntw + kConsumerWarps * kMaxK);     // [K*(D+1)]
+  const int D = int(a.D), K = int(a.K), KD = K * D, KD1 = K * (D + 1);
+
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long T = (a.N + kTP - 1) / kTP;
+  const long long t0 = blockIdx.x * a.per_block;
+  const long long t1 = t0 + a.per_block < T ? t0 + a.per_block : T;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kStages; ++i) {
+      mbar_init(full + i, 1);
+      mbar_init(empty + i, kConsumerWarps);
+    }
+    mbar_fence_init();
+  }
+  if (threadIdx.x < kConsumers) {
+    for (int i = threadIdx.x; i < kConsumerWarps * KD; i += kConsumers) accw[i] = 0.f;
+    for (int i = threadIdx.x; i < kConsumerWarps * K; i += kConsumers) cntw[i] = 0u;
+    for (int i = threadIdx.x; i < KD1; i += kConsumers) bacc[i] = 0.0;
+  }
+  __syncthreads();
+
+  if (warp == kConsumerWarps) {
+    // ------------------------------------------------------------ producer: one elected lane
+    if (lane == 0) {
+      prefetch_map(&xmap);
+      prefetch_map(&amap);
+      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
+      const unsigned bytes = unsigned(kTP * D * 4 + kASlot);
+      for (long long t = t0; t < t1; ++t) {
+        const long long i = t - t0;
+        const int slot = int(i % kStages);
+        if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
+        mbar_expect_tx(full + slot, bytes);
+        load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
+        load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
+      }
+    }
+    return;
+  }
+
+  // -------------------------------------------------------------- consumers
+  float* myacc = accw + warp * KD;
+  unsigned* mycnt = cntw + warp * K;
+  const bool dim_lane = 2 * lane < D;
+  auto flush = [&]() {  // fold the 8 warp copies into the fp64 block accumulator, zero the copies
+    consumers_sync();
+    for (int i = threadIdx.x; i < KD; i += kConsumers) {
+      double s = 0.0;
+#pragma unroll
+      for (int w = 0; w < kConsumerWarps; ++w) {
+        s += double(accw[w * KD + i]);
+        accw[w * KD + i] = 0.f;
+      }
+      const int k = i / D;
+      bacc[i + k] += s;  // row k of [K x (D+1)]
+    }
+    for (int k = threadIdx.x; k < K; k += kConsumers) {
+      unsigned c = 0;
+#pragma unroll
+      for (int w = 0; w < kConsumerWarps; ++w) {
+        c += cntw[w * K + k];
+        cntw[w * K + k] = 0u;
+      }
+      bacc[k * (D + 1) + D] += double(c);
+    }
+    consumers_sync();
+  };
+  int since = 0;
+  for (long long t = t0; t < t1; ++t) {
+    const long long i = t - t0;
+    const int slot = int(i % kStages);
+    mbar_wait(full + slot, unsigned((i / kStages) & 1));
+    const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
+    const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
+    const long long base = t * kTP;
+    const int np = a.N - base < kTP ? int(a.N - base) : kTP;  // valid points (TMA zero-fills the rest)
+    for (int p = warp; p < np; p += kConsumerWarps) {
+      const int k = at[p];
+      if (unsigned(k) >= unsigned(K)) continue;  // no group (warp-uniform)
+      if (dim_lane) {
+        const float2 xv = *reinterpret_cast<const float2*>(xt + p * D + 2 * lane);
+        float2* acc = reinterpret_cast<float2*>(myacc + k * D + 2 * lane);
+        float2 v = *acc;
+        v.x += xv.x;
+        v.y += xv.y;
+        *acc = v;
+      }
+      if (lane == 0) mycnt[k] += 1u;
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + slot);
+    if (++since == kFlushTiles) {
+      flush();
+      since = 0;
+    }
+  }
+  if (since) flush();
+
+  // ---- block result -> fp64 workspace accumulators; the last block converts (fused Split combine)
+  asm volatile("griddepcontrol.wait;" ::: "memory");  // workspace / out: after the previous grid
+  for (int i = threadIdx.x; i < KD1; i += kConsumers) {
+    const double v = bacc[i];
+    if (v != 0.0) atomicAdd(a.acc + i, v);
+  }
+  __threadfence();
+  consumers_sync();
+  if (threadIdx.x == 0) {
+    const bool last = atomicAdd(a.ticket, 1u) + 1u == gridDim.x;
+    if (last) *a.ticket = 0u;
+    flag[0] = last ? 1 : 0;
+  }
+  consumers_sync();
+  if (flag[0]) {
+    __threadfence();
+    for (int i = threadIdx.x; i < KD1; i += kConsumers) {
+      const double v = __ldcg(a.acc + i);
+      __stcg(a.acc + i, 0.0);
+      a.out[i] = float(v);
+    }
+  }
+}
+
+cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st) {
+  if (a.D % 4 != 0 || a.D < 4 || a.D > 64 || a.K < 1 || a.K > kMaxK || a.K * a.D > kMaxKD)
+    return cudaErrorInvalidValue;
+  CUtensorMap xmap, amap;
+  cudaError_t e = encode_2d(&xmap, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(a.D), unsigned(kTP));
+  if (e != cudaSuccess) return e;
+  if ((e = encode_1d(&amap, keys, CU_TENSOR_MAP_DATA_TYPE_INT32, a.N, unsigned(kTP))) != cudaSuccess) return e;
+  static bool attr_set = false;
+  if (!attr_set) {
+    e = cudaFuncSetAttribute(npp_kmupdate_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, true, xmap, amap, a);
+}
+
+}  // namespace npp

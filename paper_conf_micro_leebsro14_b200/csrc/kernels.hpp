@@ -114,4 +114,16 @@ struct RowsColsArgs {
 };
 cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int grid, cudaStream_t st);
 
+// k-means centroid update (class KU, S8 KU): x [N x D] fp32, keys [N] int32 ->
+// out [K x (D+1)] fp32 = per group (Σ x, count). Block b takes 128-point tiles [b*P, (b+1)*P).
+struct KmUpdateArgs {
+  float* out;          // [K x (D+1)]
+  double* acc;         // [K x (D+1)] fp64 accumulators (zero on entry and on exit)
+  unsigned* ticket;    // blocks done (zero on entry and on exit)
+  int64_t N, D, K;
+  int64_t per_block;   // P
+  int early_reads;     // NPP_EXEC_OVERLAP
+};
+cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st);
+
 }  // namespace npp

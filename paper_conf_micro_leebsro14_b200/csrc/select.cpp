@@ -81,7 +81,7 @@ int64_t level_chunk(int64_t N, int b, int span, int64_t factor, int vec) {
 }
 
 int acc_bytes(int pattern, int dtype) {
-  if (pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) return 8;
+  if (pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) return 8;
   return dtype == NPP_I32 ? 4 : 8;
 }
 
@@ -359,10 +359,30 @@ void r2_rowscols(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   c->claim_tiles = t.cr * t.cc;
 }
 
+// S8 KMEANS_UPDATE (class KU): 128-point tiles, contiguous ranges of P tiles, 8 warps one point at a
+// time with 2 dims per lane on x.
+bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
+  const int64_t N = n.N[0], D = n.N[1], K = n.K;
+  if (D % 4 != 0 || D < 4 || D > 64 || K < 1 || K > 256 || K * D > 2048) return false;
+  const int64_t T = cdiv(N, 128);
+  const int64_t P = cdiv(T, std::min<int64_t>(lim.sm_count, T));
+  c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
+  c->blocks[0] = 8, c->blocks[1] = 32;
+  c->persistent_grid = cdiv(T, P);
+  c->claim_tiles = P;
+  c->spans[0] = c->persistent_grid > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[0] = c->persistent_grid;
+  c->chunks[0] = c->persistent_grid > 1 ? 128 * P : N;
+  c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = D;
+  c->vec = 2;
+  c->staged = 1;
+  return true;
+}
+
 int kernel_class_of(const Nest& n, const Choice& c) {
   if (n.pattern == NPP_KMEANS_ASSIGN) return NPP_CLASS_KMEANS;
   if (n.pattern == NPP_LOGREG_GRAD) return NPP_CLASS_LOGREG;
   if (n.pattern == NPP_SUM_ROWS_COLS) return NPP_CLASS_RC;
+  if (n.pattern == NPP_KMEANS_UPDATE) return NPP_CLASS_KMUPDATE;
   return c.dims[1] == NPP_DIM_X ? NPP_CLASS_RX : NPP_CLASS_MX;
 }
 
@@ -496,6 +516,21 @@ int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
       n.acc[n.nacc++] = {0, 0x1u};  // out_rows[r]
       n.acc[n.nacc++] = {1, 0x2u};  // out_cols[c]
       n.acc[n.nacc++] = {1, 0x3u};  // m[r,c]
+      n.cols = shape[1];
+      break;
+    case NPP_KMEANS_UPDATE:  // shape {N, D, K}: groupBy over points (a Reduce into K groups), Map over dims
+      if (!need(3)) return NPP_ERR_INVALID_ARG;
+      n.L = 2;
+      n.N[0] = shape[0], n.sync[0] = true;
+      n.N[1] = shape[1], n.sync[1] = false;
+      n.K = shape[2];
+      if (n.K < 1) {
+        set_error("KMEANS_UPDATE needs K >= 1");
+        return NPP_ERR_INVALID_ARG;
+      }
+      n.acc[n.nacc++] = {1, 0x3u};  // x[i,d]
+      n.acc[n.nacc++] = {0, 0x1u};  // a[i]
+      n.acc[n.nacc++] = {1, 0x2u};  // U[k,d]
       n.cols = shape[1];
       break;
     case NPP_KMEANS_ASSIGN:  // shape {N, D, K}; levels N / K / D
@@ -633,6 +668,9 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.temp_stride[1] = c.temp_stride[1];
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
+  } else if (n.pattern == NPP_KMEANS_UPDATE && c.staged) {
+    // S9 KU: ticket (256 B) + fp64 accumulators [K x (D+1)]
+    m.workspace_bytes = 256 + 256 * cdiv(8 * n.K * (eff(n.N[1]) + 1), 256);
   } else if (n.pattern == NPP_SUM_ROWS_COLS && c.persistent_grid > 0) {
     // S9 RC: tickets [gr] + tickets [gc] (u32) + accumulators [R] + [C] of the accumulator type
     const RcTiling t = rc_tiling(n.N[0], n.N[1], dtype, lim.sm_count);
@@ -734,6 +772,13 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
     r2_rowscols(n, dtype, lim, &c);
     return record_from_choice(n, dtype, lim, c, sc, out);
   }
+  if (n.pattern == NPP_KMEANS_UPDATE) {
+    if (!r2_kmupdate(n, lim, &c)) {
+      set_error("KMEANS_UPDATE AUTO needs D % 4 == 0, 4 <= D <= 64, 1 <= K <= 256 and K*D <= 2048");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    return record_from_choice(n, dtype, lim, c, sc, out);
+  }
   if (staged_eligible(n, dtype, c))
     r2_staged(n, dtype, lim, &c);
   else
@@ -759,7 +804,8 @@ extern "C" int npp_select(int pattern, const int64_t* shape, int ndim, int dtype
   Nest n;
   st = build_nest(pattern, shape, ndim, &n);
   if (st) return st;
-  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD) && dtype != NPP_F32) {
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) &&
+      dtype != NPP_F32) {
     set_error("k-means and logreg are defined for f32");
     return NPP_ERR_UNSUPPORTED;
   }

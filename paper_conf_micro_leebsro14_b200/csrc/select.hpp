@@ -25,6 +25,7 @@ struct Nest {
   int nacc = 0;
   Access acc[kMaxAccesses];
   int64_t cols = 0;  // matrix columns (sums), for the vector-width rule of R2
+  int64_t K = 0;     // KMEANS_UPDATE: number of groups (the groupBy key range, not a nest level)
 };
 
 struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refinements

@@ -3,7 +3,7 @@
 SURVEY.md §8e / DESIGN.md §8. The outer (storage-row) dimension of every input is split into contiguous
 shards, one per rank. Where the rows are the Map level (sumRows, k-means points, logreg mini-batches)
 the shards are independent problems and no collective runs. Where the rows are the level being
-reduced (sumCols, the full-batch logreg gradient) the shard results are a cross-device Split(P) of that
+reduced (sumCols, the full-batch logreg gradient, the k-means centroid update) the shard results are a cross-device Split(P) of that
 Reduce and NCCL adds them — the only data-path collective.
 
 Every rank plans and executes its shard through libnpp.so (``compute=None``). The ``compute`` hook
@@ -63,6 +63,15 @@ def sum_cols(local: torch.Tensor, group=None, op: str = "all_reduce", dst: int =
 def kmeans_assign(local_x: torch.Tensor, centroids: torch.Tensor, group=None, compute=None):
     """Assignments of this rank's points (centroids replicated); points are independent."""
     return compute(local_x, centroids) if compute is not None else _npp().kmeans_assign(local_x, centroids)
+
+
+def kmeans_update(local_x: torch.Tensor, local_a: torch.Tensor, K: int, group=None, compute=None):
+    """Per-centroid (Σ x, count) over all ranks' points: the local [K, D+1] partial of this rank's
+    point shard, then one all-reduce of K*(D+1) floats (the groups are split across ranks: a
+    cross-device Split of the groupBy's Reduce)."""
+    u = compute(local_x, local_a, K) if compute is not None else _npp().kmeans_update(local_x, local_a, K)
+    dist.all_reduce(u, op=dist.ReduceOp.SUM, group=group)
+    return u
 
 
 def logreg_grad(local_x: torch.Tensor, local_y: torch.Tensor, w: torch.Tensor, batches: int, group=None,

@@ -19,10 +19,11 @@ OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_ALIGNMENT, ERR_WORKSPACE, ERR_NO_FEASI
 DTYPES = {"f32": 0, "i32": 1, "i64": 2}
 TORCH_DTYPES = {"f32": torch.float32, "i32": torch.int32, "i64": torch.int64}
 PATTERNS = {"SUM_ROWS": 0, "SUM_COLS": 1, "KMEANS_ASSIGN": 2, "LOGREG_GRAD": 3,
-            "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5, "SUM_ROWS_COLS": 6}
+            "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5, "SUM_ROWS_COLS": 6,
+            "KMEANS_UPDATE": 7}
 STRATEGIES = {"AUTO": 0, "LITERAL": 1, "1D": 2, "TB_T": 3, "WARP": 4}
 SPAN_ONE, SPAN_ALL, SPAN_N, SPLIT_K = 0, 1, 2, 3
-CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY, CLASS_RC = 0, 1, 2, 3, 4, 5
+CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY, CLASS_RC, CLASS_KMUPDATE = 0, 1, 2, 3, 4, 5, 6
 
 
 class NppError(RuntimeError):
@@ -240,6 +241,8 @@ class Plan:
             return (s[0] + s[1],)
         if p == "KMEANS_ASSIGN":
             return (s[0],)
+        if p == "KMEANS_UPDATE":
+            return (s[2], s[1] + 1)
         return (s[0], s[2])
 
     def out_dtype(self):
@@ -328,6 +331,14 @@ def kmeans_assign(x, c, strategy="AUTO", out=None, stream=None):
     N, D = x.shape
     p = _cached_plan("KMEANS_ASSIGN", (N, D, c.shape[0]), "f32", strategy, x.device)
     return p.execute([x, c], out if out is not None else p.new_out(), stream)
+
+
+def kmeans_update(x, a, K, out=None, stream=None):
+    """Centroid update after an assignment (groupBy a + Reduce, Table I): [K, D+1] fp32 with
+    row k = (Σ_{i: a_i = k} x_i, count_k). New centroids are U[:, :D] / U[:, D:] where the count > 0."""
+    N, D = x.shape
+    p = _cached_plan("KMEANS_UPDATE", (N, D, int(K)), "f32", "AUTO", x.device)
+    return p.execute([x, a], out if out is not None else p.new_out(), stream)
 
 
 def logreg_grad(x, y, w, B, strategy="AUTO", out=None, stream=None):

@@ -57,6 +57,8 @@ def _worker(rank, port, results):
         plo, phi = shard_range(N, WORLD, rank)
         xs, c = gen.kmeans_inputs(phi - plo, D, K, row_offset=plo)
         a = ndist.kmeans_assign(xs, c, compute=lambda x, cc: torch.from_numpy(okm.assign(x.numpy(), cc.numpy())))
+        # k-means update: each rank's [K, D+1] partial over its points, one all-reduce
+        u = ndist.kmeans_update(xs, a, K, compute=lambda x, aa, k: torch.from_numpy(okm.update(x.numpy(), aa.numpy(), k)))
         # logreg full batch: rows sharded, one all-reduce of C floats
         Rb, Cl = 200, 12
         rlo, rhi = shard_range(Rb, WORLD, rank)
@@ -64,7 +66,7 @@ def _worker(rank, port, results):
         g = ndist.logreg_grad(xl[rlo:rhi].contiguous(), yl[rlo:rhi].contiguous(), w, 1, full_batch=True,
                               compute=lambda x, y, ww, B: torch.from_numpy(olr.grad(x.numpy(), y.numpy(), ww.numpy(), B)))
         results[rank] = dict(cols=cols.numpy(), rows=rows.numpy(), cols_i=cols_i.numpy(), a=a.numpy(),
-                             g=g.numpy(), lo=lo, hi=hi)
+                             u=u.numpy(), g=g.numpy(), lo=lo, hi=hi)
     finally:
         dist.destroy_process_group()
 
@@ -97,6 +99,10 @@ def test_two_rank_gloo():
     a = np.concatenate([results[r]["a"] for r in range(WORLD)])
     x, c = gen.kmeans_inputs(301, 8, 5)
     assert a.tolist() == okm.assign(x.numpy(), c.numpy()).tolist()
+    want_u = okm.update(x.numpy(), a, 5)
+    for rank in range(WORLD):
+        assert np.allclose(results[rank]["u"], want_u, rtol=1e-12, atol=1e-9)
+        assert results[rank]["u"][:, -1].tolist() == want_u[:, -1].tolist()
     xl, yl, w = gen.logreg_inputs(1, 200, 12, seed=6)
     want_g = olr.grad(xl.numpy(), yl.numpy(), w.numpy(), 1)
     for rank in range(WORLD):

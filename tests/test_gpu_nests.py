@@ -170,3 +170,80 @@ def test_unsupported_shapes(npp, cuda_device):
     with pytest.raises(npp.NppError) as e:
         npp.Plan("KMEANS_ASSIGN", (100, 64, 3), "f32", "LITERAL")
     assert e.value.status == npp.ERR_UNSUPPORTED
+
+
+# ---------------------------------------------------------------- k-means centroid update (class KU)
+
+def _check_update(u, x, a, K):
+    """Sums within 1e-5 * Σ|x| of the fp64 oracle per element (signed data); counts exact."""
+    xn, an = x.cpu().numpy(), a.cpu().numpy()
+    want = okm.update(xn, an, K)
+    scale = okm.update_scale(xn, an, K)
+    got = u.cpu().numpy().astype(np.float64)
+    assert np.array_equal(got[:, -1], want[:, -1]), "counts"
+    err = np.abs(got[:, :-1] - want[:, :-1])
+    bad = np.argwhere(err > 1e-5 * scale + 1e-30)
+    assert bad.size == 0, (bad[:4], got[tuple(bad[0])], want[tuple(bad[0])])
+
+
+@pytest.mark.parametrize("N,D,K", [(1, 4, 1), (127, 8, 3), (129, 64, 32), (3000, 64, 32), (10007, 60, 34),
+                                   (5000, 4, 256), (70000, 16, 128), (200000, 64, 32), (33, 32, 64)])
+def test_kmeans_update_parity(npp, cuda_device, N, D, K):
+    # random keys in [-1, K] (the out-of-range ones belong to no group), ragged last tile, every
+    # warp-row / flush boundary; back-to-back executes (plain and PDL-overlapped) leave the workspace zero
+    x, _ = gen.kmeans_inputs(N, D, max(K, 1), seed=40 + K, device=cuda_device)
+    a = gen.int_uniform(41, (N,), -1, K, device=cuda_device)
+    p = npp.Plan("KMEANS_UPDATE", (N, D, K))
+    assert p.mapping == osel.select("KMEANS_UPDATE", (N, D, K), "f32", npp.limits_query(0), "AUTO")
+    assert p.mapping["kernel_class"] == npp.CLASS_KMUPDATE
+    outs = [p.execute([x, a], p.new_out()), p.execute([x, a], p.new_out(), overlap=True)]
+    torch.cuda.synchronize()
+    for u in outs:
+        _check_update(u, x, a, K)
+    assert int(p.workspace.count_nonzero()) == 0
+
+
+def test_kmeans_update_integer_exact(npp, cuda_device):
+    # integer coordinates: every partial sum is an exact fp32 integer (|U| < 2^24), so bit-exact
+    N, D, K = 50000, 64, 32
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device, integer=True)
+    a = npp.kmeans_assign(x, c)
+    u = npp.kmeans_update(x, a, K)
+    torch.cuda.synchronize()
+    assert np.array_equal(u.cpu().numpy().astype(np.float64), okm.update(x.cpu().numpy(), a.cpu().numpy(), K))
+
+
+def test_lloyd_step_full_size(npp, cuda_device):
+    # one Lloyd iteration on the BASELINE.json k-means configuration (4M x 64 x 32): assignment, then
+    # the update, both on the GPU; the update is checked against the oracle on the GPU's assignment
+    # (sampled: the first 1M points through a second plan), and the full-size update by its invariants
+    N, D, K = 1 << 22, 64, 32
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
+    a = npp.kmeans_assign(x, c)
+    u = npp.kmeans_update(x, a, K)
+    n1 = 1 << 20
+    u1 = npp.Plan("KMEANS_UPDATE", (n1, D, K)).execute([x[:n1], a[:n1]], torch.empty(K, D + 1, device=cuda_device))
+    torch.cuda.synchronize()
+    _check_update(u1, x[:n1], a[:n1], K)
+    un = u.cpu().numpy().astype(np.float64)
+    assert un[:, -1].sum() == N                                           # every point in one group
+    colsum = x.double().sum(0).cpu().numpy()                              # Σ_k U[k] = Σ_i x_i
+    assert np.all(np.abs(un[:, :-1].sum(0) - colsum) <= 1e-5 * x.double().abs().sum(0).cpu().numpy())
+    counts = torch.bincount(a.long(), minlength=K).cpu().numpy()
+    assert np.array_equal(un[:, -1], counts)
+
+
+def test_kmeans_update_plan_rules(npp, cuda_device):
+    for strategy in ("LITERAL", "1D", "TB_T", "WARP"):
+        with pytest.raises(npp.NppError) as e:
+            npp.Plan("KMEANS_UPDATE", (100, 64, 32), "f32", strategy)
+        assert e.value.status == npp.ERR_UNSUPPORTED
+    for shape in [(100, 66, 4), (100, 128, 4), (100, 64, 33), (100, 8, 257)]:
+        with pytest.raises(npp.NppError) as e:
+            npp.Plan("KMEANS_UPDATE", shape)
+        assert e.value.status == npp.ERR_UNSUPPORTED
+    p = npp.Plan("KMEANS_UPDATE", (0, 8, 3))   # no points: every group empty
+    u = p.execute([torch.empty(0, 8, device=cuda_device), torch.empty(0, dtype=torch.int32, device=cuda_device)],
+                  torch.full((3, 9), 5.0, device=cuda_device))
+    torch.cuda.synchronize()
+    assert float(u.abs().sum()) == 0.0

@@ -62,6 +62,15 @@ def test_three_level_literal(profile):
         _cmp("KMEANS_ASSIGN", (1000, 64, 32), "f32", lim, strat)
 
 
+@pytest.mark.parametrize("profile", list(PROFILES))
+def test_kmeans_update_parity(profile):
+    lim = PROFILES[profile]
+    for shape in [(1 << 22, 64, 32), (1000, 3, 5), (17, 64, 1), (64, 4, 256), (4099, 60, 34), (128, 64, 33),
+                  (1, 8, 8), (300, 128, 4), (5000, 16, 300)]:
+        for strat in SUM_STRATS:
+            _cmp("KMEANS_UPDATE", shape, "f32", lim, strat)
+
+
 def test_unknown_sizes_literal():
     for shape in [(-1, 1024), (1024, -1), (-1, -1)]:
         for pattern in ("SUM_ROWS", "SUM_COLS"):
