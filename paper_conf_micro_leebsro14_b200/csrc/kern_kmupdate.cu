@@ -9,10 +9,8 @@
 //   Consumer warp w adds points w, w+8, ... of each tile: lane l owns dims 2l, 2l+1 (float2), so a
 //   point is one conflict-free 8-byte read of the tile plus a read-modify-write of the warp's OWN
 //   fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are CAS loops on
-//   sm_100a). Points go 8 at a time: a point whose key repeats an earlier one of the 8 is added into
-//   that point's value first, so the remaining row updates are independent and overlap (the serial
-//   load-add-store chain per point was the limit: ncu short-scoreboard stalls, 405 -> 235 µs with 4
-//   distinct-key points per step);
+//   sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are independent and
+//   overlap (the serial load-add-store chain per point was the limit: ncu short-scoreboard stalls);
 //   counts come from one match.any per tile (the lowest lane of each key group adds its size). Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
 //   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
@@ -149,45 +147,46 @@ __global__ void __launch_bounds__(kThreads, 1)
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
     const unsigned same = __match_any_sync(0xffffffffu, kl);
     if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
-    // sums: 8 points at a time. Points whose key repeats an earlier key of the 8 are first added into
-    // that point's value (warp-uniform tests), so the remaining row updates have distinct rows and
-    // their read-modify-writes are independent: 8 loads, adds and stores back to back
-    constexpr int kStep = 8;
+    // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
+    // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
+    // 4 points go one after the other (the rows may coincide)
 #pragma unroll
-    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += kStep) {
-      int k[kStep];
-      float2 xv[kStep];
+    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
+      int k[4];
+      float2 xv[4];
 #pragma unroll
-      for (int q = 0; q < kStep; ++q) {
+      for (int q = 0; q < 4; ++q) {
         k[q] = __shfl_sync(0xffffffffu, kl, j0 + q);
         xv[q] = make_float2(0.f, 0.f);
         if (k[q] >= 0 && dim_lane)
           xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
       }
-#pragma unroll
-      for (int q = 1; q < kStep; ++q) {
-        bool merged = false;
-#pragma unroll
-        for (int r = 0; r < q; ++r)
-          if (!merged && k[q] >= 0 && k[r] == k[q]) {
-            xv[r].x += xv[q].x;
-            xv[r].y += xv[q].y;
-            merged = true;
-          }
-        if (merged) k[q] = -1;
-      }
       if (!dim_lane) continue;
-      float2 v[kStep];
+      const bool distinct = (k[0] != k[1] || k[0] < 0) && (k[0] != k[2] || k[0] < 0) && (k[0] != k[3] || k[0] < 0) &&
+                            (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
+      if (distinct) {
+        float2 v[4];
 #pragma unroll
-      for (int q = 0; q < kStep; ++q)
-        if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
 #pragma unroll
-      for (int q = 0; q < kStep; ++q)
-        if (k[q] >= 0) {
-          v[q].x += xv[q].x;
-          v[q].y += xv[q].y;
-          *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
-        }
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) {
+            v[q].x += xv[q].x;
+            v[q].y += xv[q].y;
+            *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
+          }
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) {
+            float2* acc = reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane);
+            float2 v = *acc;
+            v.x += xv[q].x;
+            v.y += xv[q].y;
+            *acc = v;
+          }
+      }
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(empty + slot);
