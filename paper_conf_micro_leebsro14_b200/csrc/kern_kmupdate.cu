@@ -6,12 +6,13 @@
 // 128 rows x D floats; a: 1-D box of 128 ints) stream through a 4-deep mbarrier ring, one block per
 // SM, contiguous tile ranges. The data-dependent key is why this is not a sum family: the reduction
 // target of a point is only known when its a_i arrives.
-//   Consumer warp w adds points w, w+8, ... of each tile: lane l owns dims 2l, 2l+1 (float2), so a
-//   point is one conflict-free 8-byte read of the tile plus a read-modify-write of the warp's OWN
-//   fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are CAS loops on
-//   sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are independent and
-//   overlap (the serial load-add-store chain per point was the limit: ncu short-scoreboard stalls);
-//   counts come from one match.any per tile (the lowest lane of each key group adds its size). Every 8 tiles (<= 128 points per warp accumulator, so the
+//   Consumer warp w adds points w, w+8, ... of each tile, two per step: half-warp h takes one point,
+//   lane l owns dims 4(l%16)..+3 (float4), so a point is one 16-byte read of the tile plus a 16-byte
+//   read-modify-write of the warp's OWN fp32 accumulator row k in shared memory (no atomics:
+//   shared-memory float atomics are CAS loops on sm_100a). Counts come from one match.any per tile
+//   (the lowest lane of each key group adds its size). Measured: one point per warp step with a
+//   per-point count update 405 µs; 4 points per step with independent row updates 235 µs (issue-
+//   bound: ~230 instructions per warp per tile); this layout halves the per-point instructions. Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
 //   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
 //   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
@@ -105,18 +106,24 @@ __global__ void __launch_bounds__(kThreads, 1)
   // -------------------------------------------------------------- consumers
   float* myacc = accw + warp * KD;
   unsigned* mycnt = cntw + warp * K;
-  const bool dim_lane = 2 * lane < D;
+  const int half = lane >> 4, hl = lane & 15;
+  const bool dim_lane = 4 * hl < D;
+  int krow[kMaxKD / kConsumers];  // flush: accumulator row of element tid + 256 r (no division per flush)
+#pragma unroll
+  for (int r = 0; r < kMaxKD / kConsumers; ++r) krow[r] = (int(threadIdx.x) + kConsumers * r) / D;
   auto flush = [&]() {  // fold the 8 warp copies into the fp64 block accumulator, zero the copies
     consumers_sync();
-    for (int i = threadIdx.x; i < KD; i += kConsumers) {
+#pragma unroll
+    for (int r = 0; r < kMaxKD / kConsumers; ++r) {
+      const int i = int(threadIdx.x) + kConsumers * r;
+      if (i >= KD) break;
       double s = 0.0;
 #pragma unroll
       for (int w = 0; w < kConsumerWarps; ++w) {
         s += double(accw[w * KD + i]);
         accw[w * KD + i] = 0.f;
       }
-      const int k = i / D;
-      bacc[i + k] += s;  // row k of [K x (D+1)]
+      bacc[i + krow[r]] += s;  // row k of [K x (D+1)]
     }
     for (int k = threadIdx.x; k < K; k += kConsumers) {
       unsigned c = 0;
@@ -147,45 +154,32 @@ __global__ void __launch_bounds__(kThreads, 1)
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
     const unsigned same = __match_any_sync(0xffffffffu, kl);
     if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
-    // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
-    // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
-    // 4 points go one after the other (the rows may coincide)
-#pragma unroll
-    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
-      int k[4];
-      float2 xv[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        k[q] = __shfl_sync(0xffffffffu, kl, j0 + q);
-        xv[q] = make_float2(0.f, 0.f);
-        if (k[q] >= 0 && dim_lane)
-          xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
+    // sums: the two half-warps take points 2s and 2s+1 of the warp's 16 (lane l: dims 4(l%16)..+3,
+    // one 16-byte read of the tile and one 16-byte read-modify-write of the warp's accumulator row per
+    // point). Equal keys in one step (a warp-uniform test) would make the halves update one row: the
+    // second half hands its value to the first through shuffles and skips its update.
+#pragma unroll 4
+    for (int s = 0; s < kTP / kConsumerWarps / 2; ++s) {
+      const int j = 2 * s + half;
+      int k = __shfl_sync(0xffffffffu, kl, j);
+      const int kp = __shfl_xor_sync(0xffffffffu, k, 16);
+      float4 xv = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (k >= 0 && dim_lane)
+        xv = *reinterpret_cast<const float4*>(xt + (warp + kConsumerWarps * j) * D + 4 * hl);
+      if (k == kp && k >= 0) {
+        const float ox = __shfl_xor_sync(0xffffffffu, xv.x, 16), oy = __shfl_xor_sync(0xffffffffu, xv.y, 16);
+        const float oz = __shfl_xor_sync(0xffffffffu, xv.z, 16), ow = __shfl_xor_sync(0xffffffffu, xv.w, 16);
+        if (half == 0) {
+          xv.x += ox, xv.y += oy, xv.z += oz, xv.w += ow;
+        } else {
+          k = -1;
+        }
       }
-      if (!dim_lane) continue;
-      const bool distinct = (k[0] != k[1] || k[0] < 0) && (k[0] != k[2] || k[0] < 0) && (k[0] != k[3] || k[0] < 0) &&
-                            (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
-      if (distinct) {
-        float2 v[4];
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) {
-            v[q].x += xv[q].x;
-            v[q].y += xv[q].y;
-            *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
-          }
-      } else {
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) {
-            float2* acc = reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane);
-            float2 v = *acc;
-            v.x += xv[q].x;
-            v.y += xv[q].y;
-            *acc = v;
-          }
+      if (k >= 0 && dim_lane) {
+        float4* acc = reinterpret_cast<float4*>(myacc + k * D + 4 * hl);
+        float4 v = *acc;
+        v.x += xv.x, v.y += xv.y, v.z += xv.z, v.w += xv.w;
+        *acc = v;
       }
     }
     __syncwarp();
