@@ -12,7 +12,8 @@
 //   shared-memory float atomics are CAS loops on sm_100a). Counts come from one match.any per tile
 //   (the lowest lane of each key group adds its size). Measured: one point per warp step with a
 //   per-point count update 405 µs; 4 points per step with independent row updates 235 µs (issue-
-//   bound: ~230 instructions per warp per tile); this layout halves the per-point instructions. Every 8 tiles (<= 128 points per warp accumulator, so the
+//   bound: ~230 instructions per warp per tile); half-warp points, one step at a time 279 µs (the
+//   dependent row updates serialise); half-warp points two steps at a time (this version). Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
 //   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
 //   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
@@ -156,30 +157,55 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     // sums: the two half-warps take points 2s and 2s+1 of the warp's 16 (lane l: dims 4(l%16)..+3,
     // one 16-byte read of the tile and one 16-byte read-modify-write of the warp's accumulator row per
-    // point). Equal keys in one step (a warp-uniform test) would make the halves update one row: the
-    // second half hands its value to the first through shuffles and skips its update.
-#pragma unroll 4
-    for (int s = 0; s < kTP / kConsumerWarps / 2; ++s) {
-      const int j = 2 * s + half;
-      int k = __shfl_sync(0xffffffffu, kl, j);
-      const int kp = __shfl_xor_sync(0xffffffffu, k, 16);
-      float4 xv = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (k >= 0 && dim_lane)
-        xv = *reinterpret_cast<const float4*>(xt + (warp + kConsumerWarps * j) * D + 4 * hl);
-      if (k == kp && k >= 0) {
-        const float ox = __shfl_xor_sync(0xffffffffu, xv.x, 16), oy = __shfl_xor_sync(0xffffffffu, xv.y, 16);
-        const float oz = __shfl_xor_sync(0xffffffffu, xv.z, 16), ow = __shfl_xor_sync(0xffffffffu, xv.w, 16);
-        if (half == 0) {
-          xv.x += ox, xv.y += oy, xv.z += oz, xv.w += ow;
-        } else {
-          k = -1;
+    // point). Two steps (4 points) go together: when their 4 keys differ (a warp-uniform test) the
+    // row updates are independent and overlap; otherwise the steps run one after the other, and equal
+    // keys inside one step make the second half hand its value to the first through shuffles.
+    auto point = [&](int j) -> float4 {
+      return *reinterpret_cast<const float4*>(xt + (warp + kConsumerWarps * j) * D + 4 * hl);
+    };
+    auto rmw = [&](int k, const float4& xv) {
+      float4* acc = reinterpret_cast<float4*>(myacc + k * D + 4 * hl);
+      float4 v = *acc;
+      v.x += xv.x, v.y += xv.y, v.z += xv.z, v.w += xv.w;
+      *acc = v;
+    };
+#pragma unroll 2
+    for (int s = 0; s < kTP / kConsumerWarps / 2; s += 2) {
+      const int k0 = __shfl_sync(0xffffffffu, kl, 2 * s + half);
+      const int k1 = __shfl_sync(0xffffffffu, kl, 2 * s + 2 + half);
+      const int k0p = __shfl_xor_sync(0xffffffffu, k0, 16), k1p = __shfl_xor_sync(0xffffffffu, k1, 16);
+      float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
+      if (k0 >= 0 && dim_lane) x0 = point(2 * s + half);
+      if (k1 >= 0 && dim_lane) x1 = point(2 * s + 2 + half);
+      auto ne = [](int a, int b) { return a != b || a < 0; };
+      const bool distinct = ne(k0, k0p) && ne(k0, k1) && ne(k0, k1p) && ne(k0p, k1) && ne(k0p, k1p) && ne(k1, k1p);
+      if (distinct) {
+        if (dim_lane) {
+          float4* a0 = reinterpret_cast<float4*>(myacc + (k0 < 0 ? 0 : k0) * D + 4 * hl);
+          float4* a1 = reinterpret_cast<float4*>(myacc + (k1 < 0 ? 0 : k1) * D + 4 * hl);
+          float4 v0 = *a0, v1 = *a1;
+          v0.x += x0.x, v0.y += x0.y, v0.z += x0.z, v0.w += x0.w;
+          v1.x += x1.x, v1.y += x1.y, v1.z += x1.z, v1.w += x1.w;
+          if (k0 >= 0) *a0 = v0;
+          if (k1 >= 0) *a1 = v1;
         }
-      }
-      if (k >= 0 && dim_lane) {
-        float4* acc = reinterpret_cast<float4*>(myacc + k * D + 4 * hl);
-        float4 v = *acc;
-        v.x += xv.x, v.y += xv.y, v.z += xv.z, v.w += xv.w;
-        *acc = v;
+      } else {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          int k = q ? k1 : k0;
+          const int kp = q ? k1p : k0p;
+          float4 xv = q ? x1 : x0;
+          if (k == kp && k >= 0) {  // warp-uniform: both halves hold points of row k
+            const float ox = __shfl_xor_sync(0xffffffffu, xv.x, 16), oy = __shfl_xor_sync(0xffffffffu, xv.y, 16);
+            const float oz = __shfl_xor_sync(0xffffffffu, xv.z, 16), ow = __shfl_xor_sync(0xffffffffu, xv.w, 16);
+            if (half == 0)
+              xv.x += ox, xv.y += oy, xv.z += oz, xv.w += ow;
+            else
+              k = -1;
+          }
+          if (k >= 0 && dim_lane) rmw(k, xv);
+          __syncwarp();
+        }
       }
     }
     __syncwarp();
