@@ -6,14 +6,15 @@
 // 128 rows x D floats; a: 1-D box of 128 ints) stream through a 4-deep mbarrier ring, one block per
 // SM, contiguous tile ranges. The data-dependent key is why this is not a sum family: the reduction
 // target of a point is only known when its a_i arrives.
-//   Consumer warp w adds points w, w+8, ... of each tile, two per step: half-warp h takes one point,
-//   lane l owns dims 4(l%16)..+3 (float4), so a point is one 16-byte read of the tile plus a 16-byte
-//   read-modify-write of the warp's OWN fp32 accumulator row k in shared memory (no atomics:
-//   shared-memory float atomics are CAS loops on sm_100a). Counts come from one match.any per tile
-//   (the lowest lane of each key group adds its size). Measured: one point per warp step with a
-//   per-point count update 405 µs; 4 points per step with independent row updates 235 µs (issue-
-//   bound: ~230 instructions per warp per tile); half-warp points, one step at a time 279 µs (the
-//   dependent row updates serialise); half-warp points two steps at a time (this version). Every 8 tiles (<= 128 points per warp accumulator, so the
+//   Consumer warp w adds points w, w+8, ... of each tile: lane l owns dims 2l, 2l+1 (float2), so a
+//   point is one conflict-free 8-byte read of the tile plus a read-modify-write of the warp's OWN
+//   fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are CAS loops on
+//   sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are independent and
+//   overlap (the serial load-add-store chain per point was the limit: ncu short-scoreboard stalls,
+//   405 -> 235 µs); counts come from one match.any per tile (the lowest lane of each key group adds
+//   its size). Measured and dropped: 8 points per step with repeated keys merged first (331 µs: the
+//   merge tests cost more than the overlap gains), half-warp points with float4 lanes one step
+//   (279 µs) or two steps (280 µs) at a time. Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
 //   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
 //   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
@@ -107,8 +108,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   // -------------------------------------------------------------- consumers
   float* myacc = accw + warp * KD;
   unsigned* mycnt = cntw + warp * K;
-  const int half = lane >> 4, hl = lane & 15;
-  const bool dim_lane = 4 * hl < D;
+  const bool dim_lane = 2 * lane < D;
   int krow[kMaxKD / kConsumers];  // flush: accumulator row of element tid + 256 r (no division per flush)
 #pragma unroll
   for (int r = 0; r < kMaxKD / kConsumers; ++r) krow[r] = (int(threadIdx.x) + kConsumers * r) / D;
@@ -155,57 +155,45 @@ __global__ void __launch_bounds__(kThreads, 1)
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
     const unsigned same = __match_any_sync(0xffffffffu, kl);
     if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
-    // sums: the two half-warps take points 2s and 2s+1 of the warp's 16 (lane l: dims 4(l%16)..+3,
-    // one 16-byte read of the tile and one 16-byte read-modify-write of the warp's accumulator row per
-    // point). Two steps (4 points) go together: when their 4 keys differ (a warp-uniform test) the
-    // row updates are independent and overlap; otherwise the steps run one after the other, and equal
-    // keys inside one step make the second half hand its value to the first through shuffles.
-    auto point = [&](int j) -> float4 {
-      return *reinterpret_cast<const float4*>(xt + (warp + kConsumerWarps * j) * D + 4 * hl);
-    };
-    auto rmw = [&](int k, const float4& xv) {
-      float4* acc = reinterpret_cast<float4*>(myacc + k * D + 4 * hl);
-      float4 v = *acc;
-      v.x += xv.x, v.y += xv.y, v.z += xv.z, v.w += xv.w;
-      *acc = v;
-    };
-#pragma unroll 2
-    for (int s = 0; s < kTP / kConsumerWarps / 2; s += 2) {
-      const int k0 = __shfl_sync(0xffffffffu, kl, 2 * s + half);
-      const int k1 = __shfl_sync(0xffffffffu, kl, 2 * s + 2 + half);
-      const int k0p = __shfl_xor_sync(0xffffffffu, k0, 16), k1p = __shfl_xor_sync(0xffffffffu, k1, 16);
-      float4 x0 = make_float4(0.f, 0.f, 0.f, 0.f), x1 = x0;
-      if (k0 >= 0 && dim_lane) x0 = point(2 * s + half);
-      if (k1 >= 0 && dim_lane) x1 = point(2 * s + 2 + half);
-      auto ne = [](int a, int b) { return a != b || a < 0; };
-      const bool distinct = ne(k0, k0p) && ne(k0, k1) && ne(k0, k1p) && ne(k0p, k1) && ne(k0p, k1p) && ne(k1, k1p);
+    // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
+    // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
+    // 4 points go one after the other (the rows may coincide)
+#pragma unroll
+    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
+      int k[4];
+      float2 xv[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        k[q] = __shfl_sync(0xffffffffu, kl, j0 + q);
+        xv[q] = make_float2(0.f, 0.f);
+        if (k[q] >= 0 && dim_lane)
+          xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
+      }
+      if (!dim_lane) continue;
+      const bool distinct = (k[0] != k[1] || k[0] < 0) && (k[0] != k[2] || k[0] < 0) && (k[0] != k[3] || k[0] < 0) &&
+                            (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
       if (distinct) {
-        if (dim_lane) {
-          float4* a0 = reinterpret_cast<float4*>(myacc + (k0 < 0 ? 0 : k0) * D + 4 * hl);
-          float4* a1 = reinterpret_cast<float4*>(myacc + (k1 < 0 ? 0 : k1) * D + 4 * hl);
-          float4 v0 = *a0, v1 = *a1;
-          v0.x += x0.x, v0.y += x0.y, v0.z += x0.z, v0.w += x0.w;
-          v1.x += x1.x, v1.y += x1.y, v1.z += x1.z, v1.w += x1.w;
-          if (k0 >= 0) *a0 = v0;
-          if (k1 >= 0) *a1 = v1;
-        }
+        float2 v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) {
+            v[q].x += xv[q].x;
+            v[q].y += xv[q].y;
+            *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
+          }
       } else {
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
-          int k = q ? k1 : k0;
-          const int kp = q ? k1p : k0p;
-          float4 xv = q ? x1 : x0;
-          if (k == kp && k >= 0) {  // warp-uniform: both halves hold points of row k
-            const float ox = __shfl_xor_sync(0xffffffffu, xv.x, 16), oy = __shfl_xor_sync(0xffffffffu, xv.y, 16);
-            const float oz = __shfl_xor_sync(0xffffffffu, xv.z, 16), ow = __shfl_xor_sync(0xffffffffu, xv.w, 16);
-            if (half == 0)
-              xv.x += ox, xv.y += oy, xv.z += oz, xv.w += ow;
-            else
-              k = -1;
+        for (int q = 0; q < 4; ++q)
+          if (k[q] >= 0) {
+            float2* acc = reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane);
+            float2 v = *acc;
+            v.x += xv[q].x;
+            v.y += xv[q].y;
+            *acc = v;
           }
-          if (k >= 0 && dim_lane) rmw(k, xv);
-          __syncwarp();
-        }
       }
     }
     __syncwarp();
