@@ -11,8 +11,8 @@
 //   fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are CAS loops on
 //   sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are independent and
 //   overlap (the serial load-add-store chain per point was the limit: ncu short-scoreboard stalls,
-//   405 -> 235 µs); lane 0 updates the count next to each row update (one match.any per tile for the
-//   counts measured slower: 232.8 µs). Measured and dropped: 8 points per step with repeated keys merged first (331 µs: the
+//   405 -> 235 µs); counts come from one match.any per tile (the lowest lane of each key group adds
+//   its size). Measured and dropped: 8 points per step with repeated keys merged first (331 µs: the
 //   merge tests cost more than the overlap gains), half-warp points with float4 lanes one step
 //   (279 µs) or two steps (280 µs) at a time. Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
@@ -152,6 +152,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       kl = at[warp + kConsumerWarps * lane];
       if (unsigned(kl) >= unsigned(K)) kl = -1;
     }
+    // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
+    const unsigned same = __match_any_sync(0xffffffffu, kl);
+    if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
     // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
     // 4 points go one after the other (the rows may coincide)
@@ -171,20 +174,15 @@ __global__ void __launch_bounds__(kThreads, 1)
                             (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
       if (distinct) {
         float2 v[4];
-        unsigned c[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) {
-            v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
-            if (lane == 0) c[q] = mycnt[k[q]];
-          }
+          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
 #pragma unroll
         for (int q = 0; q < 4; ++q)
           if (k[q] >= 0) {
             v[q].x += xv[q].x;
             v[q].y += xv[q].y;
             *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
-            if (lane == 0) mycnt[k[q]] = c[q] + 1u;
           }
       } else {
 #pragma unroll
@@ -195,7 +193,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             v.x += xv[q].x;
             v.y += xv[q].y;
             *acc = v;
-            if (lane == 0) mycnt[k[q]] += 1u;
           }
       }
     }
