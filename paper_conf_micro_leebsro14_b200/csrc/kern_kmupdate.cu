@@ -14,7 +14,8 @@
 //   405 -> 235 µs); counts come from one match.any per tile (the lowest lane of each key group adds
 //   its size). Measured and dropped: 8 points per step with repeated keys merged first (331 µs: the
 //   merge tests cost more than the overlap gains), half-warp points with float4 lanes one step
-//   (279 µs) or two steps (280 µs) at a time. Every 8 tiles (<= 128 points per warp accumulator, so the
+//   (279 µs) or two steps (280 µs) at a time, counts updated by lane 0 next to each row update
+//   instead of the match.any (306 µs: divergent lane-0 branches). Every 8 tiles (<= 128 points per warp accumulator, so the
 //   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
 //   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
 //   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
