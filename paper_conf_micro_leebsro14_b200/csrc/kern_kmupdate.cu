@@ -38,17 +38,15 @@ constexpr int kStages = 4;
 constexpr int kTP = 128;                  // points per tile
 constexpr int kXSlot = 32 * 1024;         // kTP * D * 4 <= 32 KB (D <= 64)
 constexpr int kASlot = kTP * 4;           // 512 B of keys
-constexpr int kPointWarps = 8;                         // warps across a tile's points
-constexpr int kHalves = 2;                             // warps across a point's dims
-constexpr int kConsumerWarps = kPointWarps * kHalves;  // 16: each owns one fp32 copy of [K x D/2]
+constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
 constexpr int kMaxKD = 2048;               // DESIGN.md S8 KU: K*D <= 2048, K <= 256
 constexpr int kMaxK = 256;
 constexpr int kFlushTiles = 8;
-constexpr int kSmemBytes = kHeader + kStages * (kXSlot + kASlot) + kConsumerWarps * (kMaxKD / kHalves) * 4 +
-                           kPointWarps * kMaxK * 4 + (kMaxKD + kMaxK) * 8;
+constexpr int kSmemBytes = kHeader + kStages * (kXSlot + kASlot) + kConsumerWarps * kMaxKD * 4 +
+                           kConsumerWarps * kMaxK * 4 + (kMaxKD + kMaxK) * 8;
 
 __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
 
@@ -63,11 +61,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   volatile int* flag = reinterpret_cast<volatile int*>(empty + kStages);
   unsigned char* xring = smem + kHeader;
   unsigned char* aring = xring + kStages * kXSlot;
-  float* accw = reinterpret_cast<float*>(aring + kStages * kASlot);  // [16][K][D/2]
-  unsigned* cntw = reinterpret_cast<unsigned*>(accw + kConsumerWarps * (kMaxKD / kHalves));  // [8][K]
-  double* bacc = reinterpret_cast<double*>(cntw + kPointWarps * kMaxK);  // [K*(D+1)]
+  float* accw = reinterpret_cast<float*>(aring + kStages * kASlot);           // [8][K*D]
+  unsigned* cntw = reinterpret_cast<unsigned*>(accw + kConsumerWarps * kMaxKD);  // [8][K]
+  double* bacc = reinterpret_cast<double*>(cntw + kConsumerWarps * kMaxK);     // [K*(D+1)]
   const int D = int(a.D), K = int(a.K), KD = K * D, KD1 = K * (D + 1);
-  const int DH = D / kHalves, KDH = K * DH;
 
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
@@ -84,8 +81,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     mbar_fence_init();
   }
   if (threadIdx.x < kConsumers) {
-    for (int i = threadIdx.x; i < kConsumerWarps * KDH; i += kConsumers) accw[i] = 0.f;
-    for (int i = threadIdx.x; i < kPointWarps * K; i += kConsumers) cntw[i] = 0u;
+    for (int i = threadIdx.x; i < kConsumerWarps * KD; i += kConsumers) accw[i] = 0.f;
+    for (int i = threadIdx.x; i < kConsumerWarps * K; i += kConsumers) cntw[i] = 0u;
     for (int i = threadIdx.x; i < KD1; i += kConsumers) bacc[i] = 0.0;
   }
   __syncthreads();
@@ -110,10 +107,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 
   // -------------------------------------------------------------- consumers
-  const int pw = warp % kPointWarps, hd = warp / kPointWarps;  // points pw + 8j, dims hd*D/2 + lane
-  float* myacc = accw + warp * KDH;
-  unsigned* mycnt = cntw + pw * K;
-  const bool dim_lane = lane < DH;
+  float* myacc = accw + warp * KD;
+  unsigned* mycnt = cntw + warp * K;
+  const bool dim_lane = 2 * lane < D;
   int krow[kMaxKD / kConsumers];  // flush: accumulator row of element tid + 256 r (no division per flush)
 #pragma unroll
   for (int r = 0; r < kMaxKD / kConsumers; ++r) krow[r] = (int(threadIdx.x) + kConsumers * r) / D;
@@ -123,21 +119,18 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int r = 0; r < kMaxKD / kConsumers; ++r) {
       const int i = int(threadIdx.x) + kConsumers * r;
       if (i >= KD) break;
-      const int k = krow[r], d = i - k * D;
-      const int h = d >= DH ? 1 : 0;
-      const int e = k * DH + d - h * DH;  // element of the half-h copies
       double s = 0.0;
 #pragma unroll
-      for (int w = 0; w < kPointWarps; ++w) {
-        s += double(accw[(w + kPointWarps * h) * KDH + e]);
-        accw[(w + kPointWarps * h) * KDH + e] = 0.f;
+      for (int w = 0; w < kConsumerWarps; ++w) {
+        s += double(accw[w * KD + i]);
+        accw[w * KD + i] = 0.f;
       }
-      bacc[i + k] += s;  // row k of [K x (D+1)]
+      bacc[i + krow[r]] += s;  // row k of [K x (D+1)]
     }
     for (int k = threadIdx.x; k < K; k += kConsumers) {
       unsigned c = 0;
 #pragma unroll
-      for (int w = 0; w < kPointWarps; ++w) {
+      for (int w = 0; w < kConsumerWarps; ++w) {
         c += cntw[w * K + k];
         cntw[w * K + k] = 0u;
       }
@@ -156,43 +149,52 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int np = a.N - base < kTP ? int(a.N - base) : kTP;  // valid points (TMA zero-fills the rest)
     // the warp's 16 points of the tile are p = warp + 8j: lane j < 16 reads key j (-1: no group)
     int kl = -1;
-    if (lane < kTP / kPointWarps && pw + kPointWarps * lane < np) {
-      kl = at[pw + kPointWarps * lane];
+    if (lane < kTP / kConsumerWarps && warp + kConsumerWarps * lane < np) {
+      kl = at[warp + kConsumerWarps * lane];
       if (unsigned(kl) >= unsigned(K)) kl = -1;
     }
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
-    if (hd == 0) {  // warp-uniform: the first dim half counts
-      const unsigned same = __match_any_sync(0xffffffffu, kl);
-      if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
-    }
+    const unsigned same = __match_any_sync(0xffffffffu, kl);
+    if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
     // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
     // 4 points go one after the other (the rows may coincide)
 #pragma unroll
-    for (int j0 = 0; j0 < kTP / kPointWarps; j0 += 4) {
+    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
       int k[4];
-      float xv[4];
+      float2 xv[4];
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         k[q] = __shfl_sync(0xffffffffu, kl, j0 + q);
-        xv[q] = 0.f;
-        if (k[q] >= 0 && dim_lane) xv[q] = xt[(pw + kPointWarps * (j0 + q)) * D + hd * DH + lane];
+        xv[q] = make_float2(0.f, 0.f);
+        if (k[q] >= 0 && dim_lane)
+          xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
       }
       if (!dim_lane) continue;
       const bool distinct = (k[0] != k[1] || k[0] < 0) && (k[0] != k[2] || k[0] < 0) && (k[0] != k[3] || k[0] < 0) &&
                             (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
       if (distinct) {
-        float v[4];
+        float2 v[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) v[q] = myacc[k[q] * DH + lane];
+          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) myacc[k[q] * DH + lane] = v[q] + xv[q];
+          if (k[q] >= 0) {
+            v[q].x += xv[q].x;
+            v[q].y += xv[q].y;
+            *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
+          }
       } else {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) myacc[k[q] * DH + lane] += xv[q];
+          if (k[q] >= 0) {
+            float2* acc = reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane);
+            float2 v = *acc;
+            v.x += xv[q].x;
+            v.y += xv[q].y;
+            *acc = v;
+          }
       }
     }
     __syncwarp();
