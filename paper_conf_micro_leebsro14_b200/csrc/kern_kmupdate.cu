@@ -139,14 +139,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     consumers_sync();
   };
   int since = 0;
-  for (long long t = t0; t < t1; ++t) {
-    const long long i = t - t0;
-    const int slot = int(i % kStages);
-    mbar_wait(full + slot, unsigned((i / kStages) & 1));
+  int slot = 0;
+  unsigned phase = 0;
+  for (long long t = t0; t < t1; ++t, slot = slot + 1 == kStages ? 0 : slot + 1, phase ^= slot == 0 ? 1u : 0u) {
+    mbar_wait(full + slot, phase);
     const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
     const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
-    const long long base = t * kTP;
-    const int np = a.N - base < kTP ? int(a.N - base) : kTP;  // valid points (TMA zero-fills the rest)
+    const int np = t + 1 < t1 || t1 * kTP <= a.N ? kTP : int(a.N - t * kTP);  // valid points (TMA zero-fills)
     // the warp's 16 points of the tile are p = warp + 8j: lane j < 16 reads key j (-1: no group)
     int kl = -1;
     if (lane < kTP / kConsumerWarps && warp + kConsumerWarps * lane < np) {
@@ -154,8 +153,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (unsigned(kl) >= unsigned(K)) kl = -1;
     }
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
+    // (after the sums below, so the match latency overlaps them)
     const unsigned same = __match_any_sync(0xffffffffu, kl);
-    if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
     // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
     // 4 points go one after the other (the rows may coincide)
@@ -197,6 +196,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
       }
     }
+    if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     __syncwarp();
     if (lane == 0) mbar_arrive(empty + slot);
     if (++since == kFlushTiles) {
