@@ -155,9 +155,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
     // (after the sums below, so the match latency overlaps them)
     const unsigned same = __match_any_sync(0xffffffffu, kl);
-    // sums: 4 points at a time. When their keys are distinct (warp-uniform test) the 4 read-modify-
-    // writes of the warp's accumulator rows are independent and issue back to back; otherwise the
-    // 4 points go one after the other (the rows may coincide)
+    // sums: 4 points at a time
 #pragma unroll
     for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
       int k[4];
@@ -170,31 +168,32 @@ __global__ void __launch_bounds__(kThreads, 1)
           xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
       }
       if (!dim_lane) continue;
-      const bool distinct = (k[0] != k[1] || k[0] < 0) && (k[0] != k[2] || k[0] < 0) && (k[0] != k[3] || k[0] < 0) &&
-                            (k[1] != k[2] || k[1] < 0) && (k[1] != k[3] || k[1] < 0) && (k[2] != k[3] || k[2] < 0);
-      if (distinct) {
-        float2 v[4];
+      // a repeated key adds its point into the first point of that key (branch-free selects), so
+      // the remaining row updates are distinct and their loads may all issue before the stores;
+      // with no branches the compiler interleaves consecutive batches
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
+      for (int q = 1; q < 4; ++q) {
+        bool done = k[q] < 0;
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) {
-            v[q].x += xv[q].x;
-            v[q].y += xv[q].y;
-            *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
-          }
-      } else {
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (k[q] >= 0) {
-            float2* acc = reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane);
-            float2 v = *acc;
-            v.x += xv[q].x;
-            v.y += xv[q].y;
-            *acc = v;
-          }
+        for (int r = 0; r < q; ++r) {
+          const bool hit = !done && k[r] == k[q];
+          xv[r].x += hit ? xv[q].x : 0.f;
+          xv[r].y += hit ? xv[q].y : 0.f;
+          done = done || hit;
+        }
+        k[q] = (k[q] >= 0 && done) ? -1 : k[q];
       }
+      float2 v[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (k[q] >= 0) v[q] = *reinterpret_cast<const float2*>(myacc + k[q] * D + 2 * lane);
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (k[q] >= 0) {
+          v[q].x += xv[q].x;
+          v[q].y += xv[q].y;
+          *reinterpret_cast<float2*>(myacc + k[q] * D + 2 * lane) = v[q];
+        }
     }
     if (kl >= 0 && __ffs(same) - 1 == lane) mycnt[kl] += unsigned(__popc(same));
     __syncwarp();
