@@ -165,3 +165,34 @@ def logreg_inputs(B, Rb, C, seed=6, batch_offset=0, device="cpu", y_zero=False):
                         device=device).to(torch.float32)
     w = uniform_f32(seed + 2, (C,), device=device, lo=-1.0 / 16, scale=1.0 / 8)
     return x, y, w
+
+
+def _pair_clz(h: torch.Tensor) -> torch.Tensor:
+    """Number of leading all-zero bit PAIRS of a 32-bit value (0..16), integer ops only."""
+    k = torch.zeros_like(h)
+    for j in range(1, 17):
+        k += (h < (1 << (32 - 2 * j))).to(h.dtype)
+    return k
+
+
+def pagerank_inputs(N, avg_deg=16, seed=7, max_deg=1024, device="cpu"):
+    """A directed multigraph of N nodes as the CSR of IN-neighbours: row n lists every w with an edge
+    w -> n (Fig 5: `n.nbrs`), plus each node's out-degree and a previous PageRank vector.
+
+    In-degrees follow a doubling-class power law (integer ops only): with k = leading zero bit pairs of
+    a hash (P(k >= j) = 4^-j) and base = dmin * 2^k, d_n = min(max_deg, base + hash' mod base), mean
+    about 2.25 * dmin, dmin = max(1, round(avg_deg / 2.25)). Neighbours are uniform over [0, N).
+    Returns (rowptr int64 [N+1], colidx int32 [E], pr float32 [N], outdeg int32 [N])."""
+    dmin = max(1, int(round(avg_deg / 2.25)))
+    i = _indices(0, N, device)
+    k = torch.clamp(_pair_clz(hash32(seed, i)), max=20)
+    base = dmin * (torch.ones_like(k) << k)
+    deg = torch.clamp(base + hash32(seed + 1, i) % base, max=max_deg)
+    rowptr = torch.zeros(N + 1, dtype=torch.int64, device=device)
+    rowptr[1:] = torch.cumsum(deg, 0)
+    E = int(rowptr[-1])
+    colidx = _empty((E,), torch.int32, device)
+    _fill(colidx, 0, lambda j: hash32(seed + 2, j) % N)
+    outdeg = torch.bincount(colidx.long(), minlength=N).to(torch.int32)
+    pr = uniform_f32(seed + 3, (N,), device=device, lo=0.5, scale=1.0) * (1.0 / N)
+    return rowptr, colidx, pr.contiguous(), outdeg
