@@ -178,6 +178,18 @@ def build_kmeans_update(npp, gen, torch, rank, world, strategy, device):
     return [item], ([out] if world > 1 else []), "k-means centroid update 4M x 64 -> 32 groups"
 
 
+def build_pagerank(npp, gen, torch, rank, world, strategy, device):
+    # one PageRank step (Fig 5) over a 4M-node power-law graph (mean in-degree ~16,
+    # cap 1024, ~63M edges); a rank owns its nodes' rows (the graph is replicated per rank here)
+    N = 1 << 22
+    rowptr, colidx, pr, outdeg = gen.pagerank_inputs(N, avg_deg=16, seed=7, max_deg=1024, device=device)
+    E = colidx.numel()
+    plan = npp.Plan("PAGERANK", (N, E), "f32", "AUTO", device=device)
+    item = Item("pagerank[4M,%dM]" % (E // 1000000), plan, [rowptr, colidx, pr, outdeg], plan.new_out(),
+                (N + 1) * 8 + E * 4 + N * 4 * 3)
+    return [item], [], "PageRank step, 4M nodes, ~63M edges"
+
+
 def build_logreg(npp, gen, torch, rank, world, strategy, device):
     # BASELINE.json config 5: [16M, 256] fp32 in B = 4096 mini-batches of 4096 rows; batches sharded
     B, Rb, C = 4096 // world, 4096, 256
@@ -203,9 +215,10 @@ def build_rowscols(npp, gen, torch, rank, world, strategy, device):
 
 # per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
 SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak",
-           "kmeans_update": "weak"}
+           "kmeans_update": "weak", "pagerank": "weak"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
-             "logreg": build_logreg, "rowscols": build_rowscols, "kmeans_update": build_kmeans_update}
+             "logreg": build_logreg, "rowscols": build_rowscols, "kmeans_update": build_kmeans_update,
+             "pagerank": build_pagerank}
 
 
 # ------------------------------------------------------------------------- reference arm (the oracle)
@@ -255,6 +268,8 @@ def config_for(args, extra):
           "sumcols_1m4k": "sumCols fp32 [1M,4K] row-sharded (BASELINE.json configs[2])",
           "kmeans": "k-means assignment 4M x 64 x 32 fp32, points sharded (BASELINE.json configs[3])",
           "logreg": "batched logreg gradient [16M,256] fp32, B=4096, batches sharded (BASELINE.json configs[4])",
+          "pagerank": "PageRank step (Fig 5) over a 4M-node power-law CSR graph, ~63M edges fp32 (SURVEY §8f "
+                      "NEXT 4)",
           "kmeans_update": "k-means centroid update 4M x 64 -> 32 groups fp32, points sharded + all-reduce "
                            "of [32, 65] (SURVEY §8f NEXT 4)",
           "rowscols": "sumRows+sumCols in ONE pass (SUM_ROWS_COLS) fp32 @ [64K,1K],[8K,8K],[1K,64K] "
@@ -272,11 +287,14 @@ def cpu_baseline(items, budget_s=12.0):
     import numpy as np
     from oracle import kmeans as okm
     from oracle import logreg as olr
+    from oracle import pagerank as opr
     from oracle import sums
     done_bytes, t_total, n = 0, 0.0, 0
     samples = []
     for it in items:
-        if it.name.startswith("kmeans_update"):  # first 1M points
+        if it.name.startswith("pagerank"):  # the whole graph (the oracle is O(E) NumPy)
+            samples.append((it.name, [x.cpu().numpy() for x in it.ins]))
+        elif it.name.startswith("kmeans_update"):  # first 1M points
             samples.append((it.name, [it.ins[0][: 1 << 20].cpu().numpy(), it.ins[1][: 1 << 20].cpu().numpy()]))
         elif it.name.startswith("kmeans"):  # first 256K points (the oracle is O(N K D) in fp64)
             samples.append((it.name, [it.ins[0][: 1 << 18].cpu().numpy(), it.ins[1].cpu().numpy()]))
@@ -289,7 +307,9 @@ def cpu_baseline(items, budget_s=12.0):
             samples.append((it.name, [it.ins[0].cpu().numpy()]))
 
     def run(name, arrs):
-        if name.startswith("kmeans_update"):
+        if name.startswith("pagerank"):
+            opr.step(*arrs)
+        elif name.startswith("kmeans_update"):
             okm.update(arrs[0], arrs[1], it_k)
         elif name.startswith("kmeans"):
             okm.assign(*arrs)

@@ -62,7 +62,15 @@ typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2 } npp_dtype;
  *   SUM_ROWS_COLS      {R,C}   ins={m[R*C]}                  out[R+C] = [Σ_c m[r,c] (r<R) | Σ_r m[r,c] (c<C)]
  *                      both outputs of the Naive Bayes counts (§VI-E) from ONE read of m;
  *                      executable with strategy AUTO (npp_select/npp_enumerate give every strategy's
- *                      record for analysis; the paper's two-kernel schedule = a SUM_ROWS and a SUM_COLS plan) */
+ *                      record for analysis; the paper's two-kernel schedule = a SUM_ROWS and a SUM_COLS plan)
+ *   KMEANS_UPDATE      {N,D,K} ins={x[N*D] f32, a[N] int32}  out[K*(D+1)] f32: row k = (Σ_{i: a_i=k} x_i, count_k)
+ *                      the centroid update after an assignment: Table I groupBy + Reduce per group;
+ *                      keys outside [0,K) belong to no group; counts exact below 2^24. AUTO only.
+ *   PAGERANK           {N,E}   ins={rowptr[N+1] int64, colidx[E] int32, pr[N] f32, outdeg[N] int32}
+ *                      out[N] f32 = (1-0.85)/N + 0.85 * Σ_{j=rowptr[n]}^{rowptr[n+1]-1} pr[w_j]/outdeg[w_j], w_j = colidx[j]
+ *                      one PageRank step (Fig 5) over the CSR of IN-neighbours; the caller
+ *                      guarantees 0 <= rowptr[n] <= rowptr[n+1] <= E, 0 <= colidx < N and outdeg >= 1 for
+ *                      every id in colidx (no device-side checks). AUTO only. */
 typedef enum {
   NPP_SUM_ROWS = 0,
   NPP_SUM_COLS = 1,
@@ -71,7 +79,8 @@ typedef enum {
   NPP_SUM_WEIGHTED_ROWS = 4,
   NPP_SUM_WEIGHTED_COLS = 5,
   NPP_SUM_ROWS_COLS = 6,
-  NPP_KMEANS_UPDATE = 7
+  NPP_KMEANS_UPDATE = 7,
+  NPP_PAGERANK = 8
 } npp_pattern;
 
 /* AUTO     = Algorithm 1 + ControlDOP + the runtime step R2 (L810-817; S8)
@@ -101,7 +110,8 @@ typedef enum {
   NPP_CLASS_LOGREG = 3,  /* 3-level: Map batches / Reduce rows / Map+Reduce columns       */
   NPP_CLASS_EMPTY = 4,   /* a zero-sized level: output zero-filled (or nothing to do)     */
   NPP_CLASS_RC = 5,      /* 2-level, both levels Reduce: row and column sums in one pass  */
-  NPP_CLASS_KMUPDATE = 6 /* groupBy + Reduce: per-centroid sums and counts                */
+  NPP_CLASS_KMUPDATE = 6,/* groupBy + Reduce: per-centroid sums and counts                */
+  NPP_CLASS_PAGERANK = 7 /* irregular inner Map+Reduce over CSR rows (Fig 5)              */
 } npp_kernel_class;
 
 /* One nest level of a mapping (§IV-A). dim: npp_dim; span: npp_span; factor: n of Span(n) or k of

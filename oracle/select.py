@@ -22,7 +22,7 @@ X, Y, Z = 0, 1, 2
 # span codes (S9 / record)
 ONE, ALL, SPAN_N, SPLIT = 0, 1, 2, 3
 # kernel classes (S9)
-RX, MX, KM, LR, EMPTY, RC, KU = 0, 1, 2, 3, 4, 5, 6
+RX, MX, KM, LR, EMPTY, RC, KU, PR = 0, 1, 2, 3, 4, 5, 6, 7
 
 SIZE_SET = [1 << i for i in range(11)]          # {1,2,4,...,1024}  Alg 1
 W_C, W_B = 8, 1                                  # DESIGN.md G3
@@ -32,7 +32,7 @@ T_BLOCK, U_MIN = 256, 8                          # DESIGN.md S8
 MAX_GRID = (1 << 31) - 1                         # DESIGN.md S3 H6
 
 PATTERNS = ("SUM_ROWS", "SUM_COLS", "KMEANS_ASSIGN", "LOGREG_GRAD",
-            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS", "KMEANS_UPDATE")
+            "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS", "KMEANS_UPDATE", "PAGERANK")
 DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8}
 
 B200 = dict(sm_count=148, max_threads_per_sm=2048, max_threads_per_block=1024,
@@ -99,6 +99,14 @@ def build_nest(pattern: str, shape) -> dict:
         levels = [(N, True), (D, False)]            # points: Reduce into K groups; dims: Map
         acc = [(1, (0, 1)), (0, (0,)), (1, (1,))]   # x[i,d], a[i], U[k,d]
         return {"pattern": pattern, "levels": levels, "accesses": acc, "K": K}
+    elif pattern == "PAGERANK":                      # Fig 5 L348-361 over the CSR of in-neighbours
+        N, E = shape
+        if E < 0:
+            raise ValueError("PAGERANK needs E >= 0")
+        inner = max(1, cdiv(E, N)) if N > 0 else 1  # the average in-degree stands for the inner size
+        levels = [(N, False), (inner, True)]         # nodes: Map; neighbours: Map + Reduce
+        acc = [(0, (0,)), (0, (0,)), (1, (0, 1)), (-1, (0, 1)), (-1, (0, 1))]  # rowptr, out, colidx, 2 gathers
+        return {"pattern": pattern, "levels": levels, "accesses": acc, "E": E}
     elif pattern == "KMEANS_ASSIGN":
         N, D, K = shape
         levels = [(N, False), (K, True), (D, True)]
@@ -153,7 +161,7 @@ def level_chunk(n: int, b: int, span: int, factor: int, vec: int = 1) -> int:
 # ------------------------------------------------------------------ S3 hard constraints
 
 def acc_bytes(pattern: str, dtype: str) -> int:
-    if pattern in ("KMEANS_ASSIGN", "LOGREG_GRAD", "KMEANS_UPDATE"):
+    if pattern in ("KMEANS_ASSIGN", "LOGREG_GRAD", "KMEANS_UPDATE", "PAGERANK"):
         return 8
     return 4 if dtype == "i32" else 8
 
@@ -409,6 +417,18 @@ def r2_rowscols(nest, dtype, lim):
     return dims, blocks, spans, factors, 1, chunks, staged, t["G"], t["cr"] * t["cc"]
 
 
+def r2_pagerank(nest, lim):
+    """DESIGN.md S8 PR: V = min(32, pow2 >= ceil(E/N)) lanes per row on x, 256/V row groups on y, rows
+    claimed in chunks of 4*256/V by min(4*SMs, chunks) blocks. Returns (dims, blocks, spans, factors,
+    vec, chunks, G, chunk)."""
+    (N, _), (inner, _) = nest["levels"]
+    V = min(32, pow2ceil(inner))
+    RPB = 256 // V
+    chunk = 4 * RPB
+    G = min(4 * lim["sm_count"], cdiv(N, chunk))
+    return (Y, X), (RPB, V), (SPAN_N, ALL), (4, 1), 1, (chunk, inner), G, chunk
+
+
 def r2_kmupdate(nest, lim):
     """DESIGN.md S8 KU: 128-point tiles, contiguous ranges of P tiles, 8 warps x 32 lanes (2 dims per lane).
     Returns (dims, blocks, spans, factors, vec, chunks, G, P)."""
@@ -511,6 +531,8 @@ def kernel_class(pattern, dims):
         return RC
     if pattern == "KMEANS_UPDATE":
         return KU
+    if pattern == "PAGERANK":
+        return PR
     return RX if dims[1] == X else MX
 
 
@@ -561,6 +583,8 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
+    if nest["pattern"] == "PAGERANK" and persistent_grid is not None:  # the row-chunk claim counter
+        rec["workspace_bytes"] = 256
     if nest["pattern"] == "KMEANS_UPDATE" and staged:  # ticket (256 B) + fp64 accumulators [K x (D+1)]
         rec["workspace_bytes"] = 256 + 256 * cdiv(8 * nest["K"] * (_eff(nest["levels"][1][0]) + 1), 256)
     if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:
@@ -625,6 +649,10 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
         b3, s3, f3, vec, chunks, G, P = r2_kmeans(nest, lim)
         return make_record(nest, dtype, lim, dims, b3, s3, f3, vec, sc, chunks, staged=1,
                            persistent_grid=G, claim_tiles=P)
+    if pattern == "PAGERANK":
+        d2, b2, s2, f2, vec, chunks, G, CH = r2_pagerank(nest, lim)
+        return make_record(nest, dtype, lim, d2, b2, s2, f2, vec, sc, chunks, staged=0,
+                           persistent_grid=G, claim_tiles=CH)
     if pattern == "KMEANS_UPDATE":
         d2, b2, s2, f2, vec, chunks, G, P = r2_kmupdate(nest, lim)
         return make_record(nest, dtype, lim, d2, b2, s2, f2, vec, sc, chunks, staged=1,

@@ -50,6 +50,7 @@ int n_inputs(int pattern) {
     case NPP_KMEANS_ASSIGN:
     case NPP_KMEANS_UPDATE: return 2;
     case NPP_LOGREG_GRAD: return 3;
+    case NPP_PAGERANK: return 4;
     default: return -1;
   }
 }
@@ -66,6 +67,7 @@ int64_t input_bytes(const npp_plan_s* p, int k) {
     case NPP_SUM_WEIGHTED_COLS: return k == 0 ? s[0] * s[1] * es : s[0] * es;
     case NPP_KMEANS_ASSIGN: return k == 0 ? s[0] * s[1] * 4 : s[2] * s[1] * 4;
     case NPP_KMEANS_UPDATE: return k == 0 ? s[0] * s[1] * 4 : s[0] * 4;
+    case NPP_PAGERANK: return k == 0 ? (s[0] + 1) * 8 : (k == 1 ? s[1] * 4 : s[0] * 4);
     case NPP_LOGREG_GRAD: return k == 0 ? s[0] * s[1] * s[2] * 4 : (k == 1 ? s[0] * s[1] * 4 : s[2] * 4);
     default: return 0;
   }
@@ -82,6 +84,7 @@ int64_t output_bytes(const npp_plan_s* p) {
     case NPP_SUM_ROWS_COLS: return (s[0] + s[1]) * es;
     case NPP_KMEANS_ASSIGN: return s[0] * 4;
     case NPP_KMEANS_UPDATE: return s[2] * (s[1] + 1) * 4;
+    case NPP_PAGERANK: return s[0] * 4;
     case NPP_LOGREG_GRAD: return s[0] * s[2] * 4;
     default: return 0;
   }
@@ -100,9 +103,10 @@ int validate_request(int pattern, const int64_t* shape, int ndim, int dtype, boo
     set_error("unknown pattern");
     return NPP_ERR_INVALID_ARG;
   }
-  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) &&
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE ||
+       pattern == NPP_PAGERANK) &&
       dtype != NPP_F32) {
-    set_error("k-means and logreg are defined for f32");
+    set_error("k-means, logreg and PageRank are defined for f32");
     return NPP_ERR_UNSUPPORTED;
   }
   *empty = false;
@@ -111,7 +115,8 @@ int validate_request(int pattern, const int64_t* shape, int ndim, int dtype, boo
       set_error("npp_plan needs known, non-negative sizes");
       return NPP_ERR_INVALID_ARG;
     }
-    if (shape[d] == 0) *empty = true;
+    // a PageRank step over N > 0 nodes without edges still writes (1 - damp) / N: only N = 0 is empty
+    if (shape[d] == 0 && !(pattern == NPP_PAGERANK && d == 1)) *empty = true;
   }
   return NPP_OK;
 }
@@ -228,6 +233,11 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
   if (pattern == NPP_KMEANS_UPDATE && strategy != NPP_MAP_AUTO) {
     delete p;
     set_error("KMEANS_UPDATE executes with strategy AUTO only (class KU)");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  if (pattern == NPP_PAGERANK && strategy != NPP_MAP_AUTO) {
+    delete p;
+    set_error("PAGERANK executes with strategy AUTO only (class PR)");
     return NPP_ERR_UNSUPPORTED;
   }
   st = get_limits(limits, &p->lim);
@@ -412,7 +422,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     return NPP_ERR_INVALID_ARG;
   }
   for (int k = 0; k < need; ++k)
-    if (!ins[k]) {
+    if (!ins[k] && !(plan->pattern == NPP_PAGERANK && k == 1 && plan->shape[1] == 0)) {  // E = 0: no colidx
       set_error("input pointer is NULL");
       return NPP_ERR_INVALID_ARG;
     }
@@ -454,6 +464,20 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     k.per_block = m.claim_tiles;
     cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);
+    return NPP_OK;
+  }
+  if (plan->pattern == NPP_PAGERANK) {  // class PR (S8 PR)
+    npp::PagerankArgs r{};
+    r.rowptr = static_cast<const long long*>(ins[0]);
+    r.colidx = static_cast<const int*>(ins[1]);
+    r.pr = static_cast<const float*>(ins[2]);
+    r.outdeg = static_cast<const int*>(ins[3]);
+    r.out = static_cast<float*>(out);
+    r.pool = static_cast<unsigned*>(workspace);
+    r.N = plan->shape[0];
+    r.damp = 0.85f;
+    cudaError_t e = npp::launch_pagerank(r, m.level[1].block, int(m.grid), st);
+    if (e != cudaSuccess) return cuda_fail("PageRank kernel launch", e);
     return NPP_OK;
   }
   if (plan->pattern == NPP_KMEANS_UPDATE) {  // class KU (S8 KU)

@@ -126,4 +126,17 @@ struct KmUpdateArgs {
 };
 cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st);
 
+// One PageRank step over the CSR of in-neighbours (class PR, S8 PR, Fig 5).
+struct PagerankArgs {
+  const long long* rowptr;  // [N+1]
+  const int* colidx;        // [E] in-neighbour ids
+  const float* pr;          // [N] previous PageRank
+  const int* outdeg;        // [N] out-degrees (>= 1 for every id that occurs in colidx)
+  float* out;               // [N]
+  unsigned* pool;           // row-chunk claim counter (zero on entry and on exit)
+  int64_t N;
+  float damp;
+};
+cudaError_t launch_pagerank(const PagerankArgs& a, int V, int grid, cudaStream_t st);
+
 }  // namespace npp

@@ -81,7 +81,9 @@ int64_t level_chunk(int64_t N, int b, int span, int64_t factor, int vec) {
 }
 
 int acc_bytes(int pattern, int dtype) {
-  if (pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) return 8;
+  if (pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE ||
+      pattern == NPP_PAGERANK)
+    return 8;
   return dtype == NPP_I32 ? 4 : 8;
 }
 
@@ -378,11 +380,29 @@ bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
   return true;
 }
 
+// S8 PAGERANK (class PR): V = min(32, pow2 >= ceil(E/N)) lanes per row on x, 256/V row groups on y,
+// rows claimed in chunks of 4*256/V by min(4*SMs, chunks) blocks.
+void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
+  const int64_t N = n.N[0], inner = n.N[1];
+  const int64_t V = std::min<int64_t>(32, pow2ceil(inner));
+  const int64_t RPB = 256 / V, chunk = 4 * RPB;
+  const int64_t units = cdiv(N, chunk);
+  c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
+  c->blocks[0] = int(RPB), c->blocks[1] = int(V);
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = 4, c->chunks[0] = chunk;
+  c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = inner;
+  c->vec = 1;
+  c->staged = 0;
+  c->persistent_grid = std::min<int64_t>(4 * int64_t(lim.sm_count), units);
+  c->claim_tiles = chunk;
+}
+
 int kernel_class_of(const Nest& n, const Choice& c) {
   if (n.pattern == NPP_KMEANS_ASSIGN) return NPP_CLASS_KMEANS;
   if (n.pattern == NPP_LOGREG_GRAD) return NPP_CLASS_LOGREG;
   if (n.pattern == NPP_SUM_ROWS_COLS) return NPP_CLASS_RC;
   if (n.pattern == NPP_KMEANS_UPDATE) return NPP_CLASS_KMUPDATE;
+  if (n.pattern == NPP_PAGERANK) return NPP_CLASS_PAGERANK;
   return c.dims[1] == NPP_DIM_X ? NPP_CLASS_RX : NPP_CLASS_MX;
 }
 
@@ -533,6 +553,23 @@ int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
       n.acc[n.nacc++] = {1, 0x2u};  // U[k,d]
       n.cols = shape[1];
       break;
+    case NPP_PAGERANK:  // shape {N, E}: Map over nodes, Map+Reduce over a node's in-neighbours (Fig 5)
+      if (!need(2)) return NPP_ERR_INVALID_ARG;
+      if (shape[1] < 0) {
+        set_error("PAGERANK needs E >= 0");
+        return NPP_ERR_INVALID_ARG;
+      }
+      n.L = 2;
+      n.N[0] = shape[0], n.sync[0] = false;
+      n.E = shape[1];
+      n.N[1] = shape[0] > 0 ? std::max<int64_t>(1, cdiv(shape[1], shape[0])) : 1, n.sync[1] = true;
+      n.acc[n.nacc++] = {0, 0x1u};   // rowptr[n]
+      n.acc[n.nacc++] = {0, 0x1u};   // out[n]
+      n.acc[n.nacc++] = {1, 0x3u};   // colidx[j]
+      n.acc[n.nacc++] = {-1, 0x3u};  // prevPR(w): a gather
+      n.acc[n.nacc++] = {-1, 0x3u};  // w.degree: a gather
+      n.cols = 0;
+      break;
     case NPP_KMEANS_ASSIGN:  // shape {N, D, K}; levels N / K / D
       if (!need(3)) return NPP_ERR_INVALID_ARG;
       n.L = 3;
@@ -668,6 +705,8 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.temp_stride[1] = c.temp_stride[1];
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
+  } else if (n.pattern == NPP_PAGERANK && c.persistent_grid > 0) {
+    m.workspace_bytes = 256;  // S9 PR: the row-chunk claim counter
   } else if (n.pattern == NPP_KMEANS_UPDATE && c.staged) {
     // S9 KU: ticket (256 B) + fp64 accumulators [K x (D+1)]
     m.workspace_bytes = 256 + 256 * cdiv(8 * n.K * (eff(n.N[1]) + 1), 256);
@@ -772,6 +811,10 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
     r2_rowscols(n, dtype, lim, &c);
     return record_from_choice(n, dtype, lim, c, sc, out);
   }
+  if (n.pattern == NPP_PAGERANK) {
+    r2_pagerank(n, lim, &c);
+    return record_from_choice(n, dtype, lim, c, sc, out);
+  }
   if (n.pattern == NPP_KMEANS_UPDATE) {
     if (!r2_kmupdate(n, lim, &c)) {
       set_error("KMEANS_UPDATE AUTO needs D % 4 == 0, 4 <= D <= 64, 1 <= K <= 256 and K*D <= 2048");
@@ -804,9 +847,10 @@ extern "C" int npp_select(int pattern, const int64_t* shape, int ndim, int dtype
   Nest n;
   st = build_nest(pattern, shape, ndim, &n);
   if (st) return st;
-  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE) &&
+  if ((pattern == NPP_KMEANS_ASSIGN || pattern == NPP_LOGREG_GRAD || pattern == NPP_KMEANS_UPDATE ||
+       pattern == NPP_PAGERANK) &&
       dtype != NPP_F32) {
-    set_error("k-means and logreg are defined for f32");
+    set_error("k-means, logreg and PageRank are defined for f32");
     return NPP_ERR_UNSUPPORTED;
   }
   return select_mapping(n, dtype, *limits, strategy, out);

@@ -26,6 +26,7 @@ struct Nest {
   Access acc[kMaxAccesses];
   int64_t cols = 0;  // matrix columns (sums), for the vector-width rule of R2
   int64_t K = 0;     // KMEANS_UPDATE: number of groups (the groupBy key range, not a nest level)
+  int64_t E = 0;     // PAGERANK: number of edges (the inner level is sized by the average ceil(E/N))
 };
 
 struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refinements

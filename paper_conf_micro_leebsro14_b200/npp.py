@@ -20,10 +20,10 @@ DTYPES = {"f32": 0, "i32": 1, "i64": 2}
 TORCH_DTYPES = {"f32": torch.float32, "i32": torch.int32, "i64": torch.int64}
 PATTERNS = {"SUM_ROWS": 0, "SUM_COLS": 1, "KMEANS_ASSIGN": 2, "LOGREG_GRAD": 3,
             "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5, "SUM_ROWS_COLS": 6,
-            "KMEANS_UPDATE": 7}
+            "KMEANS_UPDATE": 7, "PAGERANK": 8}
 STRATEGIES = {"AUTO": 0, "LITERAL": 1, "1D": 2, "TB_T": 3, "WARP": 4}
 SPAN_ONE, SPAN_ALL, SPAN_N, SPLIT_K = 0, 1, 2, 3
-CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY, CLASS_RC, CLASS_KMUPDATE = 0, 1, 2, 3, 4, 5, 6
+CLASS_RX, CLASS_MX, CLASS_KMEANS, CLASS_LOGREG, CLASS_EMPTY, CLASS_RC, CLASS_KMUPDATE, CLASS_PAGERANK = range(8)
 
 
 class NppError(RuntimeError):
@@ -243,6 +243,8 @@ class Plan:
             return (s[0],)
         if p == "KMEANS_UPDATE":
             return (s[2], s[1] + 1)
+        if p == "PAGERANK":
+            return (s[0],)
         return (s[0], s[2])
 
     def out_dtype(self):
@@ -339,6 +341,14 @@ def kmeans_update(x, a, K, out=None, stream=None):
     N, D = x.shape
     p = _cached_plan("KMEANS_UPDATE", (N, D, int(K)), "f32", "AUTO", x.device)
     return p.execute([x, a], out if out is not None else p.new_out(), stream)
+
+
+def pagerank_step(rowptr, colidx, pr, outdeg, out=None, stream=None):
+    """One PageRank step (Fig 5) over the CSR of in-neighbours: rowptr int64 [N+1], colidx
+    int32 [E], pr f32 [N], outdeg int32 [N] -> (1-0.85)/N + 0.85 * Σ_{w in nbrs(n)} pr[w]/outdeg[w]."""
+    N, E = pr.shape[0], colidx.shape[0]
+    p = _cached_plan("PAGERANK", (N, E), "f32", "AUTO", pr.device)
+    return p.execute([rowptr, colidx, pr, outdeg], out if out is not None else p.new_out(), stream)
 
 
 def logreg_grad(x, y, w, B, strategy="AUTO", out=None, stream=None):

@@ -247,3 +247,61 @@ def test_kmeans_update_plan_rules(npp, cuda_device):
                   torch.full((3, 9), 5.0, device=cuda_device))
     torch.cuda.synchronize()
     assert float(u.abs().sum()) == 0.0
+
+
+# ---------------------------------------------------------------- PageRank step (class PR, Fig 5)
+
+def _check_pr(out, rowptr, colidx, pr, outdeg):
+    from oracle import pagerank as opr
+    want = opr.step(rowptr.cpu().numpy(), colidx.cpu().numpy(), pr.cpu().numpy(), outdeg.cpu().numpy())
+    got = out.cpu().numpy().astype(np.float64)
+    err = np.abs(got - want)
+    bad = np.nonzero(err > 1e-5 * want)[0]   # every term is positive: relative 1e-5
+    assert bad.size == 0, (bad[:5], got[bad[:5]], want[bad[:5]])
+
+
+@pytest.mark.parametrize("N,avg,maxd", [(1, 3, 8), (7, 1, 4), (1000, 2, 64), (5000, 16, 1024), (20000, 5, 300),
+                                        (100000, 40, 1024), (3000, 16, 4096)])
+def test_pagerank_parity(npp, cuda_device, N, avg, maxd):
+    rowptr, colidx, pr, outdeg = gen.pagerank_inputs(N, avg_deg=avg, seed=N % 97, max_deg=maxd, device=cuda_device)
+    E = colidx.numel()
+    p = npp.Plan("PAGERANK", (N, E))
+    assert p.mapping == osel.select("PAGERANK", (N, E), "f32", npp.limits_query(0), "AUTO")
+    assert p.mapping["kernel_class"] == npp.CLASS_PAGERANK
+    outs = [p.execute([rowptr, colidx, pr, outdeg], p.new_out()),
+            p.execute([rowptr, colidx, pr, outdeg], p.new_out(), overlap=True)]
+    torch.cuda.synchronize()
+    for o in outs:
+        _check_pr(o, rowptr, colidx, pr, outdeg)
+    assert int(p.workspace.count_nonzero()) == 0   # the claim counter re-armed itself
+
+
+def test_pagerank_edge_cases(npp, cuda_device):
+    from oracle import pagerank as opr
+    # no edges: every node gets (1 - d) / N; rows of very different lengths in one chunk
+    N = 1000
+    rowptr = torch.zeros(N + 1, dtype=torch.int64, device=cuda_device)
+    out = npp.pagerank_step(rowptr, torch.empty(0, dtype=torch.int32, device=cuda_device),
+                            torch.full((N,), 1.0 / N, device=cuda_device), torch.ones(N, dtype=torch.int32, device=cuda_device))
+    torch.cuda.synchronize()
+    assert torch.allclose(out.double().cpu(), torch.full((N,), (1 - opr.DAMP) / N, dtype=torch.float64), rtol=1e-6)
+    # complete graph with uniform PageRank is a fixed point (oracle pin, now on the GPU)
+    m = 300
+    rowptr = torch.arange(0, m * m + 1, m, dtype=torch.int64, device=cuda_device)
+    colidx = torch.arange(m, dtype=torch.int32, device=cuda_device).repeat(m)
+    out = npp.pagerank_step(rowptr, colidx, torch.full((m,), 1.0 / m, device=cuda_device),
+                            torch.full((m,), m, dtype=torch.int32, device=cuda_device))
+    torch.cuda.synchronize()
+    assert torch.allclose(out.cpu(), torch.full((m,), 1.0 / m), rtol=1e-5)
+    for strategy in ("LITERAL", "1D"):
+        with pytest.raises(npp.NppError) as e:
+            npp.Plan("PAGERANK", (100, 1000), "f32", strategy)
+        assert e.value.status == npp.ERR_UNSUPPORTED
+
+
+def test_pagerank_full_size(npp, cuda_device):
+    # the bench workload: 4M nodes, power-law in-degrees (mean ~16, cap 1024), ~63M edges
+    rowptr, colidx, pr, outdeg = gen.pagerank_inputs(1 << 22, avg_deg=16, seed=7, max_deg=1024, device=cuda_device)
+    out = npp.pagerank_step(rowptr, colidx, pr, outdeg)
+    torch.cuda.synchronize()
+    _check_pr(out, rowptr, colidx, pr, outdeg)

@@ -71,6 +71,15 @@ def test_kmeans_update_parity(profile):
             _cmp("KMEANS_UPDATE", shape, "f32", lim, strat)
 
 
+@pytest.mark.parametrize("profile", list(PROFILES))
+def test_pagerank_parity(profile):
+    lim = PROFILES[profile]
+    for shape in [(1 << 22, 70000000), (1000, 0), (1, 5), (7, 7), (5000, 80000), (100, 100000), (33, 1 << 20),
+                  (1 << 20, 1 << 20)]:
+        for strat in SUM_STRATS:
+            _cmp("PAGERANK", shape, "f32", lim, strat)
+
+
 def test_unknown_sizes_literal():
     for shape in [(-1, 1024), (1024, -1), (-1, -1)]:
         for pattern in ("SUM_ROWS", "SUM_COLS"):

@@ -60,6 +60,7 @@ NAMES = {
     "kmeans": ["kmeans_assign[4M,64,32]"],
     "logreg": ["logreg_grad[16M,256]"],
     "kmeans_update": ["kmeans_update[4M,64,32]"],
+    "pagerank": ["pagerank[4M,63M]"],
     "rowscols": ["sum_rows_cols[64K,1K]", "sum_rows_cols[8K,8K]", "sum_rows_cols[1K,64K]"],
 }
 
