@@ -583,8 +583,8 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
-    if nest["pattern"] == "PAGERANK" and persistent_grid is not None:  # the row-chunk claim counter
-        rec["workspace_bytes"] = 256
+    if nest["pattern"] == "PAGERANK" and persistent_grid is not None:  # claim counter + contrib [N] f32
+        rec["workspace_bytes"] = 256 + 256 * cdiv(4 * nest["levels"][0][0], 256)
     if nest["pattern"] == "KMEANS_UPDATE" and staged:  # ticket (256 B) + fp64 accumulators [K x (D+1)]
         rec["workspace_bytes"] = 256 + 256 * cdiv(8 * nest["K"] * (_eff(nest["levels"][1][0]) + 1), 256)
     if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:

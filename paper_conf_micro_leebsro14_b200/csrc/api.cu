@@ -383,7 +383,8 @@ int64_t npp_plan_workspace_bytes(npp_plan_t plan) { return plan ? plan->map.work
 int npp_plan_launches(npp_plan_t plan) {
   if (!plan) return 0;
   if (plan->empty) return output_bytes(plan) > 0 ? 1 : 0;
-  return plan->pattern == NPP_KMEANS_ASSIGN ? 2 : 1;  // k-means: centroid pack + assignment
+  // k-means: centroid pack + assignment; PageRank: per-node contribution + the CSR kernel
+  return (plan->pattern == NPP_KMEANS_ASSIGN || plan->pattern == NPP_PAGERANK) ? 2 : 1;
 }
 
 void npp_plan_destroy(npp_plan_t plan) { delete plan; }
@@ -474,6 +475,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     r.outdeg = static_cast<const int*>(ins[3]);
     r.out = static_cast<float*>(out);
     r.pool = static_cast<unsigned*>(workspace);
+    r.contrib = reinterpret_cast<float*>(static_cast<char*>(workspace) + 256);
     r.N = plan->shape[0];
     r.damp = 0.85f;
     cudaError_t e = npp::launch_pagerank(r, m.level[1].block, int(m.grid), st);

@@ -134,6 +134,7 @@ struct PagerankArgs {
   const int* outdeg;        // [N] out-degrees (>= 1 for every id that occurs in colidx)
   float* out;               // [N]
   unsigned* pool;           // row-chunk claim counter (zero on entry and on exit)
+  float* contrib;           // [N] workspace: prevPR(w) / w.degree (Fig 5's inner map, once per node)
   int64_t N;
   float damp;
 };

@@ -706,7 +706,7 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
   } else if (n.pattern == NPP_PAGERANK && c.persistent_grid > 0) {
-    m.workspace_bytes = 256;  // S9 PR: the row-chunk claim counter
+    m.workspace_bytes = 256 + 256 * cdiv(4 * n.N[0], 256);  // S9 PR: claim counter + contrib [N] f32
   } else if (n.pattern == NPP_KMEANS_UPDATE && c.staged) {
     // S9 KU: ticket (256 B) + fp64 accumulators [K x (D+1)]
     m.workspace_bytes = 256 + 256 * cdiv(8 * n.K * (eff(n.N[1]) + 1), 256);

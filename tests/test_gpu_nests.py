@@ -273,7 +273,7 @@ def test_pagerank_parity(npp, cuda_device, N, avg, maxd):
     torch.cuda.synchronize()
     for o in outs:
         _check_pr(o, rowptr, colidx, pr, outdeg)
-    assert int(p.workspace.count_nonzero()) == 0   # the claim counter re-armed itself
+    assert int(p.workspace[:256].count_nonzero()) == 0   # the claim counter re-armed itself
 
 
 def test_pagerank_edge_cases(npp, cuda_device):
