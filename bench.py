@@ -187,6 +187,9 @@ def build_pagerank(npp, gen, torch, rank, world, strategy, device):
     plan = npp.Plan("PAGERANK", (N, E), "f32", "AUTO", device=device)
     item = Item("pagerank[4M,%dM]" % (E // 1000000), plan, [rowptr, colidx, pr, outdeg], plan.new_out(),
                 (N + 1) * 8 + E * 4 + N * 4 * 3)
+    # the random gathers bound this path: one L1tex wavefront (128-B line) per edge for contrib[w], plus
+    # the coalesced colidx / rowptr / per-node lines (DESIGN.md §6 PR)
+    item.wavefronts = E + E * 4 // 128 + (N + 1) * 8 // 128 + 3 * N * 4 // 128
     return [item], [], "PageRank step, 4M nodes, ~63M edges"
 
 
@@ -428,6 +431,7 @@ def main():
     dom_gbs = items[dom].bytes / (per_kernel_us[dom] * 1e-6) / 1e9
     traffic = ncu_traffic().get(items[dom].name)
     flops = getattr(items[dom], "flops", None)
+    wavefronts = getattr(items[dom], "wavefronts", None)
     per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9, 1),
                            "frac_of_measured": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / peak, 4),
                            "frac_of_8TBs": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / 8000.0, 4),
@@ -446,7 +450,7 @@ def main():
                           launches="programmatic dependent launch (NPP_EXEC_OVERLAP)" if overlap
                           else "serialised"),
            "per_shape": per_shape,
-           "roofline": roofline(items[dom], per_kernel_us[dom], dom_gbs, peak, peak_src, traffic, flops),
+           "roofline": roofline(items[dom], per_kernel_us[dom], dom_gbs, peak, peak_src, traffic, flops, wavefronts),
            "clocks": sampler.summary(),
            "gpu_launches": args.steps * sum(it.plan.launches for it in items)}
 
@@ -464,9 +468,16 @@ def main():
     return 0
 
 
-def roofline(item, us, gbs, peak, peak_src, traffic, flops):
+def roofline(item, us, gbs, peak, peak_src, traffic, flops, wavefronts=None):
     base = {"kernel": item.name, "traffic": traffic, "algorithmic_bytes": item.bytes, "duration_us": round(us, 2),
             "hbm_GBps": round(gbs, 1), "hbm_frac_of_measured": round(gbs / peak, 4)}
+    if wavefronts:  # random gathers: L1tex wavefront rate, ~1 per cycle per SM (B300_MICROARCH.md LDG model)
+        wf_peak = 148 * 1.965e9 / 1e9
+        achieved = wavefronts / (us * 1e-6) / 1e9
+        return dict(base, bound="l1tex", achieved=round(achieved, 2), peak=round(wf_peak, 2),
+                    unit="G wavefronts/s", frac=round(achieved / wf_peak, 4),
+                    peak_source="derived: 148 SM x 1 L1tex wavefront/clk (guide: rt_L1tex_wf ~ 1.0 cyc/wf) x 1965 MHz",
+                    algorithmic_wavefronts=wavefronts)
     if flops:  # FP32 FMA-bound (k-means): peak = 148 SMs x 128 FP32 lanes x 2 flop x 1965 MHz
         alu_peak = 148 * 128 * 2 * 1.965e9 / 1e12
         achieved = flops / (us * 1e-6) / 1e12

@@ -100,13 +100,14 @@ def build_nest(pattern: str, shape) -> dict:
         acc = [(1, (0, 1)), (0, (0,)), (1, (1,))]   # x[i,d], a[i], U[k,d]
         return {"pattern": pattern, "levels": levels, "accesses": acc, "K": K}
     elif pattern == "PAGERANK":                      # Fig 5 L348-361 over the CSR of in-neighbours
-        N, E = shape
+        N, E = shape[0], shape[1]                   # {N, E} or {rows, E, N}: L0 = the rows computed
         if E < 0:
             raise ValueError("PAGERANK needs E >= 0")
         inner = max(1, cdiv(E, N)) if N > 0 else 1  # the average in-degree stands for the inner size
         levels = [(N, False), (inner, True)]         # nodes: Map; neighbours: Map + Reduce
         acc = [(0, (0,)), (0, (0,)), (1, (0, 1)), (-1, (0, 1)), (-1, (0, 1))]  # rowptr, out, colidx, 2 gathers
-        return {"pattern": pattern, "levels": levels, "accesses": acc, "E": E}
+        return {"pattern": pattern, "levels": levels, "accesses": acc, "E": E,
+                "nodes": shape[2] if len(shape) == 3 else N}
     elif pattern == "KMEANS_ASSIGN":
         N, D, K = shape
         levels = [(N, False), (K, True), (D, True)]
@@ -584,7 +585,7 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
             tick = levels[0]["grid"] * 4
             rec["workspace_bytes"] = 256 * cdiv(part, 256) + 256 * cdiv(tick, 256)
     if nest["pattern"] == "PAGERANK" and persistent_grid is not None:  # claim counter + contrib [N] f32
-        rec["workspace_bytes"] = 256 + 256 * cdiv(4 * nest["levels"][0][0], 256)
+        rec["workspace_bytes"] = 256 + 256 * cdiv(4 * nest["nodes"], 256)
     if nest["pattern"] == "KMEANS_UPDATE" and staged:  # ticket (256 B) + fp64 accumulators [K x (D+1)]
         rec["workspace_bytes"] = 256 + 256 * cdiv(8 * nest["K"] * (_eff(nest["levels"][1][0]) + 1), 256)
     if nest["pattern"] == "SUM_ROWS_COLS" and persistent_grid is not None:

@@ -67,7 +67,7 @@ int64_t input_bytes(const npp_plan_s* p, int k) {
     case NPP_SUM_WEIGHTED_COLS: return k == 0 ? s[0] * s[1] * es : s[0] * es;
     case NPP_KMEANS_ASSIGN: return k == 0 ? s[0] * s[1] * 4 : s[2] * s[1] * 4;
     case NPP_KMEANS_UPDATE: return k == 0 ? s[0] * s[1] * 4 : s[0] * 4;
-    case NPP_PAGERANK: return k == 0 ? (s[0] + 1) * 8 : (k == 1 ? s[1] * 4 : s[0] * 4);
+    case NPP_PAGERANK: return k == 0 ? (s[0] + 1) * 8 : (k == 1 ? s[1] * 4 : (p->ndim == 3 ? s[2] : s[0]) * 4);
     case NPP_LOGREG_GRAD: return k == 0 ? s[0] * s[1] * s[2] * 4 : (k == 1 ? s[0] * s[1] * 4 : s[2] * 4);
     default: return 0;
   }
@@ -477,6 +477,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     r.pool = static_cast<unsigned*>(workspace);
     r.contrib = reinterpret_cast<float*>(static_cast<char*>(workspace) + 256);
     r.N = plan->shape[0];
+    r.Nnodes = plan->ndim == 3 ? plan->shape[2] : plan->shape[0];
     r.damp = 0.85f;
     cudaError_t e = npp::launch_pagerank(r, m.level[1].block, int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("PageRank kernel launch", e);

@@ -553,10 +553,13 @@ int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
       n.acc[n.nacc++] = {1, 0x2u};  // U[k,d]
       n.cols = shape[1];
       break;
-    case NPP_PAGERANK:  // shape {N, E}: Map over nodes, Map+Reduce over a node's in-neighbours (Fig 5)
-      if (!need(2)) return NPP_ERR_INVALID_ARG;
-      if (shape[1] < 0) {
-        set_error("PAGERANK needs E >= 0");
+    case NPP_PAGERANK:  // shape {N, E} or {rows, E, N}: Map over nodes, Map+Reduce over in-neighbours (Fig 5)
+      if (ndim != 2 && ndim != 3) {
+        set_error("PAGERANK expects {N, E} or {rows, E, N}");
+        return NPP_ERR_INVALID_ARG;
+      }
+      if (shape[1] < 0 || (ndim == 3 && shape[2] < shape[0])) {
+        set_error("PAGERANK needs E >= 0 and rows <= N");
         return NPP_ERR_INVALID_ARG;
       }
       n.L = 2;
@@ -568,7 +571,7 @@ int build_nest(int pattern, const int64_t* shape, int ndim, Nest* out) {
       n.acc[n.nacc++] = {1, 0x3u};   // colidx[j]
       n.acc[n.nacc++] = {-1, 0x3u};  // prevPR(w): a gather
       n.acc[n.nacc++] = {-1, 0x3u};  // w.degree: a gather
-      n.cols = 0;
+      n.cols = ndim == 3 ? shape[2] : shape[0];  // graph nodes (the contrib[] length)
       break;
     case NPP_KMEANS_ASSIGN:  // shape {N, D, K}; levels N / K / D
       if (!need(3)) return NPP_ERR_INVALID_ARG;
@@ -706,7 +709,7 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   if (n.pattern == NPP_LOGREG_GRAD && c.staged) {  // tickets [B] + fp64 accumulators [B x C]
     m.workspace_bytes = 256 * cdiv(4 * eff(n.N[0]), 256) + 256 * cdiv(8 * eff(n.N[0]) * eff(n.N[2]), 256);
   } else if (n.pattern == NPP_PAGERANK && c.persistent_grid > 0) {
-    m.workspace_bytes = 256 + 256 * cdiv(4 * n.N[0], 256);  // S9 PR: claim counter + contrib [N] f32
+    m.workspace_bytes = 256 + 256 * cdiv(4 * n.cols, 256);  // S9 PR: claim counter + contrib [nodes] f32
   } else if (n.pattern == NPP_KMEANS_UPDATE && c.staged) {
     // S9 KU: ticket (256 B) + fp64 accumulators [K x (D+1)]
     m.workspace_bytes = 256 + 256 * cdiv(8 * n.K * (eff(n.N[1]) + 1), 256);

@@ -74,6 +74,33 @@ def kmeans_update(local_x: torch.Tensor, local_a: torch.Tensor, K: int, group=No
     return u
 
 
+def pagerank_step(local_rowptr: torch.Tensor, local_colidx: torch.Tensor, pr: torch.Tensor, outdeg: torch.Tensor,
+                  group=None, compute=None):
+    """One PageRank step with the nodes (CSR rows) sharded: this rank's rows [lo, hi) of the in-neighbour
+    CSR (local_rowptr rebased to 0, length hi-lo+1) against the replicated previous PageRank and
+    out-degrees; the per-node contributions are computed over all N nodes, each rank writes its rows,
+    and one all-gather assembles the next [N] vector (the exchange step of the iteration)."""
+    N = pr.shape[0]
+    world, rank = _world(group)
+    lo, hi = shard_range(N, world, rank)
+    if compute is not None:
+        local = compute(local_rowptr, local_colidx, pr, outdeg, lo, hi)
+    else:
+        local = _npp().pagerank_shard(local_rowptr, local_colidx, pr, outdeg, lo, hi)
+    parts = [torch.empty(b - a, dtype=local.dtype, device=local.device)
+             for a, b in (shard_range(N, world, r) for r in range(world))]
+    if all(p.numel() == parts[0].numel() for p in parts):
+        dist.all_gather(parts, local, group=group)
+    else:  # uneven shards: gather padded buffers
+        mx = max(p.numel() for p in parts)
+        buf = torch.zeros(mx, dtype=local.dtype, device=local.device)
+        buf[: local.numel()] = local
+        padded = [torch.empty(mx, dtype=local.dtype, device=local.device) for _ in range(world)]
+        dist.all_gather(padded, buf, group=group)
+        parts = [p[: q.numel()] for p, q in zip(padded, parts)]
+    return torch.cat(parts)
+
+
 def logreg_grad(local_x: torch.Tensor, local_y: torch.Tensor, w: torch.Tensor, batches: int, group=None,
                 full_batch: bool = False, compute=None):
     """Per-mini-batch gradients of this rank's batches (independent), or with ``full_batch`` the

@@ -351,6 +351,13 @@ def pagerank_step(rowptr, colidx, pr, outdeg, out=None, stream=None):
     return p.execute([rowptr, colidx, pr, outdeg], out if out is not None else p.new_out(), stream)
 
 
+def pagerank_shard(local_rowptr, local_colidx, pr, outdeg, lo, hi, out=None, stream=None):
+    """Rows [lo, hi) of a PageRank step: the shard's CSR (rowptr rebased to 0, hi-lo+1 entries) against the
+    whole graph's pr / outdeg (PAGERANK shape {rows, E, N})."""
+    p = _cached_plan("PAGERANK", (hi - lo, local_colidx.shape[0], pr.shape[0]), "f32", "AUTO", pr.device)
+    return p.execute([local_rowptr, local_colidx, pr, outdeg], out if out is not None else p.new_out(), stream)
+
+
 def logreg_grad(x, y, w, B, strategy="AUTO", out=None, stream=None):
     n, C = x.shape
     p = _cached_plan("LOGREG_GRAD", (B, n // B, C), "f32", strategy, x.device)

@@ -65,8 +65,17 @@ def _worker(rank, port, results):
         xl, yl, w = gen.logreg_inputs(1, Rb, Cl, seed=6)
         g = ndist.logreg_grad(xl[rlo:rhi].contiguous(), yl[rlo:rhi].contiguous(), w, 1, full_batch=True,
                               compute=lambda x, y, ww, B: torch.from_numpy(olr.grad(x.numpy(), y.numpy(), ww.numpy(), B)))
+        # PageRank: node rows sharded, pr / outdeg replicated, one all-gather of the next vector
+        from oracle import pagerank as opr
+        rp, ci, prv, od = gen.pagerank_inputs(501, avg_deg=6, seed=9, max_deg=64)
+        nlo, nhi = shard_range(501, WORLD, rank)
+        lrp = rp[nlo:nhi + 1] - rp[nlo]
+        lci = ci[int(rp[nlo]):int(rp[nhi])]
+
+        prn = ndist.pagerank_step(lrp, lci, prv, od, compute=lambda lr, lc, p, d, a0, a1: torch.from_numpy(
+            opr.step(lr.numpy(), lc.numpy(), p.numpy(), d.numpy())))
         results[rank] = dict(cols=cols.numpy(), rows=rows.numpy(), cols_i=cols_i.numpy(), a=a.numpy(),
-                             u=u.numpy(), g=g.numpy(), lo=lo, hi=hi)
+                             u=u.numpy(), g=g.numpy(), pr=prn.numpy(), lo=lo, hi=hi)
     finally:
         dist.destroy_process_group()
 
@@ -103,6 +112,11 @@ def test_two_rank_gloo():
     for rank in range(WORLD):
         assert np.allclose(results[rank]["u"], want_u, rtol=1e-12, atol=1e-9)
         assert results[rank]["u"][:, -1].tolist() == want_u[:, -1].tolist()
+    from oracle import pagerank as opr
+    rp, ci, prv, od = gen.pagerank_inputs(501, avg_deg=6, seed=9, max_deg=64)
+    want_pr = opr.step(rp.numpy(), ci.numpy(), prv.numpy(), od.numpy())
+    for rank in range(WORLD):
+        assert np.allclose(results[rank]["pr"], want_pr, rtol=1e-12)
     xl, yl, w = gen.logreg_inputs(1, 200, 12, seed=6)
     want_g = olr.grad(xl.numpy(), yl.numpy(), w.numpy(), 1)
     for rank in range(WORLD):

@@ -305,3 +305,14 @@ def test_pagerank_full_size(npp, cuda_device):
     out = npp.pagerank_step(rowptr, colidx, pr, outdeg)
     torch.cuda.synchronize()
     _check_pr(out, rowptr, colidx, pr, outdeg)
+
+
+def test_pagerank_shard_rows(npp, cuda_device):
+    # the multi-GPU form: rows [lo, hi) from the shard's CSR against the whole pr / outdeg ({rows, E, N})
+    rowptr, colidx, pr, outdeg = gen.pagerank_inputs(50000, avg_deg=12, seed=5, max_deg=2000, device=cuda_device)
+    lo, hi = 12345, 40000
+    lrp = (rowptr[lo:hi + 1] - rowptr[lo]).contiguous()
+    lci = colidx[int(rowptr[lo]):int(rowptr[hi])].contiguous()
+    out = npp.pagerank_shard(lrp, lci, pr, outdeg, lo, hi)
+    torch.cuda.synchronize()
+    _check_pr(out, lrp, lci, pr, outdeg)

@@ -58,3 +58,12 @@ def test_generator_shape():
     assert 12 <= float(deg.float().mean()) <= 20               # ~avg_deg
     assert int(outdeg.sum()) == len(colidx) and int(colidx.min()) >= 0 and int(colidx.max()) < 5000
     assert torch.equal(gen.pagerank_inputs(5000, seed=7)[1], colidx)  # deterministic
+
+
+def test_shard_rows_match_full_step():
+    # rows [lo, hi) of the step from the shard's CSR alone (numNodes stays the graph's N)
+    rowptr, colidx, pr, outdeg = (t.numpy() for t in gen.pagerank_inputs(800, avg_deg=5, seed=4, max_deg=50))
+    full = opr.step(rowptr, colidx, pr, outdeg)
+    lo, hi = 300, 555
+    part = opr.step(rowptr[lo:hi + 1] - rowptr[lo], colidx[rowptr[lo]:rowptr[hi]], pr, outdeg)
+    assert np.array_equal(part, full[lo:hi])

@@ -75,7 +75,7 @@ def test_kmeans_update_parity(profile):
 def test_pagerank_parity(profile):
     lim = PROFILES[profile]
     for shape in [(1 << 22, 70000000), (1000, 0), (1, 5), (7, 7), (5000, 80000), (100, 100000), (33, 1 << 20),
-                  (1 << 20, 1 << 20)]:
+                  (1 << 20, 1 << 20), (1000, 16000, 4000), (1, 3, 1 << 22)]:
         for strat in SUM_STRATS:
             _cmp("PAGERANK", shape, "f32", lim, strat)
 
