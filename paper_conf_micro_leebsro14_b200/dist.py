@@ -2,7 +2,8 @@
 
 SURVEY.md §8e / DESIGN.md §8. The outer (storage-row) dimension of every input is split into contiguous
 shards, one per rank. Where the rows are the Map level (sumRows, k-means points, logreg mini-batches)
-the shards are independent problems and no collective runs. Where the rows are the level being
+the shards are independent problems and no collective runs (PageRank rows too, plus one all-gather
+of the next vector per step). Where the rows are the level being
 reduced (sumCols, the full-batch logreg gradient, the k-means centroid update) the shard results are a cross-device Split(P) of that
 Reduce and NCCL adds them — the only data-path collective.
 
