@@ -9,12 +9,12 @@ tail -3 $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
 tail -2 $O/smoke.log
 timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; tail -2 $O/bench.err
-for w in kmeans logreg sumcols_1m4k rowscols kmeans_update; do timeout 600 python bench.py --workload $w --steps 10 --warmup 3 > $O/bench_$w.json 2> $O/bench_$w.err; done
+for w in kmeans logreg sumcols_1m4k rowscols kmeans_update pagerank; do timeout 600 python bench.py --workload $w --steps 10 --warmup 3 > $O/bench_$w.json 2> $O/bench_$w.err; done
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > $O/bench_ref.json 2> $O/bench_ref.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:npp_ --csv --log-file $O/launches_bench.csv python bench.py --steps 2 --warmup 3 --no-mappings --no-cpu --no-e2e > $O/b_ncu.log 2>&1
 python - <<'PY'
 import json
-for w in ['bench','bench_kmeans','bench_logreg','bench_sumcols_1m4k','bench_rowscols','bench_kmeans_update','bench_ref']:
+for w in ["bench","bench_kmeans","bench_logreg","bench_sumcols_1m4k","bench_rowscols","bench_kmeans_update","bench_pagerank","bench_ref"]:
     try:
         d=json.load(open('gpurun_out/r01g/'+w+'.json'))
         r=d.get('roofline',{})
