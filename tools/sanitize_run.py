@@ -5,7 +5,9 @@
 
 Covers: staged sums (narrow/wide tiles, RX/MX, f32/i32/i64, ragged edges, pool + combiner, PDL
 overlap), weighted staged sums, the direct-load family under every strategy (Split(k) combine), the
-S10 temp family (PREALLOC layouts and MALLOC), k-means assignment, logreg gradient.
+S10 temp family (PREALLOC layouts and MALLOC), k-means assignment, logreg gradient, the one-pass
+rows+cols family (staged and direct, regions cut both ways), the k-means update, the PageRank step
+(full graph and a shard).
 """
 import os
 import sys
@@ -50,8 +52,30 @@ def main():
     npp.Plan("KMEANS_ASSIGN", (700, 96, 40)).execute([x, c], torch.empty(700, dtype=torch.int32, device=dev))
     lx, ly, lw = gen.logreg_inputs(5, 100, 256, device=dev)
     npp.Plan("LOGREG_GRAD", (5, 100, 256)).execute([lx, ly, lw], torch.empty(5, 256, device=dev))
+    n += 3
+    for dtype in ("f32", "i32", "i64"):
+        for shape in [(300, 1024), (1000, 999), (64, 9000), (5, 3)]:
+            m = (gen.uniform_f32(4, shape, device=dev) if dtype == "f32" else
+                 gen.int_uniform(5, shape, -50, 50, device=dev) if dtype == "i32" else
+                 gen.int64_wide(6, shape, device=dev))
+            p = npp.Plan("SUM_ROWS_COLS", shape, dtype)
+            p.execute([m], p.new_out())
+            p.execute([m], p.new_out(), overlap=True)
+            n += 2
+    for N, D, K in [(3000, 64, 32), (517, 8, 100), (129, 4, 1)]:
+        x, _ = gen.kmeans_inputs(N, D, K, device=dev)
+        a = gen.int_uniform(7, (N,), -1, K, device=dev)
+        p = npp.Plan("KMEANS_UPDATE", (N, D, K))
+        p.execute([x, a], p.new_out())
+        p.execute([x, a], p.new_out(), overlap=True)
+        n += 2
+    rp, ci, pr, od = gen.pagerank_inputs(3000, avg_deg=10, seed=2, max_deg=400, device=dev)
+    npp.pagerank_step(rp, ci, pr, od)
+    lo, hi = 1000, 2500
+    npp.pagerank_shard((rp[lo:hi + 1] - rp[lo]).contiguous(), ci[int(rp[lo]):int(rp[hi])].contiguous(), pr, od, lo, hi)
+    n += 2
     torch.cuda.synchronize()
-    print(f"sanitize_run ok: {n + 3} executes")
+    print(f"sanitize_run ok: {n} executes")
 
 
 if __name__ == "__main__":
