@@ -257,7 +257,11 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         const bool flush = nxt < 0 || (nxt / a.Ti) != (cur / a.Ti);
         const int slot = int(t % kStages);
         if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-        slot_tile[slot] = cur | (flush ? kFlush : 0);
+        // the tag travels through shared memory ordered by the slot's mbarriers; it is written and
+        // read with (relaxed) shared atomics so compute-sanitizer's racecheck, which does not model
+        // mbarrier ordering, sees no plain-access race
+        atomicExch(reinterpret_cast<unsigned long long*>(slot_tile + slot),
+                   static_cast<unsigned long long>(cur | (flush ? kFlush : 0)));
         constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
         mbar_expect_tx(full + slot, kTileBytes + kVBytes);
         const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
@@ -280,7 +284,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
       if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-      slot_tile[slot] = -1;
+      atomicExch(reinterpret_cast<unsigned long long*>(slot_tile + slot), ~0ull);  // -1
       mbar_arrive(full + slot);
     }
   } else if (warp == kCombinerWarp) {
@@ -361,7 +365,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     for (long long t = 0;; ++t) {
       const int slot = int(t % kStages);
       mbar_wait(full + slot, unsigned((t / kStages) & 1));
-      const long long tag = slot_tile[slot];
+      unsigned long long tag_u = 0;
+      if (lane == 0) tag_u = atomicAdd(reinterpret_cast<unsigned long long*>(slot_tile + slot), 0ull);
+      const long long tag = static_cast<long long>(__shfl_sync(0xffffffffu, tag_u, 0));
       if (tag < 0) break;
       const unsigned char* tile = tiles + slot * kTileBytes;
       const unsigned char* vs = vslots + slot * kVSlot;
