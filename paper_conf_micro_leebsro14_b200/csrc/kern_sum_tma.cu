@@ -182,13 +182,14 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   uint64_t* empty = full + kStages;
   uint64_t* fl_full = empty + kStages;        // [kFlushRing] consumer warps -> combiner
   uint64_t* fl_free = fl_full + kFlushRing;   // [kFlushRing] combiner -> consumers
-  long long* slot_tile = reinterpret_cast<long long*>(fl_free + kFlushRing);  // tile | kFlush, -1 = end
-  long long* fl_ot = slot_tile + kStages;     // [kFlushRing] outer tile of a flush, -1 = end
+  unsigned* slot_tile = reinterpret_cast<unsigned*>(fl_free + kFlushRing);  // tile | kFlush, kEnd = end
+  long long* fl_ot = reinterpret_cast<long long*>(fl_free + kFlushRing) + kStages;  // [kFlushRing] outer tile, -1 = end
   unsigned* fl_cnt = reinterpret_cast<unsigned*>(fl_ot + kFlushRing);  // tiles it contributes
   unsigned char* tiles = smem + kSmemHeader;
   unsigned char* vslots = tiles + kStages * kTileBytes;  // WT only: [kStages][kVSlot]
   Acc* accg = static_cast<Acc*>(a.acc);
-  constexpr long long kFlush = 1ll << 62;
+  constexpr unsigned kFlush = 1u << 31;  // tile ids < 2^31 - 1 (launch_sum_staged checks)
+  constexpr unsigned kEnd = 0xffffffffu;
 
   // PDL: let the next launch in the stream become resident as SMs free up (its griddepcontrol.wait
   // still orders it after this grid's completion).
@@ -260,8 +261,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         // the tag travels through shared memory ordered by the slot's mbarriers; it is written and
         // read with (relaxed) shared atomics so compute-sanitizer's racecheck, which does not model
         // mbarrier ordering, sees no plain-access race
-        atomicExch(reinterpret_cast<unsigned long long*>(slot_tile + slot),
-                   static_cast<unsigned long long>(cur | (flush ? kFlush : 0)));
+        atomicExch(slot_tile + slot, static_cast<unsigned>(cur) | (flush ? kFlush : 0u));
         constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
         mbar_expect_tx(full + slot, kTileBytes + kVBytes);
         const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
@@ -284,7 +284,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
       if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-      atomicExch(reinterpret_cast<unsigned long long*>(slot_tile + slot), ~0ull);  // -1
+      atomicExch(slot_tile + slot, kEnd);
       mbar_arrive(full + slot);
     }
   } else if (warp == kCombinerWarp) {
@@ -365,10 +365,11 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     for (long long t = 0;; ++t) {
       const int slot = int(t % kStages);
       mbar_wait(full + slot, unsigned((t / kStages) & 1));
-      unsigned long long tag_u = 0;
-      if (lane == 0) tag_u = atomicAdd(reinterpret_cast<unsigned long long*>(slot_tile + slot), 0ull);
-      const long long tag = static_cast<long long>(__shfl_sync(0xffffffffu, tag_u, 0));
-      if (tag < 0) break;
+      unsigned tag_u = 0;
+      if (lane == 0) tag_u = atomicAdd(slot_tile + slot, 0u);
+      tag_u = __shfl_sync(0xffffffffu, tag_u, 0);
+      if (tag_u == kEnd) break;
+      const long long tag = static_cast<long long>(tag_u);
       const unsigned char* tile = tiles + slot * kTileBytes;
       const unsigned char* vs = vslots + slot * kVSlot;
       if constexpr (ROWS && !WIDE) {
@@ -551,6 +552,7 @@ cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const CUtensorMap& v
 }  // namespace
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st) {
+  if (a.To * a.Ti >= 0x7fffffffll) return cudaErrorInvalidValue;  // 32-bit slot tags
   EncodeTiledFn encode = encode_fn();
   if (!encode) return cudaErrorNotSupported;
   const int esz = dtype == NPP_I64 ? 8 : 4;
