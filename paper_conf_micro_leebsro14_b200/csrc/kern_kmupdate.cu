@@ -229,139 +229,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
-// K <= 64: warp w OWNS the rows k with k % 8 == w and keeps them in fp64 registers (RPW = ceil(K/8)
-// rows x 2 dims per lane), so a point costs one shared-memory read and two register adds — no
-// read-modify-write of shared accumulators, no alias chains, no fold. Every warp scans the tile's 128
-// keys (lane j: points j, j+32, j+64, j+96), ballots the ones it owns and walks their bits. Cost of
-// the ownership split: with skewed clusters one warp carries more points (the ring's 4 slots absorb
-// ordinary imbalance).
-template <int RPW>
-__global__ void __launch_bounds__(kThreads, 1)
-    npp_kmupdate_rows_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap amap,
-                             const KmUpdateArgs a) {
-  extern __shared__ __align__(1024) unsigned char smem[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
-  uint64_t* empty = full + kStages;
-  volatile int* flag = reinterpret_cast<volatile int*>(empty + kStages);
-  unsigned char* xring = smem + kHeader;
-  unsigned char* aring = xring + kStages * kXSlot;
-  const int D = int(a.D), K = int(a.K), KD1 = K * (D + 1);
-
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long T = (a.N + kTP - 1) / kTP;
-  const long long t0 = blockIdx.x * a.per_block;
-  const long long t1 = t0 + a.per_block < T ? t0 + a.per_block : T;
-
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kStages; ++i) {
-      mbar_init(full + i, 1);
-      mbar_init(empty + i, kConsumerWarps);
-    }
-    mbar_fence_init();
-  }
-  __syncthreads();
-
-  if (warp == kConsumerWarps) {
-    // ------------------------------------------------------------ producer: one elected lane
-    if (lane == 0) {
-      prefetch_map(&xmap);
-      prefetch_map(&amap);
-      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
-      const unsigned bytes = unsigned(kTP * D * 4 + kASlot);
-      for (long long t = t0; t < t1; ++t) {
-        const long long i = t - t0;
-        const int slot = int(i % kStages);
-        if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
-        mbar_expect_tx(full + slot, bytes);
-        load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
-        load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
-      }
-    }
-    return;
-  }
-
-  // -------------------------------------------------------------- consumers
-  double acc[RPW][2];
-  unsigned cnt[RPW];
-#pragma unroll
-  for (int r = 0; r < RPW; ++r) acc[r][0] = acc[r][1] = 0.0, cnt[r] = 0u;
-  const bool dim_lane = 2 * lane < D;
-  int slot = 0;
-  unsigned phase = 0;
-  for (long long t = t0; t < t1; ++t, slot = slot + 1 == kStages ? 0 : slot + 1, phase ^= slot == 0 ? 1u : 0u) {
-    mbar_wait(full + slot, phase);
-    const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
-    const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
-    const int np = t + 1 < t1 || t1 * kTP <= a.N ? kTP : int(a.N - t * kTP);
-    int kq[4];
-    unsigned own[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int p = lane + 32 * q;
-      kq[q] = p < np ? at[p] : -1;
-      own[q] = __ballot_sync(0xffffffffu, unsigned(kq[q]) < unsigned(K) && (kq[q] & (kConsumerWarps - 1)) == warp);
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      unsigned m = own[q];
-      while (m) {
-        const int j = __ffs(m) - 1;
-        m &= m - 1;
-        const int row = __shfl_sync(0xffffffffu, kq[q], j) >> 3;  // kConsumerWarps = 8
-        float2 xv = make_float2(0.f, 0.f);
-        if (dim_lane) xv = *reinterpret_cast<const float2*>(xt + (j + 32 * q) * D + 2 * lane);
-#pragma unroll
-        for (int r = 0; r < RPW; ++r)
-          if (r == row) {
-            acc[r][0] += double(xv.x);
-            acc[r][1] += double(xv.y);
-            cnt[r] += 1u;
-          }
-      }
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty + slot);
-  }
-
-  // ---- the warp's rows -> fp64 workspace accumulators; the last block converts (fused Split combine)
-  asm volatile("griddepcontrol.wait;" ::: "memory");  // workspace / out: after the previous grid
-#pragma unroll
-  for (int r = 0; r < RPW; ++r) {
-    const int k = kConsumerWarps * r + warp;
-    if (k < K) {
-      if (dim_lane && acc[r][0] != 0.0) atomicAdd(a.acc + k * (D + 1) + 2 * lane, acc[r][0]);
-      if (dim_lane && acc[r][1] != 0.0) atomicAdd(a.acc + k * (D + 1) + 2 * lane + 1, acc[r][1]);
-      if (lane == 0 && cnt[r] != 0u) atomicAdd(a.acc + k * (D + 1) + D, double(cnt[r]));
-    }
-  }
-  __threadfence();
-  consumers_sync();
-  if (threadIdx.x == 0) {
-    const bool last = atomicAdd(a.ticket, 1u) + 1u == gridDim.x;
-    if (last) *a.ticket = 0u;
-    flag[0] = last ? 1 : 0;
-  }
-  consumers_sync();
-  if (flag[0]) {
-    __threadfence();
-    for (int i = threadIdx.x; i < KD1; i += kConsumers) {
-      const double v = __ldcg(a.acc + i);
-      __stcg(a.acc + i, 0.0);
-      a.out[i] = float(v);
-    }
-  }
-}
-
-template <typename Kern>
-cudaError_t launch_ku(Kern kern, int smem, const CUtensorMap& xmap, const CUtensorMap& amap, const KmUpdateArgs& a,
-                      int grid, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e != cudaSuccess) return e;
-  return launch_pdl(kern, grid, kThreads, smem, st, true, xmap, amap, a);
-}
-
 cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st) {
   if (a.D % 4 != 0 || a.D < 4 || a.D > 64 || a.K < 1 || a.K > kMaxK || a.K * a.D > kMaxKD)
     return cudaErrorInvalidValue;
@@ -369,12 +236,13 @@ cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* ke
   cudaError_t e = encode_2d(&xmap, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(a.D), unsigned(kTP));
   if (e != cudaSuccess) return e;
   if ((e = encode_1d(&amap, keys, CU_TENSOR_MAP_DATA_TYPE_INT32, a.N, unsigned(kTP))) != cudaSuccess) return e;
-  const int ring = kHeader + kStages * (kXSlot + kASlot);
-  if (a.K <= 8) return launch_ku(npp_kmupdate_rows_kernel<1>, ring, xmap, amap, a, grid, st);
-  if (a.K <= 16) return launch_ku(npp_kmupdate_rows_kernel<2>, ring, xmap, amap, a, grid, st);
-  if (a.K <= 32) return launch_ku(npp_kmupdate_rows_kernel<4>, ring, xmap, amap, a, grid, st);
-  if (a.K <= 64) return launch_ku(npp_kmupdate_rows_kernel<8>, ring, xmap, amap, a, grid, st);
-  return launch_ku(npp_kmupdate_kernel, kSmemBytes, xmap, amap, a, grid, st);
+  static bool attr_set = false;
+  if (!attr_set) {
+    e = cudaFuncSetAttribute(npp_kmupdate_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, true, xmap, amap, a);
 }
 
 }  // namespace npp
