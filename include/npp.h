@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define NPP_VERSION 2
+#define NPP_VERSION 3  /* 3: SUM_ROWS_COLS, KMEANS_UPDATE, PAGERANK */
 
 #if defined(__GNUC__)
 #define NPP_API __attribute__((visibility("default")))

@@ -52,7 +52,7 @@ def test_struct_layout_matches_binding(tmp_path):
         size, offs = _c_layout(tmp_path, struct, names)
         assert ctypes.sizeof(cls) == size, struct
         assert [getattr(cls, n).offset for n in names] == offs, struct
-    assert npp.lib().npp_version() == 2
+    assert npp.lib().npp_version() == 3
     assert set(npp.EXPORTS) == set(declared_symbols())
 
 
@@ -64,3 +64,24 @@ def test_no_gpu_calls_fail_cleanly():
     with pytest.raises(npp.NppError) as e:
         npp.limits_query(0)
     assert e.value.status == npp.ERR_CUDA
+
+
+@pytest.mark.skipif(shutil.which("gcc") is None, reason="gcc not available")
+def test_enum_values_match_binding(tmp_path):
+    # every pattern / kernel-class / strategy constant of the binding equals the header's enum value
+    from paper_conf_micro_leebsro14_b200 import npp
+    names = ([f"NPP_{k}" for k in npp.PATTERNS] +
+             ["NPP_CLASS_RX", "NPP_CLASS_MX", "NPP_CLASS_KMEANS", "NPP_CLASS_LOGREG", "NPP_CLASS_EMPTY",
+              "NPP_CLASS_RC", "NPP_CLASS_KMUPDATE", "NPP_CLASS_PAGERANK"] +
+             ["NPP_MAP_AUTO", "NPP_MAP_LITERAL", "NPP_MAP_1D", "NPP_MAP_TB_THREAD", "NPP_MAP_WARP"])
+    src = tmp_path / "enums.c"
+    body = "".join(f'  printf("%d\\n", (int){n});\n' for n in names)
+    src.write_text(f'#include <stdio.h>\n#include "npp.h"\nint main(void) {{\n{body}  return 0;\n}}\n')
+    exe = tmp_path / "enums"
+    subprocess.run(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    vals = [int(v) for v in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
+    want = (list(npp.PATTERNS.values()) +
+            [npp.CLASS_RX, npp.CLASS_MX, npp.CLASS_KMEANS, npp.CLASS_LOGREG, npp.CLASS_EMPTY, npp.CLASS_RC,
+             npp.CLASS_KMUPDATE, npp.CLASS_PAGERANK] +
+            [npp.STRATEGIES[k] for k in ("AUTO", "LITERAL", "1D", "TB_T", "WARP")])
+    assert vals == want
