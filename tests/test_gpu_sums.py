@@ -322,7 +322,8 @@ def test_weighted_temp_modes(npp, cuda_device, dtype):
 
 
 RC_SHAPES = [(1, 1), (3, 5), (31, 33), (33, 31), (1000, 999), (1024, 1024), (4097, 300), (300, 4097),
-             (7, 70000), (70000, 7), (2, 1 << 17), (1001, 1024), (9, 3072), (5000, 8192), (100000, 36)]
+             (7, 70000), (70000, 7), (2, 1 << 17), (1001, 1024), (9, 3072), (5000, 8192), (100000, 36),
+             (3, 1 << 21), (40, 1200004)]   # more column groups than SMs: blocks walk several regions
 
 
 def _check_rc(m, got, dtype):
