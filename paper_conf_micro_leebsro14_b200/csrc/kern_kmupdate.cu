@@ -119,13 +119,19 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int r = 0; r < kMaxKD / kConsumers; ++r) {
       const int i = int(threadIdx.x) + kConsumers * r;
       if (i >= KD) break;
-      double s = 0.0;
+      // the 8 warp copies meet in an fp32 pairwise tree (error <= 3u on top of the copies' <= 127u), then
+      // one fp64 add (8 fp64 adds per element measured slower)
+      float v[kConsumerWarps];
 #pragma unroll
       for (int w = 0; w < kConsumerWarps; ++w) {
-        s += double(accw[w * KD + i]);
+        v[w] = accw[w * KD + i];
         accw[w * KD + i] = 0.f;
       }
-      bacc[i + krow[r]] += s;  // row k of [K x (D+1)]
+#pragma unroll
+      for (int h = kConsumerWarps / 2; h >= 1; h /= 2)
+#pragma unroll
+        for (int w = 0; w < h; ++w) v[w] += v[w + h];
+      bacc[i + krow[r]] += double(v[0]);  // row k of [K x (D+1)]
     }
     for (int k = threadIdx.x; k < K; k += kConsumers) {
       unsigned c = 0;
