@@ -227,27 +227,58 @@ WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans":
 # ------------------------------------------------------------------------- reference arm (the oracle)
 
 def run_reference(args):
+    """The reference arm: the oracle as it stands (NumPy fp64, one host core) on a bounded sample of
+    the selected workload, same metric / unit / config as the npp arm."""
     world, rank, _ = dist_env()
     if rank != 0:
         return 0
-    import numpy as np
-    import torch
+    import numpy as np  # noqa: F401
+    from oracle import kmeans as okm
+    from oracle import logreg as olr
+    from oracle import pagerank as opr
     from oracle import sums
     from synth import gen
-    shapes = PAPER_SHAPES if args.workload == "paper" else [(1 << 20, 4096)]
-    # bounded sample per step: the first rows of each matrix, 4M elements per (pattern, shape)
-    sample_elems = 1 << 22
-    mats = []
-    for si, (R, C) in enumerate(shapes):
-        rows = max(1, min(R, sample_elems // C))
-        for pattern in (("SUM_ROWS", "SUM_COLS") if args.workload == "paper" else ("SUM_COLS",)):
-            seed = 300 + 2 * si + (pattern == "SUM_COLS")
-            mats.append((pattern, gen.uniform_f32(seed, (rows, C)).numpy()))
-    step_bytes = sum(m.size * 4 + (m.shape[0] if p == "SUM_ROWS" else m.shape[1]) * 4 for p, m in mats)
+    calls, desc = [], ""
+    wl = args.workload
+    if wl in ("paper", "sumcols_1m4k", "rowscols"):
+        shapes = PAPER_SHAPES if wl != "sumcols_1m4k" else [(1 << 20, 4096)]
+        sample_elems = 1 << 22   # the first rows of each matrix, 4M elements per (pattern, shape)
+        for si, (R, C) in enumerate(shapes):
+            rows = max(1, min(R, sample_elems // C))
+            pats = {"paper": ("SUM_ROWS", "SUM_COLS"), "sumcols_1m4k": ("SUM_COLS",), "rowscols": ("SUM_ROWS_COLS",)}[wl]
+            for pattern in pats:
+                seed = (300 + 2 * si + (pattern == "SUM_COLS")) if wl != "sumcols_1m4k" else 4
+                m = gen.uniform_f32(seed, (rows, C)).numpy()
+                fn = {"SUM_ROWS": sums.sum_rows, "SUM_COLS": sums.sum_cols, "SUM_ROWS_COLS": sums.sum_rows_cols}[pattern]
+                out = rows if pattern == "SUM_ROWS" else (C if pattern == "SUM_COLS" else rows + C)
+                calls.append((lambda f=fn, a=m: f(a), m.size * 4 + out * 4))
+        desc = f"first {sample_elems} elements of each matrix per step"
+    elif wl in ("kmeans", "kmeans_update"):
+        N, D, K = 1 << 16, 64, 32
+        x, c = gen.kmeans_inputs(N, D, K)
+        x, c = x.numpy(), c.numpy()
+        if wl == "kmeans":
+            calls.append((lambda: okm.assign(x, c), N * D * 4 + K * D * 4 + N * 4))
+        else:
+            a = okm.assign(x, c)
+            calls.append((lambda: okm.update(x, a, K), N * D * 4 + N * 4 + K * (D + 1) * 4))
+        desc = f"{N} points of the 4M x 64 x 32 workload per step"
+    elif wl == "logreg":
+        B, Rb, C = 16, 4096, 256
+        x, y, w = gen.logreg_inputs(B, Rb, C, seed=6)
+        x, y, w = x.numpy(), y.numpy(), w.numpy()
+        calls.append((lambda: olr.grad(x, y, w, B), B * Rb * C * 4 + B * Rb * 4 + C * 4 + B * C * 4))
+        desc = f"{B} of the 4096 mini-batches per step"
+    elif wl == "pagerank":
+        N = 1 << 20
+        rp, ci, pr, od = (t.numpy() for t in gen.pagerank_inputs(N, avg_deg=16, seed=7, max_deg=1024))
+        calls.append((lambda: opr.step(rp, ci, pr, od), (N + 1) * 8 + len(ci) * 4 + N * 12))
+        desc = f"a {N}-node graph of the same recipe per step"
+    step_bytes = sum(b for _, b in calls)
 
     def step():
-        for p, m in mats:
-            (sums.sum_rows if p == "SUM_ROWS" else sums.sum_cols)(m)
+        for f, _ in calls:
+            f()
     for _ in range(args.warmup):
         step()
     t0 = time.perf_counter()
@@ -257,10 +288,10 @@ def run_reference(args):
     value = step_bytes / dt / 1e9
     line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "impl": "reference",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": SCALING[wl], "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": config_for(args, "oracle (NumPy fp64) on host cores"),
             "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": f"first {sample_elems} elements of each of {len(mats)} matrices per step"},
+                             "sample": desc},
             "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
