@@ -36,15 +36,15 @@ namespace {
 
 using namespace tma;
 
-constexpr int kStages = 5;
+constexpr int kStages = 4;
 constexpr int kTileRows = 32;
 constexpr int kTileBytes = kTileRows * 1024;
 constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
-constexpr int kColTilesMax = 24;          // column tiles of one region (select.hpp kRcColTilesMax)
-constexpr int kColAccBytes = 48 * 1024;   // [row groups][kColTilesMax * BC] accumulators
+constexpr int kColTilesMax = 32;          // column tiles of one region (select.hpp kRcColTilesMax)
+constexpr int kColAccBytes = 64 * 1024;   // [row groups][kColTilesMax * BC] accumulators
 constexpr int kRowSumBytes = 2 * kConsumerWarps * 32 * 8;
 constexpr int kSmemBytes = kHeader + kStages * kTileBytes + kColAccBytes + kRowSumBytes;
 
