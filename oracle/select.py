@@ -423,7 +423,7 @@ def r2_pagerank(nest, lim):
     claimed by warps in chunks of 4*32/V; min(6*SMs, chunks) blocks. Returns (dims, blocks, spans, factors,
     vec, chunks, G, chunk)."""
     (N, _), (inner, _) = nest["levels"]
-    V = min(32, pow2ceil(cdiv(inner, 2)))          # two edges per lane for a row of average length
+    V = min(32, pow2ceil(cdiv(inner, 4)))          # four edges per lane for a row of average length
     RPB = 256 // V
     chunk = 4 * (32 // V)                          # a warp's claim: 4 rows per group
     G = min(6 * lim["sm_count"], cdiv(N, chunk))

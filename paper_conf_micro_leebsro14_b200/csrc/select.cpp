@@ -384,7 +384,7 @@ bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
 // rows claimed by warps in chunks of 4*32/V; min(6*SMs, chunks) blocks.
 void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], inner = n.N[1];
-  const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 2)));  // two edges per lane on average
+  const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 4)));  // four edges per lane on average
   const int64_t RPB = 256 / V, chunk = 4 * (32 / V);  // a warp's claim: 4 rows per group
   const int64_t units = cdiv(N, chunk);
   c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
