@@ -420,13 +420,13 @@ def r2_rowscols(nest, dtype, lim):
 
 def r2_pagerank(nest, lim):
     """DESIGN.md S8 PR: V = min(32, pow2 >= ceil(ceil(E/N)/2)) lanes per row on x, 256/V row groups on y, rows
-    claimed by warps in chunks of 4*32/V; min(3*SMs, chunks) blocks. Returns (dims, blocks, spans, factors,
+    claimed by warps in chunks of 4*32/V; min(4*SMs, chunks) blocks. Returns (dims, blocks, spans, factors,
     vec, chunks, G, chunk)."""
     (N, _), (inner, _) = nest["levels"]
-    V = min(32, pow2ceil(cdiv(inner, 8)))          # eight edges per lane for a row of average length
+    V = min(32, pow2ceil(cdiv(inner, 4)))          # four edges per lane for a row of average length
     RPB = 256 // V
     chunk = 4 * (32 // V)                          # a warp's claim: 4 rows per group
-    G = min(3 * lim["sm_count"], cdiv(N, chunk))
+    G = min(4 * lim["sm_count"], cdiv(N, chunk))
     return (Y, X), (RPB, V), (SPAN_N, ALL), (4, 1), 1, (chunk, inner), G, chunk
 
 

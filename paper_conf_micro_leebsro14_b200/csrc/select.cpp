@@ -381,10 +381,10 @@ bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
 }
 
 // S8 PAGERANK (class PR): V = min(32, pow2 >= ceil(ceil(E/N)/2)) lanes per row on x, 256/V row groups on y,
-// rows claimed by warps in chunks of 4*32/V; min(3*SMs, chunks) blocks.
+// rows claimed by warps in chunks of 4*32/V; min(4*SMs, chunks) blocks.
 void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], inner = n.N[1];
-  const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 8)));  // eight edges per lane on average
+  const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 4)));  // four edges per lane on average
   const int64_t RPB = 256 / V, chunk = 4 * (32 / V);  // a warp's claim: 4 rows per group
   const int64_t units = cdiv(N, chunk);
   c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
@@ -393,7 +393,7 @@ void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = inner;
   c->vec = 1;
   c->staged = 0;
-  c->persistent_grid = std::min<int64_t>(3 * int64_t(lim.sm_count), units);  // 3 x 256 threads per SM
+  c->persistent_grid = std::min<int64_t>(4 * int64_t(lim.sm_count), units);  // 4 x 256 threads per SM
   c->claim_tiles = chunk;
 }
 
