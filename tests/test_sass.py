@@ -70,3 +70,23 @@ def test_kmeans_centroids_on_uniform_datapath(sass):
 def test_packed_fma_in_kmeans(sass):
     for n in _find(sass, "npp_kmeans_tma_kernel"):
         assert sass[n]["FFMA2"] >= 2 * sass[n]["FFMA"], (n, sass[n]["FFMA2"], sass[n]["FFMA"])
+
+
+def test_new_staged_families_use_tma(sass):
+    # the one-pass rows+cols (staged variant) and the k-means update stream their tiles with TMA; the
+    # rows+cols direct variant (ragged row pitch) has no tensor map and loads with LDG instead
+    for n in _find(sass, "npp_rowscols_kernel"):
+        tma = sum(sass[n][f"UTMALDG.{d}D"] for d in (1, 2, 3))
+        if "Lb1E" in n:   # STAGED = true
+            assert tma > 0, n
+        else:
+            assert tma == 0 and sum(v for k, v in sass[n].items() if k.startswith("LDG")) > 0, n
+    for n in _find(sass, "npp_kmupdate_kernel"):
+        assert sass[n]["UTMALDG.2D"] > 0 and sass[n]["UTMALDG.1D"] > 0, n
+
+
+def test_slot_tags_use_native_shared_atomics(sass):
+    # the staged sums hand slot tags over with 32-bit shared atomics (racecheck-visible); a 64-bit form
+    # compiles to a CAS loop (ATOMS.CAST.SPIN), which the design avoids
+    for n in _find(sass, "npp_sum_tma_kernel"):
+        assert sass[n]["ATOMS.CAST.SPIN.64"] == 0 and sass[n]["ATOMS.EXCH"] > 0, (n, dict(sass[n]))
