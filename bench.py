@@ -180,17 +180,29 @@ def build_kmeans_update(npp, gen, torch, rank, world, strategy, device):
 
 def build_pagerank(npp, gen, torch, rank, world, strategy, device):
     # one PageRank step (Fig 5) over a 4M-node power-law graph (mean in-degree ~16,
-    # cap 1024, ~63M edges); a rank owns its nodes' rows (the graph is replicated per rank here)
+    # cap 1024, ~63M edges). At N > 1 rank r computes its node rows [lo, hi) from its CSR shard against
+    # the replicated previous vector, and the step ends with an all-gather of the next vector
     N = 1 << 22
     rowptr, colidx, pr, outdeg = gen.pagerank_inputs(N, avg_deg=16, seed=7, max_deg=1024, device=device)
     E = colidx.numel()
-    plan = npp.Plan("PAGERANK", (N, E), "f32", "AUTO", device=device)
-    item = Item("pagerank[4M,%dM]" % (E // 1000000), plan, [rowptr, colidx, pr, outdeg], plan.new_out(),
-                (N + 1) * 8 + E * 4 + N * 4 * 3)
-    # the random gathers bound this path: one L1tex wavefront (128-B line) per edge for contrib[w], plus
-    # the coalesced colidx / rowptr / per-node lines (DESIGN.md §6 PR)
-    item.wavefronts = E + E * 4 // 128 + (N + 1) * 8 // 128 + 3 * N * 4 // 128
-    return [item], [], "PageRank step, 4M nodes, ~63M edges"
+    if world == 1:
+        plan = npp.Plan("PAGERANK", (N, E), "f32", "AUTO", device=device)
+        item = Item("pagerank[4M,%dM]" % (E // 1000000), plan, [rowptr, colidx, pr, outdeg], plan.new_out(),
+                    (N + 1) * 8 + E * 4 + N * 4 * 3)
+        # the random gathers bound this path: one L1tex wavefront (128-B line) per edge for contrib[w], plus
+        # the coalesced colidx / rowptr / per-node lines (DESIGN.md §6 PR)
+        item.wavefronts = E + E * 4 // 128 + (N + 1) * 8 // 128 + 3 * N * 4 // 128
+        return [item], [], "PageRank step, 4M nodes, ~63M edges"
+    from paper_conf_micro_leebsro14_b200.dist import shard_range
+    lo, hi = shard_range(N, world, rank)
+    e0, e1 = int(rowptr[lo]), int(rowptr[hi])
+    lrp = (rowptr[lo:hi + 1] - e0).contiguous()
+    lci = colidx[e0:e1].contiguous()
+    plan = npp.Plan("PAGERANK", (hi - lo, e1 - e0, N), "f32", "AUTO", device=device)
+    item = Item("pagerank_shard[4M,%dM]" % (E // 1000000), plan, [lrp, lci, pr, outdeg], plan.new_out(),
+                (hi - lo + 1) * 8 + (e1 - e0) * 4 + (hi - lo) * 4 + 2 * N * 4)
+    item.gather = (world, N)
+    return [item], [], "PageRank step, 4M nodes, ~63M edges, node rows sharded + all-gather"
 
 
 def build_logreg(npp, gen, torch, rank, world, strategy, device):
@@ -218,7 +230,7 @@ def build_rowscols(npp, gen, torch, rank, world, strategy, device):
 
 # per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
 SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak",
-           "kmeans_update": "weak", "pagerank": "weak"}
+           "kmeans_update": "weak", "pagerank": "strong"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
              "logreg": build_logreg, "rowscols": build_rowscols, "kmeans_update": build_kmeans_update,
              "pagerank": build_pagerank}
@@ -405,12 +417,23 @@ def main():
     # drain (npp_execute_ex NPP_EXEC_OVERLAP); outputs still wait for the previous kernel
     overlap = not args.no_overlap
 
+    gathers = [(it, torch.empty(it.gather[1], dtype=it.out.dtype, device=device)) for it in items
+               if getattr(it, "gather", None)]
+
     def step():
         for it in items:
             it.run(stream, overlap)
         for b in reduce_bufs:
             with torch.cuda.stream(stream):
                 dist.all_reduce(b)
+        for it, full in gathers:  # PageRank shards: the next vector on every rank (uneven shards padded)
+            with torch.cuda.stream(stream):
+                n = it.out.numel()
+                mx = -(-it.gather[1] // world)
+                buf = torch.zeros(mx, dtype=it.out.dtype, device=device)
+                buf[:n] = it.out
+                parts = [torch.empty(mx, dtype=it.out.dtype, device=device) for _ in range(world)]
+                dist.all_gather(parts, buf)
 
     # one step = the six launches; at N=1 it is captured once into a CUDA graph and replayed, so the
     # timed region holds the kernels back to back without host launch gaps (streams and graphs are
