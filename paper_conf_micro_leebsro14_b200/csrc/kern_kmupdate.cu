@@ -235,176 +235,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
-// Sorted variant (the launch default): per tile, the 128 keys are counting-sorted in shared memory
-// (integer shared atomics are native: ATOMS.ADD returns each point's rank in its bin), and warp w
-// then owns the keys k = w, w+8, ...: it adds each owned key's points in REGISTERS (no read-modify-
-// write chain, no aliasing between points) and updates that key's fp64 block-accumulator row ONCE
-// per tile. Rows are owned by one warp, so the block accumulator is shared (no per-warp copies, no
-// fold). Three consumer barriers per tile (histogram, scan, scatter); bins and index lists are
-// double-buffered by tile parity and reset by their owner warp.
-constexpr int kSortSmem = kHeader + kStages * (kXSlot + kASlot) + 2 * kMaxK * 4 /*hist*/ + 2 * kMaxK * 4 /*offs*/ +
-                          2 * kTP * 2 /*idx*/ + (kMaxKD + kMaxK) * 8 /*bacc*/;
-
-__global__ void __launch_bounds__(kThreads, 1)
-    npp_kmupdate_sorted_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap amap,
-                               const KmUpdateArgs a) {
-  extern __shared__ __align__(1024) unsigned char smem[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
-  uint64_t* empty = full + kStages;
-  volatile int* flag = reinterpret_cast<volatile int*>(empty + kStages);
-  unsigned char* xring = smem + kHeader;
-  unsigned char* aring = xring + kStages * kXSlot;
-  unsigned* hist = reinterpret_cast<unsigned*>(aring + kStages * kASlot);  // [2][kMaxK]
-  unsigned* offs = hist + 2 * kMaxK;                                       // [2][kMaxK]
-  unsigned short* idx = reinterpret_cast<unsigned short*>(offs + 2 * kMaxK);  // [2][kTP]
-  double* bacc = reinterpret_cast<double*>(idx + 2 * kTP);                  // [K x (D+1)]
-  const int D = int(a.D), K = int(a.K), KD1 = K * (D + 1);
-
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long T = (a.N + kTP - 1) / kTP;
-  const long long t0 = blockIdx.x * a.per_block;
-  const long long t1 = t0 + a.per_block < T ? t0 + a.per_block : T;
-
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kStages; ++i) {
-      mbar_init(full + i, 1);
-      mbar_init(empty + i, kConsumerWarps);
-    }
-    mbar_fence_init();
-  }
-  if (threadIdx.x < kConsumers) {
-    for (int i = threadIdx.x; i < 2 * kMaxK; i += kConsumers) hist[i] = 0u;
-    for (int i = threadIdx.x; i < KD1; i += kConsumers) bacc[i] = 0.0;
-  }
-  __syncthreads();
-
-  if (warp == kConsumerWarps) {
-    // ------------------------------------------------------------ producer: one elected lane
-    if (lane == 0) {
-      prefetch_map(&xmap);
-      prefetch_map(&amap);
-      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
-      const unsigned bytes = unsigned(kTP * D * 4 + kASlot);
-      for (long long t = t0; t < t1; ++t) {
-        const long long i = t - t0;
-        const int slot = int(i % kStages);
-        if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
-        mbar_expect_tx(full + slot, bytes);
-        load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
-        load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
-      }
-    }
-    return;
-  }
-
-  // -------------------------------------------------------------- consumers
-  const bool dim_lane = 2 * lane < D;
-  int slot = 0;
-  unsigned phase = 0;
-  int b = 0;  // bins / index buffer (tile parity)
-  for (long long t = t0; t < t1;
-       ++t, slot = slot + 1 == kStages ? 0 : slot + 1, phase ^= slot == 0 ? 1u : 0u, b ^= 1) {
-    mbar_wait(full + slot, phase);
-    const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
-    const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
-    const int np = t + 1 < t1 || t1 * kTP <= a.N ? kTP : int(a.N - t * kTP);
-    unsigned* hb = hist + b * kMaxK;
-    unsigned* ob = offs + b * kMaxK;
-    unsigned short* ib = idx + b * kTP;
-    // 1. each point's rank in its key's bin
-    int k = -1;
-    unsigned r = 0;
-    if (threadIdx.x < np) {
-      k = at[threadIdx.x];
-      if (unsigned(k) < unsigned(K)) r = atomicAdd(hb + k, 1u);
-      else k = -1;
-    }
-    consumers_sync();
-    // 2. exclusive prefix of the bins (warp 0, 8 bins per lane)
-    if (warp == 0) {
-      unsigned v[kMaxK / 32], sum = 0;
-#pragma unroll
-      for (int q = 0; q < kMaxK / 32; ++q) {
-        const int kk = lane * (kMaxK / 32) + q;
-        v[q] = kk < K ? hb[kk] : 0u;
-        sum += v[q];
-      }
-      unsigned incl = sum;
-#pragma unroll
-      for (int o = 1; o < 32; o *= 2) {
-        const unsigned n = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += n;
-      }
-      unsigned run = incl - sum;
-#pragma unroll
-      for (int q = 0; q < kMaxK / 32; ++q) {
-        const int kk = lane * (kMaxK / 32) + q;
-        if (kk < K) ob[kk] = run;
-        run += v[q];
-      }
-    }
-    consumers_sync();
-    // 3. scatter the point indices, grouped by key
-    if (k >= 0) ib[ob[k] + r] = (unsigned short)threadIdx.x;
-    consumers_sync();
-    // 4. warp w adds the points of its keys in registers, then updates each key's row once
-    for (int kk = warp; kk < K; kk += kConsumerWarps) {
-      const unsigned n = hb[kk];
-      if (n == 0) continue;
-      const unsigned o = ob[kk];
-      float sx = 0.f, sy = 0.f;
-      if (dim_lane) {
-        unsigned i = 0;
-        for (; i + 4 <= n; i += 4) {
-          float2 xv[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) xv[q] = *reinterpret_cast<const float2*>(xt + int(ib[o + i + q]) * D + 2 * lane);
-#pragma unroll
-          for (int q = 0; q < 4; ++q) sx += xv[q].x, sy += xv[q].y;
-        }
-        for (; i < n; ++i) {
-          const float2 xv = *reinterpret_cast<const float2*>(xt + int(ib[o + i]) * D + 2 * lane);
-          sx += xv.x, sy += xv.y;
-        }
-        bacc[kk * (D + 1) + 2 * lane] += double(sx);
-        bacc[kk * (D + 1) + 2 * lane + 1] += double(sy);
-      }
-      if (lane == 0) {
-        bacc[kk * (D + 1) + D] += double(n);
-        hb[kk] = 0u;  // the bin is free again for tile t+2 (tile t+1's barriers order this)
-      }
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty + slot);
-  }
-
-  // ---- block result -> fp64 workspace accumulators; the last block converts (fused Split combine)
-  asm volatile("griddepcontrol.wait;" ::: "memory");
-  consumers_sync();
-  for (int i = threadIdx.x; i < KD1; i += kConsumers) {
-    const double v = bacc[i];
-    if (v != 0.0) atomicAdd(a.acc + i, v);
-  }
-  __threadfence();
-  consumers_sync();
-  if (threadIdx.x == 0) {
-    const bool last = atomicAdd(a.ticket, 1u) + 1u == gridDim.x;
-    if (last) *a.ticket = 0u;
-    flag[0] = last ? 1 : 0;
-  }
-  consumers_sync();
-  if (flag[0]) {
-    __threadfence();
-    for (int i = threadIdx.x; i < KD1; i += kConsumers) {
-      const double v = __ldcg(a.acc + i);
-      __stcg(a.acc + i, 0.0);
-      a.out[i] = float(v);
-    }
-  }
-}
-
 cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st) {
   if (a.D % 4 != 0 || a.D < 4 || a.D > 64 || a.K < 1 || a.K > kMaxK || a.K * a.D > kMaxKD)
     return cudaErrorInvalidValue;
@@ -414,11 +244,11 @@ cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* ke
   if ((e = encode_1d(&amap, keys, CU_TENSOR_MAP_DATA_TYPE_INT32, a.N, unsigned(kTP))) != cudaSuccess) return e;
   static bool attr_set = false;
   if (!attr_set) {
-    e = cudaFuncSetAttribute(npp_kmupdate_sorted_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSortSmem);
+    e = cudaFuncSetAttribute(npp_kmupdate_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  return launch_pdl(npp_kmupdate_sorted_kernel, grid, kThreads, kSortSmem, st, true, xmap, amap, a);
+  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, true, xmap, amap, a);
 }
 
 }  // namespace npp
