@@ -168,10 +168,11 @@ def build_kmeans(npp, gen, torch, rank, world, strategy, device):
 
 def build_kmeans_update(npp, gen, torch, rank, world, strategy, device):
     # the centroid update after the config-4 assignment: 4M points x 64 dims into
-    # 32 groups; keys = the assignment of the same points (computed once, outside the timed region)
+    # 32 groups; keys = the generator's cluster labels of the same points (synthetic inputs, so the
+    # cpu_baseline's oracle never consumes a CUDA result)
     N, D, K = 1 << 22, 64, 32
     x, c = gen.kmeans_inputs(N, D, K, row_offset=rank * N, device=device)
-    a = npp.kmeans_assign(x, c)
+    a = gen.int_uniform(5 + 1, (N,), 0, K - 1, dtype=torch.int32, offset=rank * N, device=device)
     plan = npp.Plan("KMEANS_UPDATE", (N, D, K), "f32", "AUTO", device=device)
     out = plan.new_out()
     item = Item("kmeans_update[4M,64,32]", plan, [x, a], out, N * D * 4 + N * 4 + K * (D + 1) * 4)

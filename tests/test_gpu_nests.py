@@ -205,26 +205,30 @@ def test_kmeans_update_parity(npp, cuda_device, N, D, K):
 
 def test_kmeans_update_integer_exact(npp, cuda_device):
     # integer coordinates: every partial sum is an exact fp32 integer (|U| < 2^24), so bit-exact
+    # (keys: the oracle's own assignment of the points — no oracle input comes from the CUDA path)
     N, D, K = 50000, 64, 32
     x, c = gen.kmeans_inputs(N, D, K, device=cuda_device, integer=True)
-    a = npp.kmeans_assign(x, c)
-    u = npp.kmeans_update(x, a, K)
+    xn = x.cpu().numpy()
+    an = okm.assign(xn, c.cpu().numpy())
+    u = npp.kmeans_update(x, torch.from_numpy(an).to(cuda_device), K)
     torch.cuda.synchronize()
-    assert np.array_equal(u.cpu().numpy().astype(np.float64), okm.update(x.cpu().numpy(), a.cpu().numpy(), K))
+    assert np.array_equal(u.cpu().numpy().astype(np.float64), okm.update(xn, an, K))
 
 
 def test_lloyd_step_full_size(npp, cuda_device):
     # one Lloyd iteration on the BASELINE.json k-means configuration (4M x 64 x 32): assignment, then
-    # the update, both on the GPU; the update is checked against the oracle on the GPU's assignment
-    # (sampled: the first 1M points through a second plan), and the full-size update by its invariants
+    # the update, both on the GPU, checked by invariants that hold for any assignment. Parity at this
+    # size uses the generator's own cluster labels z as keys (a synthetic input, not a CUDA result):
+    # the first 1M points through a second plan against the oracle
     N, D, K = 1 << 22, 64, 32
     x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
     a = npp.kmeans_assign(x, c)
     u = npp.kmeans_update(x, a, K)
     n1 = 1 << 20
-    u1 = npp.Plan("KMEANS_UPDATE", (n1, D, K)).execute([x[:n1], a[:n1]], torch.empty(K, D + 1, device=cuda_device))
+    z = gen.int_uniform(5 + 1, (n1,), 0, K - 1, dtype=torch.int32, device=cuda_device)  # kmeans_inputs' labels
+    u1 = npp.Plan("KMEANS_UPDATE", (n1, D, K)).execute([x[:n1], z], torch.empty(K, D + 1, device=cuda_device))
     torch.cuda.synchronize()
-    _check_update(u1, x[:n1], a[:n1], K)
+    _check_update(u1, x[:n1], z, K)
     un = u.cpu().numpy().astype(np.float64)
     assert un[:, -1].sum() == N                                           # every point in one group
     colsum = x.double().sum(0).cpu().numpy()                              # Σ_k U[k] = Σ_i x_i
