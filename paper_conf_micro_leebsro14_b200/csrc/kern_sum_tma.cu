@@ -307,14 +307,20 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       const unsigned ends = __ballot_sync(0xffffffffu, lane < nb && ot < 0);
       const int n = ends ? __ffs(ends) - 1 : nb;  // entries before the end marker
       const unsigned long long t_b0 = a.dbg_times ? gtimer() : 0ull;
-      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      // the ticket add is itself the release (cumulative over the consumers' accumulator adds, which
+      // the fl_full mbarrier ordered before it) and the acquire of the contributor that completes
+      // the tile; the other lanes read the accumulators after a fence only when some tile completed
       bool last = false;
       if (lane < n) {
-        const unsigned prev = atomicAdd(a.tickets + ot, cnt);
+        unsigned prev;
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;"
+                     : "=r"(prev)
+                     : "l"(a.tickets + ot), "r"(cnt)
+                     : "memory");
         last = prev + cnt == unsigned(a.Ti);
         if (last) a.tickets[ot] = 0u;
       }
-      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      if (__any_sync(0xffffffffu, last)) asm volatile("fence.acq_rel.gpu;" ::: "memory");
       if (a.dbg_times && lane == 0 && n > 0) {  // measurement knob: the last batch's phases
         a.dbg_times[bid * 8 + 4] = t_b0;
         a.dbg_times[bid * 8 + 5] = gtimer();
