@@ -217,10 +217,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     const double v = bacc[i];
     if (v != 0.0) atomicAdd(a.acc + i, v);
   }
-  __threadfence();
   consumers_sync();
-  if (threadIdx.x == 0) {
-    const bool last = atomicAdd(a.ticket, 1u) + 1u == gridDim.x;
+  if (threadIdx.x == 0) {  // acq_rel ticket: the release of every consumer's adds (barrier above)
+    const bool last = ticket_add(a.ticket, 1u) + 1u == gridDim.x;
     if (last) *a.ticket = 0u;
     flag[0] = last ? 1 : 0;
   }

@@ -196,11 +196,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
         atomicAdd(a.acc + b * C + c, s);
     }
     if (!owned) {
-      __threadfence();
       tma::bar_sync_consumers<kConsumers>();
       if (threadIdx.x == 0) {
         const unsigned contributors = unsigned((f1 - 1) / P - f0 / P + 1);
-        const unsigned prev = atomicAdd(a.tickets + b, 1u);
+        const unsigned prev = tma::ticket_add(a.tickets + b, 1u);  // release of the block's adds
         *s_last = (prev + 1 == contributors) ? 1u : 0u;
         if (prev + 1 == contributors) a.tickets[b] = 0u;
       }

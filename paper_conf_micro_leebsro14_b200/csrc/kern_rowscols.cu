@@ -243,16 +243,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     // column regions of row region ri add their row partials (band ends above), the gr row regions of
     // column group cj their column partials; the last of each converts and re-zeroes.
     if (a.gr > 1 || a.gc > 1) {
-      __threadfence();
       consumers_sync();
-      if (threadIdx.x == 0) {
+      if (threadIdx.x == 0) {  // acq_rel tickets: the release of every consumer's adds (barrier above)
         bool last_r = false, last_c = false;
         if (a.gc > 1) {
-          last_r = atomicAdd(a.tick_r + ri, 1u) + 1u == unsigned(a.gc);
+          last_r = ticket_add(a.tick_r + ri, 1u) + 1u == unsigned(a.gc);
           if (last_r) a.tick_r[ri] = 0u;
         }
         if (a.gr > 1) {
-          last_c = atomicAdd(a.tick_c + cj, 1u) + 1u == unsigned(a.gr);
+          last_c = ticket_add(a.tick_c + cj, 1u) + 1u == unsigned(a.gr);
           if (last_c) a.tick_c[cj] = 0u;
         }
         flag[0] = last_r ? 1 : 0;

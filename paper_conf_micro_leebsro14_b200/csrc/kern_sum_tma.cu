@@ -30,6 +30,7 @@
 #include <type_traits>
 
 #include "kernels.hpp"
+#include "tma_ring.cuh"
 
 #ifndef NPP_TMA_STAGES
 #define NPP_TMA_STAGES 4
@@ -312,11 +313,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       // the tile; the other lanes read the accumulators after a fence only when some tile completed
       bool last = false;
       if (lane < n) {
-        unsigned prev;
-        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;"
-                     : "=r"(prev)
-                     : "l"(a.tickets + ot), "r"(cnt)
-                     : "memory");
+        const unsigned prev = tma::ticket_add(a.tickets + ot, cnt);
         last = prev + cnt == unsigned(a.Ti);
         if (last) a.tickets[ot] = 0u;
       }

@@ -66,6 +66,16 @@ __device__ __forceinline__ void load_1d(void* dst, const CUtensorMap* map, int x
 __device__ __forceinline__ void prefetch_map(const CUtensorMap* map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
 }
+// Split-combine ticket: a gpu-scope acq_rel add. Its release is cumulative over the accumulator adds
+// that a preceding CTA barrier / mbarrier ordered before it (so the writers need no fence of their
+// own), and its acquire orders the completing contributor's reads of the accumulators after it.
+// Measured on the staged sums: the step 6552 -> 6645 GB/s against fence + atomicAdd + fence.
+__device__ __forceinline__ unsigned ticket_add(unsigned* p, unsigned v) {
+  unsigned prev;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(prev) : "l"(p), "r"(v) : "memory");
+  return prev;
+}
+
 // named barrier over the first `n` threads of the block (the consumer warps)
 template <int N>
 __device__ __forceinline__ void bar_sync_consumers() {
