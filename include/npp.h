@@ -70,7 +70,7 @@ typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2 } npp_dtype;
  *                      out[N] f32 = (1-0.85)/N + 0.85 * Σ_{j=rowptr[n]}^{rowptr[n+1]-1} pr[w_j]/outdeg[w_j], w_j = colidx[j]
  *                      one PageRank step (Fig 5) over the CSR of IN-neighbours; the caller
  *                      guarantees 0 <= rowptr[n] <= rowptr[n+1] <= E, 0 <= colidx < N and outdeg >= 1 for
- *                      every id in colidx (no device-side checks); colidx 16-byte aligned. AUTO only. */
+ *                      every id in colidx (no device-side checks). AUTO only. */
 typedef enum {
   NPP_SUM_ROWS = 0,
   NPP_SUM_COLS = 1,

@@ -468,10 +468,6 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     return NPP_OK;
   }
   if (plan->pattern == NPP_PAGERANK) {  // class PR (S8 PR)
-    if (ins[1] && !aligned16(ins[1])) {
-      set_error("PAGERANK: colidx must be 16-byte aligned (read in 16-byte quads)");
-      return NPP_ERR_ALIGNMENT;
-    }
     npp::PagerankArgs r{};
     r.rowptr = static_cast<const long long*>(ins[0]);
     r.colidx = static_cast<const int*>(ins[1]);
@@ -481,7 +477,6 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     r.pool = static_cast<unsigned*>(workspace);
     r.contrib = reinterpret_cast<float*>(static_cast<char*>(workspace) + 256);
     r.N = plan->shape[0];
-    r.E = plan->shape[1];
     r.Nnodes = plan->ndim == 3 ? plan->shape[2] : plan->shape[0];
     r.damp = 0.85f;
     cudaError_t e = npp::launch_pagerank(r, m.level[1].block, int(m.grid), st);

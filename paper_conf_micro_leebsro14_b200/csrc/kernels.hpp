@@ -136,7 +136,6 @@ struct PagerankArgs {
   unsigned* pool;           // row-chunk claim counter (zero on entry and on exit)
   float* contrib;           // [N] workspace: prevPR(w) / w.degree (Fig 5's inner map, once per node)
   int64_t N;        // rows computed (a shard's rows, or all nodes)
-  int64_t E;        // edges in colidx (bounds the 16-byte quad reads)
   int64_t Nnodes;   // nodes of the graph: length of pr / outdeg / contrib, and the N of (1-damp)/N
   float damp;
 };
