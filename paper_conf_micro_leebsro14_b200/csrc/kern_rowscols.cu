@@ -204,13 +204,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         asm volatile("griddepcontrol.wait;" ::: "memory");
         waited = true;
       }
-      if (a.gc > 1) {
-        // rows are Split across column regions anyway: every warp adds its own row partials (lane l:
-        // row rg*RPT + l) to the accumulators, no barrier per band
-        const long long row = br * kTileRows + rg * RPT + lane;
-        if (lane < RPT && row < a.R) atomicAdd(accR + row, racc);
-        continue;
-      }
       rsum[(rb * kConsumerWarps + warp) * 32 + lane] = racc;
       consumers_sync();
       if (warp == 0) {
