@@ -373,25 +373,25 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
-RC_BANDS_MAX = 128                                # DESIGN.md S8 RC: row bands of one region
+RC_COL_TILES_MAX = 32                             # DESIGN.md S8 RC: column tiles of one region
 
 
 def rc_tiling(R, C, dtype, lim):
     """DESIGN.md S8 RC region rule. The ceil(R/32) x ceil(C/BC) tile grid is cut into regions of cr row
-    bands (cr <= 128) x cc column tiles. Written as the plain double loop over gc and gr:
-    for gc in [1, min(Tc, S)], gr in [ceil(Tr/128), max(that, min(Tr, S // gc'))], with cc = ceil(Tc/gc),
+    bands x cc column tiles (cc <= 32). Written as the plain double loop over gc and gr:
+    for gc in [ceil(Tc/32), max(that, min(Tc, S))], gr in [1, min(Tr, S // gc')], with cc = ceil(Tc/gc),
     gc' = ceil(Tc/cc), cr = ceil(Tr/gr), gr' = ceil(Tr/cr), nreg = gr'*gc', G = min(S, nreg):
     minimise (ceil(nreg/G)*cr*cc, nreg, gc'), the first minimum winning.
     Returns dict(BC, Tr, Tc, cr, cc, gr, gc, nreg, G)."""
     S = lim["sm_count"]
     BC = 1024 // DTYPE_SIZE[dtype]
     Tr, Tc = cdiv(R, STAGE_ROWS), cdiv(C, BC)
-    gr_lo = cdiv(Tr, RC_BANDS_MAX)
+    gc_lo = cdiv(Tc, RC_COL_TILES_MAX)
     best, best_key = None, None
-    for gc in range(1, max(1, min(Tc, S)) + 1):
+    for gc in range(gc_lo, max(gc_lo, min(Tc, S)) + 1):
         cc = cdiv(Tc, gc)
         gce = cdiv(Tc, cc)
-        for gr in range(gr_lo, max(gr_lo, min(Tr, max(1, S // gce))) + 1):
+        for gr in range(1, min(Tr, max(1, S // gce)) + 1):
             cr = cdiv(Tr, gr)
             gre = cdiv(Tr, cr)
             nreg = gre * gce
@@ -404,19 +404,18 @@ def rc_tiling(R, C, dtype, lim):
 
 
 def r2_rowscols(nest, dtype, lim):
-    """DESIGN.md S8 RC: columns on x; 8 warps over a tile's rows, 32 lanes over its 16-byte vectors (vec =
-    16/esz when staged, else 1); the regions of rc_tiling as Split levels. Returns (dims, blocks, spans,
-    factors, vec, chunks, staged, G, claim)."""
+    """DESIGN.md S8 RC: columns on x, one thread per column of a 1 KB tile (256/BC row halves), the
+    regions of rc_tiling as Split levels. Returns (dims, blocks, spans, factors, vec, chunks, staged, G,
+    claim)."""
     (R, _), (C, _) = nest["levels"]
     t = rc_tiling(R, C, dtype, lim)
     dims = (Y, X)
-    blocks = (8, 32)
+    blocks = (256 // t["BC"], t["BC"])
     spans = (SPLIT if t["gr"] > 1 else ALL, SPLIT if t["gc"] > 1 else ALL)
     factors = (t["gr"], t["gc"])
     chunks = (STAGE_ROWS * t["cr"] if t["gr"] > 1 else R, t["BC"] * t["cc"] if t["gc"] > 1 else C)
     staged = 1 if C % (16 // DTYPE_SIZE[dtype]) == 0 else 0
-    vec = 16 // DTYPE_SIZE[dtype] if staged else 1
-    return dims, blocks, spans, factors, vec, chunks, staged, t["G"], t["cr"] * t["cc"]
+    return dims, blocks, spans, factors, 1, chunks, staged, t["G"], t["cr"] * t["cc"]
 
 
 def r2_pagerank(nest, lim):

@@ -8,24 +8,19 @@
 // both directions out of shared memory, which halves the bytes of the two-kernel schedule.
 //
 // Work split (S8 RC): the Tr x Tc tile grid is cut into gr x gc rectangular regions of
-// cr row bands (cr <= 128) x cc column tiles; block b of G takes regions [b*nreg/G, (b+1)*nreg/G).
-// Inside a region the walk is column-tile-major (all bands of a column tile, then the next):
-//   lanes: warp w owns rows 4w..4w+3 of a tile, lane l two 16-byte vectors of each (elements
-//          [4l, 4l+4) and [128+4l, ...) for 4-byte types: LDS.128, as the sumRows family);
-//   columns: a thread's 8 (4 for 8-byte types) column partials of the current column tile stay in
-//          registers across the bands (fp32 tree over the tile's 4 rows, then fp64); at the end of a
-//          column tile the eight warps meet in shared memory and the tile's columns are written (gr ==
-//          1) or added to accumulators;
-//   rows:    per tile the thread's 4 row partials go through one transposing butterfly (lane l ends
-//          with row 4w + l%4 of the tile) and lanes 0-3 add them to the region's shared-memory row
-//          accumulators (fp64, <= 4096 rows), flushed at region end.
-// A row band (column group) covered by several regions is the Split of P:L542-550: contributions meet
-// through fp64 / integer atomics and one acq_rel ticket per row region (column group) at region end;
-// the last contributor converts and re-zeroes (the combiner of P:L880-883, fused). gc == 1 rows and
-// gr == 1 columns are written directly. Without 16-B row pitch (no tensor map) the same consumers load
-// the tile straight from global memory element by element (STAGED = false; the producer warp idles).
-// (The first version — a thread per column, a 31-shuffle butterfly per tile and per-band barriers —
-// ran at 5.8-6.1 TB/s, consumer-bound.)
+// cr row bands x cc column tiles; block b of G takes regions [b*nreg/G, (b+1)*nreg/G). Inside a region
+// the walk is row-band-major:
+//   columns: thread t owns column t of every tile (two row halves for 8-byte types); its per-tile
+//            column partial (a pairwise tree over the tile's rows) is added to a shared-memory
+//            accumulator slot of the region's columns (<= 32 tiles = 64 KB), flushed at region end;
+//   rows:    each warp turns its per-thread row values into per-row partials with one transposing
+//            butterfly (lane l ends with row l), keeps them in a register across the band's column
+//            tiles, and the eight warps meet in shared memory once per band.
+// A row band (column region) covered by several regions is the Split of P:L542-550: contributions meet
+// through fp64 / integer atomics and one ticket per row region (column group), taken once at region
+// end; the last contributor converts and re-zeroes (the combiner of P:L880-883, fused). gc == 1 rows and gr == 1 columns are
+// written directly. Without 16-B row pitch (no tensor map) the same consumers load the tile straight
+// from global memory (STAGED = false; the producer warp idles).
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -48,10 +43,10 @@ constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
-constexpr int kBandsMax = 128;            // row bands of one region (select.hpp kRcBandsMax)
-constexpr int kRowAccBytes = kBandsMax * kTileRows * 8;          // region row accumulators
-constexpr int kColRedBytes = 2 * kConsumerWarps * 256 * 8;       // [2][8 warps][BC] column partials
-constexpr int kSmemBytes = kHeader + kStages * kTileBytes + kRowAccBytes + kColRedBytes;
+constexpr int kColTilesMax = 32;          // column tiles of one region (select.hpp kRcColTilesMax)
+constexpr int kColAccBytes = 64 * 1024;   // [row groups][kColTilesMax * BC] accumulators
+constexpr int kRowSumBytes = 2 * kConsumerWarps * 32 * 8;
+constexpr int kSmemBytes = kHeader + kStages * kTileBytes + kColAccBytes + kRowSumBytes;
 
 template <typename T> struct RcOps;
 template <> struct RcOps<float> {
@@ -69,19 +64,6 @@ template <> struct RcOps<int64_t> {
   using Acc = unsigned long long;
   __device__ static int64_t finish(unsigned long long a) { return int64_t(a); }
 };
-
-template <typename T> struct Vec16;
-template <> struct Vec16<float> { using type = float4; };
-template <> struct Vec16<int32_t> { using type = int4; };
-template <> struct Vec16<int64_t> { using type = longlong2; };
-template <typename S, typename V, int N>
-__device__ __forceinline__ void unpack(const V& v, S (&o)[N], int at) {
-  if constexpr (N == 2 || sizeof(S) == 8) {
-    o[at] = S(v.x), o[at + 1] = S(v.y);
-  } else {
-    o[at] = S(v.x), o[at + 1] = S(v.y), o[at + 2] = S(v.z), o[at + 3] = S(v.w);
-  }
-}
 
 // N values per lane -> the lane holds Σ over the 32 lanes of value (lane % N): log2 N transposing
 // steps (a lane keeps the half its bit selects and receives the partner's copy of it), then plain
@@ -125,17 +107,18 @@ __global__ void __launch_bounds__(kThreads, 1)
   using S = typename RcOps<T>::S;
   using Acc = typename RcOps<T>::Acc;
   constexpr int BC = 1024 / int(sizeof(T));  // columns of a tile
-  constexpr int VPL = 16 / int(sizeof(T));   // elements of a 16-byte vector
-  constexpr int EPL = 2 * VPL;               // tile columns one lane owns
-  constexpr int RPW = kTileRows / kConsumerWarps;  // tile rows one warp owns (4)
-  using V = typename Vec16<T>::type;
+  constexpr int WPG = BC / 32;               // warps across a tile's columns (8 or 4)
+  constexpr int NRG = kConsumerWarps / WPG;  // row groups (1 or 2)
+  constexpr int RPT = kTileRows / NRG;       // tile rows one thread adds (32 or 16)
+  constexpr int CAP = kColTilesMax * BC;     // column accumulators per row group
+  static_assert(NRG * CAP * int(sizeof(Acc)) <= kColAccBytes, "column accumulators exceed their region");
   extern __shared__ __align__(1024) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
   uint64_t* empty = full + kStages;
   volatile int* flag = reinterpret_cast<volatile int*>(empty + kStages);
   unsigned char* tiles = smem + kHeader;
-  Acc* rowacc = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes);                 // [kBandsMax * 32]
-  Acc* colred = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes + kRowAccBytes);  // [2][8][BC]
+  Acc* colacc = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes);  // [NRG][CAP]
+  Acc* rsum = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes + kColAccBytes);  // [2][8][32]
   Acc* accR = static_cast<Acc*>(a.accR);
   Acc* accC = static_cast<Acc*>(a.accC);
   T* out = static_cast<T*>(a.out);
@@ -154,7 +137,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     mbar_fence_init();
   }
   if (threadIdx.x < kConsumers)
-    for (int i = threadIdx.x; i < kBandsMax * kTileRows; i += kConsumers) rowacc[i] = Acc(0);
+    for (int i = threadIdx.x; i < NRG * CAP; i += kConsumers) colacc[i] = Acc(0);
   __syncthreads();
 
   if (warp == kConsumerWarps) {
@@ -167,8 +150,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         const long long ri = q / a.gc, cj = q - ri * a.gc;
         const long long b0 = ri * a.cr, b1 = b0 + a.cr < a.Tr ? b0 + a.cr : a.Tr;
         const long long c0 = cj * a.cc, c1 = c0 + a.cc < a.Tc ? c0 + a.cc : a.Tc;
-        for (long long ct = c0; ct < c1; ++ct)
-          for (long long br = b0; br < b1; ++br, ++t) {
+        for (long long br = b0; br < b1; ++br)
+          for (long long ct = c0; ct < c1; ++ct, ++t) {
             const int slot = int(t % kStages);
             if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
             mbar_expect_tx(full + slot, kTileBytes);
@@ -180,29 +163,25 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 
   // -------------------------------------------------------------- consumers
+  const int rg = warp / WPG;                 // row group: tile rows rg*RPT .. +RPT
+  const int col = (warp % WPG) * 32 + lane;  // tile column
   bool waited = false;
   long long t = 0;
-  int cb = 0;  // colred double buffer
+  int rb = 0;  // rsum double buffer
   for (long long q = q0; q < q1; ++q) {
     const long long ri = q / a.gc, cj = q - ri * a.gc;
     const long long b0 = ri * a.cr, b1 = b0 + a.cr < a.Tr ? b0 + a.cr : a.Tr;
     const long long c0 = cj * a.cc, c1 = c0 + a.cc < a.Tc ? c0 + a.cc : a.Tc;
-    for (long long ct = c0; ct < c1; ++ct) {
-      Acc cacc[EPL];
-#pragma unroll
-      for (int e = 0; e < EPL; ++e) cacc[e] = Acc(0);
-      for (long long br = b0; br < b1; ++br, ++t) {
-        S x[RPW][EPL];
+    for (long long br = b0; br < b1; ++br) {
+      Acc racc = Acc(0);
+      for (long long ct = c0; ct < c1; ++ct, ++t) {
+        S v[RPT];
         if constexpr (STAGED) {
           const int slot = int(t % kStages);
           mbar_wait(full + slot, unsigned((t / kStages) & 1));
-          const unsigned char* tile = tiles + slot * kTileBytes;
+          const T* tile = reinterpret_cast<const T*>(tiles + slot * kTileBytes);
 #pragma unroll
-          for (int rr = 0; rr < RPW; ++rr) {
-            const unsigned char* row = tile + (warp * RPW + rr) * 1024;
-            unpack(*reinterpret_cast<const V*>(row + lane * 16), x[rr], 0);
-            unpack(*reinterpret_cast<const V*>(row + 512 + lane * 16), x[rr], VPL);
-          }
+          for (int rr = 0; rr < RPT; ++rr) v[rr] = S(tile[(rg * RPT + rr) * BC + col]);
           __syncwarp();
           if (lane == 0) mbar_arrive(empty + slot);
         } else {
@@ -210,64 +189,59 @@ __global__ void __launch_bounds__(kThreads, 1)
             asm volatile("griddepcontrol.wait;" ::: "memory");
             waited = true;
           }
+          const long long c = ct * BC + col;
+          const long long r0 = br * kTileRows + rg * RPT;
           const T* m = static_cast<const T*>(a.m);
 #pragma unroll
-          for (int rr = 0; rr < RPW; ++rr) {
-            const long long r = br * kTileRows + warp * RPW + rr;
-#pragma unroll
-            for (int e = 0; e < EPL; ++e) {
-              const long long c = ct * BC + (e < VPL ? VPL * lane + e : BC / 2 + VPL * lane + e - VPL);
-              x[rr][e] = (r < a.R && c < a.C) ? S(__ldg(m + r * a.C + c)) : S(0);
-            }
-          }
+          for (int rr = 0; rr < RPT; ++rr)
+            v[rr] = (c < a.C && r0 + rr < a.R) ? S(__ldg(m + (r0 + rr) * a.C + c)) : S(0);
         }
-        // columns: the tile's 4 rows as a pairwise tree, into the thread's column accumulators
-#pragma unroll
-        for (int e = 0; e < EPL; ++e) cacc[e] += Acc((x[0][e] + x[1][e]) + (x[2][e] + x[3][e]));
-        // rows: each row's EPL elements, then one transposing butterfly over the warp
-        S rv[RPW];
-#pragma unroll
-        for (int rr = 0; rr < RPW; ++rr) rv[rr] = tree_sum(x[rr]);
-        const S rsum = transpose_reduce(rv, lane);  // lane l: row warp*4 + l%4 of this tile
-        if (lane < RPW) rowacc[(br - b0) * kTileRows + warp * RPW + lane] += Acc(rsum);
+        colacc[rg * CAP + (ct - c0) * BC + col] += Acc(tree_sum(v));
+        racc += Acc(transpose_reduce(v, lane));  // lane l: row rg*RPT + l % RPT of this band
       }
-      // ---- column-tile end: the eight warps' column partials meet in shared memory
+      // ---- band end: the warps' row partials meet in shared memory
       if (!waited) {  // out / workspace are written only after the previous grid in the stream is done
         asm volatile("griddepcontrol.wait;" ::: "memory");
         waited = true;
       }
-      Acc* cr = colred + cb * (kConsumerWarps * BC);
-#pragma unroll
-      for (int e = 0; e < EPL; ++e) cr[warp * BC + (e < VPL ? VPL * lane + e : BC / 2 + VPL * lane + e - VPL)] = cacc[e];
+      rsum[(rb * kConsumerWarps + warp) * 32 + lane] = racc;
       consumers_sync();
-      if (threadIdx.x < BC) {
-        Acc sum = Acc(0);
+      if (warp == 0) {
+        const int g = lane / RPT, li = lane % RPT;
+        Acc s = Acc(0);
 #pragma unroll
-        for (int w = 0; w < kConsumerWarps; ++w) sum += cr[w * BC + threadIdx.x];
-        const long long cg = ct * BC + threadIdx.x;
-        if (cg < a.C) {
-          if (a.gr == 1)
-            out[a.R + cg] = RcOps<T>::finish(sum);
+        for (int j = 0; j < WPG; ++j) s += rsum[(rb * kConsumerWarps + g * WPG + j) * 32 + li];
+        const long long row = br * kTileRows + lane;
+        if (row < a.R) {
+          if (a.gc == 1)
+            out[row] = RcOps<T>::finish(s);
           else
-            atomicAdd(accC + cg, sum);  // completed by the column-group ticket at region end
+            atomicAdd(accR + row, s);  // completed by the row-region ticket at region end
         }
       }
-      cb ^= 1;
+      rb ^= 1;
     }
-    // ---- region end: the region's row accumulators
+    // ---- region end: the region's column accumulators
     consumers_sync();
-    const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
-    for (long long row = rlo + threadIdx.x; row < rhi; row += kConsumers) {
-      const Acc sum = rowacc[row - rlo];
-      rowacc[row - rlo] = Acc(0);
-      if (a.gc == 1)
-        out[row] = RcOps<T>::finish(sum);
-      else
-        atomicAdd(accR + row, sum);
+    const long long ncols = (c1 - c0) * BC;
+    for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
+      Acc s = colacc[c];
+      colacc[c] = Acc(0);
+      if constexpr (NRG == 2) {
+        s += colacc[CAP + c];
+        colacc[CAP + c] = Acc(0);
+      }
+      const long long cg = c0 * BC + c;
+      if (cg < a.C) {
+        if (a.gr == 1)
+          out[a.R + cg] = RcOps<T>::finish(s);
+        else
+          atomicAdd(accC + cg, s);
+      }
     }
-    // Split combine (fused): one acq_rel ticket per region and direction. The gc column
-    // regions of row region ri add their row partials, the gr row regions of column group cj their
-    // column partials (column-tile ends above); the last of each converts and re-zeroes.
+    // Split combine (fused): one fence and one ticket per region and direction. The gc
+    // column regions of row region ri add their row partials (band ends above), the gr row regions of
+    // column group cj their column partials; the last of each converts and re-zeroes.
     if (a.gr > 1 || a.gc > 1) {
       consumers_sync();
       if (threadIdx.x == 0) {  // acq_rel tickets: the release of every consumer's adds (barrier above)
@@ -287,6 +261,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const bool last_r = flag[0] != 0, last_c = flag[1] != 0;
       if (last_r || last_c) __threadfence();
       if (last_r) {
+        const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
         for (long long row = rlo + threadIdx.x; row < rhi; row += kConsumers) {
           const Acc val = __ldcg(accR + row);
           __stcg(accR + row, Acc(0));
@@ -294,15 +269,17 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
       if (last_c) {
-        const long long clo = c0 * BC, chi = c1 * BC < a.C ? c1 * BC : a.C;
-        for (long long c = clo + threadIdx.x; c < chi; c += kConsumers) {
-          const Acc val = __ldcg(accC + c);
-          __stcg(accC + c, Acc(0));
-          out[a.R + c] = RcOps<T>::finish(val);
+        for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
+          const long long cg = c0 * BC + c;
+          if (cg < a.C) {
+            const Acc val = __ldcg(accC + cg);
+            __stcg(accC + cg, Acc(0));
+            out[a.R + cg] = RcOps<T>::finish(val);
+          }
         }
       }
     }
-    consumers_sync();  // row accumulators re-zeroed and the flags read before the next region
+    consumers_sync();  // accumulators re-zeroed and the flags read before the next region
   }
 }
 

@@ -350,13 +350,13 @@ void r2_rowscols(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const int64_t R = n.N[0], C = n.N[1];
   const RcTiling t = rc_tiling(R, C, dtype, lim.sm_count);
   c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
-  c->blocks[0] = 8, c->blocks[1] = 32;  // warps over a tile's rows, lanes over its 16-byte vectors
+  c->blocks[0] = int(256 / t.BC), c->blocks[1] = int(t.BC);
   c->spans[0] = t.gr > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[0] = t.gr;
   c->chunks[0] = t.gr > 1 ? kStageRows * t.cr : R;
   c->spans[1] = t.gc > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[1] = t.gc;
   c->chunks[1] = t.gc > 1 ? t.BC * t.cc : C;
+  c->vec = 1;
   c->staged = C % (16 / dtype_size(dtype)) == 0 ? 1 : 0;  // TMA needs a 16-B row pitch
-  c->vec = c->staged ? 16 / dtype_size(dtype) : 1;        // staged: 16-byte shared-memory vectors
   c->persistent_grid = t.G;
   c->claim_tiles = t.cr * t.cc;
 }
@@ -452,7 +452,7 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   return t;
 }
 
-// S8 RC region rule: over gc in [1, min(Tc, S)] and gr in [ceil(Tr/128), max(that, min(Tr, S/gc'))]
+// S8 RC region rule: over gc in [ceil(Tc/32), max(that, min(Tc, S))] and gr in [1, min(Tr, S/gc')]
 // (gc', gr' the region counts after rounding the region sizes cc = ceil(Tc/gc), cr = ceil(Tr/gr)),
 // minimise (ceil(nreg/G) * cr * cc = tiles of the busiest block, nreg, gc'); first minimum wins.
 RcTiling rc_tiling(int64_t R, int64_t C, int dtype, int sm_count) {
@@ -461,13 +461,13 @@ RcTiling rc_tiling(int64_t R, int64_t C, int dtype, int sm_count) {
   best.BC = 1024 / dtype_size(dtype);
   best.Tr = cdiv(R, kStageRows);
   best.Tc = cdiv(C, best.BC);
-  const int64_t gr_lo = cdiv(best.Tr, kRcBandsMax);
-  const int64_t gc_hi = std::max<int64_t>(1, std::min(best.Tc, S));
+  const int64_t gc_lo = cdiv(best.Tc, kRcColTilesMax);
+  const int64_t gc_hi = std::max(gc_lo, std::min(best.Tc, S));
   int64_t kc = -1, kn = 0, kg = 0;
-  for (int64_t gc = 1; gc <= gc_hi; ++gc) {
+  for (int64_t gc = gc_lo; gc <= gc_hi; ++gc) {
     const int64_t cc = cdiv(best.Tc, gc), gce = cdiv(best.Tc, cc);
-    const int64_t gr_hi = std::max(gr_lo, std::min(best.Tr, std::max<int64_t>(1, S / gce)));
-    for (int64_t gr = gr_lo; gr <= gr_hi; ++gr) {
+    const int64_t gr_hi = std::min(best.Tr, std::max<int64_t>(1, S / gce));
+    for (int64_t gr = 1; gr <= gr_hi; ++gr) {
       const int64_t cr = cdiv(best.Tr, gr), gre = cdiv(best.Tr, cr);
       const int64_t nreg = gre * gce, G = std::min(S, nreg);
       const int64_t cost = cdiv(nreg, G) * cr * cc;
