@@ -425,9 +425,9 @@ def r2_pagerank(nest, lim):
     (N, _), (inner, _) = nest["levels"]
     V = min(32, pow2ceil(cdiv(inner, 4)))          # four edges per lane for a row of average length
     RPB = 256 // V
-    chunk = 8 * (32 // V)                          # a warp's claim: 8 rows per group
+    chunk = 4 * (32 // V)                          # a warp's claim: 4 rows per group
     G = min(4 * lim["sm_count"], cdiv(N, chunk))
-    return (Y, X), (RPB, V), (SPAN_N, ALL), (8, 1), 1, (chunk, inner), G, chunk
+    return (Y, X), (RPB, V), (SPAN_N, ALL), (4, 1), 1, (chunk, inner), G, chunk
 
 
 def r2_kmupdate(nest, lim):

@@ -385,11 +385,11 @@ bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
 void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], inner = n.N[1];
   const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 4)));  // four edges per lane on average
-  const int64_t RPB = 256 / V, chunk = 8 * (32 / V);  // a warp's claim: 8 rows per group
+  const int64_t RPB = 256 / V, chunk = 4 * (32 / V);  // a warp's claim: 4 rows per group
   const int64_t units = cdiv(N, chunk);
   c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
   c->blocks[0] = int(RPB), c->blocks[1] = int(V);
-  c->spans[0] = NPP_SPAN_N, c->factors[0] = 8, c->chunks[0] = chunk;
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = 4, c->chunks[0] = chunk;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = inner;
   c->vec = 1;
   c->staged = 0;
