@@ -212,3 +212,46 @@ def test_r2_invariants(pat, shape, dtype):
         if lv["dim"] == S.X and lv["span"] == S.SPLIT:
             assert lv["chunk"] % r["vec"] == 0
     assert r["vec"] in (1, 16 // S.DTYPE_SIZE[dtype])
+
+
+# ---------------------------------------------------------------- NEXT rows: hand-computed records
+
+def test_rowscols_regions_by_hand():
+    # DESIGN.md S8 RC on B200 (S = 148): [8K,8K] f32 has Tr = 256 bands x Tc = 32 tiles; gc = 4 column
+    # groups of 8 tiles and gr = 37 row regions of 7 bands give 148 regions of <= 56 tiles (the fair share
+    # is 8192/148 = 55.35); [64K,1K]: 147 row regions of 14 bands, all 4 column tiles (rows written
+    # directly); [1K,64K]: 4 x 37 regions of 8 bands x 7 tiles
+    t = S.rc_tiling(8192, 8192, "f32", S.B200)
+    assert (t["Tr"], t["Tc"], t["cr"], t["cc"], t["gr"], t["gc"], t["G"]) == (256, 32, 7, 8, 37, 4, 148)
+    t = S.rc_tiling(65536, 1024, "f32", S.B200)
+    assert (t["cr"], t["cc"], t["gr"], t["gc"], t["G"]) == (14, 4, 147, 1, 147)
+    t = S.rc_tiling(1024, 65536, "f32", S.B200)
+    assert (t["cr"], t["cc"], t["gr"], t["gc"], t["G"]) == (8, 7, 4, 37, 148)
+    rec = S.select("SUM_ROWS_COLS", (8192, 8192), "f32", S.B200, "AUTO")
+    assert rec["kernel_class"] == S.RC and rec["staged"] == 1 and rec["grid"] == 148
+    assert [lv["span"] for lv in rec["levels"]] == [S.SPLIT, S.SPLIT]
+    assert [lv["factor"] for lv in rec["levels"]] == [37, 4]
+    assert [lv["chunk"] for lv in rec["levels"]] == [32 * 7, 256 * 8]
+    # tickets [37] + [4] (256 B each), accumulators [8192] + [8192] fp64
+    assert rec["workspace_bytes"] == 256 + 256 + 8192 * 8 + 8192 * 8
+
+
+def test_kmeans_update_record_by_hand():
+    # 4M points / 128 = 32768 tiles over 148 SMs: P = 222 tiles per block, G = ceil(32768/222) = 148;
+    # workspace = 256-B ticket + 32 x 65 fp64 accumulators rounded up to 256 B
+    rec = S.select("KMEANS_UPDATE", (1 << 22, 64, 32), "f32", S.B200, "AUTO")
+    assert rec["kernel_class"] == S.KU and rec["grid"] == 148 and rec["claim_tiles"] == 222
+    assert rec["levels"][0]["chunk"] == 128 * 222 and rec["levels"][0]["factor"] == 148
+    assert rec["workspace_bytes"] == 256 + 256 * -(-32 * 65 * 8 // 256)
+
+
+def test_pagerank_record_by_hand():
+    # mean in-degree ceil(63710769 / 4194304) = 16 -> V = pow2 >= 16/4 = 4 lanes per row, 64 row groups
+    # per block, warp claims of 4 rows x 8 groups = 32 rows, min(4 x 148, 131072) = 592 blocks;
+    # workspace = claim counter + contrib [4M] f32
+    rec = S.select("PAGERANK", (1 << 22, 63710769), "f32", S.B200, "AUTO")
+    assert rec["kernel_class"] == S.PR and rec["staged"] == 0
+    assert [lv["block"] for lv in rec["levels"]] == [64, 4]
+    assert rec["levels"][0]["chunk"] == 32 and rec["levels"][0]["grid"] == (1 << 22) // 32
+    assert rec["grid"] == 592 and rec["levels"][1]["chunk"] == 16
+    assert rec["workspace_bytes"] == 256 + 4 * (1 << 22)
