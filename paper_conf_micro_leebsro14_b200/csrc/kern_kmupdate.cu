@@ -152,13 +152,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
     const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
     const int np = t + 1 < t1 || t1 * kTP <= a.N ? kTP : int(a.N - t * kTP);  // valid points (TMA zero-fills)
-    // the warp's 16 points of the tile are p = 16w + j (contiguous): lane j < 16 reads key j (-1: no
-    // group) for the counts; the sums read each batch's 4 keys with one broadcast 16-byte load
-    constexpr int PPW = kTP / kConsumerWarps;
-    const int pw0 = PPW * warp;
+    // the warp's 16 points of the tile are p = warp + 8j: lane j < 16 reads key j (-1: no group)
     int kl = -1;
-    if (lane < PPW && pw0 + lane < np) {
-      kl = at[pw0 + lane];
+    if (lane < kTP / kConsumerWarps && warp + kConsumerWarps * lane < np) {
+      kl = at[warp + kConsumerWarps * lane];
       if (unsigned(kl) >= unsigned(K)) kl = -1;
     }
     // counts: lanes holding equal keys meet in match.any; the lowest of them adds the group's size
@@ -166,17 +163,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     const unsigned same = __match_any_sync(0xffffffffu, kl);
     // sums: 4 points at a time
 #pragma unroll
-    for (int j0 = 0; j0 < PPW; j0 += 4) {
+    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
       int k[4];
       float2 xv[4];
 #pragma unroll
-      const int4 kv = *reinterpret_cast<const int4*>(at + pw0 + j0);  // same address for all lanes
-      k[0] = kv.x, k[1] = kv.y, k[2] = kv.z, k[3] = kv.w;
-#pragma unroll
       for (int q = 0; q < 4; ++q) {
-        if (pw0 + j0 + q >= np || unsigned(k[q]) >= unsigned(K)) k[q] = -1;
+        k[q] = __shfl_sync(0xffffffffu, kl, j0 + q);
         xv[q] = make_float2(0.f, 0.f);
-        if (k[q] >= 0 && dim_lane) xv[q] = *reinterpret_cast<const float2*>(xt + (pw0 + j0 + q) * D + 2 * lane);
+        if (k[q] >= 0 && dim_lane)
+          xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
       }
       if (!dim_lane) continue;
       // a repeated key adds its point into the first point of that key (branch-free selects), so
