@@ -373,7 +373,7 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
-RC_COL_TILES_MAX = 16                             # DESIGN.md S8 RC: column tiles of one region
+RC_COL_TILES_MAX = 32                             # DESIGN.md S8 RC: column tiles of one region
 
 
 def rc_tiling(R, C, dtype, lim):

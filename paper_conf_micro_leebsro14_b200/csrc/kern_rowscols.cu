@@ -43,7 +43,7 @@ constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
-constexpr int kColTilesMax = 16;          // column tiles of one region (select.hpp kRcColTilesMax)
+constexpr int kColTilesMax = 32;          // column tiles of one region (select.hpp kRcColTilesMax)
 constexpr int kColAccBytes = 64 * 1024;   // [row groups][kColTilesMax * BC] accumulators
 constexpr int kRowSumBytes = 2 * kConsumerWarps * 32 * 8;
 constexpr int kSmemBytes = kHeader + kStages * kTileBytes + kColAccBytes + kRowSumBytes;
@@ -64,11 +64,6 @@ template <> struct RcOps<int64_t> {
   using Acc = unsigned long long;
   __device__ static int64_t finish(unsigned long long a) { return int64_t(a); }
 };
-
-template <typename T> struct Pair;  // two adjacent tile elements in one 8- or 16-byte shared-memory read
-template <> struct Pair<float> { using type = float2; };
-template <> struct Pair<int32_t> { using type = int2; };
-template <> struct Pair<int64_t> { using type = longlong2; };
 
 // N values per lane -> the lane holds Σ over the 32 lanes of value (lane % N): log2 N transposing
 // steps (a lane keeps the half its bit selects and receives the partner's copy of it), then plain
@@ -112,10 +107,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   using S = typename RcOps<T>::S;
   using Acc = typename RcOps<T>::Acc;
   constexpr int BC = 1024 / int(sizeof(T));  // columns of a tile
-  constexpr int CPT = 2;                     // adjacent columns one thread owns (one 8- or 16-byte read)
-  constexpr int WPG = BC / (32 * CPT);       // warps across a tile's columns (4 or 2)
-  constexpr int NRG = kConsumerWarps / WPG;  // row groups (2 or 4)
-  constexpr int RPT = kTileRows / NRG;       // tile rows one thread adds (16 or 8)
+  constexpr int WPG = BC / 32;               // warps across a tile's columns (8 or 4)
+  constexpr int NRG = kConsumerWarps / WPG;  // row groups (1 or 2)
+  constexpr int RPT = kTileRows / NRG;       // tile rows one thread adds (32 or 16)
   constexpr int CAP = kColTilesMax * BC;     // column accumulators per row group
   static_assert(NRG * CAP * int(sizeof(Acc)) <= kColAccBytes, "column accumulators exceed their region");
   extern __shared__ __align__(1024) unsigned char smem[];
@@ -169,8 +163,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 
   // -------------------------------------------------------------- consumers
-  const int rg = warp / WPG;                        // row group: tile rows rg*RPT .. +RPT
-  const int col = CPT * ((warp % WPG) * 32 + lane);  // the thread's first tile column
+  const int rg = warp / WPG;                 // row group: tile rows rg*RPT .. +RPT
+  const int col = (warp % WPG) * 32 + lane;  // tile column
   bool waited = false;
   long long t = 0;
   int rb = 0;  // rsum double buffer
@@ -181,16 +175,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (long long br = b0; br < b1; ++br) {
       Acc racc = Acc(0);
       for (long long ct = c0; ct < c1; ++ct, ++t) {
-        S v[CPT][RPT];
+        S v[RPT];
         if constexpr (STAGED) {
           const int slot = int(t % kStages);
           mbar_wait(full + slot, unsigned((t / kStages) & 1));
           const T* tile = reinterpret_cast<const T*>(tiles + slot * kTileBytes);
 #pragma unroll
-          for (int rr = 0; rr < RPT; ++rr) {
-            const typename Pair<T>::type pr = *reinterpret_cast<const typename Pair<T>::type*>(tile + (rg * RPT + rr) * BC + col);
-            v[0][rr] = S(pr.x), v[1][rr] = S(pr.y);
-          }
+          for (int rr = 0; rr < RPT; ++rr) v[rr] = S(tile[(rg * RPT + rr) * BC + col]);
           __syncwarp();
           if (lane == 0) mbar_arrive(empty + slot);
         } else {
@@ -198,22 +189,15 @@ __global__ void __launch_bounds__(kThreads, 1)
             asm volatile("griddepcontrol.wait;" ::: "memory");
             waited = true;
           }
+          const long long c = ct * BC + col;
           const long long r0 = br * kTileRows + rg * RPT;
           const T* m = static_cast<const T*>(a.m);
 #pragma unroll
-          for (int cc2 = 0; cc2 < CPT; ++cc2) {
-            const long long c = ct * BC + col + cc2;
-#pragma unroll
-            for (int rr = 0; rr < RPT; ++rr)
-              v[cc2][rr] = (c < a.C && r0 + rr < a.R) ? S(__ldg(m + (r0 + rr) * a.C + c)) : S(0);
-          }
+          for (int rr = 0; rr < RPT; ++rr)
+            v[rr] = (c < a.C && r0 + rr < a.R) ? S(__ldg(m + (r0 + rr) * a.C + c)) : S(0);
         }
-#pragma unroll
-        for (int cc2 = 0; cc2 < CPT; ++cc2) colacc[rg * CAP + (ct - c0) * BC + col + cc2] += Acc(tree_sum(v[cc2]));
-        S rv[RPT];
-#pragma unroll
-        for (int rr = 0; rr < RPT; ++rr) rv[rr] = v[0][rr] + v[1][rr];
-        racc += Acc(transpose_reduce(rv, lane));  // lane l: row rg*RPT + l % RPT of this band
+        colacc[rg * CAP + (ct - c0) * BC + col] += Acc(tree_sum(v));
+        racc += Acc(transpose_reduce(v, lane));  // lane l: row rg*RPT + l % RPT of this band
       }
       // ---- band end: the warps' row partials meet in shared memory
       if (!waited) {  // out / workspace are written only after the previous grid in the stream is done
@@ -241,11 +225,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     consumers_sync();
     const long long ncols = (c1 - c0) * BC;
     for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
-      Acc s = Acc(0);
-#pragma unroll
-      for (int g = 0; g < NRG; ++g) {
-        s += colacc[g * CAP + c];
-        colacc[g * CAP + c] = Acc(0);
+      Acc s = colacc[c];
+      colacc[c] = Acc(0);
+      if constexpr (NRG == 2) {
+        s += colacc[CAP + c];
+        colacc[CAP + c] = Acc(0);
       }
       const long long cg = c0 * BC + c;
       if (cg < a.C) {

@@ -69,7 +69,7 @@ StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count);
 // S8 RC (SUM_ROWS_COLS): the Tr x Tc grid of 32-row x 1 KB tiles is cut into gr x gc regions of cr row
 // bands x cc column tiles (cc <= kRcColTilesMax: a region's column accumulators fit shared memory);
 // G = min(SMs, nreg) blocks take contiguous region ranges.
-constexpr int64_t kRcColTilesMax = 16;
+constexpr int64_t kRcColTilesMax = 32;
 struct RcTiling {
   int64_t BC, Tr, Tc, cr, cc, gr, gc, nreg, G;
 };
