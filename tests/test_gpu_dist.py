@@ -60,3 +60,42 @@ def test_fake_multigpu_row_shards(cuda_device, P):
     full = gen.small_int_f32(4, (R, C), 0, 15).numpy()
     assert np.array_equal(sum(p for p in parts_c).cpu().numpy(), sums.sum_cols(full))   # exact data
     assert np.array_equal(torch.cat(parts_r).double().cpu().numpy(), sums.sum_rows(full))
+
+
+def test_nccl_world1_kmeans_update_and_pagerank(nccl_group, cuda_device):
+    # the NEXT rows' exchange steps through NCCL (world 1): the k-means update all-reduce and the
+    # PageRank all-gather of the next vector, against the oracle
+    from oracle import kmeans as okm
+    from oracle import pagerank as opr
+    from paper_conf_micro_leebsro14_b200 import dist as ndist
+    x, _ = gen.kmeans_inputs(20000, 64, 32, device=cuda_device)
+    a = gen.int_uniform(6, (20000,), 0, 31, device=cuda_device)
+    u = ndist.kmeans_update(x, a, 32)
+    torch.cuda.synchronize()
+    want = okm.update(x.cpu().numpy(), a.cpu().numpy(), 32)
+    assert np.array_equal(u.cpu().numpy()[:, -1], want[:, -1])
+    assert np.allclose(u.cpu().numpy()[:, :-1], want[:, :-1], rtol=1e-5, atol=1e-3)
+    rp, ci, pr, od = gen.pagerank_inputs(30000, avg_deg=10, seed=8, max_deg=500, device=cuda_device)
+    nxt = ndist.pagerank_step(rp, ci, pr, od)
+    torch.cuda.synchronize()
+    want = opr.step(rp.cpu().numpy(), ci.cpu().numpy(), pr.cpu().numpy(), od.cpu().numpy())
+    assert np.all(np.abs(nxt.cpu().numpy() - want) <= 1e-5 * want)
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_fake_multigpu_pagerank_shards(cuda_device, P):
+    # P node-row shards computed one after another on one GPU reassemble the full step
+    from oracle import pagerank as opr
+    from paper_conf_micro_leebsro14_b200 import npp
+    from paper_conf_micro_leebsro14_b200.dist import shard_range
+    N = 40000
+    rp, ci, pr, od = gen.pagerank_inputs(N, avg_deg=12, seed=9, max_deg=800, device=cuda_device)
+    parts = []
+    for rank in range(P):
+        lo, hi = shard_range(N, P, rank)
+        e0, e1 = int(rp[lo]), int(rp[hi])
+        parts.append(npp.pagerank_shard((rp[lo:hi + 1] - e0).contiguous(), ci[e0:e1].contiguous(), pr, od, lo, hi))
+    torch.cuda.synchronize()
+    want = opr.step(rp.cpu().numpy(), ci.cpu().numpy(), pr.cpu().numpy(), od.cpu().numpy())
+    got = torch.cat(parts).cpu().numpy()
+    assert np.all(np.abs(got - want) <= 1e-5 * want)
