@@ -196,29 +196,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int rr = 0; rr < RPT; ++rr)
             v[rr] = (c < a.C && r0 + rr < a.R) ? S(__ldg(m + (r0 + rr) * a.C + c)) : S(0);
         }
-        if constexpr (NRG == 1) {
-          // last band of the region: the column slot is final, so it leaves now (spread over the
-          // band's tiles instead of bunched at the region end)
-          const Acc cv = colacc[(ct - c0) * BC + col] + Acc(tree_sum(v));
-          if (br + 1 == b1) {
-            colacc[(ct - c0) * BC + col] = Acc(0);
-            const long long cg = ct * BC + col;
-            if (cg < a.C) {
-              if (!waited) {
-                asm volatile("griddepcontrol.wait;" ::: "memory");
-                waited = true;
-              }
-              if (a.gr == 1)
-                out[a.R + cg] = RcOps<T>::finish(cv);
-              else
-                atomicAdd(accC + cg, cv);
-            }
-          } else {
-            colacc[(ct - c0) * BC + col] = cv;
-          }
-        } else {
-          colacc[rg * CAP + (ct - c0) * BC + col] += Acc(tree_sum(v));
-        }
+        colacc[rg * CAP + (ct - c0) * BC + col] += Acc(tree_sum(v));
         racc += Acc(transpose_reduce(v, lane));  // lane l: row rg*RPT + l % RPT of this band
       }
       // ---- band end: the warps' row partials meet in shared memory
@@ -243,10 +221,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       rb ^= 1;
     }
-    // ---- region end: the region's column accumulators (2 row groups: summed here; 1: already sent)
+    // ---- region end: the region's column accumulators
     consumers_sync();
     const long long ncols = (c1 - c0) * BC;
-    for (long long c = threadIdx.x; NRG > 1 && c < ncols; c += kConsumers) {
+    for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
       Acc s = colacc[c];
       colacc[c] = Acc(0);
       if constexpr (NRG == 2) {
