@@ -545,10 +545,11 @@ def roofline(item, us, gbs, peak, peak_src, traffic, flops, wavefronts=None):
 
 
 def mapping_brief(m):
-    sp = {0: "Span(1)", 1: "Span(all)", 2: "Span(n)", 3: "Split(k)"}
+    def span(l):
+        return {0: "Span(1)", 1: "Span(all)", 2: f"Span({l['factor']})", 3: f"Split({l['factor']})"}[l["span"]]
     dims = "xyz"
-    return "; ".join(f"L{i}:{dims[l['dim']]},{l['block']},{sp[l['span']].replace('n', str(l['factor'])) if l['span'] == 2 else sp[l['span']].replace('k', str(l['factor']))}"
-                     for i, l in enumerate(m["levels"])) + f"; vec={m['vec']}; grid={m['grid']}"
+    return "; ".join(f"L{i}:{dims[l['dim']]},{l['block']},{span(l)}" for i, l in enumerate(m["levels"])) + \
+        f"; vec={m['vec']}; grid={m['grid']}"
 
 
 def e2e_host(items, torch, stream, world, dist, steps=3):
