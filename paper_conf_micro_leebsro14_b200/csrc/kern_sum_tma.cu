@@ -174,9 +174,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   using Acc = typename SOps<T>::Acc;
   using V = typename V16<T>::type;
   constexpr int BC = 1024 / int(sizeof(T));     // columns of one 1 KB chunk
-  constexpr int NCH = WIDE ? 4 : 1;             // chunks per tile row: tile = RT rows x NCH KB
-  constexpr int RT = kTileRows / NCH;           // tile rows (narrow 32, wide 8)
-  constexpr int W = NCH * BC;                   // tile columns
+  // RX: WIDE = 8 rows x 4 KB tiles. MX: WIDE = narrow strips, 128 rows x 256 B (a static split of
+  // whole strips then never cuts one: no Split combine at all)
+  constexpr bool MXN = WIDE && !ROWS;
+  constexpr int NCH = (WIDE && ROWS) ? 4 : 1;   // chunks per tile row: tile = RT rows x NCH KB
+  constexpr int RT = MXN ? 128 : kTileRows / NCH;  // tile rows (narrow 32, wide 8, MX-narrow 128)
+  constexpr int W = MXN ? 256 / int(sizeof(T)) : NCH * BC;  // tile columns
   constexpr int OUT_PER_TILE = ROWS ? RT : W;   // outputs of one outer tile (band / strip)
   extern __shared__ __align__(1024) unsigned char smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);
@@ -199,7 +202,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long bid = blockIdx.x, G = gridDim.x;
   const long long total = a.To * a.Ti;
-  const long long s0 = bid * a.static_tiles / G, s1 = (bid + 1) * a.static_tiles / G;  // static range
+  // static range (MX-narrow: whole strips, so no strip is ever cut)
+  const long long s0 = MXN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
+  const long long s1 = MXN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
   const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order
 
   if (threadIdx.x == 0) {
@@ -277,10 +282,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
             tma_load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
           }
         }
-        if constexpr (WIDE)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
+        if constexpr (WIDE && ROWS)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
           tma_load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
         else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
-          tma_load_2d(tiles + slot * kTileBytes, &map, ch * BC, y, full + slot);
+          tma_load_2d(tiles + slot * kTileBytes, &map, MXN ? int(ot * W) : ch * BC, y, full + slot);
         cur = nxt;
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
@@ -356,10 +361,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     if (a.dbg_times && lane == 0) a.dbg_times[bid * 8 + 2] = gtimer();
   } else {
     // ------------------------------------------------------------ consumers
-    constexpr int kGroups = ROWS ? 1 : 256 / BC;  // MX row groups (1 for 4-byte types, 2 for 8-byte)
+    constexpr int kGroups = ROWS ? 1 : 256 / W;   // MX row groups (1 / 2 for 4- / 8-byte; MX-narrow 4 / 8)
     constexpr int kRowsPer = RT / kGroups;        // MX rows of a tile one thread adds
-    const int col = threadIdx.x % BC;
-    const int rg = threadIdx.x / BC;
+    const int col = threadIdx.x % W;
+    const int rg = threadIdx.x / W;
     // RX narrow: rows 4w..4w+3; RX wide: acc[0] = row w; MX: acc[k] = column col of chunk k
     Acc acc[4] = {0, 0, 0, 0};
     unsigned n_acc = 0;         // tiles of the current outer tile accumulated since the last flush
@@ -469,6 +474,19 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       constexpr int NV = ROWS ? (WIDE ? 1 : 4) : NCH;
       const unsigned contributed = n_acc;
       n_acc = 0;
+      if (MXN && whole) {  // the row groups of a whole strip meet in shared memory, one write per column
+        Acc* red = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes);  // [kGroups][W]
+        red[rg * W + col] = val[0];
+        consumers_sync();
+        if (threadIdx.x < W) {
+          Acc s = Acc(0);
+#pragma unroll
+          for (int g = 0; g < kGroups; ++g) s += red[g * W + threadIdx.x];
+          if (ot * W + threadIdx.x < a.C) static_cast<T*>(a.out)[ot * W + threadIdx.x] = SOps<T>::finish(s);
+        }
+        consumers_sync();
+        continue;
+      }
       if (whole && kGroups == 1) {
 #pragma unroll
         for (int i = 0; i < NV; ++i)
@@ -526,7 +544,7 @@ cudaError_t launch_typed(const CUtensorMap& map, const CUtensorMap& vmap, const 
                          cudaStream_t st) {
   static bool attr_set = false;
   auto kern = npp_sum_tma_kernel<T, ROWS, WIDE, WT>;
-  const int smem = WT ? kSmemBytesW : kSmemBytes;
+  const int smem = (WT ? kSmemBytesW : kSmemBytes) + ((WIDE && !ROWS) ? 2048 : 0);  // MX-narrow: group sums
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
@@ -543,7 +561,8 @@ cudaError_t launch_w(bool rows, const CUtensorMap& map, const CUtensorMap& vmap,
   if (rows)
     return a.wide ? launch_typed<T, true, true, WT>(map, vmap, a, grid, st)
                   : launch_typed<T, true, false, WT>(map, vmap, a, grid, st);
-  return launch_typed<T, false, false, WT>(map, vmap, a, grid, st);
+  return a.wide ? launch_typed<T, false, true, WT>(map, vmap, a, grid, st)
+                : launch_typed<T, false, false, WT>(map, vmap, a, grid, st);
 }
 
 template <typename T>
@@ -565,7 +584,14 @@ cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedA
                                  : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
                                                     : CU_TENSOR_MAP_DATA_TYPE_INT64;
   CUresult r;
-  if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (row pitch is a multiple of 4 KB)
+  if (a.wide && !rows) {  // MX-narrow strips: {C, R}, box 128 rows x 256 B
+    const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
+    const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
+    const cuuint32_t box[2] = {cuuint32_t(256 / esz), 128};
+    const cuuint32_t estr[2] = {1, 1};
+    r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  } else if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (row pitch is a multiple of 4 KB)
     const cuuint64_t dims[3] = {bc, cuuint64_t(a.C) / bc, cuuint64_t(a.R)};
     const cuuint64_t strides[2] = {1024, cuuint64_t(a.C) * esz};
     const cuuint32_t box[3] = {cuuint32_t(bc), 4, cuuint32_t(kTileRows / 4)};

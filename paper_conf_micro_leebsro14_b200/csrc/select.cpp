@@ -242,10 +242,10 @@ void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
     c->chunks[1] = t.Ti > 1 ? t.W : n.N[1];
     c->vec = 16 / dtype_size(dtype);
   } else {  // one thread per column of each 1 KB chunk (W / BC chunks per tile row)
-    c->blocks[0] = int(t.BC);
-    c->blocks[1] = int(256 / t.BC);
-    c->spans[0] = t.wide ? NPP_SPAN_N : NPP_SPAN_ONE;
-    c->factors[0] = t.W / t.BC;
+    c->blocks[0] = int(t.wide ? t.W : t.BC);
+    c->blocks[1] = int(256 / c->blocks[0]);
+    c->spans[0] = NPP_SPAN_ONE;
+    c->factors[0] = 1;
     c->chunks[0] = t.W;
     c->chunks[1] = t.Ti > 1 ? t.BR : n.N[1];
     c->vec = 1;
@@ -442,6 +442,11 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   t.wide = is_rows_pattern(pattern) && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
   t.BR = t.wide ? 8 : kStageRows;
   t.W = t.wide ? 4 * t.BC : t.BC;
+  if (!is_rows_pattern(pattern) && getenv("NPP_EXP_MXN") && C * esz >= 65536 && cdiv(R, 128) <= 8) {
+    t.wide = true;  // EXPERIMENT: MX-narrow strips of 128 rows x 256 B
+    t.BR = 128;
+    t.W = 256 / esz;
+  }
   if (is_rows_pattern(pattern)) {
     t.To = cdiv(R, t.BR);
     t.Ti = cdiv(C, t.W);
