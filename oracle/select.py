@@ -329,6 +329,8 @@ def staged_tiles(nest, dtype):
     C = I if rows else O
     wide = rows and (C * esz) % 4096 == 0
     BR, W = (8, 4 * BC) if wide else (STAGE_ROWS, BC)
+    if nest["pattern"] == "SUM_COLS" and C * esz >= 65536 and cdiv(I, 128) <= WHOLE_UNIT_MAX:
+        BR, W = 128, 256 // esz     # MX-narrow strips: whole-strip static split, no strip is ever cut
     if rows:
         return BR, BC, W, cdiv(O, BR), cdiv(I, W)
     return BR, BC, W, cdiv(O, W), cdiv(I, BR)
@@ -364,10 +366,10 @@ def r2_staged(nest, dtype, lim):
         factors = (1 if wide else 4, Ti)
         chunks = (BR, W if Ti > 1 else I)
         vec = 16 // esz
-    else:                                 # one thread per column of each 1 KB chunk (W/BC chunks)
-        blocks = (BC, 256 // BC)
-        spans = (SPAN_N if wide else ONE, ALL if Ti == 1 else SPLIT)
-        factors = (W // BC, Ti)
+    else:                                 # one thread per column of a tile (W columns, 256/W row groups)
+        blocks = (W, 256 // W)
+        spans = (ONE, ALL if Ti == 1 else SPLIT)
+        factors = (1, Ti)
         chunks = (W, BR if Ti > 1 else I)
         vec = 1
     return blocks, spans, factors, vec, chunks, G, CL

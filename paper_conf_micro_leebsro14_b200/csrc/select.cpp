@@ -442,9 +442,11 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   t.wide = is_rows_pattern(pattern) && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
   t.BR = t.wide ? 8 : kStageRows;
   t.W = t.wide ? 4 * t.BC : t.BC;
-  if (!is_rows_pattern(pattern) && getenv("NPP_EXP_MXN") && C * esz >= 65536 && cdiv(R, 128) <= 8) {
-    t.wide = true;  // EXPERIMENT: MX-narrow strips of 128 rows x 256 B
-    t.BR = 128;
+  if (pattern == NPP_SUM_COLS && C * esz >= 65536 && cdiv(R, kStageRowsNarrowMx) <= kWholeUnitMax) {
+    // MX-narrow strips (S8): 128 rows x 256 B tiles, so an outer strip is <= 8 tiles, the pool unit is a
+    // whole strip and the static split is aligned to whole strips: no strip is ever cut (no combine)
+    t.wide = true;
+    t.BR = kStageRowsNarrowMx;
     t.W = 256 / esz;
   }
   if (is_rows_pattern(pattern)) {

@@ -48,6 +48,7 @@ struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refi
 void temp_layout(const struct Nest& n, Choice* c);
 
 constexpr int kStageRows = 32;  // BR of the staged family (S8): tiles of 32 rows x 1 KB
+constexpr int64_t kStageRowsNarrowMx = 128;  // BR of the MX-narrow strips (S8): tiles of 128 rows x 256 B
 constexpr int64_t kPoolDiv = 8;       // S8 balance rule: about 1/kPoolDiv of the tiles form the shared pool
 constexpr int64_t kPoolUnit = 4;      // S8 balance rule: pool claim unit when outer tiles are long
 constexpr int64_t kWholeUnitMax = 8;  // S8 balance rule: outer tiles of <= 8 tiles are claimed whole

@@ -1,3 +1,4 @@
+"""MX-narrow strips (SUM_COLS, row pitch >= 64 KB, R <= 1024): parity on ragged shapes, back-to-back and PDL executes, workspace left zero."""
 import sys, os
 sys.path.insert(0, os.environ.get("GRAFT_REPO_ROOT", "/root/repo"))
 import numpy as np, torch
