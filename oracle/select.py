@@ -329,6 +329,8 @@ def staged_tiles(nest, dtype):
     C = I if rows else O
     wide = rows and (C * esz) % 4096 == 0
     BR, W = (8, 4 * BC) if wide else (STAGE_ROWS, BC)
+    if nest["pattern"] == "SUM_ROWS" and (C * esz) % 32768 == 0 and 65536 <= C * esz <= 32768 * WHOLE_UNIT_MAX:
+        BR, W = 1, 32 * BC          # RX one-row tiles: whole-row static split, no row is ever cut
     if nest["pattern"] == "SUM_COLS" and C * esz >= 65536 and cdiv(I, 128) <= WHOLE_UNIT_MAX:
         BR, W = 128, 256 // esz     # MX-narrow strips: whole-strip static split, no strip is ever cut
     if rows:

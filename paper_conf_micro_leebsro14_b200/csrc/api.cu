@@ -541,7 +541,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     s.static_tiles = bal.Ts;
     s.unit = bal.U;
     s.early_reads = overlap ? 1 : 0;
-    s.wide = t.wide ? 1 : 0;
+    s.wide = t.r1 ? 2 : (t.wide ? 1 : 0);
     s.pool = static_cast<unsigned*>(workspace);  // S9 staged workspace: [256 B pool][tickets][acc]
     s.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + 256);
     s.acc = static_cast<char*>(workspace) + 256 + ((t.To * 4 + 255) / 256) * 256;

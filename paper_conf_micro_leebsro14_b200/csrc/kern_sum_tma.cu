@@ -167,7 +167,7 @@ __device__ __forceinline__ A warp_sum(A v) {
 // WT: weighted sums (sumWeightedRows / sumWeightedCols, Fig 15) fused: the zipWith
 // product m·v is formed in registers from the staged tile and the tile's slice of v (staged by a 1-D
 // TMA box on the same mbarrier), so no inner allocation exists at all (§V-A taken to its limit).
-template <typename T, bool ROWS, bool WIDE, bool WT>
+template <typename T, bool ROWS, bool WIDE, bool WT, bool R1>
 __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_constant__ CUtensorMap map,
                                                                   const __grid_constant__ CUtensorMap vmap,
                                                                   StagedArgs a) {
@@ -176,9 +176,11 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   constexpr int BC = 1024 / int(sizeof(T));     // columns of one 1 KB chunk
   // RX: WIDE = 8 rows x 4 KB tiles. MX: WIDE = narrow strips, 128 rows x 256 B (a static split of
   // whole strips then never cuts one: no Split combine at all)
+  // RX R1: one-row tiles of 32 KB (a row of 64-256 KB is <= 8 tiles: whole rows balance, no cuts)
   constexpr bool MXN = WIDE && !ROWS;
-  constexpr int NCH = (WIDE && ROWS) ? 4 : 1;   // chunks per tile row: tile = RT rows x NCH KB
-  constexpr int RT = MXN ? 128 : kTileRows / NCH;  // tile rows (narrow 32, wide 8, MX-narrow 128)
+  constexpr bool ALIGN = MXN || R1;             // static split aligned to whole outer tiles
+  constexpr int NCH = R1 ? 32 : ((WIDE && ROWS) ? 4 : 1);  // chunks per tile row: tile = RT rows x NCH KB
+  constexpr int RT = MXN ? 128 : (R1 ? 1 : kTileRows / NCH);  // tile rows (32, wide 8, R1 1, MX-narrow 128)
   constexpr int W = MXN ? 256 / int(sizeof(T)) : NCH * BC;  // tile columns
   constexpr int OUT_PER_TILE = ROWS ? RT : W;   // outputs of one outer tile (band / strip)
   extern __shared__ __align__(1024) unsigned char smem[];
@@ -203,8 +205,8 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   const long long bid = blockIdx.x, G = gridDim.x;
   const long long total = a.To * a.Ti;
   // static range (MX-narrow: whole strips, so no strip is ever cut)
-  const long long s0 = MXN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
-  const long long s1 = MXN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
+  const long long s0 = ALIGN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
+  const long long s1 = ALIGN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
   const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order
 
   if (threadIdx.x == 0) {
@@ -459,7 +461,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         }
       } else if constexpr (ROWS) {
         val[0] = warp_sum(acc[0]);
-        oidx[0] = ot * RT + warp;
+        oidx[0] = R1 ? ot : ot * RT + warp;  // R1: every warp holds a piece of the one row
         mine[0] = lane == 0 && oidx[0] < a.R;
         acc[0] = 0;
       } else {
@@ -474,6 +476,19 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       constexpr int NV = ROWS ? (WIDE ? 1 : 4) : NCH;
       const unsigned contributed = n_acc;
       n_acc = 0;
+      if (R1 && whole) {  // the eight warps' pieces of a whole row meet in shared memory
+        Acc* red = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes);  // [8]
+        if (lane == 0) red[warp] = val[0];
+        consumers_sync();
+        if (threadIdx.x == 0) {
+          Acc s = Acc(0);
+#pragma unroll
+          for (int w = 0; w < kConsumerWarps; ++w) s += red[w];
+          if (ot < a.R) static_cast<T*>(a.out)[ot] = SOps<T>::finish(s);
+        }
+        consumers_sync();
+        continue;
+      }
       if (MXN && whole) {  // the row groups of a whole strip meet in shared memory, one write per column
         Acc* red = reinterpret_cast<Acc*>(tiles + kStages * kTileBytes);  // [kGroups][W]
         red[rg * W + col] = val[0];
@@ -487,7 +502,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         consumers_sync();
         continue;
       }
-      if (whole && kGroups == 1) {
+      if (whole && kGroups == 1 && !R1) {
 #pragma unroll
         for (int i = 0; i < NV; ++i)
           if (mine[i]) static_cast<T*>(a.out)[oidx[i]] = SOps<T>::finish(val[i]);
@@ -539,12 +554,12 @@ EncodeTiledFn encode_fn() {
   return fn;
 }
 
-template <typename T, bool ROWS, bool WIDE, bool WT>
+template <typename T, bool ROWS, bool WIDE, bool WT, bool R1 = false>
 cudaError_t launch_typed(const CUtensorMap& map, const CUtensorMap& vmap, const StagedArgs& a, int grid,
                          cudaStream_t st) {
   static bool attr_set = false;
-  auto kern = npp_sum_tma_kernel<T, ROWS, WIDE, WT>;
-  const int smem = (WT ? kSmemBytesW : kSmemBytes) + ((WIDE && !ROWS) ? 2048 : 0);  // MX-narrow: group sums
+  auto kern = npp_sum_tma_kernel<T, ROWS, WIDE, WT, R1>;
+  const int smem = (WT ? kSmemBytesW : kSmemBytes) + (((WIDE && !ROWS) || R1) ? 2048 : 0);  // group sums
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
@@ -559,8 +574,9 @@ cudaError_t launch_w(bool rows, const CUtensorMap& map, const CUtensorMap& vmap,
   // wide tiles are selected for sumRows only (S8); the MX-wide path of the kernel template (4 KB
   // column strips) measured slower than 1 KB strips because of the larger combine per cut strip
   if (rows)
-    return a.wide ? launch_typed<T, true, true, WT>(map, vmap, a, grid, st)
-                  : launch_typed<T, true, false, WT>(map, vmap, a, grid, st);
+    return a.wide == 2 ? launch_typed<T, true, true, false, true>(map, vmap, a, grid, st)
+           : a.wide    ? launch_typed<T, true, true, WT>(map, vmap, a, grid, st)
+                       : launch_typed<T, true, false, WT>(map, vmap, a, grid, st);
   return a.wide ? launch_typed<T, false, true, WT>(map, vmap, a, grid, st)
                 : launch_typed<T, false, false, WT>(map, vmap, a, grid, st);
 }
@@ -594,7 +610,7 @@ cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedA
   } else if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (row pitch is a multiple of 4 KB)
     const cuuint64_t dims[3] = {bc, cuuint64_t(a.C) / bc, cuuint64_t(a.R)};
     const cuuint64_t strides[2] = {1024, cuuint64_t(a.C) * esz};
-    const cuuint32_t box[3] = {cuuint32_t(bc), 4, cuuint32_t(kTileRows / 4)};
+    const cuuint32_t box[3] = {cuuint32_t(bc), a.wide == 2 ? 32u : 4u, a.wide == 2 ? 1u : cuuint32_t(kTileRows / 4)};
     const cuuint32_t estr[3] = {1, 1, 1};
     r = encode(&map, dt, 3, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);

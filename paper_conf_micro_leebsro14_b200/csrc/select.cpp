@@ -442,6 +442,14 @@ StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   t.wide = is_rows_pattern(pattern) && (C * esz) % 4096 == 0;  // MX measured faster with 1 KB strips
   t.BR = t.wide ? 8 : kStageRows;
   t.W = t.wide ? 4 * t.BC : t.BC;
+  if (pattern == NPP_SUM_ROWS && (C * esz) % 32768 == 0 && C * esz >= 65536 && C * esz <= 32768 * kWholeUnitMax) {
+    // RX one-row tiles (S8): 1 row x 32 KB, a row is 2-8 tiles, the pool unit is a whole row and the
+    // static split is aligned to whole rows: no row is ever cut (no combine)
+    t.wide = true;
+    t.r1 = true;
+    t.BR = 1;
+    t.W = 32 * t.BC;
+  }
   if (pattern == NPP_SUM_COLS && C * esz >= 65536 && cdiv(R, kStageRowsNarrowMx) <= kWholeUnitMax) {
     // MX-narrow strips (S8): 128 rows x 256 B tiles, so an outer strip is <= 8 tiles, the pool unit is a
     // whole strip and the static split is aligned to whole strips: no strip is ever cut (no combine)

@@ -60,6 +60,7 @@ struct StagedTiling {
   int64_t BR, BC, W;  // tile rows, chunk columns, tile columns
   int64_t To, Ti;     // tiles along the outer / inner level
   bool wide;
+  bool r1 = false;    // SUM_ROWS one-row tiles of 32 KB (row pitch 64-256 KB, a multiple of 32 KB)
 };
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype);
 struct StagedBalance {
