@@ -132,6 +132,29 @@ def test_overlap_back_to_back(npp, cuda_device, dtype):
         assert int(p.workspace.count_nonzero()) == 0, p.shape
 
 
+@pytest.mark.parametrize("pattern,shapes", [
+    # SUM_ROWS, row pitch 64-256 KB and a multiple of 32 KB: one-row 32 KB tiles, whole rows (DESIGN S8 RX rule)
+    ("SUM_ROWS", [(1024, 65536), (1000, 16384), (3, 65536), (4099, 24576), (1, 65536)]),
+    # SUM_COLS, row pitch >= 64 KB and <= 1024 rows: MX-narrow strips, whole strips (DESIGN S8 MX-narrow rule)
+    ("SUM_COLS", [(1024, 65536), (1000, 70000), (777, 16384), (129, 65536), (1, 1 << 20), (1024, 65540)]),
+])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+def test_large_pitch_whole_tile_rules(npp, cuda_device, pattern, shapes, dtype):
+    # the large-pitch staged rules never cut a row / strip: back-to-back and PDL executes match the
+    # oracle and leave the workspace (pool counter, tickets) zero
+    for i, s in enumerate(shapes):
+        if dtype == "i64" and s[1] % 2 == 0:
+            s = (s[0], s[1] // 2)
+        m = _make(dtype, s, 60 + i, cuda_device)
+        p = npp.Plan(pattern, s, dtype)
+        o1 = p.execute([m], p.new_out())
+        o2 = p.execute([m], p.new_out(), overlap=True)
+        torch.cuda.synchronize()
+        check(pattern, m, o1, dtype)
+        check(pattern, m, o2, dtype)
+        assert int(p.workspace.count_nonzero()) == 0, (s, dtype)
+
+
 def test_large_sumcols_sampled(npp, cuda_device):
     # [1M, 4K] fp32 (16 GiB, 2^32 elements: 64-bit indexing); sampled columns recomputed by the oracle
     R, C = 1 << 20, 4096
