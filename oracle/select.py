@@ -340,17 +340,19 @@ def staged_tiles(nest, dtype):
 
 POOL_DIV = 8                                      # DESIGN.md S8 balance rule
 POOL_UNIT = 4
+POOL_UNIT_SHORT = 8                               # outer tiles of 9..512 tiles
+POOL_UNIT_SHORT_TI_MAX = 512
 WHOLE_UNIT_MAX = 8
 
 
 def balance(To, Ti, lim):
     """DESIGN.md S8 balance rule over T = To*Ti tiles: G = min(SMs, T) persistent blocks; pool claim
-    unit U = Ti if Ti <= 8 else 4; Ts = U*floor((T - floor(T/8))/U) tiles split statically (block b
+    unit U = Ti if Ti <= 8, else 8 if Ti <= 512, else 4; Ts = U*floor((T - floor(T/8))/U) tiles split statically (block b
     streams [b*Ts/G, (b+1)*Ts/G)); the units of [Ts, T) are claimed in order by whichever block is
     free. Returns (G, U, Ts)."""
     T = To * Ti
     G = min(lim["sm_count"], T)
-    U = Ti if Ti <= WHOLE_UNIT_MAX else POOL_UNIT
+    U = Ti if Ti <= WHOLE_UNIT_MAX else (POOL_UNIT_SHORT if Ti <= POOL_UNIT_SHORT_TI_MAX else POOL_UNIT)
     return G, U, U * ((T - T // POOL_DIV) // U)
 
 

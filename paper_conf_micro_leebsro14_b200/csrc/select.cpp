@@ -414,7 +414,9 @@ void set_error(const std::string& msg) { g_error = msg; }
 
 // S8 balance rule (S8): G = min(SMs, T) persistent blocks over T tiles in order. The pool
 // unit is U = Ti when an outer tile has at most kWholeUnitMax tiles (a claim then covers whole outer
-// tiles), else kPoolUnit. Ts = U * floor((T - floor(T / kPoolDiv)) / U) tiles are split statically:
+// tiles), else kPoolUnitShort for outer tiles of at most kPoolUnitShortTiMax tiles (fewer contributors
+// per cut outer tile: sumCols [8K,8K] 43.3 -> 42.6 us, profiles/r01/unit/sweep.log) and kPoolUnit
+// beyond (sumCols [64K,1K] is 0.35 us slower with 8). Ts = U * floor((T - floor(T / kPoolDiv)) / U) tiles are split statically:
 // block b streams [b*Ts/G, (b+1)*Ts/G); the units of [Ts, T) are claimed in order from a counter by
 // whichever block is free, which absorbs the per-SM bandwidth differences of a static split.
 // (NPP_POOL_DIV / NPP_POOL_UNIT override the constants for measurements; tests never set them.)
@@ -425,12 +427,12 @@ StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count) {
   }();
   static const int64_t unit = [] {
     const char* e = getenv("NPP_POOL_UNIT");
-    return e ? std::max<int64_t>(1, atoll(e)) : kPoolUnit;
+    return e ? std::max<int64_t>(1, atoll(e)) : int64_t(0);
   }();
   StagedBalance b;
   const int64_t T = To * Ti;
   b.G = std::min<int64_t>(sm_count, T);
-  b.U = Ti <= kWholeUnitMax ? Ti : unit;
+  b.U = Ti <= kWholeUnitMax ? Ti : (unit ? unit : (Ti <= kPoolUnitShortTiMax ? kPoolUnitShort : kPoolUnit));
   b.Ts = b.U * ((T - T / div) / b.U);
   return b;
 }

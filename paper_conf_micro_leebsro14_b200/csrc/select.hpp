@@ -51,6 +51,8 @@ constexpr int kStageRows = 32;  // BR of the staged family (S8): tiles of 32 row
 constexpr int64_t kStageRowsNarrowMx = 128;  // BR of the MX-narrow strips (S8): tiles of 128 rows x 256 B
 constexpr int64_t kPoolDiv = 8;       // S8 balance rule: about 1/kPoolDiv of the tiles form the shared pool
 constexpr int64_t kPoolUnit = 4;      // S8 balance rule: pool claim unit when outer tiles are long
+constexpr int64_t kPoolUnitShort = 8;  // S8 balance rule: pool claim unit when outer tiles are 9-512 tiles
+constexpr int64_t kPoolUnitShortTiMax = 512;
 constexpr int64_t kWholeUnitMax = 8;  // S8 balance rule: outer tiles of <= 8 tiles are claimed whole
 
 // S8 staged-family tiling shared with the kernels: a tile is BR rows x W columns (32 KB) made of

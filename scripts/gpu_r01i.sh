@@ -1,7 +1,7 @@
 #!/bin/bash
 # verify the RX one-row SUM_ROWS tiles (fd755de) and refresh the paper-step bench line + ncu evidence
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
-O=gpurun_out/r01i
+O=${OUT:-gpurun_out/r01i}
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $O/nvsmi.txt 2>&1
 timeout 300 python tools/check_r1_rows.py > $O/check_r1_rows.log 2>&1; echo "check rc=$?" >> $O/check_r1_rows.log
@@ -20,7 +20,7 @@ python - <<'PY'
 import json
 for w in ["bench","bench_rowscols","bench_ref"]:
     try:
-        d=json.load(open('gpurun_out/r01i/'+w+'.json'))
+        d=json.load(open(''+__import__("os").environ.get("OUT","gpurun_out/r01i")+'/'+w+'.json'))
         r=d.get('roofline',{})
         print(w, d['value'], d['unit'], 'frac', r.get('frac'), 'clk', d.get('clocks',{}).get('sm_mhz'), d.get('clocks',{}).get('reasons'))
     except Exception as e:
