@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define NPP_VERSION 3  /* 3: SUM_ROWS_COLS, KMEANS_UPDATE, PAGERANK */
+#define NPP_VERSION 4  /* 3: SUM_ROWS_COLS, KMEANS_UPDATE, PAGERANK; 4: static_tiles, NPP_EXEC_NO_PDL, traces */
 
 #if defined(__GNUC__)
 #define NPP_API __attribute__((visibility("default")))
@@ -70,7 +70,7 @@ typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2 } npp_dtype;
  *                      out[N] f32 = (1-0.85)/N + 0.85 * Σ_{j=rowptr[n]}^{rowptr[n+1]-1} pr[w_j]/outdeg[w_j], w_j = colidx[j]
  *                      one PageRank step (Fig 5) over the CSR of IN-neighbours; the caller
  *                      guarantees 0 <= rowptr[n] <= rowptr[n+1] <= E, 0 <= colidx < N and outdeg >= 1 for
- *                      every id in colidx (no device-side checks). AUTO only. */
+ *                      every id in colidx (no device-side checks). AUTO only; E < 2^31. */
 typedef enum {
   NPP_SUM_ROWS = 0,
   NPP_SUM_COLS = 1,
@@ -148,6 +148,8 @@ typedef struct {
   int32_t temp;           /* npp_temp: the weighted sums' inner allocation (S10) */
   int32_t reserved2;
   int64_t temp_stride[2]; /* PREALLOC: element strides of the temp buffer along (outer, inner) */
+  int64_t static_tiles;   /* staged sums: the first Ts tiles (outer-major order) are split statically over the
+                             grid, the rest form the claim pool of units of claim_tiles (S8); else 0 */
 } npp_mapping;
 
 /* Hardware limits the selector's hard constraints and ControlDOP read (L658-662, L799-803).
@@ -233,12 +235,16 @@ NPP_API int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void*
 
 /* Execution flags of npp_execute_ex. */
 #define NPP_EXEC_OVERLAP 1u
+#define NPP_EXEC_NO_PDL 2u
 /* npp_execute with flags. NPP_EXEC_OVERLAP: the caller asserts that no work enqueued earlier on
  * `stream` writes this call's inputs (e.g. inputs resident before the preceding kernel started); the
  * staged (TMA) kernels are then launched as programmatic dependent launches (sm_90+ PDL): their blocks
  * start streaming the inputs while the previous kernel on the stream drains, and they write `out` and
  * the workspace only after that kernel has completed (griddepcontrol.wait). Other plans ignore the
- * flag. Unknown flag bits: NPP_ERR_INVALID_ARG. Otherwise identical to npp_execute. */
+ * flag. NPP_EXEC_NO_PDL: launch every kernel as a plain stream-ordered launch (no programmatic dependent
+ * launch attribute at all: the kernel's blocks become resident only after the previous kernel completed;
+ * used to time one kernel in isolation). OVERLAP together with NO_PDL, or unknown flag bits:
+ * NPP_ERR_INVALID_ARG. Otherwise identical to npp_execute. */
 NPP_API int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace,
                            void* stream, unsigned flags);
 
@@ -247,6 +253,21 @@ NPP_API int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, vo
  * into `host_out` and synchronises `stream` before returning. */
 NPP_API int npp_execute_host(npp_plan_t plan, const void* const* host_ins, int n_in, void* host_out,
                      void* const* dev_ins, void* dev_out, void* workspace, void* stream);
+
+/* Tiles of the plan's schedule (white-box tests of the runtime rule, S8): To*Ti for a staged
+ * sum (outer-major tile order), B*ceil(Rb/32) for LOGREG_GRAD, ceil(N/TP) for KMEANS_ASSIGN (TP = 256 if
+ * D <= 64 else 128), ceil(N/128) for KMEANS_UPDATE, the number of regions for SUM_ROWS_COLS; 0 for plans
+ * without a tile schedule (direct-load families, PAGERANK, empty plans). */
+NPP_API int64_t npp_plan_tiles(npp_plan_t plan);
+
+/* npp_execute that also records the schedule: `trace` is a caller-owned DEVICE int32 array of
+ * 2*npp_plan_tiles(plan) entries, the second half zero-filled by the caller. For every tile t the kernel
+ * writes trace[t] = index of the block that loaded it and adds 1 to trace[n + t] per load (so a correct
+ * schedule leaves every trace[n + t] == 1). Enqueue only, like npp_execute; the trace costs one store and
+ * one atomic per tile. Errors: as npp_execute; NPP_ERR_UNSUPPORTED if the plan has no tile schedule;
+ * NPP_ERR_INVALID_ARG if trace is NULL. */
+NPP_API int npp_execute_traced(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace,
+                               void* stream, int32_t* trace);
 
 /* Number of kernel launches one npp_execute of this plan enqueues (0 for an empty plan). */
 NPP_API int npp_plan_launches(npp_plan_t plan);

@@ -379,6 +379,12 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
+def r2_staged_static(nest, dtype, lim) -> int:
+    """Ts of the balance rule for a staged sum: the tiles split statically (the rest is the pool)."""
+    _, _, _, To, Ti = staged_tiles(nest, dtype)
+    return balance(To, Ti, lim)[2]
+
+
 RC_COL_TILES_MAX = 32                             # DESIGN.md S8 RC: column tiles of one region
 
 
@@ -557,7 +563,7 @@ def temp_layout(nest, dims):
 
 
 def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chunks=None, staged=0,
-                persistent_grid=None, claim_tiles=0, temp=(TEMP_NONE, (0, 0))):
+                persistent_grid=None, claim_tiles=0, temp=(TEMP_NONE, (0, 0)), static_tiles=0):
     L = len(blocks)
     levels = []
     for l in range(L):
@@ -575,7 +581,7 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
                levels=levels, score=score_, dop=mapping_dop(nest, blocks, spans, factors),
                threads=grid * prod(blocks), grid=grid, block=block3,
                smem_bytes=smem_model(nest, dtype, blocks), workspace_bytes=0, claim_tiles=claim_tiles,
-               temp=temp[0], temp_stride=[temp[1][0], temp[1][1]])
+               temp=temp[0], temp_stride=[temp[1][0], temp[1][1]], static_tiles=static_tiles)
     if nest["pattern"] == "LOGREG_GRAD" and staged:  # tickets [B] + fp64 accumulators [B x C]
         B, C = _eff(nest["levels"][0][0]), _eff(nest["levels"][2][0])
         rec["workspace_bytes"] = 256 * cdiv(4 * B, 256) + 256 * cdiv(8 * B * C, 256)
@@ -671,6 +677,6 @@ def select(pattern: str, shape, dtype: str, lim: dict, strategy: str = "AUTO") -
     if staged_eligible(nest, dtype, dims):
         b2, s2, f2, vec, chunks, G, CL = r2_staged(nest, dtype, lim)
         return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks, staged=1,
-                           persistent_grid=G, claim_tiles=CL)
+                           persistent_grid=G, claim_tiles=CL, static_tiles=r2_staged_static(nest, dtype, lim))
     b2, s2, f2, vec, chunks = r2_sums(nest, dtype, lim, dims)
     return make_record(nest, dtype, lim, dims, b2, s2, f2, vec, sc, chunks)

@@ -9,14 +9,31 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <mutex>
+#include <set>
 #include <string>
+#include <tuple>
 
 #include "kernels.hpp"
 #include "select.hpp"
 
 namespace npp {
 extern thread_local std::string g_error;
+
+cudaError_t ensure_smem_attr(const void* func, int smem_bytes) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  static std::mutex mu;
+  static std::set<std::tuple<const void*, int, int>> done;  // (kernel, device, bytes) already set
+  std::lock_guard<std::mutex> lock(mu);
+  const auto key = std::make_tuple(func, dev, smem_bytes);
+  if (done.count(key)) return cudaSuccess;
+  e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  if (e == cudaSuccess) done.insert(key);
+  return e;
 }
+}  // namespace npp
 
 struct npp_plan_s {
   int pattern = 0;
@@ -134,39 +151,6 @@ int get_limits(const npp_limits* limits, npp_limits* out) {
 
 inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
-void debug_print_times(const unsigned long long* dbg, int G, cudaStream_t st) {
-  static unsigned long long h[4096 * 8];
-  if (G > 4096) return;
-  cudaStreamSynchronize(st);
-  cudaMemcpy(h, dbg, size_t(G) * 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
-  cudaMemset(const_cast<unsigned long long*>(dbg), 0, size_t(G) * 8 * sizeof(unsigned long long));
-  unsigned long long t0 = ~0ull;
-  for (int b = 0; b < G; ++b) t0 = h[b * 8] < t0 ? h[b * 8] : t0;
-  double mx[3] = {0, 0, 0}, mn[3] = {1e30, 1e30, 1e30}, sm[3] = {0, 0, 0};
-  double fence_ticket = 0, convert = 0, flushes = 0, last_n = 0;
-  int nb = 0;
-  for (int b = 0; b < G; ++b) {
-    for (int i = 0; i < 3; ++i) {
-      const double v = double(h[b * 8 + i] - t0) / 1e3;
-      mx[i] = v > mx[i] ? v : mx[i];
-      mn[i] = v < mn[i] ? v : mn[i];
-      sm[i] += v;
-    }
-    if (h[b * 8 + 4]) {
-      fence_ticket += double(h[b * 8 + 5] - h[b * 8 + 4]) / 1e3;
-      convert += double(h[b * 8 + 2] - h[b * 8 + 5]) / 1e3;
-      last_n += double(h[b * 8 + 7]);
-      ++nb;
-    }
-    flushes += double(h[b * 8 + 6]);
-  }
-  std::fprintf(stderr,
-               "npp times(us) G=%d start[%.2f..%.2f] stream_end[%.2f avg %.2f max %.2f] combiner_end[%.2f avg %.2f "
-               "max %.2f] last batch: fence+ticket %.2f, convert+exit %.2f, size %.2f; flushes/block %.2f\n",
-               G, mn[0], mx[0], mn[1], sm[1] / G, mx[1], mn[2], sm[2] / G, mx[2], nb ? fence_ticket / nb : 0.0,
-               nb ? convert / nb : 0.0, nb ? last_n / nb : 0.0, flushes / G);
-}
-
 }  // namespace
 
 extern "C" {
@@ -238,6 +222,11 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
   if (pattern == NPP_PAGERANK && strategy != NPP_MAP_AUTO) {
     delete p;
     set_error("PAGERANK executes with strategy AUTO only (class PR)");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  if (pattern == NPP_PAGERANK && ndim >= 2 && shape[1] >= (int64_t(1) << 31)) {
+    delete p;
+    set_error("PAGERANK plans need E < 2^31 edges (the kernel keeps 32-bit edge offsets inside a row chunk)");
     return NPP_ERR_UNSUPPORTED;
   }
   st = get_limits(limits, &p->lim);
@@ -312,6 +301,15 @@ int npp_plan_with_mapping(int pattern, const int64_t* shape, int ndim, int dtype
   if (!npp::is_sum_pattern(pattern)) {
     set_error("explicit mappings are executable for the 2-level sum families only");
     return NPP_ERR_UNSUPPORTED;
+  }
+  // class RX (inner Reduce on x) finishes a row with xor-shuffles over min(b_x, 32) lanes: the x block must
+  // be a power of two <= 32 or a multiple of 32, or two rows would share (or lose) lanes of one warp
+  if (c.dims[1] == NPP_DIM_X) {
+    const int bx = c.blocks[1];
+    if (!((bx <= 32 && (bx & (bx - 1)) == 0) || bx % 32 == 0)) {
+      set_error("explicit RX mapping: the x-level block must be a power of two <= 32 or a multiple of 32");
+      return NPP_ERR_UNSUPPORTED;
+    }
   }
   // vector width: only on the x level when it is the stride-1 level of m and C % vec == 0
   const int v0 = 16 / npp::dtype_size(dtype);
@@ -389,17 +387,23 @@ int npp_plan_launches(npp_plan_t plan) {
 
 void npp_plan_destroy(npp_plan_t plan) { delete plan; }
 
-int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream) {
-  return npp_execute_ex(plan, ins, n_in, out, workspace, stream, 0u);
-}
+}  // extern "C"
 
-int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream,
-                   unsigned flags) {
-  if (flags & ~NPP_EXEC_OVERLAP) {
+namespace {
+
+// npp_execute_ex / npp_execute_traced: `trace` (device, may be NULL) receives the tile schedule
+int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream,
+                 unsigned flags, int* trace) {
+  if (flags & ~(NPP_EXEC_OVERLAP | NPP_EXEC_NO_PDL)) {
     set_error("unknown npp_execute_ex flag bits");
     return NPP_ERR_INVALID_ARG;
   }
+  if ((flags & NPP_EXEC_OVERLAP) && (flags & NPP_EXEC_NO_PDL)) {
+    set_error("NPP_EXEC_OVERLAP needs a programmatic dependent launch (not NPP_EXEC_NO_PDL)");
+    return NPP_ERR_INVALID_ARG;
+  }
   const bool overlap = (flags & NPP_EXEC_OVERLAP) != 0;
+  const int pdl = (flags & NPP_EXEC_NO_PDL) ? 0 : 1;
   if (!plan) {
     set_error("plan is NULL");
     return NPP_ERR_INVALID_ARG;
@@ -451,6 +455,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     g.per_block = m.claim_tiles;
     g.tickets = static_cast<unsigned*>(workspace);
     g.acc = reinterpret_cast<double*>(static_cast<char*>(workspace) + ((4 * g.B + 255) / 256) * 256);
+    g.trace = trace;
     cudaError_t e = npp::launch_logreg(g, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("logreg kernel launch", e);
     return NPP_OK;
@@ -463,6 +468,7 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     k.D = plan->shape[1];
     k.K = plan->shape[2];
     k.per_block = m.claim_tiles;
+    k.trace = trace;
     cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);
     return NPP_OK;
@@ -493,6 +499,8 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     u.K = plan->shape[2];
     u.per_block = m.claim_tiles;
     u.early_reads = overlap ? 1 : 0;
+    u.pdl = pdl;
+    u.trace = trace;
     cudaError_t e = npp::launch_kmupdate(u, static_cast<const float*>(ins[0]), static_cast<const int*>(ins[1]),
                                          int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("k-means update kernel launch", e);
@@ -516,6 +524,8 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     r.accR = ws + o_ar;
     r.accC = ws + o_ac;
     r.early_reads = overlap ? 1 : 0;
+    r.pdl = pdl;
+    r.trace = trace;
     cudaError_t e = npp::launch_rowscols(plan->dtype, m.staged != 0, r, int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("rows+cols kernel launch", e);
     return NPP_OK;
@@ -541,21 +551,13 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
     s.static_tiles = bal.Ts;
     s.unit = bal.U;
     s.early_reads = overlap ? 1 : 0;
+    s.pdl = pdl;
+    s.trace = trace;
     s.wide = t.r1 ? 2 : (t.wide ? 1 : 0);
     s.pool = static_cast<unsigned*>(workspace);  // S9 staged workspace: [256 B pool][tickets][acc]
     s.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + 256);
     s.acc = static_cast<char*>(workspace) + 256 + ((t.To * 4 + 255) / 256) * 256;
-    // measurement knob: NPP_DEBUG_TIMES=1 prints per-phase block timestamps (synchronises the stream)
-    static unsigned long long* dbg = nullptr;
-    const bool want_times = getenv("NPP_DEBUG_TIMES") != nullptr;
-    if (want_times && !dbg) {
-      if (cudaMalloc(&dbg, 4096 * 8 * sizeof(unsigned long long)) != cudaSuccess) dbg = nullptr;
-      else cudaMemset(dbg, 0, 4096 * 8 * sizeof(unsigned long long));
-    }
-    s.dbg_times = want_times ? dbg : nullptr;
-    const int G = int(m.grid);
-    cudaError_t e = npp::launch_sum_staged(plan->dtype, rows, ins[0], s, G, st);
-    if (s.dbg_times && e == cudaSuccess) debug_print_times(dbg, G, st);
+    cudaError_t e = npp::launch_sum_staged(plan->dtype, rows, ins[0], s, int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("staged kernel launch", e);
     return NPP_OK;
   }
@@ -598,6 +600,49 @@ int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out,
   cudaError_t e = npp::launch_sum(plan->dtype, m.kernel_class, m.vec, weighted, a, st);
   if (e != cudaSuccess) return cuda_fail("kernel launch", e);
   return NPP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int npp_execute(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream) {
+  return execute_impl(plan, ins, n_in, out, workspace, stream, 0u, nullptr);
+}
+
+int npp_execute_ex(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream,
+                   unsigned flags) {
+  return execute_impl(plan, ins, n_in, out, workspace, stream, flags, nullptr);
+}
+
+int64_t npp_plan_tiles(npp_plan_t plan) {
+  if (!plan || plan->empty) return 0;
+  const npp_mapping& m = plan->map;
+  const int64_t* s = plan->shape;
+  switch (m.kernel_class) {
+    case NPP_CLASS_RX:
+    case NPP_CLASS_MX:
+      if (!m.staged) return 0;
+      return m.level[0].grid * m.level[1].grid;  // To x Ti (S9: chunk = one tile per level)
+    case NPP_CLASS_LOGREG: return s[0] * ((s[1] + 31) / 32);
+    case NPP_CLASS_KMEANS: return (s[0] + (s[1] <= 64 ? 255 : 127)) / (s[1] <= 64 ? 256 : 128);
+    case NPP_CLASS_KMUPDATE: return (s[0] + 127) / 128;
+    case NPP_CLASS_RC: return m.level[0].grid * m.level[1].grid;
+    default: return 0;
+  }
+}
+
+int npp_execute_traced(npp_plan_t plan, const void* const* ins, int n_in, void* out, void* workspace, void* stream,
+                       int32_t* trace) {
+  if (!trace) {
+    set_error("trace is NULL");
+    return NPP_ERR_INVALID_ARG;
+  }
+  if (npp_plan_tiles(plan) <= 0) {
+    set_error("npp_execute_traced: the plan has no tile schedule (staged families only)");
+    return NPP_ERR_UNSUPPORTED;
+  }
+  return execute_impl(plan, ins, n_in, out, workspace, stream, 0u, trace);
 }
 
 int npp_execute_host(npp_plan_t plan, const void* const* host_ins, int n_in, void* host_out,

@@ -133,6 +133,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 
   const long long n_tiles = r1 - r0;
   auto issue = [&](long long t, int slot) {  // tile t of the block's range into slot t % kStages
+    if (a.trace) {  // white-box schedule trace (npp_execute_traced)
+      a.trace[r0 + t] = int(bid);
+      atomicAdd(a.trace + T + r0 + t, 1);
+    }
     tma::mbar_expect_tx(full + slot, unsigned(stage_bytes));
     for (int bx = 0; bx < nb; ++bx)
       tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
@@ -282,7 +286,7 @@ cudaEvent_t g_km_done[64] = {};
 
 cudaError_t launch_tp(void (*kern)(const CUtensorMap, KmeansArgs), const CUtensorMap& map, const KmeansArgs& a,
                       int grid, size_t smem, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  cudaError_t e = ensure_smem(kern, int(smem));
   if (e != cudaSuccess) return e;
   kern<<<grid, kThreads, smem, st>>>(map, a);
   return cudaGetLastError();

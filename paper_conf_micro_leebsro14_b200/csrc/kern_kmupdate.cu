@@ -101,6 +101,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         mbar_expect_tx(full + slot, bytes);
         load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
         load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
+        if (a.trace) {
+          a.trace[t] = int(blockIdx.x);
+          atomicAdd(a.trace + T + t, 1);
+        }
       }
     }
     return;
@@ -241,13 +245,8 @@ cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* ke
   cudaError_t e = encode_2d(&xmap, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(a.D), unsigned(kTP));
   if (e != cudaSuccess) return e;
   if ((e = encode_1d(&amap, keys, CU_TENSOR_MAP_DATA_TYPE_INT32, a.N, unsigned(kTP))) != cudaSuccess) return e;
-  static bool attr_set = false;
-  if (!attr_set) {
-    e = cudaFuncSetAttribute(npp_kmupdate_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
-  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, true, xmap, amap, a);
+  if ((e = ensure_smem(npp_kmupdate_kernel, kSmemBytes)) != cudaSuccess) return e;
+  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, a.pdl != 0, xmap, amap, a);
 }
 
 }  // namespace npp

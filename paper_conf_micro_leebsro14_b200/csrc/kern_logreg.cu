@@ -92,6 +92,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
         tma::mbar_expect_tx(full + slot, tile_bytes + kYBox * 4);
         tma::load_2d(tiles + slot * kTileBytes, &map, 0, int(row0), full + slot);
         tma::load_1d(y_ring + slot * kYSlot, &ymap, int(row0 & ~3ll), full + slot);
+        if (a.trace) {
+          a.trace[cur] = int(bid);
+          atomicAdd(a.trace + total + cur, 1);
+        }
         if (++j == Ti) j = 0, ++b;
         if (++slot == kStages) slot = 0, ph ^= 1u;
       }
@@ -217,15 +221,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
 }
 
 cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStream_t st) {
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(npp_logreg_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  cudaError_t e = ensure_smem(npp_logreg_tma_kernel, kSmemBytes);
+  if (e != cudaSuccess) return e;
   CUtensorMap map;
-  cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.B * a.Rb, a.C, unsigned(a.C),
+  e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.B * a.Rb, a.C, unsigned(a.C),
                                  unsigned(kTileRows));
   if (e != cudaSuccess) return e;
   CUtensorMap ymap;

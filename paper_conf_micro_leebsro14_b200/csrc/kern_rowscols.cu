@@ -169,6 +169,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   long long t = 0;
   int rb = 0;  // rsum double buffer
   for (long long q = q0; q < q1; ++q) {
+    if (a.trace && threadIdx.x == 0) {  // white-box schedule trace: who took region q
+      a.trace[q] = int(blockIdx.x);
+      atomicAdd(a.trace + a.nreg + q, 1);
+    }
     const long long ri = q / a.gc, cj = q - ri * a.gc;
     const long long b0 = ri * a.cr, b1 = b0 + a.cr < a.Tr ? b0 + a.cr : a.Tr;
     const long long c0 = cj * a.cc, c1 = c0 + a.cc < a.Tc ? c0 + a.cc : a.Tc;
@@ -288,14 +292,10 @@ namespace {
 
 template <typename T, bool STAGED>
 cudaError_t launch_typed(const CUtensorMap& map, const RowsColsArgs& a, int grid, cudaStream_t st) {
-  static bool attr_set = false;
   auto kern = npp_rowscols_kernel<T, STAGED>;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
-  return launch_pdl(kern, grid, kThreads, kSmemBytes, st, true, map, a);
+  cudaError_t e = ensure_smem(kern, kSmemBytes);
+  if (e != cudaSuccess) return e;
+  return launch_pdl(kern, grid, kThreads, kSmemBytes, st, a.pdl != 0, map, a);
 }
 
 template <typename T>

@@ -54,62 +54,12 @@ constexpr int kSmemBytes = kSmemHeader + kStages * kTileBytes;
 constexpr int kVSlot = 4096;  // weighted sums: the tile's slice of v (<= 4 KB) per ring slot
 constexpr int kSmemBytesW = kSmemBytes + kStages * kVSlot;
 
-__device__ __forceinline__ unsigned smem_u32(const void* p) {
-  return static_cast<unsigned>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n NPP_WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra NPP_WAIT_%=;\n}" ::"r"(smem_u32(b)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          smem_u32(dst)),
-      "l"(map), "r"(x), "r"(y), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
-  unsigned ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
-      : "=r"(ok)
-      : "r"(smem_u32(b)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-__device__ __forceinline__ void tma_load_1d(void* dst, const CUtensorMap* map, int x, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(map), "r"(x), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int x, int y, int z, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
-          smem_u32(dst)),
-      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
-__device__ __forceinline__ unsigned long long gtimer() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
+using tma::mbar_arrive;
+using tma::mbar_expect_tx;
+using tma::mbar_init;
+using tma::mbar_test;
+using tma::mbar_wait;
+__device__ __forceinline__ void consumers_sync() { tma::bar_sync_consumers<kConsumers>(); }
 
 template <typename T> struct SOps;
 template <> struct SOps<float> {
@@ -218,21 +168,15 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       mbar_init(fl_full + i, kConsumerWarps);
       mbar_init(fl_free + i, 1);
     }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    if (a.dbg_times) {
-      unsigned smid;
-      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-      a.dbg_times[bid * 8 + 0] = gtimer();
-      a.dbg_times[bid * 8 + 3] = smid;
-    }
+    tma::mbar_fence_init();
   }
   __syncthreads();
 
   if (warp == kProducerWarp) {
     // ------------------------------------------------------------ producer: one elected lane
     if (lane == 0) {
-      asm volatile("prefetch.tensormap [%0];" ::"l"(&map) : "memory");
-      if constexpr (WT) asm volatile("prefetch.tensormap [%0];" ::"l"(&vmap) : "memory");
+      tma::prefetch_map(&map);
+      if constexpr (WT) tma::prefetch_map(&vmap);
       long long sn = s0, u_cur = 0, u_end = 0;
       // Every launch is a programmatic dependent launch: this block may already be resident while the
       // previous kernel in the stream drains. Unless the caller asserted NPP_EXEC_OVERLAP (inputs not
@@ -270,6 +214,10 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         // read with (relaxed) shared atomics so compute-sanitizer's racecheck, which does not model
         // mbarrier ordering, sees no plain-access race
         atomicExch(slot_tile + slot, static_cast<unsigned>(cur) | (flush ? kFlush : 0u));
+        if (a.trace) {  // white-box schedule trace (npp_execute_traced): who streamed tile cur
+          a.trace[cur] = int(bid);
+          atomicAdd(a.trace + total + cur, 1);
+        }
         constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
         mbar_expect_tx(full + slot, kTileBytes + kVBytes);
         const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
@@ -279,15 +227,15 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
           if constexpr (ROWS) {
 #pragma unroll
             for (int q = 0; q < NCH; ++q)
-              tma_load_1d(vslots + slot * kVSlot + q * 1024, &vmap, (ch + q) * BC, full + slot);
+              tma::load_1d(vslots + slot * kVSlot + q * 1024, &vmap, (ch + q) * BC, full + slot);
           } else {
-            tma_load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
+            tma::load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
           }
         }
         if constexpr (WIDE && ROWS)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
-          tma_load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
+          tma::load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
         else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
-          tma_load_2d(tiles + slot * kTileBytes, &map, MXN ? int(ot * W) : ch * BC, y, full + slot);
+          tma::load_2d(tiles + slot * kTileBytes, &map, MXN ? int(ot * W) : ch * BC, y, full + slot);
         cur = nxt;
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
@@ -307,14 +255,13 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       mbar_wait(fl_full + int(k % kFlushRing), unsigned((k / kFlushRing) & 1));
       int nb = 1;
       while (nb < kFlushRing &&
-             mbar_try(fl_full + int((k + nb) % kFlushRing), unsigned(((k + nb) / kFlushRing) & 1)))
+             mbar_test(fl_full + int((k + nb) % kFlushRing), unsigned(((k + nb) / kFlushRing) & 1)))
         ++nb;
       const int i = int((k + lane) % kFlushRing);
       const long long ot = lane < nb ? fl_ot[i] : -1;
       const unsigned cnt = lane < nb ? fl_cnt[i] : 0u;
       const unsigned ends = __ballot_sync(0xffffffffu, lane < nb && ot < 0);
       const int n = ends ? __ffs(ends) - 1 : nb;  // entries before the end marker
-      const unsigned long long t_b0 = a.dbg_times ? gtimer() : 0ull;
       // the ticket add is itself the release (cumulative over the consumers' accumulator adds, which
       // the fl_full mbarrier ordered before it) and the acquire of the contributor that completes
       // the tile; the other lanes read the accumulators after a fence only when some tile completed
@@ -325,12 +272,6 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         if (last) a.tickets[ot] = 0u;
       }
       if (__any_sync(0xffffffffu, last)) asm volatile("fence.acq_rel.gpu;" ::: "memory");
-      if (a.dbg_times && lane == 0 && n > 0) {  // measurement knob: the last batch's phases
-        a.dbg_times[bid * 8 + 4] = t_b0;
-        a.dbg_times[bid * 8 + 5] = gtimer();
-        a.dbg_times[bid * 8 + 6] += n;
-        a.dbg_times[bid * 8 + 7] = n;
-      }
       unsigned lasts = __ballot_sync(0xffffffffu, last);
       while (lasts) {  // every contribution to these outer tiles is in: read (L2), convert, re-zero
         const int j = __ffs(lasts) - 1;
@@ -360,7 +301,6 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       k += n;
       if (ends) break;
     }
-    if (a.dbg_times && lane == 0) a.dbg_times[bid * 8 + 2] = gtimer();
   } else {
     // ------------------------------------------------------------ consumers
     constexpr int kGroups = ROWS ? 1 : 256 / W;   // MX row groups (1 / 2 for 4- / 8-byte; MX-narrow 4 / 8)
@@ -532,40 +472,19 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       mbar_arrive(fl_full + fi);
     }
   }
-  if (a.dbg_times && threadIdx.x == 0) a.dbg_times[bid * 8 + 1] = gtimer();
 }
 
 // ====================================================================================== host side
 namespace {
 
-typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
-                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_fn() {
-  static EncodeTiledFn fn = [] {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess)
-      return static_cast<EncodeTiledFn>(nullptr);
-    return reinterpret_cast<EncodeTiledFn>(p);
-  }();
-  return fn;
-}
-
 template <typename T, bool ROWS, bool WIDE, bool WT, bool R1 = false>
 cudaError_t launch_typed(const CUtensorMap& map, const CUtensorMap& vmap, const StagedArgs& a, int grid,
                          cudaStream_t st) {
-  static bool attr_set = false;
   auto kern = npp_sum_tma_kernel<T, ROWS, WIDE, WT, R1>;
   const int smem = (WT ? kSmemBytesW : kSmemBytes) + (((WIDE && !ROWS) || R1) ? 2048 : 0);  // group sums
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
-  return launch_pdl(kern, grid, kThreads, smem, st, true, map, vmap, a);
+  cudaError_t e = ensure_smem(kern, smem);
+  if (e != cudaSuccess) return e;
+  return launch_pdl(kern, grid, kThreads, smem, st, a.pdl != 0, map, vmap, a);
 }
 
 template <typename T, bool WT>
@@ -591,49 +510,28 @@ cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const CUtensorMap& v
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st) {
   if (a.To * a.Ti >= 0x7fffffffll) return cudaErrorInvalidValue;  // 32-bit slot tags
-  EncodeTiledFn encode = encode_fn();
-  if (!encode) return cudaErrorNotSupported;
   const int esz = dtype == NPP_I64 ? 8 : 4;
   const cuuint64_t bc = cuuint64_t(1024 / esz);
-  CUtensorMap map;
   const CUtensorMapDataType dt = dtype == NPP_F32   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                  : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
                                                     : CU_TENSOR_MAP_DATA_TYPE_INT64;
-  CUresult r;
+  CUtensorMap map;
+  cudaError_t e;
   if (a.wide && !rows) {  // MX-narrow strips: {C, R}, box 128 rows x 256 B
-    const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
-    const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
-    const cuuint32_t box[2] = {cuuint32_t(256 / esz), 128};
-    const cuuint32_t estr[2] = {1, 1};
-    r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  } else if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (row pitch is a multiple of 4 KB)
+    e = tma::encode_2d(&map, m, dt, esz, a.R, a.C, unsigned(256 / esz), 128u);
+  } else if (a.wide) {  // {1 KB chunk, chunks per row, rows}; box 8 rows x 4 KB (or R1: 1 row x 32 KB)
     const cuuint64_t dims[3] = {bc, cuuint64_t(a.C) / bc, cuuint64_t(a.R)};
     const cuuint64_t strides[2] = {1024, cuuint64_t(a.C) * esz};
     const cuuint32_t box[3] = {cuuint32_t(bc), a.wide == 2 ? 32u : 4u, a.wide == 2 ? 1u : cuuint32_t(kTileRows / 4)};
-    const cuuint32_t estr[3] = {1, 1, 1};
-    r = encode(&map, dt, 3, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    e = tma::encode_nd(&map, m, dt, 3, dims, strides, box);
   } else {  // {C, R}; box 32 rows x 1 KB
-    const cuuint64_t dims[2] = {cuuint64_t(a.C), cuuint64_t(a.R)};
-    const cuuint64_t strides[1] = {cuuint64_t(a.C) * esz};
-    const cuuint32_t box[2] = {cuuint32_t(bc), cuuint32_t(kTileRows)};
-    const cuuint32_t estr[2] = {1, 1};
-    r = encode(&map, dt, 2, const_cast<void*>(m), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    e = tma::encode_2d(&map, m, dt, esz, a.R, a.C, unsigned(bc), unsigned(kTileRows));
   }
-  if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  if (e != cudaSuccess) return e;
   CUtensorMap vmap;  // weighted: 1-D map over v (C elements for sumRows, R for sumCols)
   std::memset(&vmap, 0, sizeof vmap);
-  if (a.v) {
-    const cuuint64_t vd[1] = {cuuint64_t(rows ? a.C : a.R)};
-    const cuuint64_t vs[1] = {vd[0] * esz};
-    const cuuint32_t vb[1] = {cuuint32_t(rows ? bc : kTileRows)};
-    const cuuint32_t ve[1] = {1};
-    r = encode(&vmap, dt, 1, const_cast<void*>(a.v), vd, vs, vb, ve, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  }
+  if (a.v && (e = tma::encode_1d(&vmap, a.v, dt, rows ? a.C : a.R, unsigned(rows ? bc : kTileRows))) != cudaSuccess)
+    return e;
   switch (dtype) {
     case NPP_F32: return launch_dtype<float>(rows, map, vmap, a, grid, st);
     case NPP_I32: return launch_dtype<int32_t>(rows, map, vmap, a, grid, st);

@@ -10,6 +10,14 @@
 
 namespace npp {
 
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is per device: set it once per (kernel, device) under a
+// lock (the first launch on each device of a process that drives several GPUs sets its own).
+cudaError_t ensure_smem_attr(const void* func, int smem_bytes);
+template <typename... Params>
+cudaError_t ensure_smem(void (*kern)(Params...), int smem_bytes) {
+  return ensure_smem_attr(reinterpret_cast<const void*>(kern), smem_bytes);
+}
+
 // Launch `kern` on `st`; with `overlap` as a programmatic dependent launch (PDL): its blocks may become
 // resident while the previous kernel in the stream drains; the kernel orders itself after that kernel
 // with `griddepcontrol.wait` (before its first read, or — NPP_EXEC_OVERLAP — before its first write).
@@ -67,8 +75,9 @@ struct StagedArgs {
   int64_t static_tiles; // Ts
   int64_t unit;         // U: pool claim unit (tiles)
   int early_reads;      // NPP_EXEC_OVERLAP: stream the inputs before the previous kernel completes
-  int wide;             // tiles of 8 rows x 4 KB (row pitch a multiple of 4 KB), else 32 rows x 1 KB
-  unsigned long long* dbg_times;  // measurement knob (NPP_DEBUG_TIMES): [grid x 4] globaltimer stamps
+  int wide;             // 1: tiles of 8 rows x 4 KB (RX) / 128 rows x 256 B (MX-narrow); 2: RX one-row 32 KB tiles
+  int pdl;              // launch as a programmatic dependent launch (npp_execute_ex without NPP_EXEC_NO_PDL)
+  int* trace;           // npp_execute_traced: [2 x To*Ti] block of each tile, loads per tile (else NULL)
 };
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st);
@@ -83,6 +92,7 @@ struct LogregArgs {
   int64_t B, Rb, C;
   int64_t Ti;          // 32-row tiles per batch
   int64_t per_block;   // P: block b streams tiles [b*P, (b+1)*P) of the batch-major order
+  int* trace;          // npp_execute_traced: [2 x B*Ti] block of each tile, loads per tile (else NULL)
 };
 cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStream_t st);
 
@@ -91,7 +101,8 @@ struct KmeansArgs {
   const float* c;      // [K x D]
   int* assign;         // [N]
   int64_t N, D, K;
-  int64_t per_block;   // P: block b handles 128-point tiles [b*P, (b+1)*P)
+  int64_t per_block;   // P: block b handles TP-point tiles [b*P, (b+1)*P)
+  int* trace;          // npp_execute_traced: [2 x T] block of each tile, loads per tile (else NULL)
 };
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st);
 
@@ -111,6 +122,8 @@ struct RowsColsArgs {
   int64_t gr, gc;      // regions along rows / columns
   int64_t nreg;        // gr * gc
   int early_reads;     // NPP_EXEC_OVERLAP
+  int pdl;             // programmatic dependent launch (not NPP_EXEC_NO_PDL)
+  int* trace;          // npp_execute_traced: [2 x nreg] block of each region, visits per region (else NULL)
 };
 cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int grid, cudaStream_t st);
 
@@ -123,6 +136,8 @@ struct KmUpdateArgs {
   int64_t N, D, K;
   int64_t per_block;   // P
   int early_reads;     // NPP_EXEC_OVERLAP
+  int pdl;             // programmatic dependent launch (not NPP_EXEC_NO_PDL)
+  int* trace;          // npp_execute_traced: [2 x T] block of each 128-point tile, loads per tile (else NULL)
 };
 cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st);
 

@@ -231,6 +231,7 @@ void r2_staged(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   const StagedTiling t = staged_tiling(n.pattern, R, n.cols, dtype);
   const StagedBalance bal = staged_balance(t.To, t.Ti, lim.sm_count);
   c->claim_tiles = bal.U;
+  c->static_tiles = bal.Ts;
   c->persistent_grid = bal.G;
   c->staged = 1;
   if (rows) {  // 8 warps; narrow: 4 rows per warp, wide: 1 row per warp
@@ -720,6 +721,7 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
   m.workspace_bytes = 0;
   m.staged = c.staged;
   m.claim_tiles = c.claim_tiles;
+  m.static_tiles = c.static_tiles;
   m.temp = c.temp;
   m.temp_stride[0] = c.temp_stride[0];
   m.temp_stride[1] = c.temp_stride[1];

@@ -39,6 +39,7 @@ struct Choice {  // one point of the candidate space plus its ControlDOP/R2 refi
   int staged = 0;  // 1: TMA-staged tile family (S8)
   int64_t persistent_grid = 0;  // staged: blocks launched (0: product of the level grids)
   int64_t claim_tiles = 0;      // staged: tiles per dynamic claim
+  int64_t static_tiles = 0;     // staged sums: tiles split statically before the claim pool (Ts)
   int temp = NPP_TEMP_NONE;     // weighted sums: inner allocation (S10)
   int64_t temp_stride[2] = {0, 0};
 };

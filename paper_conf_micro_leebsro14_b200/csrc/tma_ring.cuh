@@ -43,6 +43,16 @@ __device__ __forceinline__ bool mbar_try(uint64_t* b, unsigned parity) {
       : "memory");
   return ok != 0;
 }
+// non-blocking probe of a phase (mbarrier.test_wait): polls a batch of ready entries without sleeping
+__device__ __forceinline__ bool mbar_test(uint64_t* b, unsigned parity) {
+  unsigned ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
 // whole-warp wait whose exit is a vote: the compiler sees the warp converged after it (the phase
 // cannot flip back while these threads still hold the buffer), so uniform-datapath code may follow
 __device__ __forceinline__ void mbar_wait_warp(uint64_t* b, unsigned parity) {
@@ -61,6 +71,13 @@ __device__ __forceinline__ void load_1d(void* dst, const CUtensorMap* map, int x
       "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2}], [%3];" ::"r"(
           smem_u32(dst)),
       "l"(map), "r"(x), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void load_3d(void* dst, const CUtensorMap* map, int x, int y, int z, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
+          smem_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
       : "memory");
 }
 __device__ __forceinline__ void prefetch_map(const CUtensorMap* map) {
@@ -112,6 +129,18 @@ inline cudaError_t encode_2d(CUtensorMap* map, const void* base, CUtensorMapData
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = encode(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                       swizzle, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+// rank-n map (n <= 3) with explicit dims / byte strides (strides[i] for dims 1..n-1) and box
+inline cudaError_t encode_nd(CUtensorMap* map, const void* base, CUtensorMapDataType dt, int rank, const cuuint64_t* dims,
+                             const cuuint64_t* strides, const cuuint32_t* box) {
+  EncodeTiledFn encode = encoder();
+  if (!encode) return cudaErrorNotSupported;
+  const cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = encode(map, dt, cuuint32_t(rank), const_cast<void*>(base), dims, strides, box, estr,
+                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 

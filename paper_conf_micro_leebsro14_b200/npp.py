@@ -44,7 +44,8 @@ class Mapping(ctypes.Structure):
                 ("dop", ctypes.c_int64), ("threads", ctypes.c_int64), ("grid", ctypes.c_int64),
                 ("block", ctypes.c_int32 * 3), ("smem_bytes", ctypes.c_int32),
                 ("workspace_bytes", ctypes.c_int64), ("claim_tiles", ctypes.c_int64),
-                ("temp", ctypes.c_int32), ("reserved2", ctypes.c_int32), ("temp_stride", ctypes.c_int64 * 2)]
+                ("temp", ctypes.c_int32), ("reserved2", ctypes.c_int32), ("temp_stride", ctypes.c_int64 * 2),
+                ("static_tiles", ctypes.c_int64)]
 
 
 class Limits(ctypes.Structure):
@@ -56,12 +57,13 @@ class Limits(ctypes.Structure):
                 ("smem_per_block", ctypes.c_int64)]
 
 
-EXEC_OVERLAP = 1  # npp.h NPP_EXEC_OVERLAP
+EXEC_OVERLAP, EXEC_NO_PDL = 1, 2  # npp.h NPP_EXEC_OVERLAP / NPP_EXEC_NO_PDL
 TEMP_NONE, TEMP_MALLOC, TEMP_PREALLOC = 0, 1, 2  # npp.h npp_temp
 
 EXPORTS = ("npp_version", "npp_last_error", "npp_limits_query", "npp_select", "npp_plan",
            "npp_plan_with_mapping", "npp_plan_mapping", "npp_plan_workspace_bytes", "npp_execute",
-           "npp_execute_ex", "npp_execute_host", "npp_enumerate", "npp_plan_launches", "npp_plan_destroy")
+           "npp_execute_ex", "npp_execute_host", "npp_enumerate", "npp_plan_launches", "npp_plan_destroy",
+           "npp_plan_tiles", "npp_execute_traced")
 
 
 def _load():
@@ -86,6 +88,9 @@ def _load():
     lib.npp_execute_ex.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, P, P, ctypes.c_uint]
     lib.npp_execute_host.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, ctypes.POINTER(P), P, P, P]
     lib.npp_plan_launches.argtypes = [P]
+    lib.npp_plan_tiles.argtypes = [P]
+    lib.npp_plan_tiles.restype = ctypes.c_int64
+    lib.npp_execute_traced.argtypes = [P, ctypes.POINTER(P), ctypes.c_int, P, P, P, P]
     lib.npp_enumerate.argtypes = [ctypes.c_int, I64P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(Limits),
                                   ctypes.c_void_p, ctypes.c_int64]
     lib.npp_enumerate.restype = ctypes.c_int64
@@ -138,7 +143,7 @@ def mapping_to_dict(m: Mapping) -> dict:
                 score=m.score,
                 dop=m.dop, threads=m.threads, grid=m.grid, block=list(m.block), smem_bytes=m.smem_bytes,
                 workspace_bytes=m.workspace_bytes, claim_tiles=m.claim_tiles, temp=m.temp,
-                temp_stride=[m.temp_stride[0], m.temp_stride[1]])
+                temp_stride=[m.temp_stride[0], m.temp_stride[1]], static_tiles=m.static_tiles)
 
 
 def mapping_from_dict(d: dict) -> Mapping:
@@ -255,18 +260,35 @@ class Plan:
     def new_out(self):
         return torch.empty(self.out_shape(), dtype=self.out_dtype(), device=self.device)
 
-    def execute(self, ins, out, stream=None, workspace=None, overlap=False):
+    def execute(self, ins, out, stream=None, workspace=None, overlap=False, pdl=True):
         """Enqueue on `stream` (default: torch's current stream). Inputs must be contiguous device tensors.
         overlap=True is npp_execute_ex(NPP_EXEC_OVERLAP): the caller asserts no earlier work on the
-        stream writes `ins` (the staged kernels then start while the previous kernel drains)."""
+        stream writes `ins` (the staged kernels then start while the previous kernel drains).
+        pdl=False is NPP_EXEC_NO_PDL: plain stream-ordered launches (isolated kernel timing)."""
         for t in ins:
             if not t.is_contiguous():
                 raise ValueError("inputs must be contiguous")
         arr = (ctypes.c_void_p * len(ins))(*[t.data_ptr() for t in ins])
         ws = workspace if workspace is not None else self.workspace
-        _check(_lib.npp_execute_ex(self._h, arr, len(ins), _ptr(out), _ptr(ws), _stream_handle(stream),
-                                   EXEC_OVERLAP if overlap else 0))
+        flags = (EXEC_OVERLAP if overlap else 0) | (0 if pdl else EXEC_NO_PDL)
+        _check(_lib.npp_execute_ex(self._h, arr, len(ins), _ptr(out), _ptr(ws), _stream_handle(stream), flags))
         return out
+
+    @property
+    def tiles(self) -> int:
+        """npp_plan_tiles: tiles (or regions) of the plan's schedule, 0 if it has none."""
+        return int(_lib.npp_plan_tiles(self._h))
+
+    def execute_traced(self, ins, out, stream=None):
+        """npp_execute_traced: execute and return (block of each tile, loads of each tile) as int32 tensors
+        on the device (white-box check of the runtime rule's schedule, S8)."""
+        n = self.tiles
+        trace = torch.zeros(2 * max(n, 1), dtype=torch.int32, device=self.device)
+        trace[:n] = -1
+        arr = (ctypes.c_void_p * len(ins))(*[t.data_ptr() for t in ins])
+        _check(_lib.npp_execute_traced(self._h, arr, len(ins), _ptr(out), _ptr(self.workspace),
+                                       _stream_handle(stream), _ptr(trace)))
+        return trace[:n], trace[n:2 * n]
 
     def execute_host(self, host_ins, host_out, dev_ins, dev_out, stream=None):
         """End-to-end: H2D copy of host_ins into dev_ins, execute, D2H into host_out, synchronise."""
@@ -282,8 +304,13 @@ class Plan:
 _PLAN_CACHE: dict = {}
 
 
-def _cached_plan(pattern, shape, dtype, strategy, device):
-    key = (pattern, tuple(shape), dtype, strategy, str(device))
+def _cached_plan(pattern, shape, dtype, strategy, device, stream=None):
+    """One plan (and so one workspace) per (pattern, shape, dtype, strategy, device, STREAM): executes on
+    one stream are ordered, so they may share a workspace; executes on different streams get their own
+    (npp.h: concurrent executes need distinct workspaces)."""
+    with torch.cuda.device(device):
+        sh = _stream_handle(stream).value
+    key = (pattern, tuple(shape), dtype, strategy, str(device), sh)
     p = _PLAN_CACHE.get(key)
     if p is None:
         p = Plan(pattern, shape, dtype, strategy, device=device)
@@ -300,13 +327,13 @@ def _dtype_name(t: torch.Tensor) -> str:
 
 def sum_rows(m: torch.Tensor, strategy: str = "AUTO", out=None, stream=None) -> torch.Tensor:
     """m mapRows { r => r reduce + } (Fig 1) on a contiguous [R, C] CUDA tensor."""
-    p = _cached_plan("SUM_ROWS", m.shape, _dtype_name(m), strategy, m.device)
+    p = _cached_plan("SUM_ROWS", m.shape, _dtype_name(m), strategy, m.device, stream)
     return p.execute([m], out if out is not None else p.new_out(), stream)
 
 
 def sum_cols(m: torch.Tensor, strategy: str = "AUTO", out=None, stream=None) -> torch.Tensor:
     """m mapCols { c => c reduce + } (Fig 1)."""
-    p = _cached_plan("SUM_COLS", m.shape, _dtype_name(m), strategy, m.device)
+    p = _cached_plan("SUM_COLS", m.shape, _dtype_name(m), strategy, m.device, stream)
     return p.execute([m], out if out is not None else p.new_out(), stream)
 
 
@@ -314,24 +341,26 @@ def sum_rows_cols(m: torch.Tensor, out=None, stream=None):
     """Both Naive Bayes counts (§VI-E) in one pass over m: returns (row sums, column
     sums), views of one [R + C] output (SUM_ROWS_COLS, strategy AUTO)."""
     R = m.shape[0]
-    p = _cached_plan("SUM_ROWS_COLS", m.shape, _dtype_name(m), "AUTO", m.device)
+    p = _cached_plan("SUM_ROWS_COLS", m.shape, _dtype_name(m), "AUTO", m.device, stream)
     o = p.execute([m], out if out is not None else p.new_out(), stream)
     return o[:R], o[R:]
 
 
 def sum_weighted_rows(m, v, strategy="AUTO", out=None, stream=None):
-    p = _cached_plan("SUM_WEIGHTED_ROWS", m.shape, _dtype_name(m), strategy, m.device)
+    p = _cached_plan("SUM_WEIGHTED_ROWS", m.shape, _dtype_name(m), strategy, m.device, stream)
     return p.execute([m, v], out if out is not None else p.new_out(), stream)
 
 
 def sum_weighted_cols(m, v, strategy="AUTO", out=None, stream=None):
-    p = _cached_plan("SUM_WEIGHTED_COLS", m.shape, _dtype_name(m), strategy, m.device)
+    p = _cached_plan("SUM_WEIGHTED_COLS", m.shape, _dtype_name(m), strategy, m.device, stream)
     return p.execute([m, v], out if out is not None else p.new_out(), stream)
 
 
 def kmeans_assign(x, c, strategy="AUTO", out=None, stream=None):
     N, D = x.shape
-    p = _cached_plan("KMEANS_ASSIGN", (N, D, c.shape[0]), "f32", strategy, x.device)
+    if c.dim() != 2 or c.shape[1] != D:
+        raise ValueError("kmeans_assign: centroids must be [K, D] with the points' D")
+    p = _cached_plan("KMEANS_ASSIGN", (N, D, c.shape[0]), "f32", strategy, x.device, stream)
     return p.execute([x, c], out if out is not None else p.new_out(), stream)
 
 
@@ -339,7 +368,9 @@ def kmeans_update(x, a, K, out=None, stream=None):
     """Centroid update after an assignment (groupBy a + Reduce, Table I): [K, D+1] fp32 with
     row k = (Σ_{i: a_i = k} x_i, count_k). New centroids are U[:, :D] / U[:, D:] where the count > 0."""
     N, D = x.shape
-    p = _cached_plan("KMEANS_UPDATE", (N, D, int(K)), "f32", "AUTO", x.device)
+    if a.dtype != torch.int32 or a.numel() != N:
+        raise ValueError("kmeans_update: keys must be an int32 vector with one key per point")
+    p = _cached_plan("KMEANS_UPDATE", (N, D, int(K)), "f32", "AUTO", x.device, stream)
     return p.execute([x, a], out if out is not None else p.new_out(), stream)
 
 
@@ -347,18 +378,23 @@ def pagerank_step(rowptr, colidx, pr, outdeg, out=None, stream=None):
     """One PageRank step (Fig 5) over the CSR of in-neighbours: rowptr int64 [N+1], colidx
     int32 [E], pr f32 [N], outdeg int32 [N] -> (1-0.85)/N + 0.85 * Σ_{w in nbrs(n)} pr[w]/outdeg[w]."""
     N, E = pr.shape[0], colidx.shape[0]
-    p = _cached_plan("PAGERANK", (N, E), "f32", "AUTO", pr.device)
+    p = _cached_plan("PAGERANK", (N, E), "f32", "AUTO", pr.device, stream)
     return p.execute([rowptr, colidx, pr, outdeg], out if out is not None else p.new_out(), stream)
 
 
 def pagerank_shard(local_rowptr, local_colidx, pr, outdeg, lo, hi, out=None, stream=None):
     """Rows [lo, hi) of a PageRank step: the shard's CSR (rowptr rebased to 0, hi-lo+1 entries) against the
     whole graph's pr / outdeg (PAGERANK shape {rows, E, N})."""
-    p = _cached_plan("PAGERANK", (hi - lo, local_colidx.shape[0], pr.shape[0]), "f32", "AUTO", pr.device)
+    p = _cached_plan("PAGERANK", (hi - lo, local_colidx.shape[0], pr.shape[0]), "f32", "AUTO", pr.device, stream)
     return p.execute([local_rowptr, local_colidx, pr, outdeg], out if out is not None else p.new_out(), stream)
 
 
 def logreg_grad(x, y, w, B, strategy="AUTO", out=None, stream=None):
+    """g[b, j] = Σ_{i in batch b} x_ij (σ(x_i·w) − y_i) over B equal mini-batches of the rows of x."""
     n, C = x.shape
-    p = _cached_plan("LOGREG_GRAD", (B, n // B, C), "f32", strategy, x.device)
+    if B < 1 or n % B != 0:
+        raise ValueError(f"logreg_grad: {n} rows do not split into {B} equal mini-batches")
+    if y.numel() != n or w.numel() != C:
+        raise ValueError("logreg_grad: y needs one label per row and w one weight per column")
+    p = _cached_plan("LOGREG_GRAD", (B, n // B, C), "f32", strategy, x.device, stream)
     return p.execute([x, y, w], out if out is not None else p.new_out(), stream)

@@ -52,7 +52,7 @@ def test_struct_layout_matches_binding(tmp_path):
         size, offs = _c_layout(tmp_path, struct, names)
         assert ctypes.sizeof(cls) == size, struct
         assert [getattr(cls, n).offset for n in names] == offs, struct
-    assert npp.lib().npp_version() == 3
+    assert npp.lib().npp_version() == 4
     assert set(npp.EXPORTS) == set(declared_symbols())
 
 
