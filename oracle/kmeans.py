@@ -4,8 +4,11 @@ The nest (BASELINE.json config 4; the triply nested form of PAPER.md L606-610, r
 MSMBuilder clustering case study L1256-1271):
     points mapRows { x_i => (0 until K) argmin { k => (x_i zipWith c_k)((a,b) => (a-b)^2) reduce + } }
 i.e.  a[i] = min{ k : Σ_d (x[i,d] − c[k,d])² is minimal }   — ties go to the lowest k (G20).
-fp64: the difference of two fp32 values and its square are exact in fp64, so the literal evaluator's
-``math.fsum`` distance is the correctly rounded exact distance.
+The paper has no k-means and fixes no precision, so the decision is taken in fp64 as written (DESIGN.md
+reading G25): d(i,k) = Σ_{d=0}^{D-1} (x_id − c_kd)² evaluated left to right in IEEE fp64 — each
+difference, square and add rounded to nearest, no fused multiply-add — and a[i] is the lowest k whose
+d(i,k) is minimal. (This equals the exact-real argmin except when two exact distances lie within the
+fp64 rounding error of each other, ~D·2^-53 relative; tests pin that against exact rationals.)
 
 The centroid update that follows an assignment is Table I's groupBy (L292) followed
 by a Reduce per group:
@@ -20,6 +23,15 @@ import math
 import numpy as np
 
 
+def distance_literal(xi, ck) -> float:
+    """d = Σ_d (x_d − c_d)² left to right in fp64 (Python floats are IEEE doubles; every op rounds)."""
+    d = 0.0
+    for a, b in zip(xi, ck):
+        t = float(a) - float(b)
+        d = d + t * t
+    return d
+
+
 def assign_literal(x: np.ndarray, c: np.ndarray) -> list:
     """Pure-Python triple loop, outer Map over points, argmin over centroids, Reduce over dims."""
     xs, cs = x.tolist(), c.tolist()
@@ -27,7 +39,7 @@ def assign_literal(x: np.ndarray, c: np.ndarray) -> list:
     for xi in xs:
         best_k, best_d = -1, None
         for k, ck in enumerate(cs):
-            d = math.fsum((float(a) - float(b)) ** 2 for a, b in zip(xi, ck))
+            d = distance_literal(xi, ck)
             if best_d is None or d < best_d:       # strict: the first (lowest) k wins ties
                 best_k, best_d = k, d
         out.append(best_k)
@@ -35,12 +47,17 @@ def assign_literal(x: np.ndarray, c: np.ndarray) -> list:
 
 
 def distances(x: np.ndarray, c: np.ndarray, chunk: int = 4096) -> np.ndarray:
-    """d[i,k] = Σ_d (x[i,d] − c[k,d])² in fp64 (NumPy reduction as the library primitive)."""
+    """d[i,k] = Σ_d (x[i,d] − c[k,d])², the same fp64 operations in the same order as
+    distance_literal (one elementwise subtract, square and add per d, over all (i, k) at once)."""
     x64, c64 = x.astype(np.float64), c.astype(np.float64)
     out = np.empty((x.shape[0], c.shape[0]), dtype=np.float64)
     for s in range(0, x.shape[0], chunk):
-        diff = x64[s:s + chunk, None, :] - c64[None, :, :]
-        out[s:s + chunk] = np.add.reduce(diff * diff, axis=2)
+        xs = x64[s:s + chunk]
+        acc = np.zeros((xs.shape[0], c.shape[0]), dtype=np.float64)
+        for d in range(x.shape[1]):
+            t = xs[:, None, d] - c64[None, :, d]
+            acc += t * t
+        out[s:s + chunk] = acc
     return out
 
 

@@ -64,6 +64,57 @@ def test_random_data_vs_cdist():
     assert kmeans.assign_literal(x[:40], c) == a[:40].tolist()
 
 
+def test_vectorised_distances_bitwise_literal():
+    # the vectorised oracle performs the literal's fp64 operations in the literal's order (G25)
+    rng = np.random.default_rng(5)
+    for D, K in [(64, 32), (7, 5), (128, 3)]:
+        x = (rng.standard_normal((40, D)) * rng.choice([1e-3, 1.0, 1e3], size=(40, D))).astype(np.float32)
+        c = (rng.standard_normal((K, D)) * 4).astype(np.float32)
+        d = kmeans.distances(x, c)
+        for i in range(0, 40, 7):
+            for k in range(K):
+                assert d[i, k] == kmeans.distance_literal(x[i].tolist(), c[k].tolist())
+
+
+def test_fp64_decision_is_the_exact_argmin_away_from_ties():
+    # pin of reading G25 against exact rational arithmetic: |d64 - d| <= D * 2^-52 * d (each of the D
+    # squares and adds rounds once, differences of fp32 values are exact in fp64 at these magnitudes),
+    # and the fp64 argmin is the exact argmin whenever the exact margin exceeds twice that bound
+    from fractions import Fraction
+    rng = np.random.default_rng(6)
+    D, K = 16, 6
+    x = rng.uniform(-8, 8, (60, D)).astype(np.float32)
+    c = rng.uniform(-8, 8, (K, D)).astype(np.float32)
+    d64 = kmeans.distances(x, c)
+    a = kmeans.assign(x, c)
+    for i in range(60):
+        exact = [sum((Fraction(float(p)) - Fraction(float(q))) ** 2 for p, q in zip(x[i], c[k])) for k in range(K)]
+        for k in range(K):
+            assert abs(Fraction(d64[i, k]) - exact[k]) <= Fraction(D, 2 ** 52) * exact[k]
+        order = sorted(range(K), key=lambda k: (exact[k], k))
+        margin = exact[order[1]] - exact[order[0]]
+        if margin > Fraction(2 * D, 2 ** 52) * exact[order[1]]:
+            assert a[i] == order[0]
+
+
+def test_exact_midpoint_ties_go_to_lowest_index():
+    # dyadic coordinates: x = (c_a + c_b)/2 is exactly equidistant from c_a and c_b, and every fp64
+    # operation on these values is exact, so the tie is real and the lower index wins (G20)
+    rng = np.random.default_rng(7)
+    D, K = 64, 32
+    c = (rng.integers(-64, 64, (K, D)) / 4.0).astype(np.float32)
+    pairs = [(3, 17), (20, 5), (0, 31), (9, 8)]
+    x = np.stack([(c[p] + c[q]) / 2 for p, q in pairs]).astype(np.float32)
+    d = kmeans.distances(x, c)
+    for row, (p, q) in enumerate(pairs):
+        assert d[row, p] == d[row, q]
+    a = kmeans.assign(x, c)
+    for row, (p, q) in enumerate(pairs):
+        if d[row].min() == d[row, p]:
+            assert a[row] == min(p, q)
+    assert kmeans.assign_literal(x, c) == a.tolist()
+
+
 # ------------------------------------------------------------------ logistic-regression gradient
 
 def test_w_zero_closed_form():
