@@ -10,9 +10,9 @@
 #include <cstdio>
 #include <cstdlib>
 #include <mutex>
-#include <set>
+#include <map>
 #include <string>
-#include <tuple>
+#include <utility>
 
 #include "kernels.hpp"
 #include "select.hpp"
@@ -24,13 +24,15 @@ cudaError_t ensure_smem_attr(const void* func, int smem_bytes) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
+  // the attribute is an upper bound: keep the largest value set so far per (kernel, device), raise it
+  // when a launch needs more (a smaller later value would break launches that need the larger one)
   static std::mutex mu;
-  static std::set<std::tuple<const void*, int, int>> done;  // (kernel, device, bytes) already set
+  static std::map<std::pair<const void*, int>, int> cur;
   std::lock_guard<std::mutex> lock(mu);
-  const auto key = std::make_tuple(func, dev, smem_bytes);
-  if (done.count(key)) return cudaSuccess;
+  int& have = cur[std::make_pair(func, dev)];
+  if (have >= smem_bytes) return cudaSuccess;
   e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-  if (e == cudaSuccess) done.insert(key);
+  if (e == cudaSuccess) have = smem_bytes;
   return e;
 }
 }  // namespace npp

@@ -62,7 +62,10 @@ def test_staged_sum_schedule(npp, cuda_device, pattern, shape, dtype):
         assert np.array_equal(blk[:Ts], own[:Ts]), "static part differs from the record's ranges"
         for s0, s1 in pool_units(T, Ts, U):
             assert len(set(blk[s0:s1].tolist())) == 1, "a pool unit was split between blocks"
-        assert set(blk.tolist()) == set(range(G))
+        ranges = static_ranges(G, Ts, Ti, align)
+        # every block with static tiles takes part (blocks with an empty static range may find the
+        # pool already drained: small shapes with Ts < G)
+        assert {b for b, (s0, s1) in enumerate(ranges) if s1 > s0} <= set(blk.tolist())
         m_np = m.cpu().numpy()
         want = sums.sum_rows(m_np) if pattern == "SUM_ROWS" else sums.sum_cols(m_np)
         got = out.cpu().numpy()
