@@ -38,15 +38,15 @@ constexpr int kSets = NPP_KM_SETS;
 constexpr int kConsumerWarps = 8;                 // per set
 constexpr int kConsumers = kConsumerWarps * 32;   // per set
 constexpr int kThreads = kSets * kConsumers;      // no producer warp: see the refill below
-constexpr int kSmemHeader = 1024;
+constexpr int kSmemHeader = 128;
 constexpr int kMaxStageBytes = 64 * 1024;
 constexpr int kSmemLimit = 227 * 1024;
 constexpr int kConstFloats = 16384;  // DESIGN.md S8: 32·⌈K/32⌉·D ≤ 16384
 
 
-// centroids as pairs: km_pairs[(k/2)·D + d] = (c[k & ~1][d], c[k | 1][d]), padded rows zero. One
-// packed FFMA2 then advances the dot products of two centroids with one (broadcast) x element, so
-// each accumulator half ends as a whole dot product (no final add of even/odd halves).
+// centroids as pairs of −2c: km_pairs[(k/2)·D + d] = (−2c[k & ~1][d], −2c[k | 1][d]), padded rows zero
+// (the scaling by −2 is exact). One packed FFMA2 advances two centroids' chains with one (broadcast) x
+// element; a chain starts at ||c_k||², so each accumulator half ends as the score ||c_k||² − 2 x·c_k.
 __constant__ float2 km_pairs[kConstFloats / 2];
 __device__ float2 km_pack_buf[kConstFloats / 2];  // staging for the copy into the constant bank
 
@@ -55,14 +55,15 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int k2 = i / D, d = i - k2 * D;
     const int k = 2 * k2;
-    km_pack_buf[i] = make_float2(k < K ? c[k * D + d] : 0.f, k + 1 < K ? c[(k + 1) * D + d] : 0.f);
+    km_pack_buf[i] = make_float2(k < K ? -2.f * c[k * D + d] : 0.f, k + 1 < K ? -2.f * c[(k + 1) * D + d] : 0.f);
   }
 }
 
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
 __host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
-  return 1024 /* alignment pad */ + kSmemHeader + km_kpad(K) * 4 + kSets * 2 * 3 * int64_t(tp) * 8;
+  // alignment pad + barriers + ||c||² + exchange words [3 slots][4 groups][tp]
+  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kMaxStages) * 4 * tp * 8;
 }
 // ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
 __host__ __device__ inline int km_stages(int64_t K, int tp) {
@@ -83,38 +84,43 @@ __device__ __forceinline__ void ffma2(float2& acc, const float2 a, const float2 
 
 }  // namespace
 
+// 12-bit monotone codes of non-negative floats (the top 12 bits below the sign: 8 exponent + 4 mantissa
+// bits), rounded up or down, so a bound survives the packing into the exchange word (2^-4 relative)
+__device__ __forceinline__ unsigned code_up(float v) { return (__float_as_uint(v) + 0x7ffffu) >> 19; }
+__device__ __forceinline__ unsigned code_down(float v) { return (__float_as_uint(v) & 0x7fffffffu) >> 19; }
+__device__ __forceinline__ float decode12(unsigned c) { return __uint_as_float(c << 19); }
+
 // PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
 // groups; a tile is TP = PPT·256/G points.
 template <int PPT, int CPT>
 __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const KmeansArgs& a) {
   const CUtensorMap& map = *mapp;
   constexpr int G = 32 / CPT;
+  static_assert(G == 4, "the exchange word packs four centroid groups");
   constexpr int LP = kConsumers / G;  // threads (and point lanes) per centroid group
   constexpr int TP = PPT * LP;        // points per tile
   extern __shared__ __align__(1024) unsigned char smem[];
   const int nb = km_boxes(a.D);
   const int stage_bytes = nb * TP * 128;
   const int kStages = km_stages(a.K, TP);  // ring depth (2 or 3)
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
-  uint64_t* empty = full + kMaxStages;
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
-  unsigned char* ring = smem + pad + kSmemHeader;
+  unsigned char* ring = smem + pad;
   const int D = int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
-  float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp]
-  // minima of groups 1..G-1 handed to group 0: [set][2 (tile parity)][G-1 <= 3][TP]
-  float* xs_s = cn + Kp;
-  int* xs_k = reinterpret_cast<int*>(xs_s + kSets * 2 * 3 * TP);
+  float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp] ||c_k||², +inf padded
+  // per ring slot: each group's (best score, packed {k, margin code, norm code}) per point
+  uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kMaxStages][G][TP]
+  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kMaxStages * G * TP);
+  unsigned* released = reinterpret_cast<unsigned*>(full + kMaxStages);  // [kStages] warps done with the slot
 
-  // warp index broadcast from lane 0: ptxas then knows the producer/consumer split is warp-
-  // uniform and may use the uniform datapath (LDCU) for the centroid reads after it
+  // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
+  // uniform datapath (LDCU) for the centroid reads after it
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
   const long long bid = blockIdx.x;
   const long long T = (a.N + TP - 1) / TP;
   const long long P = a.per_block;
   const long long r0 = bid * P, r1 = (T < r0 + P) ? T : r0 + P;
 
-  unsigned* released = reinterpret_cast<unsigned*>(empty);  // [kStages] warps done with the slot
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       tma::mbar_init(full + i, 1);
@@ -122,7 +128,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     }
     tma::mbar_fence_init();
   }
-  // ||c_k||² (fp32 FMA chain over d); padded rows (zero) get +inf and are never selected
+  // ||c_k||² (fp32 FMA chain over d); padded rows get +inf and are never selected
   for (int k = threadIdx.x; k < Kp; k += kThreads) {
     float s = 0.f;
     if (k < K)
@@ -130,6 +136,15 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     cn[k] = k < K ? s : __int_as_float(0x7f800000);
   }
   __syncthreads();
+  // near-tie bound (DESIGN.md §5 k-means): every fp32 score s_k = fl(||c_k||² − 2 x·c_k) is within
+  // γ_{2D+2} (||x|| + ||c_k||)² of its exact value, and the fp64 distance as written (G25) within
+  // (D+3) 2^-53 (||x|| + ||c_k||)² of the exact distance; a point whose fp32 margin exceeds twice
+  // the sum is decided by its fp32 winner, every other point is recomputed in fp64
+  float cmax = 0.f;
+  for (int k = 0; k < K; ++k) cmax = fmaxf(cmax, cn[k]);
+  const float sqrt_cm = __fsqrt_ru(__fmul_ru(cmax, 1.0001f));  // cn carries γ_D relative error
+  const float g2d = float(2 * D + 2) * 5.9604645e-8f;                  // (2D+2) u, u = 2^-24
+  const float coef = 2.02f * (g2d / (1.f - g2d) + float(D + 3) * 1.1102230e-16f);
 
   const long long n_tiles = r1 - r0;
   auto issue = [&](long long t, int slot) {  // tile t of the block's range into slot t % kStages
@@ -147,7 +162,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     for (int t = 0; t < kStages && t < n_tiles; ++t) issue(t, t);
   }
 
-  // ------------------------------------------------------------------ consumers
   // centroid group; redux.sync lands in a uniform register, so ptxas treats g as warp-uniform and
   // keeps the centroid reads on the uniform datapath (LDCU)
   const int set = int(__reduce_min_sync(0xffffffffu, unsigned(warp / kConsumerWarps)));
@@ -157,24 +171,28 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // of 8, so every point of the thread has the key lt & 7
   const unsigned key = unsigned(lt & 7);
   const int nd4 = D / 4;
+  const int q0 = g * nd4 / G, q1 = (g + 1) * nd4 / G;  // the group's quarter of the dims for ||x||²
   // slot = t % kStages and round = t / kStages advance incrementally (no 64-bit division per tile)
   int slot = set % kStages;
   unsigned round = unsigned(set / kStages);
   for (long long t = set; t < n_tiles; t += kSets) {
     tma::mbar_wait_warp(full + slot, round & 1u);
-    const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
-    float bs[PPT];
+    const unsigned char* sbase = ring + slot * kMaxStageBytes;
+    const unsigned char* tile = sbase + lt * 128;
+    float bs[PPT], s2[PPT];
     int bk[PPT];
 #pragma unroll
-    for (int i = 0; i < PPT; ++i) bs[i] = __int_as_float(0x7f800000), bk[i] = 0x7fffffff;
+    for (int i = 0; i < PPT; ++i) bs[i] = s2[i] = __int_as_float(0x7f800000), bk[i] = 0;
     for (int kc = 0; kc < Kp; kc += 32) {
       const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
-      float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1
+      float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1; starts at (||c||², ||c'||²)
 #pragma unroll
-      for (int i = 0; i < PPT; ++i)
+      for (int p = 0; p < CPT / 2; ++p) {
+        const float2 nkp = *reinterpret_cast<const float2*>(cn + k0 + 2 * p);
 #pragma unroll
-        for (int p = 0; p < CPT / 2; ++p) acc[i][p] = make_float2(0.f, 0.f);
-      const float2* cq = km_pairs + (k0 >> 1) * D;
+        for (int i = 0; i < PPT; ++i) acc[i][p] = nkp;
+      }
+      const float2* cq = km_pairs + (k0 >> 1) * D;  // pairs of −2c: the chain ends at the score
 #pragma unroll 2
       for (int d4 = 0; d4 < nd4; ++d4) {
         const unsigned char* xb = tile + (d4 >> 3) * (TP * 128) + ((unsigned(d4 & 7) ^ key) << 4);
@@ -199,55 +217,105 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const int k = k0 + 2 * p + h;
-          const float nk = cn[k];
 #pragma unroll
           for (int i = 0; i < PPT; ++i) {
-            const float s = fmaf(-2.f, h ? acc[i][p].y : acc[i][p].x, nk);
-            if (s < bs[i]) bs[i] = s, bk[i] = k;
+            const float sc = h ? acc[i][p].y : acc[i][p].x;
+            s2[i] = fminf(s2[i], fmaxf(sc, bs[i]));  // the runner-up over every other k
+            if (sc < bs[i]) bs[i] = sc, bk[i] = k;
           }
         }
       }
     }
-    const long long base = (r0 + t) * TP;
-    if (G == 1) {
+    // the group's share of ||x||² and its exchange word per point: (best score, {k, margin, norm})
+    uint2* ex = xch + (slot * G + g) * TP;
 #pragma unroll
-      for (int i = 0; i < PPT; ++i) {
-        const long long gi = base + lt + LP * i;
-        if (gi < a.N) a.assign[gi] = bk[i];
+    for (int i = 0; i < PPT; ++i) {
+      float2 n2 = make_float2(0.f, 0.f);
+      for (int d4 = q0; d4 < q1; ++d4) {
+        const float4 v = *reinterpret_cast<const float4*>(tile + (d4 >> 3) * (TP * 128) + LP * 128 * i +
+                                                          ((unsigned(d4 & 7) ^ key) << 4));
+        ffma2(n2, make_float2(v.x, v.y), make_float2(v.x, v.y));
+        ffma2(n2, make_float2(v.z, v.w), make_float2(v.z, v.w));
       }
-    } else {  // groups 1.. hand their minima to group 0 (double-buffered by tile parity)
-      const int par = int(((t - set) / kSets) & 1);  // kSets is a compile-time constant
-      float* ss = xs_s + (set * 2 + par) * 3 * TP;
-      int* sk = xs_k + (set * 2 + par) * 3 * TP;
-      if (g > 0) {
-#pragma unroll
-        for (int i = 0; i < PPT; ++i) ss[(g - 1) * TP + lt + LP * i] = bs[i], sk[(g - 1) * TP + lt + LP * i] = bk[i];
-      }
-      asm volatile("bar.sync %0, %1;" ::"r"(1 + set), "n"(kConsumers) : "memory");  // this set only
-      if (g == 0) {
-#pragma unroll
-        for (int i = 0; i < PPT; ++i) {
-          float s = bs[i];
-          int k = bk[i];
-#pragma unroll
-          for (int h = 1; h < G; ++h) {
-            const float s2 = ss[(h - 1) * TP + lt + LP * i];
-            const int k2 = sk[(h - 1) * TP + lt + LP * i];
-            if (s2 < s || (s2 == s && k2 < k)) s = s2, k = k2;
-          }
-          const long long gi = base + lt + LP * i;
-          if (gi < a.N) a.assign[gi] = k;
-        }
-      }
+      const float margin = __fsub_rd(s2[i], bs[i]);
+      ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
+                                                               code_up(__fadd_ru(n2.x, n2.y)));
     }
-    // release the slot: the last of the 8 warps to finish with it refills it with tile t+kStages
-    // (nobody waits on an "empty" barrier). Every x value the warp read is already consumed, the
-    // fences order those reads and the counter before the TMA (async proxy) overwrites the slot.
+    // release the slot: the last of the 8 warps to finish with it merges the four groups' words, writes
+    // the tile's assignments and refills the slot with tile t+kStages (nobody waits on a barrier).
     __syncwarp();
+    unsigned last = 0;
     if (lane == 0) {
       __threadfence_block();
-      if (atomicAdd(released + slot, 1u) == kConsumerWarps - 1) {
-        __threadfence_block();
+      last = atomicAdd(released + slot, 1u) == kConsumerWarps - 1;
+    }
+    if (__shfl_sync(0xffffffffu, last, 0)) {
+      __threadfence_block();
+      const uint2* exs = xch + slot * G * TP;
+      const long long base = (r0 + t) * TP;
+      unsigned need64 = 0;  // bit j: point lane + 32 j is a near tie
+#pragma unroll 2
+      for (int j = 0; j < TP / 32; ++j) {
+        const int pt = lane + 32 * j;
+        uint2 w[G];
+#pragma unroll
+        for (int h = 0; h < G; ++h) w[h] = exs[h * TP + pt];
+        int hw = 0;
+#pragma unroll
+        for (int h = 1; h < G; ++h) {  // lowest (score, k): groups interleave centroids, so k decides ties
+          const float sh = __uint_as_float(w[h].x), sw = __uint_as_float(w[hw].x);
+          if (sh < sw || (sh == sw && (w[h].y >> 24) < (w[hw].y >> 24))) hw = h;
+        }
+        const float sb = __uint_as_float(w[hw].x);
+        float margin = decode12((w[hw].y >> 12) & 0xfffu);
+        float xn = 0.f;
+#pragma unroll
+        for (int h = 0; h < G; ++h) {
+          if (h != hw) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
+          xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
+        }
+        const float r = __fadd_ru(__fsqrt_ru(xn), sqrt_cm);
+        const float thr = __fmul_ru(coef, __fmul_ru(r, r));
+        const long long gi = base + pt;
+        if (margin > thr) {
+          if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
+        } else if (gi < a.N) {
+          need64 |= 1u << j;
+        }
+      }
+      // near ties: the fp64 distance as written (G25), one warp per point, lane = centroid
+      for (int j = 0; j < TP / 32; ++j) {
+        unsigned m = __ballot_sync(0xffffffffu, (need64 >> j) & 1u);
+        while (m) {
+          const int src = __ffs(m) - 1;
+          m &= m - 1;
+          const int pt = src + 32 * j;
+          const unsigned char* xr = sbase + pt * 128;
+          const unsigned kx = unsigned(pt & 7);
+          double best = __longlong_as_double(0x7ff0000000000000ll);
+          int bestk = 0x7fffffff;
+          for (int k = lane; k < K; k += 32) {
+            const float* ck = a.c + (long long)k * D;
+            double dist = 0.0;
+            for (int d = 0; d < D; ++d) {
+              const float xd = *reinterpret_cast<const float*>(xr + (d >> 5) * (TP * 128) +
+                                                               ((unsigned((d >> 2) & 7) ^ kx) << 4) + (d & 3) * 4);
+              const double df = __dsub_rn(double(xd), double(__ldg(ck + d)));
+              dist = __dadd_rn(dist, __dmul_rn(df, df));
+            }
+            if (dist < best) best = dist, bestk = k;  // k increases per lane: first minimum
+          }
+#pragma unroll
+          for (int off = 16; off >= 1; off >>= 1) {
+            const double ob = __shfl_xor_sync(0xffffffffu, best, off);
+            const int ok = __shfl_xor_sync(0xffffffffu, bestk, off);
+            if (ob < best || (ob == best && ok < bestk)) best = ob, bestk = ok;
+          }
+          if (lane == 0) a.assign[base + pt] = bestk;
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {
         released[slot] = 0;
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         if (t + kStages < n_tiles) issue(t + kStages, slot);

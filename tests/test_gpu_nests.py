@@ -2,10 +2,10 @@
 through the C-ABI against the fp64 oracle.
 
 Tolerances:
-  logreg  |g - g64| <= 1e-5 * Σ_i|x_ij e_i| + 2^-20 * Σ_i|x_ij|   (fp32 terms; fp32 residual e_i)
-  kmeans  integer-valued data: bit-exact (every fp32 distance is exact, ties -> lowest k);
-          random data: d64(x_i, c_a) - min_k d64(x_i, c_k) <= 2^-16 (|x_i|² + |c_a|² + |c_o|²)
-          (the fp32 expansion ||c||² - 2x·c can only swap near-ties within that bound)
+  logreg  |g - g64| <= 1e-5 * Σ_i|x_ij e_i|   (z and e_i in fp64, fp32 products and 4-term sums)
+  kmeans  index-exact on every input: the decision is the fp64 distance as written (DESIGN.md G25);
+          the kernel's fp32 screen settles only points whose margin beats its rigorous error bound
+          and recomputes the rest in fp64 with the oracle's operations
 """
 import numpy as np
 import pytest
@@ -28,9 +28,9 @@ def npp(cuda_device):
 def _check_logreg(g, x, y, w, B):
     xn, yn, wn = x.cpu().numpy(), y.cpu().numpy(), w.cpu().numpy()
     want = olr.grad(xn, yn, wn, B)
-    s_rel, s_abs = olr.grad_scales(xn, yn, wn, B)
+    s_rel, _ = olr.grad_scales(xn, yn, wn, B)
     err = np.abs(g.cpu().numpy().astype(np.float64) - want)
-    tol = 1e-5 * s_rel + 2.0 ** -20 * s_abs
+    tol = 1e-5 * s_rel
     bad = np.argwhere(err > tol)
     assert bad.size == 0, (bad[:4], err[tuple(bad[0])], tol[tuple(bad[0])])
 
@@ -61,8 +61,9 @@ def test_logreg_y_zero_and_w_zero(npp, cuda_device):
     assert torch.allclose(g0.double(), want, rtol=1e-6, atol=0)
 
 
-def test_logreg_full_size_sampled(npp, cuda_device):
-    # BASELINE.json config 5: [16M, 256] fp32 (16 GiB), B = 4096 batches of 4096 rows
+def test_logreg_full_size(npp, cuda_device):
+    # BASELINE.json config 5: [16M, 256] fp32 (16 GiB), B = 4096 batches of 4096 rows; every batch's
+    # gradient is compared with the oracle (64 batches at a time)
     B, Rb, C = 4096, 4096, 256
     free, _ = torch.cuda.mem_get_info()
     if free < 24 * (1 << 30):
@@ -71,23 +72,11 @@ def test_logreg_full_size_sampled(npp, cuda_device):
     p = npp.Plan("LOGREG_GRAD", (B, Rb, C), "f32", "AUTO")
     g = p.execute([x, y, w], p.new_out())
     torch.cuda.synchronize()
-    for b in (0, 1, 1777, 4094, 4095):
-        rows = slice(b * Rb, (b + 1) * Rb)
-        _check_logreg(g[b:b + 1], x[rows], y[rows], w, 1)
+    nb = 64
+    for b0 in range(0, B, nb):
+        rows = slice(b0 * Rb, (b0 + nb) * Rb)
+        _check_logreg(g[b0:b0 + nb], x[rows], y[rows], w, nb)
     del x
-
-
-def _check_kmeans_valid(a, x, c):
-    xn, cn = x.cpu().numpy(), c.cpu().numpy()
-    d = okm.distances(xn, cn)
-    best = d.min(axis=1)
-    a = a.cpu().numpy().astype(np.int64)
-    chosen = d[np.arange(len(a)), a]
-    o = okm.assign(xn, cn).astype(np.int64)
-    scale = (xn.astype(np.float64) ** 2).sum(1) + (cn.astype(np.float64) ** 2).sum(1)[a] + \
-        (cn.astype(np.float64) ** 2).sum(1)[o]
-    assert np.all(chosen - best <= 2.0 ** -16 * scale)
-    return float(np.mean(a == o))
 
 
 @pytest.mark.parametrize("N,D,K", [(10000, 64, 32), (1000, 12, 5), (4099, 128, 96), (127, 4, 1),
@@ -101,27 +90,65 @@ def test_kmeans_integer_data_exact(npp, cuda_device, N, D, K):
     assert a.cpu().numpy().tolist() == okm.assign(x.cpu().numpy(), c.cpu().numpy()).tolist()
 
 
-@pytest.mark.parametrize("N,D,K", [(50000, 64, 32), (3000, 16, 7)])
-def test_kmeans_random_data(npp, cuda_device, N, D, K):
+@pytest.mark.parametrize("N,D,K", [(50000, 64, 32), (3000, 16, 7), (20000, 128, 200), (7777, 4, 3)])
+def test_kmeans_random_data_exact(npp, cuda_device, N, D, K):
     x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
     p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
     a = p.execute([x, c], p.new_out())
     torch.cuda.synchronize()
-    agree = _check_kmeans_valid(a, x, c)
-    assert agree > 0.999
+    assert np.array_equal(a.cpu().numpy(), okm.assign(x.cpu().numpy(), c.cpu().numpy()))
 
 
-def test_kmeans_full_size_sampled(npp, cuda_device):
-    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids
+def test_kmeans_unclustered_data_exact(npp, cuda_device):
+    # points uniform in the centroids' box (no cluster structure): many small margins, so the fp64
+    # recheck of near ties runs often
+    N, D, K = 60000, 64, 32
+    _, c = gen.kmeans_inputs(16, D, K, device=cuda_device)
+    x = gen.uniform_f32(31, (N, D), lo=-8.0, scale=16.0, device=cuda_device)
+    a = npp.kmeans_assign(x, c)
+    torch.cuda.synchronize()
+    assert np.array_equal(a.cpu().numpy(), okm.assign(x.cpu().numpy(), c.cpu().numpy()))
+
+
+def test_kmeans_exact_and_near_ties(npp, cuda_device):
+    # dyadic midpoints of centroid pairs are exactly equidistant (the lower index wins), and points
+    # nudged by one ulp towards either side of a midpoint are decided by the fp64 distances
+    N, D, K = 4096, 64, 32
+    g = torch.Generator().manual_seed(9)
+    c = (torch.randint(-64, 64, (K, D), generator=g).float() / 4.0)
+    pa = torch.randint(0, K, (N,), generator=g)
+    pb = (pa + torch.randint(1, K, (N,), generator=g)) % K
+    x = (c[pa] + c[pb]) / 2
+    nudge = torch.randint(0, 3, (N, 1), generator=g).float() - 1.0  # one ulp towards c_b, none, towards c_a
+    direction = torch.sign(c[pb] - c[pa]) * nudge
+    inf = torch.full_like(x, float("inf"))
+    x = torch.nextafter(x, torch.where(direction > 0, inf, torch.where(direction < 0, -inf, x)))
+    x, c = x.contiguous().to(cuda_device), c.contiguous().to(cuda_device)
+    a = npp.kmeans_assign(x, c)
+    torch.cuda.synchronize()
+    want = okm.assign(x.cpu().numpy(), c.cpu().numpy())
+    assert np.array_equal(a.cpu().numpy(), want)
+    # the exact ties really occur and go to the lower index
+    ties = (nudge.squeeze(1) == 0).numpy()
+    d = okm.distances(x.cpu().numpy(), c.cpu().numpy())
+    exact_tie = ties & (d[np.arange(N), pa.numpy()] == d.min(1))
+    assert exact_tie.sum() > 100
+    assert np.all(want[exact_tie] == np.minimum(pa.numpy(), pb.numpy())[exact_tie])
+
+
+def test_kmeans_full_size_exact(npp, cuda_device):
+    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids, every assignment checked
     N, D, K = 1 << 22, 64, 32
     x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
     p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
     a = p.execute([x, c], p.new_out())
     torch.cuda.synchronize()
-    idx = torch.cat([torch.arange(0, 4096), torch.arange(N - 4096, N),
-                     torch.randint(0, N, (12000,), generator=torch.Generator().manual_seed(3))]).to(cuda_device)
-    agree = _check_kmeans_valid(a.index_select(0, idx), x.index_select(0, idx), c)
-    assert agree > 0.999
+    a = a.cpu().numpy()
+    cn = c.cpu().numpy()
+    step = 1 << 19
+    for s0 in range(0, N, step):
+        want = okm.assign(x[s0:s0 + step].cpu().numpy(), cn)
+        assert np.array_equal(a[s0:s0 + step], want), s0
 
 
 def test_kmeans_two_streams_distinct_centroids(npp, cuda_device):
