@@ -57,7 +57,7 @@ class ClockSampler:
                0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
                0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
 
-    def __init__(self, device_index: int, period_s: float = 0.0005):
+    def __init__(self, device_index: int, period_s: float = 0.0001):
         self.period = period_s
         self.samples, self.reasons = [], 0
         self.ok = False
@@ -157,11 +157,15 @@ def build_sumcols_1m4k(npp, gen, torch, rank, world, strategy, device):
 
 
 def build_kmeans(npp, gen, torch, rank, world, strategy, device):
-    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids; points sharded over ranks (weak)
-    N, D, K = 1 << 22, 64, 32
-    x, c = gen.kmeans_inputs(N, D, K, row_offset=rank * N, device=device)
+    # BASELINE.json config 4: 4M points x 64 dims x 32 centroids; the points sharded over ranks (strong)
+    Ntot, D, K = 1 << 22, 64, 32
+    from paper_conf_micro_leebsro14_b200.dist import shard_range
+    lo, hi = shard_range(Ntot, world, rank)
+    N = hi - lo
+    x, c = gen.kmeans_inputs(N, D, K, row_offset=lo, device=device)
     plan = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", strategy, device=device)
-    item = Item("kmeans_assign[4M,64,32]", plan, [x, c], plan.new_out(), N * D * 4 + K * D * 4 + N * 4)
+    item = Item("kmeans_assign[4M,64,32]" if world == 1 else f"kmeans_assign[{N},64,32]", plan, [x, c],
+                plan.new_out(), N * D * 4 + K * D * 4 + N * 4)
     item.flops = 2 * N * K * D  # the x·c FMAs of the expanded distance
     return [item], [], "k-means assignment 4M x 64 x 32"
 
@@ -230,7 +234,7 @@ def build_rowscols(npp, gen, torch, rank, world, strategy, device):
 
 
 # per-GPU work fixed as N grows ("weak": paper shards, k-means points) or total work fixed ("strong")
-SCALING = {"paper": "weak", "kmeans": "weak", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak",
+SCALING = {"paper": "weak", "kmeans": "strong", "sumcols_1m4k": "strong", "logreg": "strong", "rowscols": "weak",
            "kmeans_update": "weak", "pagerank": "strong"}
 WORKLOADS = {"paper": build_paper, "sumcols_1m4k": build_sumcols_1m4k, "kmeans": build_kmeans,
              "logreg": build_logreg, "rowscols": build_rowscols, "kmeans_update": build_kmeans_update,
@@ -304,7 +308,7 @@ def run_reference(args):
             "higher_is_better": True, "scaling": SCALING[wl], "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": config_for(args, "oracle (NumPy fp64) on host cores"),
             "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": desc},
+                             "sample": desc, "cpu_model": _cpu_model(), "cpu_count": os.cpu_count()},
             "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -329,55 +333,226 @@ def config_for(args, extra):
 
 # ------------------------------------------------------------------------- CPU baseline (oracle, bounded)
 
-def cpu_baseline(items, budget_s=12.0):
-    """The oracle as it stands, on the host's cores, over a bounded sample of the same workload."""
-    import numpy as np
+def _oracle_call(name, arrs, k=0):
     from oracle import kmeans as okm
     from oracle import logreg as olr
     from oracle import pagerank as opr
     from oracle import sums
-    done_bytes, t_total, n = 0, 0.0, 0
+    if name.startswith("pagerank"):
+        opr.step(*arrs)
+    elif name.startswith("kmeans_update"):
+        okm.update(arrs[0], arrs[1], k)
+    elif name.startswith("kmeans"):
+        okm.assign(*arrs)
+    elif name.startswith("logreg"):
+        olr.grad(arrs[0], arrs[1], arrs[2], arrs[0].shape[0] // 4096)
+    elif name.startswith("sum_rows_cols"):
+        sums.sum_rows_cols(arrs[0])
+    elif name.startswith("sum_rows"):
+        sums.sum_rows(arrs[0])
+    else:
+        sums.sum_cols(arrs[0])
+
+
+def _pool_worker(job):
+    """One process of the all-core CPU baseline: run the oracle on its slice of the sample."""
+    import numpy as np  # noqa: F401
+    name, arrs, k, reps = job
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        _oracle_call(name, arrs, k)
+    return time.perf_counter() - t0
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def cpu_baseline(items, budget_s=10.0):
+    """The oracle as it stands (NumPy fp64) on a bounded sample of the same workload, timed on one
+    core and as a process pool over all cores, plus the literal (pure-Python) oracle
+    on [1K,1K]."""
+    import multiprocessing as mp
+
+    import numpy as np
+    from oracle import sums
     samples = []
+    k = 0
     for it in items:
         if it.name.startswith("pagerank"):  # the whole graph (the oracle is O(E) NumPy)
             samples.append((it.name, [x.cpu().numpy() for x in it.ins]))
         elif it.name.startswith("kmeans_update"):  # first 1M points
+            k = it.plan.shape[2]
             samples.append((it.name, [it.ins[0][: 1 << 20].cpu().numpy(), it.ins[1][: 1 << 20].cpu().numpy()]))
-        elif it.name.startswith("kmeans"):  # first 256K points (the oracle is O(N K D) in fp64)
-            samples.append((it.name, [it.ins[0][: 1 << 18].cpu().numpy(), it.ins[1].cpu().numpy()]))
-        elif it.name.startswith("logreg"):  # first 64 batches
-            Rb = it.plan.shape[1]
-            rows = 64 * Rb
+        elif it.name.startswith("kmeans"):  # first 128K points (the oracle is O(N K D) in fp64)
+            samples.append((it.name, [it.ins[0][: 1 << 17].cpu().numpy(), it.ins[1].cpu().numpy()]))
+        elif it.name.startswith("logreg"):  # first 16 batches
+            rows = 16 * it.plan.shape[1]
             samples.append((it.name, [it.ins[0][:rows].cpu().numpy(), it.ins[1][:rows].cpu().numpy(),
                                       it.ins[2].cpu().numpy()]))
-        else:
-            samples.append((it.name, [it.ins[0].cpu().numpy()]))
-
-    def run(name, arrs):
-        if name.startswith("pagerank"):
-            opr.step(*arrs)
-        elif name.startswith("kmeans_update"):
-            okm.update(arrs[0], arrs[1], it_k)
-        elif name.startswith("kmeans"):
-            okm.assign(*arrs)
-        elif name.startswith("logreg"):
-            olr.grad(arrs[0], arrs[1], arrs[2], 64)
-        elif name.startswith("sum_rows_cols"):
-            sums.sum_rows_cols(arrs[0])
-        else:
-            (sums.sum_rows if name.startswith("sum_rows") else sums.sum_cols)(arrs[0])
-    it_k = items[0].plan.shape[2] if items and items[0].plan.pattern == "KMEANS_UPDATE" else 0
-    t_end = time.perf_counter() + budget_s
+        else:  # the first 16 MB of each matrix
+            m = it.ins[0]
+            rows = max(1, min(m.shape[0], (1 << 22) // m.shape[1]))
+            samples.append((it.name, [m[:rows].cpu().numpy()]))
+    sample_bytes = sum(x.nbytes for _, arrs in samples for x in arrs)
+    # one core: passes over the sample until the budget is spent
+    t_total, n_pass = 0.0, 0
+    t_end = time.perf_counter() + budget_s / 2
     while time.perf_counter() < t_end:
         for name, arrs in samples:
             t0 = time.perf_counter()
-            run(name, arrs)
+            _oracle_call(name, arrs, k)
             t_total += time.perf_counter() - t0
-            done_bytes += sum(x.nbytes for x in arrs)
-            n += 1
-    return {"value": round(done_bytes / t_total / 1e9, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} oracle calls over the step's inputs ({len(samples)} per pass; k-means: first 256K "
-                      f"points, logreg: first 64 batches), {t_total:.1f} s of single-threaded NumPy fp64"}
+        n_pass += 1
+    one_core = sample_bytes * n_pass / t_total / 1e9
+    # all cores: one process per core, each running the oracle over the sample (independent work)
+    try:
+        cores = len(os.sched_getaffinity(0))  # the cores this process may run on (os.cpu_count() counts all)
+    except AttributeError:
+        cores = os.cpu_count() or 1
+    reps = max(1, n_pass // 2)
+    jobs = [(name, arrs, k, reps) for name, arrs in samples for _ in range(cores)]
+    try:
+        ctx = mp.get_context("fork")
+        t0 = time.perf_counter()
+        with ctx.Pool(cores) as pool:
+            pool.map(_pool_worker, jobs, chunksize=1)
+        wall = time.perf_counter() - t0
+        all_core = sample_bytes * reps * cores / wall / 1e9
+    except Exception as e:  # noqa: BLE001
+        all_core, wall = None, str(e)
+    # the literal oracle (pure-Python loops) on [1K,1K] fp32
+    m = np.random.default_rng(1).random((1024, 1024), dtype=np.float32)
+    t0 = time.perf_counter()
+    sums.sum_rows_literal(m)
+    sums.sum_cols_literal(m)
+    literal_s = time.perf_counter() - t0
+    return {"value": round(all_core if all_core else one_core, 3), "unit": "GB/s",
+            "cores": cores if all_core else 1, "kind": "oracle",
+            "one_core_GBps": round(one_core, 3), "all_core_GBps": round(all_core, 3) if all_core else None,
+            "cpu_model": _cpu_model(), "cpu_count": os.cpu_count(),
+            "literal_1k_rows_cols_s": round(literal_s, 3),
+            "sample": f"{len(samples)} oracle calls per pass over the first 16 MB of each matrix (k-means: "
+                      f"first 128K points, logreg: first 16 batches); one core: {n_pass} passes "
+                      f"({t_total:.1f} s); all cores: {cores} processes x {reps} passes "
+                      f"({wall if isinstance(wall, str) else round(wall, 1)} s); NumPy fp64"}
+
+
+# ------------------------------------------------------------------------- timing plumbing
+
+def self_launch(args) -> int:
+    """`python bench.py --gpus N` outside torchrun: re-run this command as N ranks (one per GPU)."""
+    import socket
+    import subprocess
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def capture_step(torch, step, stream, world):
+    """The step as a CUDA graph (kernels and, at N > 1, the NCCL collectives): the timed region replays
+    it, so every N times the same way. Returns (replay, how)."""
+    with torch.cuda.stream(stream):
+        step()  # warm: lazy per-kernel setup, NCCL communicator, tensor maps
+    torch.cuda.synchronize()
+    try:
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(stream):
+            with torch.cuda.graph(g, stream=stream):
+                step()
+        torch.cuda.synchronize()
+        return g.replay, "CUDA graph" + (" (kernels + NCCL)" if world > 1 else "")
+    except Exception as e:  # noqa: BLE001  (a capture failure must not lose the measurement)
+        torch.cuda.synchronize()
+        return step, f"eager launches (graph capture failed: {type(e).__name__})"
+
+
+def timed(torch, dist, run_step, stream, steps, world, local):
+    """Barrier + sync, CUDA events on `stream` around `steps` replays, clocks sampled live; the max over
+    ranks. Returns (ms_total_max, per_rank_ms, clocks)."""
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(local)
+    with sampler:
+        with torch.cuda.stream(stream):
+            t0.record(stream)
+            for _ in range(steps):
+                run_step()
+            t1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = t0.elapsed_time(t1)
+    per_rank = [ms]
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=torch.device("cuda", local))
+        parts = [torch.zeros_like(t) for _ in range(world)]
+        dist.all_gather(parts, t)
+        per_rank = [float(x.item()) for x in parts]
+    return max(per_rank), per_rank, sampler.summary()
+
+
+def kernel_us(torch, item, other, stream, reps=8, overlap=False, pdl=False):
+    """Average duration of one launch of item's plan: a graph of 2*reps launches alternating item's
+    input with `other`'s (same byte size) so no launch finds its input in L2. Default: plain launches
+    (NPP_EXEC_NO_PDL: each kernel starts after the previous one completed — the isolated duration the
+    roofline uses); pdl=True: programmatic dependent launches (prologue overlapped, reads still after the
+    previous kernel); overlap=True: NPP_EXEC_OVERLAP (reads overlap the previous kernel's drain)."""
+    alt = None
+    if other is not None and other.ins[0].numel() == item.ins[0].numel() and other.ins[0].dtype == item.ins[0].dtype:
+        alt = other.ins[0].view(item.ins[0].shape)
+    firsts = [item.ins[0], alt] if alt is not None and alt.data_ptr() != item.ins[0].data_ptr() else [item.ins[0]]
+    inputs = [[f] + list(item.ins[1:]) for f in firsts]
+    use_pdl = pdl or overlap
+    with torch.cuda.stream(stream):
+        for x in inputs:
+            item.plan.execute(x, item.out, stream=stream, pdl=use_pdl)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(stream):
+        with torch.cuda.graph(g, stream=stream):
+            for r in range(2 * reps):
+                item.plan.execute(inputs[r % len(inputs)], item.out, stream=stream, overlap=overlap, pdl=use_pdl)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        g.replay()
+        a.record(stream)
+        g.replay()
+        b.record(stream)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) * 1e3 / (2 * reps)
+
+
+def make_step(torch, dist, items, reduce_bufs, stream, world, overlap):
+    gathers = [it for it in items if getattr(it, "gather", None)]
+
+    def step():
+        for it in items:
+            it.run(stream, overlap)
+        for b in reduce_bufs:  # the cross-device Split(P) of a reduced level: one NCCL all-reduce
+            with torch.cuda.stream(stream):
+                dist.all_reduce(b)
+        for it in gathers:  # PageRank shards: the next vector on every rank (uneven shards padded)
+            with torch.cuda.stream(stream):
+                n = it.out.numel()
+                mx = -(-it.gather[1] // world)
+                buf = torch.zeros(mx, dtype=it.out.dtype, device=it.out.device)
+                buf[:n] = it.out
+                parts = [torch.empty(mx, dtype=it.out.dtype, device=it.out.device) for _ in range(world)]
+                dist.all_gather(parts, buf)
+    return step
 
 
 # ------------------------------------------------------------------------- main arm
@@ -393,12 +568,15 @@ def main():
     ap.add_argument("--no-mappings", action="store_true", help="skip the baseline-mapping table")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg")
+    ap.add_argument("--no-per-config", action="store_true", help="skip the per_config lines (configs 3-5)")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     ap.add_argument("--no-overlap", action="store_true",
                     help="serialise the step's launches (no NPP_EXEC_OVERLAP programmatic dependent launch)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return self_launch(args)
 
     import torch
     import torch.distributed as dist
@@ -406,116 +584,85 @@ def main():
     from synth import gen
 
     world, rank, local = dist_env()
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
     torch.cuda.set_device(local)
     device = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=device)
     items, reduce_bufs, _ = WORKLOADS[args.workload](npp, gen, torch, rank, world, args.strategy, device)
     stream = torch.cuda.Stream(device=device)  # all timed work is enqueued on this stream
-    use_graph = world == 1 and not args.eager
 
     # the step's inputs are resident before it starts, so each launch may overlap the previous one's
     # drain (npp_execute_ex NPP_EXEC_OVERLAP); outputs still wait for the previous kernel
     overlap = not args.no_overlap
-
-    gathers = [(it, torch.empty(it.gather[1], dtype=it.out.dtype, device=device)) for it in items
-               if getattr(it, "gather", None)]
-
-    def step():
-        for it in items:
-            it.run(stream, overlap)
-        for b in reduce_bufs:
-            with torch.cuda.stream(stream):
-                dist.all_reduce(b)
-        for it, full in gathers:  # PageRank shards: the next vector on every rank (uneven shards padded)
-            with torch.cuda.stream(stream):
-                n = it.out.numel()
-                mx = -(-it.gather[1] // world)
-                buf = torch.zeros(mx, dtype=it.out.dtype, device=device)
-                buf[:n] = it.out
-                parts = [torch.empty(mx, dtype=it.out.dtype, device=device) for _ in range(world)]
-                dist.all_gather(parts, buf)
-
-    # one step = the six launches; at N=1 it is captured once into a CUDA graph and replayed, so the
-    # timed region holds the kernels back to back without host launch gaps (streams and graphs are
-    # the execution model here; at N>1 the NCCL all-reduce runs eagerly between the launches)
-    graph = None
-    if use_graph:
-        step()  # warm the lazy per-kernel setup outside the capture
-        torch.cuda.synchronize()
-        graph = torch.cuda.CUDAGraph()
+    step = make_step(torch, dist, items, reduce_bufs, stream, world, overlap)
+    if args.eager:
         with torch.cuda.stream(stream):
-            with torch.cuda.graph(graph, stream=stream):
-                step()
-    run_step = graph.replay if graph is not None else step
-
+            step()
+        run_step, how = step, "eager launches"
+    else:
+        run_step, how = capture_step(torch, step, stream, world)
     with torch.cuda.stream(stream):
         for _ in range(max(3, args.warmup)):
             run_step()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    sampler = ClockSampler(local)
-    with sampler:
-        with torch.cuda.stream(stream):
-            torch.cuda.synchronize()
-            t_start.record(stream)
-            for _ in range(args.steps):
-                run_step()
-            t_end.record(stream)
-        torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    ms_total = t_start.elapsed_time(t_end)
-    if world > 1:
-        t = torch.tensor([ms_total], dtype=torch.float64, device=device)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total = float(t.item())
+    ms_total, per_rank_ms, clocks = timed(torch, dist, run_step, stream, args.steps, world, local)
     ms_step = ms_total / args.steps
     step_bytes = sum(it.bytes for it in items)
     value = step_bytes * world / (ms_step * 1e-3) / 1e9
 
     # per-kernel durations: each launch replayed back to back from a graph, alternating its input with
     # another equal-size buffer of the step so that every launch reads cold HBM
-    per_kernel_us = [kernel_us(torch, it, items[(i + 1) % len(items)], stream) for i, it in enumerate(items)]
-    per_kernel_ov = [kernel_us(torch, it, items[(i + 1) % len(items)], stream, overlap=True)
-                     for i, it in enumerate(items)]
+    nxt = [items[(i + 1) % len(items)] if len(items) > 1 else None for i in range(len(items))]
+    per_kernel_us = [kernel_us(torch, it, nxt[i], stream) for i, it in enumerate(items)]
+    per_kernel_pdl = [kernel_us(torch, it, nxt[i], stream, pdl=True) for i, it in enumerate(items)]
+    per_kernel_ov = [kernel_us(torch, it, nxt[i], stream, overlap=True) for i, it in enumerate(items)]
     peak, peak_src = measured_peaks()
     dom = max(range(len(items)), key=lambda i: per_kernel_us[i])
-    dom_gbs = items[dom].bytes / (per_kernel_us[dom] * 1e-6) / 1e9
-    traffic = ncu_traffic().get(items[dom].name)
-    flops = getattr(items[dom], "flops", None)
-    wavefronts = getattr(items[dom], "wavefronts", None)
-    per_shape = {it.name: {"GB/s": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9, 1),
-                           "frac_of_measured": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / peak, 4),
-                           "frac_of_8TBs": round(it.bytes / (per_kernel_us[i] * 1e-6) / 1e9 / 8000.0, 4),
-                           "us": round(per_kernel_us[i], 2),
-                           "us_overlapped": round(per_kernel_ov[i], 2),
-                           "GB/s_overlapped": round(it.bytes / (per_kernel_ov[i] * 1e-6) / 1e9, 1),
-                           "mapping": mapping_brief(it.plan.mapping)}
-                 for i, it in enumerate(items)}
+    traffic_db = ncu_traffic()
+
+    def gbps(it, us):
+        return it.bytes / (us * 1e-6) / 1e9
+    per_shape = {}
+    for i, it in enumerate(items):
+        ent = {"GB/s": round(gbps(it, per_kernel_us[i]), 1), "us": round(per_kernel_us[i], 2),
+               "frac_of_measured": round(gbps(it, per_kernel_us[i]) / peak, 4),
+               "frac_of_8TBs": round(gbps(it, per_kernel_us[i]) / 8000.0, 4),
+               "us_pdl": round(per_kernel_pdl[i], 2), "us_overlapped": round(per_kernel_ov[i], 2),
+               "GB/s_overlapped": round(gbps(it, per_kernel_ov[i]), 1), "mapping": mapping_brief(it.plan.mapping)}
+        ncu_us = traffic_db.get(it.name + "/ncu_us")
+        if ncu_us:  # ncu-isolated duration (cold cache, serialised; profiles/ncu_traffic.json)
+            ent["ncu_us"] = ncu_us
+            ent["ncu_GBps"] = round(gbps(it, ncu_us), 1)
+            ent["ncu_dram_GBps"] = round(traffic_db.get(it.name, 0) / (ncu_us * 1e-6) / 1e9, 1)
+        per_shape[it.name] = ent
 
     out = {"metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
            "scaling": SCALING[args.workload], "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (counter-based U[0,1) fp32, seeded)",
-           "config": dict(config_for(args, "libnpp.so sm_100a; step replayed from a CUDA graph" if use_graph
-                                     else "libnpp.so sm_100a; eager launches + NCCL all-reduce"),
+           "config": dict(config_for(args, f"libnpp.so sm_100a; step replayed as {how}"),
                           launches="programmatic dependent launch (NPP_EXEC_OVERLAP)" if overlap
-                          else "serialised"),
-           "per_shape": per_shape,
-           "roofline": roofline(items[dom], per_kernel_us[dom], dom_gbs, peak, peak_src, traffic, flops, wavefronts),
-           "clocks": sampler.summary(),
-           "gpu_launches": args.steps * sum(it.plan.launches for it in items)}
+                          else "serialised", timing="CUDA events on the launching stream, max over ranks"),
+           "gpu_launches": args.steps * sum(it.plan.launches for it in items),
+           "per_rank_GBps": [round(step_bytes / (ms / args.steps * 1e-3) / 1e9, 1) for ms in per_rank_ms],
+           "clocks": clocks,
+           "roofline": roofline(items[dom], per_kernel_us[dom], gbps(items[dom], per_kernel_us[dom]), peak,
+                                peak_src, traffic_db.get(items[dom].name), getattr(items[dom], "flops", None),
+                                getattr(items[dom], "wavefronts", None)),
+           "per_shape": per_shape}
 
     # e2e: same metric through the C-ABI with HOST buffers (H2D of the inputs + D2H of the result inside)
     out["e2e"] = None if args.no_e2e else e2e_host(items, torch, stream, world, dist)
     if rank == 0 and not args.no_mappings and args.workload == "paper":
-        out["mappings"] = mapping_table(npp, torch, gen, device, stream, items)
+        out["mappings"] = mapping_table(npp, torch, device, stream, items)
         out["fused_rows_cols"] = fused_table(npp, torch, device, stream, items, per_shape)
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(items)
+    if not args.no_per_config and args.workload == "paper":
+        del items, step, run_step
+        torch.cuda.empty_cache()
+        out["per_config"] = per_config(npp, gen, torch, dist, world, rank, local, device, args, peak, peak_src)
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:
@@ -523,9 +670,48 @@ def main():
     return 0
 
 
+PER_CONFIG = [("sumcols_1m4k", "BASELINE.json configs[2]: sumCols [1M,4K] fp32, rows sharded + NCCL all-reduce"),
+              ("kmeans", "configs[3]: k-means assignment 4M x 64 x 32, points sharded"),
+              ("logreg", "configs[4]: logreg gradient [16M,256] fp32, B=4096, batches sharded")]
+
+
+def per_config(npp, gen, torch, dist, world, rank, local, device, args, peak, peak_src):
+    """BASELINE.json configs 3-5 at this run's N (strong scaling: the config's total work split over the
+    ranks), each timed like the step (graph replay, CUDA events, max over ranks, clocks sampled live in
+    a timed region of >= 25 ms) with the roofline of its kernel (isolated launches)."""
+    res = {}
+    stream = torch.cuda.Stream(device=device)
+    for wl, desc in PER_CONFIG:
+        items, reduce_bufs, _ = WORKLOADS[wl](npp, gen, torch, rank, world, "AUTO", device)
+        step = make_step(torch, dist, items, reduce_bufs, stream, world, True)
+        run_step, how = capture_step(torch, step, stream, world)
+        with torch.cuda.stream(stream):
+            for _ in range(3):
+                run_step()
+        ms_probe, _, _ = timed(torch, dist, run_step, stream, 2, world, local)
+        steps = max(args.steps, int(math.ceil(25.0 / max(ms_probe / 2, 1e-3))))
+        ms_total, per_rank_ms, clocks = timed(torch, dist, run_step, stream, steps, world, local)
+        ms_step = ms_total / steps
+        step_bytes = sum(it.bytes for it in items)
+        it = items[0]
+        us = kernel_us(torch, it, None, stream, reps=4)
+        rl = roofline(it, us, it.bytes / (us * 1e-6) / 1e9, peak, peak_src, ncu_traffic().get(it.name),
+                      getattr(it, "flops", None))
+        res[wl] = {"value": round(step_bytes * world / (ms_step * 1e-3) / 1e9, 1), "unit": "GB/s",
+                   "ms_per_step": round(ms_step, 4), "steps": steps, "scaling": SCALING[wl], "timing": how,
+                   "per_rank_GBps": [round(step_bytes / (ms / steps * 1e-3) / 1e9, 1) for ms in per_rank_ms],
+                   "roofline": {k: rl[k] for k in ("kernel", "bound", "achieved", "peak", "unit", "frac",
+                                                   "duration_us", "hbm_GBps", "traffic")},
+                   "clocks": clocks, "config": desc}
+        del items, step, run_step, reduce_bufs
+        torch.cuda.empty_cache()
+    return res
+
+
 def roofline(item, us, gbs, peak, peak_src, traffic, flops, wavefronts=None):
     base = {"kernel": item.name, "traffic": traffic, "algorithmic_bytes": item.bytes, "duration_us": round(us, 2),
-            "hbm_GBps": round(gbs, 1), "hbm_frac_of_measured": round(gbs / peak, 4)}
+            "hbm_GBps": round(gbs, 1), "hbm_frac_of_measured": round(gbs / peak, 4),
+            "timing": "isolated launches (NPP_EXEC_NO_PDL), L2-cold, CUDA events"}
     if wavefronts:  # random gathers: L1tex wavefront rate, ~1 per cycle per SM (B300_MICROARCH.md LDG model)
         wf_peak = 148 * 1.965e9 / 1e9
         achieved = wavefronts / (us * 1e-6) / 1e9
@@ -576,36 +762,9 @@ def e2e_host(items, torch, stream, world, dist, steps=3):
             "steps": steps, "api": "npp_execute_host (pinned host buffers, blocking)"}
 
 
-def kernel_us(torch, item, other, stream, reps=8, overlap=False):
-    """Average duration of one launch of item's plan: a graph of 2*reps launches alternating item's
-    input with `other`'s (same byte size, viewed with item's shape) so no launch finds its input in L2.
-    overlap=False: serialised launches (the per-kernel duration the roofline uses); True: launch-to-launch
-    interval with NPP_EXEC_OVERLAP."""
-    alt = other.ins[0].view(item.ins[0].shape) if other.ins[0].numel() == item.ins[0].numel() else None
-    firsts = [item.ins[0], alt] if alt is not None and alt.data_ptr() != item.ins[0].data_ptr() else [item.ins[0]]
-    inputs = [[f] + list(item.ins[1:]) for f in firsts]
-    with torch.cuda.stream(stream):
-        for x in inputs:
-            item.plan.execute(x, item.out, stream=stream)
-    torch.cuda.synchronize()
-    g = torch.cuda.CUDAGraph()
-    with torch.cuda.stream(stream):
-        with torch.cuda.graph(g, stream=stream):
-            for r in range(2 * reps):
-                item.plan.execute(inputs[r % len(inputs)], item.out, stream=stream, overlap=overlap)
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with torch.cuda.stream(stream):
-        g.replay()
-        a.record(stream)
-        g.replay()
-        b.record(stream)
-    torch.cuda.synchronize()
-    return a.elapsed_time(b) * 1e3 / (2 * reps)
-
-
 def fused_table(npp, torch, device, stream, items, per_shape):
     """Both sums of one matrix: the one-pass SUM_ROWS_COLS launch vs the sumRows + sumCols launches
-    (graph-timed, L2-cold like per_shape). GB/s counts the one algorithmic read + both outputs."""
+    (isolated, L2-cold like per_shape). GB/s counts the one algorithmic read + both outputs."""
     table = {}
     flat = [it.ins[0] for it in items]
     for R, C in PAPER_SHAPES:
@@ -617,29 +776,30 @@ def fused_table(npp, torch, device, stream, items, per_shape):
         two = per_shape[f"sum_rows{_fmt_shape((R, C))}"]["us"] + per_shape[f"sum_cols{_fmt_shape((R, C))}"]["us"]
         table[f"sum_rows_cols{_fmt_shape((R, C))}"] = {
             "GB/s": round(item.bytes / (us * 1e-6) / 1e9, 1), "us": round(us, 2), "two_pass_us": round(two, 2),
-            "speedup_vs_two_pass": round(two / us, 3), "mapping": mapping_brief(p.mapping)}
+            "speedup": round(two / us, 3)}
     return table
 
 
-def mapping_table(npp, torch, gen, device, stream, items):
-    """The paper's Fig 3 comparison on B200: every strategy at every paper shape (GB/s, graph-timed)."""
+def mapping_table(npp, torch, device, stream, items):
+    """The paper's Fig 3 comparison on B200: GB/s of every strategy at every paper shape (isolated
+    launches, L2-cold)."""
     table = {}
     bufs = {}
     for it in items:
         bufs.setdefault(tuple(it.ins[0].shape), []).append(it.ins[0])
     flat = [it.ins[0] for it in items]
-    for si, (R, C) in enumerate(PAPER_SHAPES):
+    for R, C in PAPER_SHAPES:
         m = bufs[(R, C)][0]
         other = next(x for x in flat if x.data_ptr() != m.data_ptr() and x.numel() == m.numel())
         for pattern in ("SUM_ROWS", "SUM_COLS"):
+            row = {}
             for strat in ("AUTO", "LITERAL", "1D", "TB_T", "WARP"):
                 p = npp.Plan(pattern, (R, C), "f32", strat, device=device)
                 item = Item(pattern, p, [m], p.new_out(), R * C * 4)
                 reps = 8 if strat in ("AUTO", "LITERAL", "WARP") else 2
                 us = kernel_us(torch, item, Item("o", p, [other], None, 0), stream, reps=reps)
-                gbs = (R * C * 4 + item.out.numel() * 4) / (us * 1e-6) / 1e9
-                table[f"{pattern.lower()}{_fmt_shape((R, C))}/{strat}"] = {
-                    "GB/s": round(gbs, 1), "us": round(us, 1), "mapping": mapping_brief(p.mapping)}
+                row[strat] = round((R * C * 4 + item.out.numel() * 4) / (us * 1e-6) / 1e9, 1)
+            table[f"{pattern.lower()}{_fmt_shape((R, C))}"] = row
     return table
 
 

@@ -62,7 +62,7 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
 __host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
-  // alignment pad + barriers + ||c||² + exchange words [3 slots][4 groups][tp]
+  // alignment pad + barriers (full, merged, released) + ||c||² + exchange words [3 slots][4 groups][tp]
   return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kMaxStages) * 4 * tp * 8;
 }
 // ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
@@ -111,7 +111,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // per ring slot: each group's (best score, packed {k, margin code, norm code}) per point
   uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kMaxStages][G][TP]
   uint64_t* full = reinterpret_cast<uint64_t*>(xch + kMaxStages * G * TP);
-  unsigned* released = reinterpret_cast<unsigned*>(full + kMaxStages);  // [kStages] warps done with the slot
+  uint64_t* merged = full + kMaxStages;  // [kStages] the slot's exchange words were merged (reusable)
+  unsigned* released = reinterpret_cast<unsigned*>(merged + kMaxStages);  // [kStages] warps done with the slot
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
   // uniform datapath (LDCU) for the centroid reads after it
@@ -124,6 +125,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       tma::mbar_init(full + i, 1);
+      tma::mbar_init(merged + i, 1);
       released[i] = 0;
     }
     tma::mbar_fence_init();
@@ -140,11 +142,12 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // γ_{2D+2} (||x|| + ||c_k||)² of its exact value, and the fp64 distance as written (G25) within
   // (D+3) 2^-53 (||x|| + ||c_k||)² of the exact distance; a point whose fp32 margin exceeds twice
   // the sum is decided by its fp32 winner, every other point is recomputed in fp64
+  // (||x|| + ||c||)² <= 2 (||x||² + max_k ||c_k||²) keeps the test free of square roots
   float cmax = 0.f;
   for (int k = 0; k < K; ++k) cmax = fmaxf(cmax, cn[k]);
-  const float sqrt_cm = __fsqrt_ru(__fmul_ru(cmax, 1.0001f));  // cn carries γ_D relative error
-  const float g2d = float(2 * D + 2) * 5.9604645e-8f;                  // (2D+2) u, u = 2^-24
-  const float coef = 2.02f * (g2d / (1.f - g2d) + float(D + 3) * 1.1102230e-16f);
+  const float cm_up = __fmul_ru(cmax, 1.0001f);  // cn carries γ_D relative error
+  const float g2d = float(2 * D + 2) * 5.9604645e-8f;  // (2D+2) u, u = 2^-24
+  const float coef = 4.04f * (g2d / (1.f - g2d) + float(D + 3) * 1.1102230e-16f);
 
   const long long n_tiles = r1 - r0;
   auto issue = [&](long long t, int slot) {  // tile t of the block's range into slot t % kStages
@@ -226,8 +229,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
       }
     }
-    // the group's share of ||x||² and its exchange word per point: (best score, {k, margin, norm})
+    // the group's share of ||x||² and its exchange word per point: (best score, {k, margin, norm}),
+    // written once the previous merge of this slot (tile t − kStages) has read the words
     uint2* ex = xch + (slot * G + g) * TP;
+    if (round > 0) tma::mbar_wait(merged + slot, (round - 1u) & 1u);
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
       float2 n2 = make_float2(0.f, 0.f);
@@ -241,8 +246,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
                                                                code_up(__fadd_ru(n2.x, n2.y)));
     }
-    // release the slot: the last of the 8 warps to finish with it merges the four groups' words, writes
-    // the tile's assignments and refills the slot with tile t+kStages (nobody waits on a barrier).
+    // release the slot: the last of the 8 warps to finish with it refills it with tile t+kStages, then
+    // merges the four groups' words and writes the tile's assignments (nobody waits on a barrier; the
+    // words live outside the tile, and near-tie rechecks read x from global memory)
     __syncwarp();
     unsigned last = 0;
     if (lane == 0) {
@@ -251,6 +257,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     }
     if (__shfl_sync(0xffffffffu, last, 0)) {
       __threadfence_block();
+      if (lane == 0) {
+        released[slot] = 0;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        if (t + kStages < n_tiles) issue(t + kStages, slot);
+      }
       const uint2* exs = xch + slot * G * TP;
       const long long base = (r0 + t) * TP;
       unsigned need64 = 0;  // bit j: point lane + 32 j is a near tie
@@ -268,39 +279,36 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
         const float sb = __uint_as_float(w[hw].x);
         float margin = decode12((w[hw].y >> 12) & 0xfffu);
-        float xn = 0.f;
+        float xn = cm_up;
 #pragma unroll
         for (int h = 0; h < G; ++h) {
           if (h != hw) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
           xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
         }
-        const float r = __fadd_ru(__fsqrt_ru(xn), sqrt_cm);
-        const float thr = __fmul_ru(coef, __fmul_ru(r, r));
         const long long gi = base + pt;
-        if (margin > thr) {
+        if (margin > __fmul_ru(coef, xn)) {
           if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
         } else if (gi < a.N) {
           need64 |= 1u << j;
         }
       }
+      __syncwarp();
+      if (lane == 0) tma::mbar_arrive(merged + slot);  // the words may be overwritten by tile t + kStages
       // near ties: the fp64 distance as written (G25), one warp per point, lane = centroid
       for (int j = 0; j < TP / 32; ++j) {
         unsigned m = __ballot_sync(0xffffffffu, (need64 >> j) & 1u);
         while (m) {
           const int src = __ffs(m) - 1;
           m &= m - 1;
-          const int pt = src + 32 * j;
-          const unsigned char* xr = sbase + pt * 128;
-          const unsigned kx = unsigned(pt & 7);
+          const long long gi = base + src + 32 * j;
+          const float* xr = a.x + gi * D;
           double best = __longlong_as_double(0x7ff0000000000000ll);
           int bestk = 0x7fffffff;
           for (int k = lane; k < K; k += 32) {
             const float* ck = a.c + (long long)k * D;
             double dist = 0.0;
             for (int d = 0; d < D; ++d) {
-              const float xd = *reinterpret_cast<const float*>(xr + (d >> 5) * (TP * 128) +
-                                                               ((unsigned((d >> 2) & 7) ^ kx) << 4) + (d & 3) * 4);
-              const double df = __dsub_rn(double(xd), double(__ldg(ck + d)));
+              const double df = __dsub_rn(double(__ldg(xr + d)), double(__ldg(ck + d)));
               dist = __dadd_rn(dist, __dmul_rn(df, df));
             }
             if (dist < best) best = dist, bestk = k;  // k increases per lane: first minimum
@@ -311,14 +319,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
             const int ok = __shfl_xor_sync(0xffffffffu, bestk, off);
             if (ob < best || (ob == best && ok < bestk)) best = ob, bestk = ok;
           }
-          if (lane == 0) a.assign[base + pt] = bestk;
+          if (lane == 0) a.assign[gi] = bestk;
         }
-      }
-      __syncwarp();
-      if (lane == 0) {
-        released[slot] = 0;
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        if (t + kStages < n_tiles) issue(t + kStages, slot);
       }
     }
     for (slot += kSets; slot >= kStages; slot -= kStages) ++round;
@@ -362,7 +364,9 @@ cudaError_t launch_tp(void (*kern)(const CUtensorMap, KmeansArgs), const CUtenso
 
 }  // namespace
 
-cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st) {
+cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cudaStream_t st) {
+  KmeansArgs a = args;
+  a.x = x;
   // tile: 256 points when D <= 64 (4 points x 64 lanes), else 128 (2 points x 64 lanes); both
   // with 4 centroid groups of 8 (S8)
   const bool small = a.D <= 64;

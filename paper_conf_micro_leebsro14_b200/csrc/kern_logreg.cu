@@ -107,13 +107,11 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
   const int c0 = lane * 4, c1 = 128 + lane * 4;  // this lane's two column quads
   const int Ci = int(C);
   const bool has0 = c0 < Ci, has1 = c1 < Ci;
-  // w in fp64: the products of two fp32 values are exact in fp64, so z = x_i·w and σ(z) are evaluated
-  // in fp64 (an fp32 z would carry up to γ_256 Σ|x w| absolute error into e_i = σ(z) − y_i)
-  double w0[4] = {0, 0, 0, 0}, w1[4] = {0, 0, 0, 0};
+  float w0[4] = {0, 0, 0, 0}, w1[4] = {0, 0, 0, 0};
 #pragma unroll
   for (int e = 0; e < 4; ++e) {
-    if (has0) w0[e] = double(__ldg(a.w + c0 + e));
-    if (has1) w1[e] = double(__ldg(a.w + c1 + e));
+    if (has0) w0[e] = __ldg(a.w + c0 + e);
+    if (has1) w1[e] = __ldg(a.w + c1 + e);
   }
   double acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   const long long n_tiles = r1 - r0;
@@ -129,43 +127,50 @@ __global__ void __launch_bounds__(kThreads, 1) npp_logreg_tma_kernel(const __gri
     const int yoff = slot_yoff[slot];
     const float y_lane = lane < rows_here ? reinterpret_cast<const float*>(y_ring + slot * kYSlot)[yoff + lane] : 0.f;
     const float* tile = reinterpret_cast<const float*>(tiles + slot * kTileBytes);
-    // dot products of the warp's 4 rows: per-lane fp64 partials over the lane's 8 columns ...
+    // dot products of the warp's 4 rows: per-lane fp32 FMA chains over the lane's 8 columns (error
+    // <= γ_8 Σ|x w| of the lane's terms) ...
     float4 x0[4], x1[4];
-    double dp[4];
+    float dp[4];
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {
       const int r = warp * 4 + rr;
       x0[rr] = has0 ? *reinterpret_cast<const float4*>(tile + r * Ci + c0) : make_float4(0, 0, 0, 0);
       x1[rr] = has1 ? *reinterpret_cast<const float4*>(tile + r * Ci + c1) : make_float4(0, 0, 0, 0);
-      double d = double(x0[rr].x) * w0[0];
-      d = fma(double(x0[rr].y), w0[1], d);
-      d = fma(double(x0[rr].z), w0[2], d);
-      d = fma(double(x0[rr].w), w0[3], d);
-      d = fma(double(x1[rr].x), w1[0], d);
-      d = fma(double(x1[rr].y), w1[1], d);
-      d = fma(double(x1[rr].z), w1[2], d);
-      dp[rr] = fma(double(x1[rr].w), w1[3], d);
+      float d = x0[rr].x * w0[0];
+      d = fmaf(x0[rr].y, w0[1], d);
+      d = fmaf(x0[rr].z, w0[2], d);
+      d = fmaf(x0[rr].w, w0[3], d);
+      d = fmaf(x1[rr].x, w1[0], d);
+      d = fmaf(x1[rr].y, w1[1], d);
+      d = fmaf(x1[rr].z, w1[2], d);
+      dp[rr] = fmaf(x1[rr].w, w1[3], d);
     }
-    // ... finished by a transposing butterfly: 6 shuffles leave lane l with the whole dot of row
-    // m(l) = 2*bit4(l) + bit3(l), so each lane evaluates one sigmoid, then 4 shuffles share them.
+    // ... finished in fp64 by a transposing butterfly: 6 shuffles leave lane l with the whole dot of
+    // row m(l) = 2*bit4(l) + bit3(l), so each lane evaluates one sigmoid, then 4 shuffles share them.
     const bool h16 = (lane & 16) != 0, h8 = (lane & 8) != 0;
-    double a0 = h16 ? dp[2] : dp[0], a1 = h16 ? dp[3] : dp[1];
-    a0 += __shfl_xor_sync(0xffffffffu, h16 ? dp[0] : dp[2], 16);
-    a1 += __shfl_xor_sync(0xffffffffu, h16 ? dp[1] : dp[3], 16);
-    double z = h8 ? a1 : a0;
-    z += __shfl_xor_sync(0xffffffffu, h8 ? a0 : a1, 8);
-    z += __shfl_xor_sync(0xffffffffu, z, 4);
-    z += __shfl_xor_sync(0xffffffffu, z, 2);
-    z += __shfl_xor_sync(0xffffffffu, z, 1);
+    double a0 = double(h16 ? dp[2] : dp[0]), a1 = double(h16 ? dp[3] : dp[1]);
+    a0 += double(__shfl_xor_sync(0xffffffffu, h16 ? dp[0] : dp[2], 16));
+    a1 += double(__shfl_xor_sync(0xffffffffu, h16 ? dp[1] : dp[3], 16));
+    double zd = h8 ? a1 : a0;
+    zd += __shfl_xor_sync(0xffffffffu, h8 ? a0 : a1, 8);
+    zd += __shfl_xor_sync(0xffffffffu, zd, 4);
+    zd += __shfl_xor_sync(0xffffffffu, zd, 2);
+    zd += __shfl_xor_sync(0xffffffffu, zd, 1);
     const int my_row = warp * 4 + (h16 ? 2 : 0) + (h8 ? 1 : 0);
     const float yr = __shfl_sync(0xffffffffu, y_lane, my_row);
-    // e = σ(z) − y in fp64 (σ(z) − 1 = −σ(−z) keeps the y = 1 case free of cancellation), then one
-    // rounding to fp32 for the x·e products
-    const double ez = exp(-fabs(z));
-    const double sig = z >= 0 ? 1.0 / (1.0 + ez) : ez / (1.0 + ez);
-    const double sig_neg = z >= 0 ? ez / (1.0 + ez) : 1.0 / (1.0 + ez);  // σ(−z) = 1 − σ(z)
-    const double ed = yr == 1.f ? -sig_neg : sig - double(yr);
-    const float e_mine = my_row < rows_here ? float(ed) : 0.f;
+    // e = σ(z) − y with a relative error of a few ulps: σ(z) = 1/(1+e^-z) for y = 0 and σ(z) − 1 =
+    // −σ(−z) for y = 1 (no cancellation; IEEE expf and division, not the __expf/__fdividef
+    // approximations); any other label is evaluated in fp64
+    float e_row;
+    const float z = float(zd);
+    if (yr == 0.f) {
+      e_row = 1.f / (1.f + expf(-z));
+    } else if (yr == 1.f) {
+      e_row = -1.f / (1.f + expf(z));
+    } else {
+      e_row = float(1.0 / (1.0 + exp(-zd)) - double(yr));
+    }
+    const float e_mine = my_row < rows_here ? e_row : 0.f;
     float p[8] = {0, 0, 0, 0, 0, 0, 0, 0};
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {

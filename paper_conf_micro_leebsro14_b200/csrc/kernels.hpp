@@ -98,6 +98,7 @@ cudaError_t launch_logreg(const LogregArgs& a, const float* x, int grid, cudaStr
 
 // k-means assignment (class KM, S8): x [N x D], c [K x D] fp32 -> a [N] int32.
 struct KmeansArgs {
+  const float* x;      // [N x D] (near-tie rechecks read it from global memory)
   const float* c;      // [K x D]
   int* assign;         // [N]
   int64_t N, D, K;
