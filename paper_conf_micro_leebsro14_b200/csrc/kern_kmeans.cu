@@ -236,12 +236,14 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
       float2 n2 = make_float2(0.f, 0.f);
+#ifndef NPP_KM_NO_NORM  // measurement variant: skip the norm share (the bound is then wrong)
       for (int d4 = q0; d4 < q1; ++d4) {
         const float4 v = *reinterpret_cast<const float4*>(tile + (d4 >> 3) * (TP * 128) + LP * 128 * i +
                                                           ((unsigned(d4 & 7) ^ key) << 4));
         ffma2(n2, make_float2(v.x, v.y), make_float2(v.x, v.y));
         ffma2(n2, make_float2(v.z, v.w), make_float2(v.z, v.w));
       }
+#endif
       const float margin = __fsub_rd(s2[i], bs[i]);
       ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
                                                                code_up(__fadd_ru(n2.x, n2.y)));
@@ -286,11 +288,17 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
           xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
         }
         const long long gi = base + pt;
+#if defined(NPP_KM_NO_RECHECK)  // measurement variant: the fp32 winner for every point
+        if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
+#elif defined(NPP_KM_MARK_FLAGS)  // measurement variant: near ties reported as -1 - winner
+        if (gi < a.N) a.assign[gi] = margin > __fmul_ru(coef, xn) ? int(w[hw].y >> 24) : -1 - int(w[hw].y >> 24);
+#else
         if (margin > __fmul_ru(coef, xn)) {
           if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
         } else if (gi < a.N) {
           need64 |= 1u << j;
         }
+#endif
       }
       __syncwarp();
       if (lane == 0) tma::mbar_arrive(merged + slot);  // the words may be overwritten by tile t + kStages
