@@ -47,7 +47,7 @@ constexpr int kConstFloats = 16384;  // DESIGN.md S8: 32·⌈K/32⌉·D ≤ 1638
 // centroids as pairs of −2c: km_pairs[(k/2)·D + d] = (−2c[k & ~1][d], −2c[k | 1][d]), padded rows zero
 // (the scaling by −2 is exact). One packed FFMA2 advances two centroids' chains with one (broadcast) x
 // element; a chain starts at ||c_k||², so each accumulator half ends as the score ||c_k||² − 2 x·c_k.
-__constant__ float2 km_pairs[kConstFloats / 2];
+__constant__ __align__(16) float2 km_pairs[kConstFloats / 2];
 __device__ float2 km_pack_buf[kConstFloats / 2];  // staging for the copy into the constant bank
 
 __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int Kp, int D) {
@@ -62,8 +62,9 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
 __host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
-  // alignment pad + barriers (full, merged, released) + ||c||² + exchange words [3 slots][4 groups][tp]
-  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kMaxStages) * 4 * tp * 8;
+  // alignment pad + barriers (full, written, merged, released) + ||c||² + exchange words
+  // [kSets x 2 parities][4 groups][tp]
+  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kSets) * 2 * 4 * tp * 8;
 }
 // ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
 __host__ __device__ inline int km_stages(int64_t K, int tp) {
@@ -99,6 +100,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   static_assert(G == 4, "the exchange word packs four centroid groups");
   constexpr int LP = kConsumers / G;  // threads (and point lanes) per centroid group
   constexpr int TP = PPT * LP;        // points per tile
+  constexpr int MPW = TP / kConsumerWarps;  // points of a tile each warp of the set merges (32 or 16)
+  static_assert(MPW <= 32 && TP % kConsumerWarps == 0, "a warp merges at most 32 points of a tile");
   extern __shared__ __align__(1024) unsigned char smem[];
   const int nb = km_boxes(a.D);
   const int stage_bytes = nb * TP * 128;
@@ -108,11 +111,12 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   unsigned char* ring = smem + pad;
   const int D = int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
   float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp] ||c_k||², +inf padded
-  // per ring slot: each group's (best score, packed {k, margin code, norm code}) per point
-  uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kMaxStages][G][TP]
-  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kMaxStages * G * TP);
-  uint64_t* merged = full + kMaxStages;  // [kStages] the slot's exchange words were merged (reusable)
-  unsigned* released = reinterpret_cast<unsigned*>(merged + kMaxStages);  // [kStages] warps done with the slot
+  // exchange words per (set, tile parity): each group's (best score, {k, margin code, norm code}) per point
+  uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kSets * 2][G][TP]
+  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * 2 * G * TP);  // [kMaxStages] tile landed
+  uint64_t* written = full + kMaxStages;        // [kSets * 2] the 8 warps wrote their words
+  uint64_t* merged = written + kSets * 2;       // [kSets * 2] the 8 warps merged their share
+  unsigned* released = reinterpret_cast<unsigned*>(merged + kSets * 2);  // [kStages] warps done with a slot
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
   // uniform datapath (LDCU) for the centroid reads after it
@@ -125,8 +129,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       tma::mbar_init(full + i, 1);
-      tma::mbar_init(merged + i, 1);
       released[i] = 0;
+    }
+    for (int i = 0; i < kSets * 2; ++i) {
+      tma::mbar_init(written + i, kConsumerWarps);
+      tma::mbar_init(merged + i, kConsumerWarps);
     }
     tma::mbar_fence_init();
   }
@@ -140,9 +147,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   __syncthreads();
   // near-tie bound (DESIGN.md §5 k-means): every fp32 score s_k = fl(||c_k||² − 2 x·c_k) is within
   // γ_{2D+2} (||x|| + ||c_k||)² of its exact value, and the fp64 distance as written (G25) within
-  // (D+3) 2^-53 (||x|| + ||c_k||)² of the exact distance; a point whose fp32 margin exceeds twice
-  // the sum is decided by its fp32 winner, every other point is recomputed in fp64
-  // (||x|| + ||c||)² <= 2 (||x||² + max_k ||c_k||²) keeps the test free of square roots
+  // (D+3) 2^-53 (||x|| + ||c_k||)² of the exact distance; a point whose fp32 margin exceeds twice the
+  // sum is decided by its fp32 winner, every other point is recomputed in fp64. (||x|| + ||c||)² <=
+  // 2 (||x||² + max_k ||c_k||²) keeps the test free of square roots.
   float cmax = 0.f;
   for (int k = 0; k < K; ++k) cmax = fmaxf(cmax, cn[k]);
   const float cm_up = __fmul_ru(cmax, 1.0001f);  // cn carries γ_D relative error
@@ -168,20 +175,87 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // centroid group; redux.sync lands in a uniform register, so ptxas treats g as warp-uniform and
   // keeps the centroid reads on the uniform datapath (LDCU)
   const int set = int(__reduce_min_sync(0xffffffffu, unsigned(warp / kConsumerWarps)));
-  const int g = int(__reduce_min_sync(0xffffffffu, unsigned((warp % kConsumerWarps) / (kConsumerWarps / G))));
+  const int wis = warp % kConsumerWarps;  // warp in set: merges points MPW·wis .. MPW·wis + MPW − 1
+  const int g = int(__reduce_min_sync(0xffffffffu, unsigned(wis / (kConsumerWarps / G))));
   const int lt = threadIdx.x % LP;  // point lane: points lt + LP·i
   // 128-byte swizzle: 16-byte chunk j of tile row p lives at chunk j ^ (p & 7); LP is a multiple
   // of 8, so every point of the thread has the key lt & 7
   const unsigned key = unsigned(lt & 7);
   const int nd4 = D / 4;
   const int q0 = g * nd4 / G, q1 = (g + 1) * nd4 / G;  // the group's quarter of the dims for ||x||²
+
+  // merge of this warp's MPW points of tile t (area ar, its use u): the four groups' words give the
+  // winner (lowest score, then lowest k), the margin to the runner-up (a lower bound) and ||x||² (an
+  // upper bound); proven points are written, the rest recomputed in fp64 exactly as the oracle does
+  auto merge_share = [&](long long t, int ar, unsigned u) {
+    tma::mbar_wait(written + ar, u & 1u);
+    const uint2* exs = xch + ar * G * TP;
+    const bool mine = lane < MPW;
+    const int pt = MPW * wis + (mine ? lane : 0);
+    uint2 w[G];
+#pragma unroll
+    for (int h = 0; h < G; ++h) w[h] = exs[h * TP + pt];
+    __syncwarp();
+    if (lane == 0) tma::mbar_arrive(merged + ar);  // the words may be overwritten (use u + 1)
+    int hw = 0;
+#pragma unroll
+    for (int h = 1; h < G; ++h) {  // lowest (score, k): groups interleave centroids, so k decides ties
+      const float sh = __uint_as_float(w[h].x), sw = __uint_as_float(w[hw].x);
+      if (sh < sw || (sh == sw && (w[h].y >> 24) < (w[hw].y >> 24))) hw = h;
+    }
+    const float sb = __uint_as_float(w[hw].x);
+    float margin = decode12((w[hw].y >> 12) & 0xfffu);
+    float xn = cm_up;
+#pragma unroll
+    for (int h = 0; h < G; ++h) {
+      if (h != hw) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
+      xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
+    }
+    const long long gi = (r0 + t) * TP + pt;
+    const bool proven = margin > __fmul_ru(coef, xn);
+    const bool valid = mine && gi < a.N;
+#if defined(NPP_KM_NO_RECHECK)  // measurement variant: the fp32 winner for every point
+    if (valid) a.assign[gi] = int(w[hw].y >> 24);
+    return;
+#elif defined(NPP_KM_MARK_FLAGS)  // measurement variant: near ties reported as -1 - winner
+    if (valid) a.assign[gi] = proven ? int(w[hw].y >> 24) : -1 - int(w[hw].y >> 24);
+    return;
+#endif
+    if (proven && valid) a.assign[gi] = int(w[hw].y >> 24);
+    unsigned m = __ballot_sync(0xffffffffu, !proven && valid);
+    while (m) {  // near ties: the fp64 distance as written (G25), the warp on one point, lane = centroid
+      const int src = __ffs(m) - 1;
+      m &= m - 1;
+      const long long gs = (r0 + t) * TP + MPW * wis + src;
+      const float* xr = a.x + gs * D;
+      double best = __longlong_as_double(0x7ff0000000000000ll);
+      int bestk = 0x7fffffff;
+      for (int k = lane; k < K; k += 32) {
+        const float* ck = a.c + (long long)k * D;
+        double dist = 0.0;
+        for (int d = 0; d < D; ++d) {
+          const double df = __dsub_rn(double(__ldg(xr + d)), double(__ldg(ck + d)));
+          dist = __dadd_rn(dist, __dmul_rn(df, df));
+        }
+        if (dist < best) best = dist, bestk = k;  // k increases per lane: first minimum
+      }
+#pragma unroll
+      for (int off = 16; off >= 1; off >>= 1) {
+        const double ob = __shfl_xor_sync(0xffffffffu, best, off);
+        const int ok = __shfl_xor_sync(0xffffffffu, bestk, off);
+        if (ob < best || (ob == best && ok < bestk)) best = ob, bestk = ok;
+      }
+      if (lane == 0) a.assign[gs] = bestk;
+    }
+  };
+
   // slot = t % kStages and round = t / kStages advance incrementally (no 64-bit division per tile)
   int slot = set % kStages;
   unsigned round = unsigned(set / kStages);
+  long long pend = -1;  // this set's previous tile, merged after the current one is computed
   for (long long t = set; t < n_tiles; t += kSets) {
     tma::mbar_wait_warp(full + slot, round & 1u);
-    const unsigned char* sbase = ring + slot * kMaxStageBytes;
-    const unsigned char* tile = sbase + lt * 128;
+    const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
     float bs[PPT], s2[PPT];
     int bk[PPT];
 #pragma unroll
@@ -229,10 +303,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
       }
     }
-    // the group's share of ||x||² and its exchange word per point: (best score, {k, margin, norm}),
-    // written once the previous merge of this slot (tile t − kStages) has read the words
-    uint2* ex = xch + (slot * G + g) * TP;
-    if (round > 0) tma::mbar_wait(merged + slot, (round - 1u) & 1u);
+    // the group's share of ||x||², then the words of tile t into area (set, tile parity) — once the
+    // set's merge of tile t − 2·kSets has read them
+    const int ar = set * 2 + int((t / kSets) & 1);
+    const unsigned u = unsigned(t / (2 * kSets));
+    float xn[PPT];
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
       float2 n2 = make_float2(0.f, 0.f);
@@ -244,95 +319,34 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         ffma2(n2, make_float2(v.z, v.w), make_float2(v.z, v.w));
       }
 #endif
-      const float margin = __fsub_rd(s2[i], bs[i]);
-      ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
-                                                               code_up(__fadd_ru(n2.x, n2.y)));
+      xn[i] = __fadd_ru(n2.x, n2.y);
     }
-    // release the slot: the last of the 8 warps to finish with it refills it with tile t+kStages, then
-    // merges the four groups' words and writes the tile's assignments (nobody waits on a barrier; the
-    // words live outside the tile, and near-tie rechecks read x from global memory)
+    // the x tile is consumed: release the slot (the last of the 8 warps refills it with t + kStages)
     __syncwarp();
-    unsigned last = 0;
     if (lane == 0) {
       __threadfence_block();
-      last = atomicAdd(released + slot, 1u) == kConsumerWarps - 1;
-    }
-    if (__shfl_sync(0xffffffffu, last, 0)) {
-      __threadfence_block();
-      if (lane == 0) {
+      if (atomicAdd(released + slot, 1u) == kConsumerWarps - 1) {
+        __threadfence_block();
         released[slot] = 0;
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         if (t + kStages < n_tiles) issue(t + kStages, slot);
       }
-      const uint2* exs = xch + slot * G * TP;
-      const long long base = (r0 + t) * TP;
-      unsigned need64 = 0;  // bit j: point lane + 32 j is a near tie
-#pragma unroll 2
-      for (int j = 0; j < TP / 32; ++j) {
-        const int pt = lane + 32 * j;
-        uint2 w[G];
-#pragma unroll
-        for (int h = 0; h < G; ++h) w[h] = exs[h * TP + pt];
-        int hw = 0;
-#pragma unroll
-        for (int h = 1; h < G; ++h) {  // lowest (score, k): groups interleave centroids, so k decides ties
-          const float sh = __uint_as_float(w[h].x), sw = __uint_as_float(w[hw].x);
-          if (sh < sw || (sh == sw && (w[h].y >> 24) < (w[hw].y >> 24))) hw = h;
-        }
-        const float sb = __uint_as_float(w[hw].x);
-        float margin = decode12((w[hw].y >> 12) & 0xfffu);
-        float xn = cm_up;
-#pragma unroll
-        for (int h = 0; h < G; ++h) {
-          if (h != hw) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
-          xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
-        }
-        const long long gi = base + pt;
-#if defined(NPP_KM_NO_RECHECK)  // measurement variant: the fp32 winner for every point
-        if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
-#elif defined(NPP_KM_MARK_FLAGS)  // measurement variant: near ties reported as -1 - winner
-        if (gi < a.N) a.assign[gi] = margin > __fmul_ru(coef, xn) ? int(w[hw].y >> 24) : -1 - int(w[hw].y >> 24);
-#else
-        if (margin > __fmul_ru(coef, xn)) {
-          if (gi < a.N) a.assign[gi] = int(w[hw].y >> 24);
-        } else if (gi < a.N) {
-          need64 |= 1u << j;
-        }
-#endif
-      }
-      __syncwarp();
-      if (lane == 0) tma::mbar_arrive(merged + slot);  // the words may be overwritten by tile t + kStages
-      // near ties: the fp64 distance as written (G25), one warp per point, lane = centroid
-      for (int j = 0; j < TP / 32; ++j) {
-        unsigned m = __ballot_sync(0xffffffffu, (need64 >> j) & 1u);
-        while (m) {
-          const int src = __ffs(m) - 1;
-          m &= m - 1;
-          const long long gi = base + src + 32 * j;
-          const float* xr = a.x + gi * D;
-          double best = __longlong_as_double(0x7ff0000000000000ll);
-          int bestk = 0x7fffffff;
-          for (int k = lane; k < K; k += 32) {
-            const float* ck = a.c + (long long)k * D;
-            double dist = 0.0;
-            for (int d = 0; d < D; ++d) {
-              const double df = __dsub_rn(double(__ldg(xr + d)), double(__ldg(ck + d)));
-              dist = __dadd_rn(dist, __dmul_rn(df, df));
-            }
-            if (dist < best) best = dist, bestk = k;  // k increases per lane: first minimum
-          }
-#pragma unroll
-          for (int off = 16; off >= 1; off >>= 1) {
-            const double ob = __shfl_xor_sync(0xffffffffu, best, off);
-            const int ok = __shfl_xor_sync(0xffffffffu, bestk, off);
-            if (ob < best || (ob == best && ok < bestk)) best = ob, bestk = ok;
-          }
-          if (lane == 0) a.assign[gi] = bestk;
-        }
-      }
     }
+    if (u > 0) tma::mbar_wait(merged + ar, (u - 1u) & 1u);
+    uint2* ex = xch + (ar * G + g) * TP;
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+      const float margin = __fsub_rd(s2[i], bs[i]);
+      ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]),
+                                   (unsigned(bk[i]) << 24) | (code_down(margin) << 12) | code_up(xn[i]));
+    }
+    __syncwarp();
+    if (lane == 0) tma::mbar_arrive(written + ar);
+    if (pend >= 0) merge_share(pend, set * 2 + int((pend / kSets) & 1), unsigned(pend / (2 * kSets)));
+    pend = t;
     for (slot += kSets; slot >= kStages; slot -= kStages) ++round;
   }
+  if (pend >= 0) merge_share(pend, set * 2 + int((pend / kSets) & 1), unsigned(pend / (2 * kSets)));
 }
 
 // One wrapper per tile shape, each with its own register cap: the cap is what keeps ptxas on the
