@@ -356,6 +356,19 @@ def balance(To, Ti, lim):
     return G, U, U * ((T - T // POOL_DIV) // U)
 
 
+def pool_claims(T, Ts, U, Ti, G):
+    """DESIGN.md S8 claim order of the pool [Ts, T): units of U tiles, except that when U < Ti the last
+    F = min(G, T - Ts) tiles are claimed one at a time. Returns the list of claimed [start, end) ranges
+    in claim order."""
+    F = min(G, T - Ts) if U < Ti else 0
+    out = []
+    for c in range(Ts, T - F, U):
+        out.append((c, min(T - F, c + U)))
+    for j in range(F):
+        out.append((T - F + j, T - F + j + 1))
+    return out
+
+
 def r2_staged(nest, dtype, lim):
     """DESIGN.md S8, staged family: persistent blocks (one per SM) stream BR x W tiles in outer-major
     order (static range + pool, balance()); the inner level is Split(Ti)."""

@@ -45,8 +45,12 @@ def static_ranges(G, Ts, Ti, align):
     return out
 
 
-def pool_units(T, Ts, U):
-    return [(c, min(T, c + U)) for c in range(Ts, T, U)]
+def pool_units(T, Ts, U, Ti, G):
+    """The claim-pool ranges of [Ts, T) in claim order (S8): units of U tiles, the last
+    F = min(G, T - Ts) tiles one at a time when U < Ti."""
+    F = min(G, T - Ts) if U < Ti else 0
+    big = [(c, min(T - F, c + U)) for c in range(Ts, T - F, U)]
+    return big + [(t, t + 1) for t in range(T - F, T)]
 
 
 def contiguous_ranges(T, P, G):

@@ -60,7 +60,7 @@ def test_staged_sum_schedule(npp, cuda_device, pattern, shape, dtype):
         assert np.all(cnt == 1), f"tiles loaded != once: {np.nonzero(cnt != 1)[0][:8]}"
         own = _owners(static_ranges(G, Ts, Ti, align), T)
         assert np.array_equal(blk[:Ts], own[:Ts]), "static part differs from the record's ranges"
-        for s0, s1 in pool_units(T, Ts, U):
+        for s0, s1 in pool_units(T, Ts, U, Ti, G):
             assert len(set(blk[s0:s1].tolist())) == 1, "a pool unit was split between blocks"
         ranges = static_ranges(G, Ts, Ti, align)
         # every block with static tiles takes part (blocks with an empty static range may find the

@@ -60,7 +60,12 @@ def _check_staged_sum(pattern, shape, dtype, lim, rec):
     assert all(s0 <= s1 for s0, s1 in ranges)
     sizes = [s1 - s0 for s0, s1 in ranges]
     assert max(sizes) - min(sizes) <= (Ti if align else 1), "balanced static split"
-    units = pool_units(T, Ts, U)
+    units = pool_units(T, Ts, U, Ti, G)
+    assert units == S.pool_claims(T, Ts, U, Ti, G)
+    # the blocks end within one tile of each other when outer tiles may be cut: the final claims are
+    # single tiles, at least one per block (or every pool tile)
+    if U < Ti:
+        assert all(e - s0 == 1 for s0, e in units[-min(G, T - Ts):])
     # exact cover of [0, T)
     seen = [0] * T
     for s0, s1 in ranges + units:

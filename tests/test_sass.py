@@ -35,6 +35,8 @@ def sass():
         m = re.match(r"\s+/\*[0-9a-f]+\*/\s+(?:@!?U?P\w+\s+)?([A-Z][A-Z0-9_.]*)", line)
         if m and name:
             funcs[name][m.group(1)] += 1
+            if m.group(1).startswith("LDC") and "c[0x3]" in line:  # user __constant__ bank (not params)
+                funcs[name][m.group(1) + "@bank3"] += 1
     return funcs
 
 
@@ -64,7 +66,7 @@ def test_kmeans_centroids_on_uniform_datapath(sass):
         # every centroid operand pair comes from a uniform register: ~one LDCU.64 per 2·PPT FFMA2,
         # and no per-thread constant loads in the inner loop
         assert c["LDCU.64"] + 2 * c["LDCU.128"] >= ffma2 // 8, (n, dict(c))
-        assert c["LDC.64"] <= 16, (n, c["LDC.64"])
+        assert c["LDC.64@bank3"] + c["LDC@bank3"] + c["LDC.128@bank3"] == 0, (n, dict(c))
 
 
 def test_packed_fma_in_kmeans(sass):
