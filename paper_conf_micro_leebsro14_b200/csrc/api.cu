@@ -6,6 +6,7 @@
 // paper's split between a static decision and launch-time parameters.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -552,6 +553,13 @@ int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, v
     const npp::StagedBalance bal = npp::staged_balance(t.To, t.Ti, plan->lim.sm_count);
     s.static_tiles = bal.Ts;
     s.unit = bal.U;
+    {  // S8 claim order: units of U, then the last F = min(G, T - Ts) tiles singly when U < Ti
+      const int64_t T = t.To * t.Ti, G = m.grid;
+      const int64_t F = bal.U < t.Ti ? std::min<int64_t>(G, T - bal.Ts) : 0;
+      s.tail_start = T - F;
+      s.big_units = (s.tail_start - bal.Ts + bal.U - 1) / bal.U;
+      s.claims = s.big_units + F;
+    }
     s.early_reads = overlap ? 1 : 0;
     s.pdl = pdl;
     s.trace = trace;

@@ -157,7 +157,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   // static range (MX-narrow: whole strips, so no strip is ever cut)
   const long long s0 = ALIGN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
   const long long s1 = ALIGN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
-  const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order
+  const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order, then single tiles
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
@@ -192,15 +192,19 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
           waited = true;
         }
         const unsigned k = atomicAdd(a.pool, 1u);
-        const long long c = a.static_tiles + (long long)k * U;
-        if (c >= total) {
-          // every producer makes exactly one failing claim, so the counter ends at units + G: the
+        if ((long long)k >= a.claims) {
+          // every producer makes exactly one failing claim, so the counter ends at claims + G: the
           // block taking the last value re-arms it for the next launch
-          if ((long long)k + 1 == (total - a.static_tiles + U - 1) / U + G) a.pool[0] = 0u;
+          if ((long long)k + 1 == a.claims + G) a.pool[0] = 0u;
           return -1;
         }
-        u_cur = c;
-        u_end = (c + U < total) ? c + U : total;
+        if ((long long)k < a.big_units) {  // units of U tiles, then the tail's single tiles (S8)
+          u_cur = a.static_tiles + (long long)k * U;
+          u_end = (u_cur + U < a.tail_start) ? u_cur + U : a.tail_start;
+        } else {
+          u_cur = a.tail_start + ((long long)k - a.big_units);
+          u_end = u_cur + 1;
+        }
         return u_cur++;
       };
       long long cur = next_tile();

@@ -74,6 +74,9 @@ struct StagedArgs {
   int64_t To, Ti;      // tiles along the outer / inner level
   int64_t static_tiles; // Ts
   int64_t unit;         // U: pool claim unit (tiles)
+  int64_t tail_start;   // T - F: the pool's last F tiles are claimed one at a time (S8)
+  int64_t big_units;    // claims of U tiles before the tail: ceil((tail_start - Ts) / U)
+  int64_t claims;       // big_units + F
   int early_reads;      // NPP_EXEC_OVERLAP: stream the inputs before the previous kernel completes
   int wide;             // 1: tiles of 8 rows x 4 KB (RX) / 128 rows x 256 B (MX-narrow); 2: RX one-row 32 KB tiles
   int pdl;              // launch as a programmatic dependent launch (npp_execute_ex without NPP_EXEC_NO_PDL)

@@ -33,10 +33,12 @@ for step in "$@"; do
           --clock-control none -k regex:npp_ --csv --log-file "$O/items_$w.csv" \
           python tools/profile_items.py $w > "$O/items_$w.log" 2>&1
       done ;;
-    full:*)
-      IFS=: read -r _ rx wl <<< "$step"
-      timeout 1200 ncu --set full --clock-control none --import-source on -k "regex:$rx" -s 4 -c 3 \
-        -o "$O/full_${wl}" python tools/profile_items.py "$wl" > "$O/full_${wl}.log" 2>&1 ;;
+    full:*)  # full:<kernel-regex>:<workload>[:<skip>[:<count>]] (skip/count of the matching launches)
+      IFS=: read -r _ rx wl sk ct <<< "$step"
+      timeout 1200 ncu --set full --clock-control none --import-source on -k "regex:$rx" -s "${sk:-4}" -c "${ct:-3}" \
+        -o "$O/full_${wl}" python tools/profile_items.py "$wl" > "$O/full_${wl}.log" 2>&1
+      ncu -i "$O/full_${wl}.ncu-rep" --page details --csv > "$O/full_${wl}_details.csv" 2>/dev/null
+      ncu -i "$O/full_${wl}.ncu-rep" --page raw --csv > "$O/full_${wl}_raw.csv" 2>/dev/null ;;
     san)
       for tool in memcheck racecheck synccheck initcheck; do
         timeout 1500 compute-sanitizer --tool $tool --error-exitcode 1 python tools/sanitize_run.py \
