@@ -38,7 +38,8 @@ constexpr int kSets = NPP_KM_SETS;
 constexpr int kConsumerWarps = 8;                 // per set
 constexpr int kConsumers = kConsumerWarps * 32;   // per set
 constexpr int kThreads = kSets * kConsumers;      // no producer warp: see the refill below
-constexpr int kSmemHeader = 128;
+constexpr int kSmemHeader = 256;
+constexpr int kMaxBoxes = 4;  // D <= 128: four 32-float boxes per point row
 constexpr int kMaxStageBytes = 64 * 1024;
 constexpr int kSmemLimit = 227 * 1024;
 constexpr int kConstFloats = 16384;  // DESIGN.md S8: 32·⌈K/32⌉·D ≤ 16384
@@ -92,8 +93,9 @@ __device__ __forceinline__ unsigned code_down(float v) { return (__float_as_uint
 __device__ __forceinline__ float decode12(unsigned c) { return __uint_as_float(c << 19); }
 
 // PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
-// groups; a tile is TP = PPT·256/G points.
-template <int PPT, int CPT>
+// groups; a tile is TP = PPT·256/G points. DT = D when it is known at compile time (the d loop is then
+// unrolled with immediate centroid offsets), 0 for any D.
+template <int PPT, int CPT, int DT>
 __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const KmeansArgs& a) {
   const CUtensorMap& map = *mapp;
   constexpr int G = 32 / CPT;
@@ -103,20 +105,21 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   constexpr int MPW = TP / kConsumerWarps;  // points of a tile each warp of the set merges (32 or 16)
   static_assert(MPW <= 32 && TP % kConsumerWarps == 0, "a warp merges at most 32 points of a tile");
   extern __shared__ __align__(1024) unsigned char smem[];
-  const int nb = km_boxes(a.D);
-  const int stage_bytes = nb * TP * 128;
+  const int D = DT ? DT : int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
+  const int nb = DT ? (DT + kBoxCols - 1) / kBoxCols : km_boxes(a.D);
   const int kStages = km_stages(a.K, TP);  // ring depth (2 or 3)
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
   unsigned char* ring = smem + pad;
-  const int D = int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
   float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp] ||c_k||², +inf padded
   // exchange words per (set, tile parity): each group's (best score, {k, margin code, norm code}) per point
   uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kSets * 2][G][TP]
-  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * 2 * G * TP);  // [kMaxStages] tile landed
-  uint64_t* written = full + kMaxStages;        // [kSets * 2] the 8 warps wrote their words
-  uint64_t* merged = written + kSets * 2;       // [kSets * 2] the 8 warps merged their share
-  unsigned* released = reinterpret_cast<unsigned*>(merged + kSets * 2);  // [kStages] warps done with a slot
+  // the ring is tracked per 32-float box of a slot, so a box is refilled as soon as the 8 warps of its set
+  // are past it (a 64-dim tile frees its first half mid-tile: more lead for the next loads)
+  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * 2 * G * TP);  // [kMaxStages][kMaxBoxes]
+  uint64_t* written = full + kMaxStages * kMaxBoxes;  // [kSets * 2] the 8 warps wrote their words
+  uint64_t* merged = written + kSets * 2;             // [kSets * 2] the 8 warps merged their share
+  unsigned* released = reinterpret_cast<unsigned*>(merged + kSets * 2);  // [kMaxStages][kMaxBoxes]
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
   // uniform datapath (LDCU) for the centroid reads after it
@@ -127,7 +130,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const long long r0 = bid * P, r1 = (T < r0 + P) ? T : r0 + P;
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kStages; ++i) {
+    for (int i = 0; i < kMaxStages * kMaxBoxes; ++i) {
       tma::mbar_init(full + i, 1);
       released[i] = 0;
     }
@@ -157,19 +160,19 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const float coef = 4.04f * (g2d / (1.f - g2d) + float(D + 3) * 1.1102230e-16f);
 
   const long long n_tiles = r1 - r0;
-  auto issue = [&](long long t, int slot) {  // tile t of the block's range into slot t % kStages
-    if (a.trace) {  // white-box schedule trace (npp_execute_traced)
+  auto issue_box = [&](long long t, int slot, int bx) {  // box bx of tile t of the range into slot t % kStages
+    if (a.trace && bx == 0) {  // white-box schedule trace (npp_execute_traced)
       a.trace[r0 + t] = int(bid);
       atomicAdd(a.trace + T + r0 + t, 1);
     }
-    tma::mbar_expect_tx(full + slot, unsigned(stage_bytes));
-    for (int bx = 0; bx < nb; ++bx)
-      tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
-                   full + slot);
+    tma::mbar_expect_tx(full + slot * kMaxBoxes + bx, unsigned(TP * 128));
+    tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
+                 full + slot * kMaxBoxes + bx);
   };
   if (threadIdx.x == 0) {
     tma::prefetch_map(&map);
-    for (int t = 0; t < kStages && t < n_tiles; ++t) issue(t, t);
+    for (int t = 0; t < kStages && t < n_tiles; ++t)
+      for (int bx = 0; bx < nb; ++bx) issue_box(t, t, bx);
   }
 
   // centroid group; redux.sync lands in a uniform register, so ptxas treats g as warp-uniform and
@@ -180,7 +183,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const int lt = threadIdx.x % LP;  // point lane: points lt + LP·i
   // 128-byte swizzle: 16-byte chunk j of tile row p lives at chunk j ^ (p & 7); LP is a multiple
   // of 8, so every point of the thread has the key lt & 7
-  const unsigned key = unsigned(lt & 7);
+  const unsigned key4 = unsigned(lt & 7) << 4;
   const int nd4 = D / 4;
   const int q0 = g * nd4 / G, q1 = (g + 1) * nd4 / G;  // the group's quarter of the dims for ||x||²
 
@@ -254,14 +257,15 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   unsigned round = unsigned(set / kStages);
   long long pend = -1;  // this set's previous tile, merged after the current one is computed
   for (long long t = set; t < n_tiles; t += kSets) {
-    tma::mbar_wait_warp(full + slot, round & 1u);
     const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
     float bs[PPT], s2[PPT];
     int bk[PPT];
+    float2 n2[PPT];  // the group's share of ||x||² (even / odd dims)
 #pragma unroll
-    for (int i = 0; i < PPT; ++i) bs[i] = s2[i] = __int_as_float(0x7f800000), bk[i] = 0;
+    for (int i = 0; i < PPT; ++i) bs[i] = s2[i] = __int_as_float(0x7f800000), bk[i] = 0, n2[i] = make_float2(0.f, 0.f);
     for (int kc = 0; kc < Kp; kc += 32) {
       const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
+      const bool last_chunk = kc + 32 >= Kp;
       float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1; starts at (||c||², ||c'||²)
 #pragma unroll
       for (int p = 0; p < CPT / 2; ++p) {
@@ -270,21 +274,55 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         for (int i = 0; i < PPT; ++i) acc[i][p] = nkp;
       }
       const float2* cq = km_pairs + (k0 >> 1) * D;  // pairs of −2c: the chain ends at the score
+#pragma unroll 1
+      for (int bx = 0; bx < nb; ++bx) {
+        uint64_t* fb = full + slot * kMaxBoxes + bx;
+        if (kc == 0) tma::mbar_wait_warp(fb, round & 1u);
+        const unsigned char* tb = tile + bx * (TP * 128);
+        const int jn = DT ? ((DT / 4 - 8 * bx) < 8 ? (DT / 4 - 8 * bx) : 8) : min(8, nd4 - 8 * bx);
 #pragma unroll 2
-      for (int d4 = 0; d4 < nd4; ++d4) {
-        const unsigned char* xb = tile + (d4 >> 3) * (TP * 128) + ((unsigned(d4 & 7) ^ key) << 4);
-        float4 xv[PPT];
+        for (int j = 0; j < jn; ++j) {
+          const int d4 = 8 * bx + j;
+          const unsigned char* xb = tb + ((unsigned(j) << 4) ^ key4);
+          float4 xv[PPT];
 #pragma unroll
-        for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
+          for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
 #pragma unroll
-        for (int p = 0; p < CPT / 2; ++p) {
+          for (int p = 0; p < CPT / 2; ++p) {
 #pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            const float2 cv = cq[p * D + 4 * d4 + q];  // warp-uniform
+            for (int q = 0; q < 4; ++q) {
+              const float2 cv = cq[p * D + 4 * d4 + q];  // warp-uniform
+#pragma unroll
+              for (int i = 0; i < PPT; ++i) {
+                const float xs = q == 0 ? xv[i].x : q == 1 ? xv[i].y : q == 2 ? xv[i].z : xv[i].w;
+                ffma2(acc[i][p], make_float2(xs, xs), cv);
+              }
+            }
+          }
+        }
+        if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
+          const int lo = max(q0, 8 * bx), hi = min(q1, 8 * bx + jn);
+          for (int d4 = lo; d4 < hi; ++d4) {
 #pragma unroll
             for (int i = 0; i < PPT; ++i) {
-              const float xs = q == 0 ? xv[i].x : q == 1 ? xv[i].y : q == 2 ? xv[i].z : xv[i].w;
-              ffma2(acc[i][p], make_float2(xs, xs), cv);
+#ifndef NPP_KM_NO_NORM  // measurement variant: skip the norm share (the bound is then wrong)
+              const float4 v = *reinterpret_cast<const float4*>(tb + LP * 128 * i + ((unsigned(d4 - 8 * bx) << 4) ^ key4));
+              ffma2(n2[i], make_float2(v.x, v.y), make_float2(v.x, v.y));
+              ffma2(n2[i], make_float2(v.z, v.w), make_float2(v.z, v.w));
+#endif
+            }
+          }
+        }
+        if (last_chunk) {  // the set is past this box of the slot: the last warp refills it (tile t + kStages)
+          __syncwarp();
+          if (lane == 0) {
+            __threadfence_block();
+            unsigned* rel = released + slot * kMaxBoxes + bx;
+            if (atomicAdd(rel, 1u) == kConsumerWarps - 1) {
+              __threadfence_block();
+              *rel = 0;
+              asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+              if (t + kStages < n_tiles) issue_box(t + kStages, slot, bx);
             }
           }
         }
@@ -303,42 +341,17 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
       }
     }
-    // the group's share of ||x||², then the words of tile t into area (set, tile parity) — once the
-    // set's merge of tile t − 2·kSets has read them
+    // the words of tile t into area (set, tile parity) — once the set's merge of tile t − 2·kSets has
+    // read them
     const int ar = set * 2 + int((t / kSets) & 1);
     const unsigned u = unsigned(t / (2 * kSets));
-    float xn[PPT];
-#pragma unroll
-    for (int i = 0; i < PPT; ++i) {
-      float2 n2 = make_float2(0.f, 0.f);
-#ifndef NPP_KM_NO_NORM  // measurement variant: skip the norm share (the bound is then wrong)
-      for (int d4 = q0; d4 < q1; ++d4) {
-        const float4 v = *reinterpret_cast<const float4*>(tile + (d4 >> 3) * (TP * 128) + LP * 128 * i +
-                                                          ((unsigned(d4 & 7) ^ key) << 4));
-        ffma2(n2, make_float2(v.x, v.y), make_float2(v.x, v.y));
-        ffma2(n2, make_float2(v.z, v.w), make_float2(v.z, v.w));
-      }
-#endif
-      xn[i] = __fadd_ru(n2.x, n2.y);
-    }
-    // the x tile is consumed: release the slot (the last of the 8 warps refills it with t + kStages)
-    __syncwarp();
-    if (lane == 0) {
-      __threadfence_block();
-      if (atomicAdd(released + slot, 1u) == kConsumerWarps - 1) {
-        __threadfence_block();
-        released[slot] = 0;
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        if (t + kStages < n_tiles) issue(t + kStages, slot);
-      }
-    }
     if (u > 0) tma::mbar_wait(merged + ar, (u - 1u) & 1u);
     uint2* ex = xch + (ar * G + g) * TP;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
       const float margin = __fsub_rd(s2[i], bs[i]);
-      ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]),
-                                   (unsigned(bk[i]) << 24) | (code_down(margin) << 12) | code_up(xn[i]));
+      ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
+                                                               code_up(__fadd_ru(n2[i].x, n2[i].y)));
     }
     __syncwarp();
     if (lane == 0) tma::mbar_arrive(written + ar);
@@ -360,12 +373,13 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #endif
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
                                                                          KmeansArgs a) {
-  kmeans_body<4, 8>(&map, a);  // D <= 64: 256-point tiles
+  kmeans_body<4, 8, 0>(&map, a);  // D <= 64: 256-point tiles
 }
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D128) npp_kmeans_tma_kernel_d128(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
-  kmeans_body<2, 8>(&map, a);  // 64 < D <= 128: 128-point tiles
+  kmeans_body<2, 8, 0>(&map, a);  // 64 < D <= 128: 128-point tiles
 }
+
 
 namespace {
 
@@ -416,7 +430,8 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   if ((e = cudaGetSymbolAddress(&pack, km_pack_buf)) != cudaSuccess) return e;
   e = cudaMemcpyToSymbolAsync(km_pairs, pack, size_t(Kp) * D * 4, 0, cudaMemcpyDeviceToDevice, st);
   if (e != cudaSuccess) return e;
-  e = launch_tp(small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128, map, a, grid, smem, st);
+  auto kern = small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128;
+  e = launch_tp(kern, map, a, grid, smem, st);
   if (e != cudaSuccess) return e;
   if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);
   return e;
