@@ -19,6 +19,7 @@
 // The path is FP32-FMA-bound: 2·N·K·D flops against 4·D bytes of x per point.
 #include <cstdint>
 #include <mutex>
+#include <type_traits>
 
 #include "kernels.hpp"
 #include "tma_ring.cuh"
@@ -63,7 +64,7 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
 __host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
-  // alignment pad + barriers (full, written, merged, released) + ||c||² + exchange words
+  // alignment pad + barriers (full, released) + ||c||² + exchange words
   // [kSets x 2 parities][4 groups][tp]
   return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kSets) * 2 * 4 * tp * 8;
 }
@@ -117,9 +118,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // the ring is tracked per 32-float box of a slot, so a box is refilled as soon as the 8 warps of its set
   // are past it (a 64-dim tile frees its first half mid-tile: more lead for the next loads)
   uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * 2 * G * TP);  // [kMaxStages][kMaxBoxes]
-  uint64_t* written = full + kMaxStages * kMaxBoxes;  // [kSets * 2] the 8 warps wrote their words
-  uint64_t* merged = written + kSets * 2;             // [kSets * 2] the 8 warps merged their share
-  unsigned* released = reinterpret_cast<unsigned*>(merged + kSets * 2);  // [kMaxStages][kMaxBoxes]
+  unsigned* released = reinterpret_cast<unsigned*>(full + kMaxStages * kMaxBoxes);  // [kMaxStages][kMaxBoxes]
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
   // uniform datapath (LDCU) for the centroid reads after it
@@ -133,10 +132,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     for (int i = 0; i < kMaxStages * kMaxBoxes; ++i) {
       tma::mbar_init(full + i, 1);
       released[i] = 0;
-    }
-    for (int i = 0; i < kSets * 2; ++i) {
-      tma::mbar_init(written + i, kConsumerWarps);
-      tma::mbar_init(merged + i, kConsumerWarps);
     }
     tma::mbar_fence_init();
   }
@@ -187,19 +182,16 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const int nd4 = D / 4;
   const int q0 = g * nd4 / G, q1 = (g + 1) * nd4 / G;  // the group's quarter of the dims for ||x||²
 
-  // merge of this warp's MPW points of tile t (area ar, its use u): the four groups' words give the
-  // winner (lowest score, then lowest k), the margin to the runner-up (a lower bound) and ||x||² (an
-  // upper bound); proven points are written, the rest recomputed in fp64 exactly as the oracle does
-  auto merge_share = [&](long long t, int ar, unsigned u) {
-    tma::mbar_wait(written + ar, u & 1u);
+  // merge of this warp's MPW points of tile t (area ar): the four groups' words give the winner
+  // (lowest score, then lowest k), the margin to the runner-up (a lower bound) and ||x||² (an upper
+  // bound); proven points are written, the rest recomputed in fp64 exactly as the oracle does
+  auto merge_share = [&](long long t, int ar) {
     const uint2* exs = xch + ar * G * TP;
     const bool mine = lane < MPW;
     const int pt = MPW * wis + (mine ? lane : 0);
     uint2 w[G];
 #pragma unroll
     for (int h = 0; h < G; ++h) w[h] = exs[h * TP + pt];
-    __syncwarp();
-    if (lane == 0) tma::mbar_arrive(merged + ar);  // the words may be overwritten (use u + 1)
     int hw = 0;
 #pragma unroll
     for (int h = 1; h < G; ++h) {  // lowest (score, k): groups interleave centroids, so k decides ties
@@ -233,9 +225,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       const float* xr = a.x + gs * D;
       double best = __longlong_as_double(0x7ff0000000000000ll);
       int bestk = 0x7fffffff;
+#pragma unroll 1
       for (int k = lane; k < K; k += 32) {
         const float* ck = a.c + (long long)k * D;
         double dist = 0.0;
+#pragma unroll 4
         for (int d = 0; d < D; ++d) {
           const double df = __dsub_rn(double(__ldg(xr + d)), double(__ldg(ck + d)));
           dist = __dadd_rn(dist, __dmul_rn(df, df));
@@ -255,7 +249,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // slot = t % kStages and round = t / kStages advance incrementally (no 64-bit division per tile)
   int slot = set % kStages;
   unsigned round = unsigned(set / kStages);
-  long long pend = -1;  // this set's previous tile, merged after the current one is computed
   for (long long t = set; t < n_tiles; t += kSets) {
     const unsigned char* tile = ring + slot * kMaxStageBytes + lt * 128;
     float bs[PPT], s2[PPT];
@@ -267,12 +260,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
       const bool last_chunk = kc + 32 >= Kp;
       float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1; starts at (||c||², ||c'||²)
+      float2 nkp[CPT / 2];
 #pragma unroll
-      for (int p = 0; p < CPT / 2; ++p) {
-        const float2 nkp = *reinterpret_cast<const float2*>(cn + k0 + 2 * p);
-#pragma unroll
-        for (int i = 0; i < PPT; ++i) acc[i][p] = nkp;
-      }
+      for (int p = 0; p < CPT / 2; ++p) nkp[p] = *reinterpret_cast<const float2*>(cn + k0 + 2 * p);
       const float2* cq = km_pairs + (k0 >> 1) * D;  // pairs of −2c: the chain ends at the score
 #pragma unroll 1
       for (int bx = 0; bx < nb; ++bx) {
@@ -280,8 +270,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         if (kc == 0) tma::mbar_wait_warp(fb, round & 1u);
         const unsigned char* tb = tile + bx * (TP * 128);
         const int jn = DT ? ((DT / 4 - 8 * bx) < 8 ? (DT / 4 - 8 * bx) : 8) : min(8, nd4 - 8 * bx);
-#pragma unroll 2
-        for (int j = 0; j < jn; ++j) {
+        // one 4-dim step of the thread's dot products; the very first starts the chains at ||c||²
+        auto step = [&](int j, auto first) {
           const int d4 = 8 * bx + j;
           const unsigned char* xb = tb + ((unsigned(j) << 4) ^ key4);
           float4 xv[PPT];
@@ -295,11 +285,20 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #pragma unroll
               for (int i = 0; i < PPT; ++i) {
                 const float xs = q == 0 ? xv[i].x : q == 1 ? xv[i].y : q == 2 ? xv[i].z : xv[i].w;
+                if constexpr (decltype(first)::value) {
+                  if (q == 0) {
+                    acc[i][p] = nkp[p];
+                  }
+                }
                 ffma2(acc[i][p], make_float2(xs, xs), cv);
               }
             }
           }
-        }
+        };
+        int j = 0;
+        if (bx == 0) step(j++, std::true_type{});
+#pragma unroll 1
+        for (; j < jn; ++j) step(j, std::false_type{});
         if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
           const int lo = max(q0, 8 * bx), hi = min(q1, 8 * bx + jn);
           for (int d4 = lo; d4 < hi; ++d4) {
@@ -341,11 +340,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
       }
     }
-    // the words of tile t into area (set, tile parity) — once the set's merge of tile t − 2·kSets has
-    // read them
+    // the words of tile t into area (set, tile parity); the set's barrier then lets every warp merge
+    // its share of the tile (the area is rewritten two tiles later, after the next barrier)
     const int ar = set * 2 + int((t / kSets) & 1);
-    const unsigned u = unsigned(t / (2 * kSets));
-    if (u > 0) tma::mbar_wait(merged + ar, (u - 1u) & 1u);
     uint2* ex = xch + (ar * G + g) * TP;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
@@ -353,13 +350,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       ex[lt + LP * i] = make_uint2(__float_as_uint(bs[i]), (unsigned(bk[i]) << 24) | (code_down(margin) << 12) |
                                                                code_up(__fadd_ru(n2[i].x, n2[i].y)));
     }
-    __syncwarp();
-    if (lane == 0) tma::mbar_arrive(written + ar);
-    if (pend >= 0) merge_share(pend, set * 2 + int((pend / kSets) & 1), unsigned(pend / (2 * kSets)));
-    pend = t;
+    asm volatile("bar.sync %0, %1;" ::"r"(1 + set), "n"(kConsumers) : "memory");  // this set only
+    merge_share(t, ar);
     for (slot += kSets; slot >= kStages; slot -= kStages) ++round;
   }
-  if (pend >= 0) merge_share(pend, set * 2 + int((pend / kSets) & 1), unsigned(pend / (2 * kSets)));
 }
 
 // One wrapper per tile shape, each with its own register cap: the cap is what keeps ptxas on the
@@ -374,6 +368,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
                                                                          KmeansArgs a) {
   kmeans_body<4, 8, 0>(&map, a);  // D <= 64: 256-point tiles
+}
+__global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64_exact(
+    const __grid_constant__ CUtensorMap map, KmeansArgs a) {
+  kmeans_body<4, 8, 64>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
 }
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D128) npp_kmeans_tma_kernel_d128(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
@@ -430,7 +428,7 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   if ((e = cudaGetSymbolAddress(&pack, km_pack_buf)) != cudaSuccess) return e;
   e = cudaMemcpyToSymbolAsync(km_pairs, pack, size_t(Kp) * D * 4, 0, cudaMemcpyDeviceToDevice, st);
   if (e != cudaSuccess) return e;
-  auto kern = small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128;
+  auto kern = a.D == 64 ? npp_kmeans_tma_kernel_d64_exact : small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128;
   e = launch_tp(kern, map, a, grid, smem, st);
   if (e != cudaSuccess) return e;
   if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);

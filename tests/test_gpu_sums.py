@@ -431,3 +431,38 @@ def test_rows_cols_plan_rules(npp, cuda_device):
                       torch.full((sum(shape),), 7, dtype=torch.int32, device=cuda_device))
         torch.cuda.synchronize()
         assert int(o.abs().sum()) == 0
+
+
+@pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"])
+def test_every_enumerated_mapping_executes_correctly(npp, cuda_device, pattern):
+    # the Fig 17 space: every hard-feasible Algorithm 1 candidate that npp_enumerate lists
+    # runs through npp_plan_with_mapping and matches the oracle, at two small shapes per nest (a ragged
+    # one and a skewed one in the spirit of the paper's (50, 20K))
+    lim = npp.limits_query(0)
+    rows = pattern in ("SUM_ROWS", "SUM_WEIGHTED_ROWS")
+    weighted = "WEIGHTED" in pattern
+    for shape, dtype in [((97, 1003), "i32"), ((50, 20000), "f32")]:
+        m = _make(dtype, shape, 61, cuda_device)
+        v = _make(dtype, (shape[1] if rows else shape[0],), 62, cuda_device) if weighted else None
+        m_np = m.cpu().numpy()
+        if weighted:
+            v_np = v.cpu().numpy()
+            want = (sums.sum_weighted_rows(m_np, v_np) if rows else sums.sum_weighted_cols(m_np, v_np))
+        else:
+            want = _oracle("SUM_ROWS" if rows else "SUM_COLS", m_np)
+        recs = npp.enumerate_mappings(pattern, shape, dtype, lim)
+        assert len(recs) > 50
+        for rec in recs:
+            p = npp.Plan(pattern, shape, dtype, mapping=rec)
+            out = p.execute([m, v] if weighted else [m], p.new_out())
+            torch.cuda.synchronize()
+            g = out.cpu().numpy()
+            if dtype == "f32":
+                scale = np.abs(want) if not weighted else None
+                if weighted:
+                    a_np = np.abs(m_np.astype(np.float64)) * (np.abs(v_np.astype(np.float64))[None, :] if rows
+                                                               else np.abs(v_np.astype(np.float64))[:, None])
+                    scale = a_np.sum(1) if rows else a_np.sum(0)
+                assert np.all(np.abs(g.astype(np.float64) - want) <= 1e-5 * scale), rec["levels"]
+            else:
+                assert np.array_equal(g.astype(np.int64), np.asarray(want).astype(np.int64)), rec["levels"]

@@ -9,12 +9,16 @@ LITERAL (the selector's pick), TB/T, warp-based and 1D are timed as markers.
     python tools/sweep_fig17.py --summarize gpurun_out/fig17.json    # markdown summary (no GPU)
 
 Timing: CUDA events around a graph of launches alternating two distinct 256 MiB inputs (L2-cold),
-median of 3 replays; algorithmic bytes = R*C*4 + outputs*4.
+median of 3 replays; algorithmic bytes = R*C*4 + outputs*4. Every mapping is first executed once and its
+output checked against the oracle (|out - oracle| <= 1e-5 * Σ|terms|); a mapping that fails is recorded
+with "valid": false and not timed.
 """
 from __future__ import annotations
 
 import argparse
 import json
+
+import numpy as np
 import os
 import statistics
 import sys
@@ -23,7 +27,7 @@ import time
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
-SHAPES = [(65536, 1024), (8192, 8192), (1024, 65536)]
+SHAPES = [(65536, 1024), (8192, 8192), (1024, 65536), (50, 20000)]  # + the paper's skewed shape (L1362-1363)
 SPAN = {0: "1", 1: "all", 2: "n", 3: "split"}
 
 
@@ -88,10 +92,13 @@ def run(args):
     result = {"device": torch.cuda.get_device_name(0), "limits": lim, "rows": []}
     os.makedirs(os.path.dirname(os.path.abspath(args.out)), exist_ok=True)
     log = open(args.out + "l", "w")  # <out>l: one JSON row per measured mapping
+    from oracle import sums
     for (R, C) in shapes:
         ma = gen.uniform_f32(3, (R, C), device=dev)
         mb = gen.uniform_f32(4, (R, C), device=dev)
+        ma_np = ma.cpu().numpy()
         for pattern in ("SUM_ROWS", "SUM_COLS"):
+            want = sums.sum_rows(ma_np) if pattern == "SUM_ROWS" else sums.sum_cols(ma_np)  # U[0,1): Σ|terms| = sum
             nbytes = R * C * 4 + (R if pattern == "SUM_ROWS" else C) * 4
             cands = npp.enumerate_mappings(pattern, (R, C), "f32", lim)
             entries = [("candidate", c) for c in cands]
@@ -104,12 +111,17 @@ def run(args):
                 else:
                     plan = npp.Plan(pattern, (R, C), "f32", mapping=rec, device=dev)
                 out = plan.new_out()
-                us = time_plan(torch, plan, [ma], [mb], out, stream)
+                with torch.cuda.stream(stream):
+                    plan.execute([ma], out, stream=stream)
+                torch.cuda.synchronize()
+                valid = bool(np.all(np.abs(out.cpu().numpy().astype(np.float64) - want) <= 1e-5 * want))
+                us = time_plan(torch, plan, [ma], [mb], out, stream) if valid else float("nan")
                 m = plan.mapping
                 row = {
                     "pattern": pattern, "shape": [R, C], "kind": kind, "score": m["score"], "dop": m["dop"],
                     "grid": m["grid"], "block": m["block"], "mapping": brief(m), "staged": m["staged"],
-                    "us": round(us, 2), "GB/s": round(nbytes / (us * 1e-6) / 1e9, 1)}
+                    "valid": valid, "us": round(us, 2),
+                    "GB/s": round(nbytes / (us * 1e-6) / 1e9, 1) if valid else 0.0}
                 result["rows"].append(row)
                 log.write(json.dumps(row) + "\n")  # incremental: a cut-off run keeps what it measured
                 log.flush()
@@ -150,12 +162,14 @@ def summarize(result):
         k = (r["pattern"], tuple(r["shape"]))
         if k not in keys:
             keys.append(k)
-    lines = ["| nest | candidates | best candidate GB/s (score, mapping) | LITERAL GB/s (score) | LITERAL rank | "
+    n_bad = sum(1 for r in rows if not r.get("valid", True))
+    lines = [f"validated against the oracle: {len(rows) - n_bad} of {len(rows)} mappings correct", "",
+             "| nest | candidates | best candidate GB/s (score, mapping) | LITERAL GB/s (score) | LITERAL rank | "
              "AUTO GB/s | TB/T | warp | 1D | Spearman(score, GB/s) | false negatives (C) |",
              "|---|---|---|---|---|---|---|---|---|---|---|"]
     for pattern, shape in keys:
         sel = [r for r in rows if r["pattern"] == pattern and tuple(r["shape"]) == shape]
-        cand = [r for r in sel if r["kind"] == "candidate"]
+        cand = [r for r in sel if r["kind"] == "candidate" and r.get("valid", True)]
         mk = {r["kind"]: r for r in sel if r["kind"] != "candidate"}
         if not cand:
             continue
