@@ -192,31 +192,34 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     uint2 w[G];
 #pragma unroll
     for (int h = 0; h < G; ++h) w[h] = exs[h * TP + pt];
-    int hw = 0;
+    // winner: lowest (score, k) — groups interleave centroids, so k decides ties (no dynamic indexing of
+    // w[], which would put it in local memory)
+    float sb = __uint_as_float(w[0].x);
+    unsigned wy = w[0].y;
 #pragma unroll
-    for (int h = 1; h < G; ++h) {  // lowest (score, k): groups interleave centroids, so k decides ties
-      const float sh = __uint_as_float(w[h].x), sw = __uint_as_float(w[hw].x);
-      if (sh < sw || (sh == sw && (w[h].y >> 24) < (w[hw].y >> 24))) hw = h;
+    for (int h = 1; h < G; ++h) {
+      const float sh = __uint_as_float(w[h].x);
+      if (sh < sb || (sh == sb && (w[h].y >> 24) < (wy >> 24))) sb = sh, wy = w[h].y;
     }
-    const float sb = __uint_as_float(w[hw].x);
-    float margin = decode12((w[hw].y >> 12) & 0xfffu);
+    // margin to the runner-up: the winner group's own runner-up, and every other group's best
+    float margin = decode12((wy >> 12) & 0xfffu);
     float xn = cm_up;
 #pragma unroll
     for (int h = 0; h < G; ++h) {
-      if (h != hw) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
+      if (w[h].y != wy || w[h].x != __float_as_uint(sb)) margin = fminf(margin, __fsub_rd(__uint_as_float(w[h].x), sb));
       xn = __fadd_ru(xn, decode12(w[h].y & 0xfffu));
     }
     const long long gi = (r0 + t) * TP + pt;
     const bool proven = margin > __fmul_ru(coef, xn);
     const bool valid = mine && gi < a.N;
 #if defined(NPP_KM_NO_RECHECK)  // measurement variant: the fp32 winner for every point
-    if (valid) a.assign[gi] = int(w[hw].y >> 24);
+    if (valid) a.assign[gi] = int(wy >> 24);
     return;
 #elif defined(NPP_KM_MARK_FLAGS)  // measurement variant: near ties reported as -1 - winner
-    if (valid) a.assign[gi] = proven ? int(w[hw].y >> 24) : -1 - int(w[hw].y >> 24);
+    if (valid) a.assign[gi] = proven ? int(wy >> 24) : -1 - int(wy >> 24);
     return;
 #endif
-    if (proven && valid) a.assign[gi] = int(w[hw].y >> 24);
+    if (proven && valid) a.assign[gi] = int(wy >> 24);
     unsigned m = __ballot_sync(0xffffffffu, !proven && valid);
     while (m) {  // near ties: the fp64 distance as written (G25), the warp on one point, lane = centroid
       const int src = __ffs(m) - 1;
@@ -297,7 +300,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         };
         int j = 0;
         if (bx == 0) step(j++, std::true_type{});
-#pragma unroll 1
+#pragma unroll 2
         for (; j < jn; ++j) step(j, std::false_type{});
         if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
           const int lo = max(q0, 8 * bx), hi = min(q1, 8 * bx + jn);
