@@ -266,6 +266,12 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       float2 nkp[CPT / 2];
 #pragma unroll
       for (int p = 0; p < CPT / 2; ++p) nkp[p] = *reinterpret_cast<const float2*>(cn + k0 + 2 * p);
+      if constexpr (DT == 0) {
+#pragma unroll
+        for (int i = 0; i < PPT; ++i)
+#pragma unroll
+          for (int p = 0; p < CPT / 2; ++p) acc[i][p] = nkp[p];
+      }
       const float2* cq = km_pairs + (k0 >> 1) * D;  // pairs of −2c: the chain ends at the score
 #pragma unroll 1
       for (int bx = 0; bx < nb; ++bx) {
@@ -299,7 +305,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
           }
         };
         int j = 0;
-        if (bx == 0) step(j++, std::true_type{});
+        if constexpr (DT != 0) {  // peeled first step (the generic-D path keeps the copies: its uniform
+          if (bx == 0) step(j++, std::true_type{});  // datapath does not survive the peel)
+        }
 #pragma unroll 2
         for (; j < jn; ++j) step(j, std::false_type{});
         if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
