@@ -50,6 +50,19 @@ def main():
     npp.Plan("KMEANS_ASSIGN", (5000, 64, 32)).execute([x, c], torch.empty(5000, dtype=torch.int32, device=dev))
     x, c = gen.kmeans_inputs(700, 96, 40, device=dev)
     npp.Plan("KMEANS_ASSIGN", (700, 96, 40)).execute([x, c], torch.empty(700, dtype=torch.int32, device=dev))
+    # near ties: exact midpoints of centroid pairs run the fp64 recheck path (D = 64 and D = 32 kernels)
+    for D in (64, 32):
+        cc = (torch.randint(-64, 64, (32, D), generator=torch.Generator().manual_seed(D)).float() / 4.0).to(dev)
+        xx = ((cc[torch.arange(600) % 32] + cc[(torch.arange(600) * 7 + 3) % 32]) / 2).contiguous()
+        npp.Plan("KMEANS_ASSIGN", (600, D, 32)).execute([xx, cc], torch.empty(600, dtype=torch.int32, device=dev))
+        n += 1
+    # traced schedules and plain (non-PDL) launches
+    mt = gen.uniform_f32(7, (4097, 300), device=dev)
+    for pattern in ("SUM_ROWS", "SUM_COLS", "SUM_ROWS_COLS"):
+        p = npp.Plan(pattern, (4097, 300), "f32", "AUTO")
+        p.execute_traced([mt], p.new_out())
+        p.execute([mt], p.new_out(), pdl=False)
+        n += 2
     lx, ly, lw = gen.logreg_inputs(5, 100, 256, device=dev)
     npp.Plan("LOGREG_GRAD", (5, 100, 256)).execute([lx, ly, lw], torch.empty(5, 256, device=dev))
     n += 3
