@@ -58,6 +58,7 @@ NAMES = {
     "paper": ["sum_rows[64K,1K]", "sum_cols[64K,1K]", "sum_rows[8K,8K]", "sum_cols[8K,8K]", "sum_rows[1K,64K]",
               "sum_cols[1K,64K]"],
     "kmeans": ["kmeans_assign[4M,64,32]"],
+    "sumcols_1m4k": ["sum_cols[1M,4K]"],
     "logreg": ["logreg_grad[16M,256]"],
     "kmeans_update": ["kmeans_update[4M,64,32]"],
     "pagerank": ["pagerank[4M,63M]"],
