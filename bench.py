@@ -705,6 +705,25 @@ def per_config(npp, gen, torch, dist, world, rank, local, device, args, peak, pe
                    "clocks": clocks, "config": desc}
         del items, step, run_step, reduce_bufs
         torch.cuda.empty_cache()
+        if world > 1 and wl == "sumcols_1m4k":
+            # strong scaling of config 3: the whole [1M,4K] on rank 0 alone (the other ranks wait at the
+            # barrier), the same graph-timed way, against this run's N-rank time
+            t1_ms = None
+            if rank == 0:
+                items1, _, _ = WORKLOADS[wl](npp, gen, torch, 0, 1, "AUTO", device)
+                step1 = make_step(torch, dist, items1, [], stream, 1, True)
+                run1, _ = capture_step(torch, step1, stream, 1)
+                with torch.cuda.stream(stream):
+                    for _ in range(3):
+                        run1()
+                t1_total, _, _ = timed(torch, dist, run1, stream, steps, 1, local)
+                t1_ms = t1_total / steps
+                del items1, step1, run1
+                torch.cuda.empty_cache()
+            dist.barrier()
+            if rank == 0:
+                res[wl]["T1_ms"] = round(t1_ms, 4)
+                res[wl]["T1_over_P_TP"] = round(t1_ms / (world * ms_step), 4)
     return res
 
 

@@ -238,10 +238,19 @@ int npp_plan(int pattern, const int64_t* shape, int ndim, int dtype, int strateg
     delete p;
     return st;
   }
-  if ((p->map.kernel_class == NPP_CLASS_KMEANS || p->map.kernel_class == NPP_CLASS_LOGREG) && !p->map.staged) {
+  if (p->map.kernel_class == NPP_CLASS_LOGREG && !p->map.staged) {
     delete p;
-    set_error("3-level nests execute through their staged (AUTO) kernel families only");
+    set_error("LOGREG_GRAD executes through its staged (AUTO) kernel family only");
     return NPP_ERR_UNSUPPORTED;
+  }
+  if (p->map.kernel_class == NPP_CLASS_KMEANS && !p->map.staged) {  // direct executor: no Split
+    for (int l = 0; l < p->map.nlevels; ++l)
+      if (p->map.level[l].span == NPP_SPLIT_K) {
+        delete p;
+        set_error("KMEANS_ASSIGN mappings with Split(k) on a reduce level are not executable (AUTO or a mapping "
+                  "without Split)");
+        return NPP_ERR_UNSUPPORTED;
+      }
   }
   if (pattern == NPP_SUM_ROWS_COLS && strategy != NPP_MAP_AUTO) {  // (also checked before selection)
     delete p;
@@ -301,8 +310,30 @@ int npp_plan_with_mapping(int pattern, const int64_t* shape, int ndim, int dtype
     set_error("forced mapping violates a hard constraint (Table II / device limits)");
     return NPP_ERR_NO_FEASIBLE_MAPPING;
   }
+  if (pattern == NPP_KMEANS_ASSIGN) {  // the direct 3-level executor (kern_kmeans_direct.cu): no Split, no vec
+    for (int l = 0; l < nest.L; ++l)
+      if (c.spans[l] == NPP_SPLIT_K) {
+        set_error("KMEANS_ASSIGN mappings with Split(k) on a reduce level are not executable");
+        return NPP_ERR_UNSUPPORTED;
+      }
+    if (forced->vec > 1 || forced->temp != NPP_TEMP_NONE) {
+      set_error("KMEANS_ASSIGN mappings take vec = 1 and no temp");
+      return NPP_ERR_UNSUPPORTED;
+    }
+    npp_plan_s* p = new npp_plan_s();
+    p->pattern = pattern;
+    p->dtype = dtype;
+    p->strategy = -1;
+    p->ndim = ndim;
+    for (int d = 0; d < ndim; ++d) p->shape[d] = shape[d];
+    p->lim = lim;
+    c.vec = 1;
+    npp::record_from_choice(nest, dtype, lim, c, npp::score(nest, lim, c), &p->map);
+    *out = p;
+    return NPP_OK;
+  }
   if (!npp::is_sum_pattern(pattern)) {
-    set_error("explicit mappings are executable for the 2-level sum families only");
+    set_error("explicit mappings are executable for the 2-level sum families and KMEANS_ASSIGN only");
     return NPP_ERR_UNSUPPORTED;
   }
   // class RX (inner Reduce on x) finishes a row with xor-shuffles over min(b_x, 32) lanes: the x block must
@@ -384,8 +415,8 @@ int64_t npp_plan_workspace_bytes(npp_plan_t plan) { return plan ? plan->map.work
 int npp_plan_launches(npp_plan_t plan) {
   if (!plan) return 0;
   if (plan->empty) return output_bytes(plan) > 0 ? 1 : 0;
-  // k-means: centroid pack + assignment; PageRank: per-node contribution + the CSR kernel
-  return (plan->pattern == NPP_KMEANS_ASSIGN || plan->pattern == NPP_PAGERANK) ? 2 : 1;
+  // k-means (staged): centroid pack + assignment; PageRank: per-node contribution + the CSR kernel
+  return ((plan->pattern == NPP_KMEANS_ASSIGN && plan->map.staged) || plan->pattern == NPP_PAGERANK) ? 2 : 1;
 }
 
 void npp_plan_destroy(npp_plan_t plan) { delete plan; }
@@ -461,6 +492,23 @@ int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, v
     g.trace = trace;
     cudaError_t e = npp::launch_logreg(g, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("logreg kernel launch", e);
+    return NPP_OK;
+  }
+  if (plan->pattern == NPP_KMEANS_ASSIGN && !m.staged) {  // class KM, direct executor (LITERAL / explicit)
+    npp::KmDirectArgs k{};
+    k.x = static_cast<const float*>(ins[0]);
+    k.c = static_cast<const float*>(ins[1]);
+    k.assign = static_cast<int*>(out);
+    k.N = plan->shape[0];
+    k.D = int(plan->shape[1]);
+    k.K = int(plan->shape[2]);
+    for (int l = 0; l < 3; ++l) {
+      k.dim[l] = m.level[l].dim;
+      k.blk[l] = m.level[l].block;
+    }
+    k.chunk0 = m.level[0].chunk;
+    cudaError_t e = npp::launch_kmeans_direct(k, int(m.level[0].grid), st);
+    if (e != cudaSuccess) return cuda_fail("kmeans direct kernel launch", e);
     return NPP_OK;
   }
   if (plan->pattern == NPP_KMEANS_ASSIGN) {  // class KM (S8)
@@ -635,7 +683,9 @@ int64_t npp_plan_tiles(npp_plan_t plan) {
       if (!m.staged) return 0;
       return m.level[0].grid * m.level[1].grid;  // To x Ti (S9: chunk = one tile per level)
     case NPP_CLASS_LOGREG: return s[0] * ((s[1] + 31) / 32);
-    case NPP_CLASS_KMEANS: return (s[0] + (s[1] <= 64 ? 255 : 127)) / (s[1] <= 64 ? 256 : 128);
+    case NPP_CLASS_KMEANS:
+      if (!m.staged) return 0;
+      return (s[0] + (s[1] <= 64 ? 255 : 127)) / (s[1] <= 64 ? 256 : 128);
     case NPP_CLASS_KMUPDATE: return (s[0] + 127) / 128;
     case NPP_CLASS_RC: return m.level[0].grid * m.level[1].grid;
     default: return 0;

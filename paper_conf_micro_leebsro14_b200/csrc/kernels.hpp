@@ -110,6 +110,21 @@ struct KmeansArgs {
 };
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st);
 
+// k-means assignment under a LITERAL / caller-given mapping with Span(all) reduce levels (class KM,
+// staged = 0; kern_kmeans_direct.cu): per level l = 0 (points), 1 (centroids), 2 (dims) the CUDA dim and
+// threads of the record; level 0's chunk (points per block); grid = ceil(N / chunk0) blocks.
+struct KmDirectArgs {
+  const float* x;      // [N x D]
+  const float* c;      // [K x D]
+  int* assign;         // [N]
+  int64_t N;
+  int D, K;
+  int dim[3];
+  int blk[3];
+  int64_t chunk0;
+};
+cudaError_t launch_kmeans_direct(const KmDirectArgs& a, int grid, cudaStream_t st);
+
 // sumRows + sumCols of one matrix in one pass (class RC, S8 RC): the ceil(R/32) x ceil(C/BC)
 // tile grid is cut into regions of cr row bands x cc column tiles, gr x gc of them in row-region-major
 // order; block b of G takes regions [b*nreg/G, (b+1)*nreg/G). out = [R row sums | C column sums].

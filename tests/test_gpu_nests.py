@@ -194,8 +194,14 @@ def test_unsupported_shapes(npp, cuda_device):
     with pytest.raises(npp.NppError) as e:
         npp.Plan("KMEANS_ASSIGN", (100, 6, 3), "f32", "AUTO")
     assert e.value.status == npp.ERR_UNSUPPORTED
+    # the direct 3-level family executes mappings without Split; a Split on a reduce level is unsupported
+    lit = npp.Plan("KMEANS_ASSIGN", (100, 64, 3), "f32", "LITERAL").mapping
+    split = dict(lit, levels=[lit["levels"][0], lit["levels"][1], dict(lit["levels"][2], span=npp.SPLIT_K, factor=2)])
     with pytest.raises(npp.NppError) as e:
-        npp.Plan("KMEANS_ASSIGN", (100, 64, 3), "f32", "LITERAL")
+        npp.Plan("KMEANS_ASSIGN", (100, 64, 3), "f32", mapping=split)
+    assert e.value.status == npp.ERR_UNSUPPORTED
+    with pytest.raises(npp.NppError) as e:
+        npp.Plan("LOGREG_GRAD", (4, 64, 256), "f32", "LITERAL")
     assert e.value.status == npp.ERR_UNSUPPORTED
 
 
@@ -347,3 +353,40 @@ def test_pagerank_shard_rows(npp, cuda_device):
     out = npp.pagerank_shard(lrp, lci, pr, outdeg, lo, hi)
     torch.cuda.synchronize()
     _check_pr(out, lrp, lci, pr, outdeg)
+
+
+@pytest.mark.parametrize("N,D,K", [(5000, 64, 32), (3000, 100, 33), (777, 8, 5), (1 << 18, 64, 32)])
+def test_kmeans_literal_mapping_exact(npp, cuda_device, N, D, K):
+    # strategy LITERAL: Algorithm 1 + ControlDOP exactly (e.g. L0 = (y, 1, Span(n)), L1 = (z, 16, all),
+    # L2 = (x, 64, all)), executed by the direct 3-level family; index-exact like AUTO
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
+    p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "LITERAL")
+    assert p.mapping == osel.select("KMEANS_ASSIGN", (N, D, K), "f32", npp.limits_query(0), "LITERAL")
+    assert p.mapping["staged"] == 0 and p.launches == 1
+    a = p.execute([x, c], p.new_out())
+    torch.cuda.synchronize()
+    assert np.array_equal(a.cpu().numpy(), okm.assign(x.cpu().numpy(), c.cpu().numpy()))
+
+
+@pytest.mark.parametrize("N,D,K", [(300, 8, 5), (200, 64, 32)])
+def test_kmeans_every_enumerated_mapping(npp, cuda_device, N, D, K):
+    # the Fig 17 space of the three-level nest: every hard-feasible Algorithm 1 candidate without Split
+    # executes through npp_plan_with_mapping and returns the oracle's assignment; Split candidates are
+    # rejected as unsupported
+    x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
+    x[:16] = (c[torch.arange(16, device=cuda_device) % K] + c[(torch.arange(16, device=cuda_device) + 1) % K]) / 2
+    want = okm.assign(x.cpu().numpy(), c.cpu().numpy())
+    recs = npp.enumerate_mappings("KMEANS_ASSIGN", (N, D, K), "f32", npp.limits_query(0))
+    ran = 0
+    for rec in recs:
+        if any(l["span"] == npp.SPLIT_K for l in rec["levels"]):
+            with pytest.raises(npp.NppError) as e:
+                npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", mapping=rec)
+            assert e.value.status == npp.ERR_UNSUPPORTED
+            continue
+        p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", mapping=rec)
+        a = p.execute([x, c], p.new_out())
+        torch.cuda.synchronize()
+        assert np.array_equal(a.cpu().numpy(), want), rec["levels"]
+        ran += 1
+    assert ran > 500
