@@ -17,6 +17,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import re
 
 import numpy as np
 import os
@@ -130,9 +131,59 @@ def run(args):
                   flush=True)
         del ma, mb
         torch.cuda.empty_cache()
+    if args.kmeans:
+        sweep_kmeans(torch, npp, gen, dev, lim, stream, result, log, args)
     with open(args.out, "w") as f:
         json.dump(result, f)
     print(summarize(result))
+
+
+KM_SHAPE = (1 << 16, 64, 32)  # config 4's D and K; N reduced so the slowest mappings finish in seconds
+
+
+def sweep_kmeans(torch, npp, gen, dev, lim, stream, result, log, args, per_band=25):
+    """The three-level nest (k-means assignment): a score-stratified sample of the Algorithm 1 candidates
+    without Split (the direct executor's space), each validated against the oracle, then timed; AUTO and
+    LITERAL as markers. Validation is exact equality of the assignments."""
+    import random
+
+    from oracle import kmeans as okm
+    N, D, K = KM_SHAPE
+    xa, c = gen.kmeans_inputs(N, D, K, device=dev)
+    xb, _ = gen.kmeans_inputs(N, D, K, row_offset=N, device=dev)
+    want = okm.assign(xa.cpu().numpy(), c.cpu().numpy())
+    nbytes = N * D * 4 + K * D * 4 + N * 4
+    cands = [r for r in npp.enumerate_mappings("KMEANS_ASSIGN", KM_SHAPE, "f32", lim)
+             if not any(l["span"] == 3 for l in r["levels"])]
+    rng = random.Random(17)
+    bands = {}
+    for r in cands:
+        bands.setdefault(r["score"], []).append(r)
+    sample = []
+    for sc in sorted(bands):
+        rng.shuffle(bands[sc])
+        sample += bands[sc][:per_band]
+    entries = [("candidate", r) for r in sample] + [("AUTO", None), ("LITERAL", None)]
+    t0 = time.perf_counter()
+    for kind, rec in entries:
+        plan = (npp.Plan("KMEANS_ASSIGN", KM_SHAPE, "f32", kind, device=dev) if rec is None
+                else npp.Plan("KMEANS_ASSIGN", KM_SHAPE, "f32", mapping=rec, device=dev))
+        out = plan.new_out()
+        with torch.cuda.stream(stream):
+            plan.execute([xa, c], out, stream=stream)
+        torch.cuda.synchronize()
+        valid = bool(np.array_equal(out.cpu().numpy(), want))
+        us = time_plan(torch, plan, [xa, c], [xb, c], out, stream) if valid else float("nan")
+        m = plan.mapping
+        row = {"pattern": "KMEANS_ASSIGN", "shape": list(KM_SHAPE), "kind": kind, "score": m["score"],
+               "dop": m["dop"], "grid": m["grid"], "block": m["block"], "mapping": brief(m), "staged": m["staged"],
+               "valid": valid, "us": round(us, 2), "GB/s": round(nbytes / (us * 1e-6) / 1e9, 1) if valid else 0.0,
+               "TFLOP/s": round(2 * N * K * D / (us * 1e-6) / 1e12, 2) if valid else 0.0}
+        result["rows"].append(row)
+        log.write(json.dumps(row) + "\n")
+        log.flush()
+    print(f"KMEANS_ASSIGN {KM_SHAPE}: {len(entries)} mappings of {len(cands)} without Split "
+          f"in {time.perf_counter() - t0:.1f} s", flush=True)
 
 
 def _spearman(xs, ys):
@@ -153,6 +204,51 @@ def _spearman(xs, ys):
     num = sum((a - mx) * (b - my) for a, b in zip(rx, ry))
     den = (sum((a - mx) ** 2 for a in rx) * sum((b - my) ** 2 for b in ry)) ** 0.5
     return num / den if den else 0.0
+
+
+def calibrate(rows):
+    """Refit the intrinsic weights (G3: W_C coalescing, W_B minimum block size; P:L1402-1411 asks for
+    tuning them from measurements): for each nest, recompute every timed candidate's soft-constraint
+    score under a grid of (W_C, W_B) with the oracle's score terms and report the Spearman rank
+    correlation of score and measured speed, and whether the top-scoring mapping would change."""
+    from oracle import select as S
+    lim = S.B200
+    grid = [(wc, wb) for wc in (1, 2, 4, 8, 16, 32, 64) for wb in (0, 1, 2, 4, 8)]
+    out = ["| nest | (W_C, W_B) | Spearman(score, speed) | time of the top-scored mapping / fastest time |",
+           "|---|---|---|---|"]
+    keys = []
+    for r in rows:
+        k = (r["pattern"], tuple(r["shape"]))
+        if k not in keys:
+            keys.append(k)
+    for pattern, shape in keys:
+        cand = [r for r in rows if (r["pattern"], tuple(r["shape"])) == (pattern, shape) and
+                r["kind"] == "candidate" and r.get("valid", True) and r["us"] == r["us"]]
+        if len(cand) < 3:
+            continue
+        nest = S.build_nest(pattern, shape)
+        speed = [-r["us"] for r in cand]
+        best = min(r["us"] for r in cand)
+        res = []
+        for wc, wb in grid:
+            S.W_C, S.W_B = wc, wb
+            sc = [S.score(nest, lim, _dims(r), _blocks(r)) for r in cand]
+            top = max(range(len(cand)), key=lambda i: (sc[i], -cand[i]["us"]))
+            res.append(((wc, wb), _spearman(sc, speed), cand[top]["us"] / best))
+        S.W_C, S.W_B = 8, 1
+        cur = next(x for x in res if x[0] == (8, 1))
+        fit = max(res, key=lambda x: (x[1], -x[2]))
+        for tag, (w, rho, ratio) in (("current", cur), ("best fit", fit)):
+            out.append(f"| {pattern.lower()}{list(shape)} | {tag} {w} | {rho:.3f} | {ratio:.2f} |")
+    return "\n".join(out)
+
+
+def _dims(r):
+    return tuple("xyz".index(tok[0]) for tok in r["mapping"].split())
+
+
+def _blocks(r):
+    return tuple(int(re.match(r"[xyz](\d+)", tok).group(1)) for tok in r["mapping"].split())
 
 
 def summarize(result):
@@ -192,8 +288,12 @@ if __name__ == "__main__":
     ap.add_argument("--out", default="gpurun_out/fig17.json")
     ap.add_argument("--shapes", default="")
     ap.add_argument("--summarize", default="")
+    ap.add_argument("--kmeans", action="store_true", help="also sweep the k-means nest (direct executor)")
+    ap.add_argument("--calibrate", default="", help="fit W_C/W_B to a sweep's jsonl (no GPU)")
     a = ap.parse_args()
-    if a.summarize:
+    if a.calibrate:
+        print(calibrate([json.loads(l) for l in open(a.calibrate) if l.strip()]))
+    elif a.summarize:
         if a.summarize.endswith(".jsonl"):
             print(summarize({"rows": [json.loads(l) for l in open(a.summarize) if l.strip()]}))
         else:
