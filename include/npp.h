@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define NPP_VERSION 4  /* 3: SUM_ROWS_COLS, KMEANS_UPDATE, PAGERANK; 4: static_tiles, NPP_EXEC_NO_PDL, traces */
+#define NPP_VERSION 4  /* 3: SUM_ROWS_COLS, KMEANS_UPDATE, PAGERANK; 4: static_tiles, NPP_EXEC_NO_PDL, traces, F64 */
 
 #if defined(__GNUC__)
 #define NPP_API __attribute__((visibility("default")))
@@ -49,7 +49,8 @@ typedef enum {
   NPP_ERR_CUDA = -6                  /* a CUDA runtime call or kernel launch failed */
 } npp_status;
 
-typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2 } npp_dtype;
+/* F64: the sums in double (the fp64 of Fig 9's generated kernel), accumulated in fp64 */
+typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2, NPP_F64 = 3 } npp_dtype;
 
 /* Patterns (shape, inputs, output) — Fig 1, Fig 15, BASELINE.json configs 4-5.
  *   SUM_ROWS           {R,C}   ins={m[R*C]}                  out[R]  = Σ_c m[r,c]

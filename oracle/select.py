@@ -33,7 +33,7 @@ MAX_GRID = (1 << 31) - 1                         # DESIGN.md S3 H6
 
 PATTERNS = ("SUM_ROWS", "SUM_COLS", "KMEANS_ASSIGN", "LOGREG_GRAD",
             "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS", "SUM_ROWS_COLS", "KMEANS_UPDATE", "PAGERANK")
-DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8}
+DTYPE_SIZE = {"f32": 4, "i32": 4, "i64": 8, "f64": 8}
 
 B200 = dict(sm_count=148, max_threads_per_sm=2048, max_threads_per_block=1024,
             max_block_dim=(1024, 1024, 64), warp_size=32, max_blocks_per_sm=32,

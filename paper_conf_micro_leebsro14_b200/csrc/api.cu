@@ -115,7 +115,7 @@ int validate_request(int pattern, const int64_t* shape, int ndim, int dtype, boo
     set_error("shape must hold 2 or 3 sizes");
     return NPP_ERR_INVALID_ARG;
   }
-  if (dtype < NPP_F32 || dtype > NPP_I64) {
+  if (dtype < NPP_F32 || dtype > NPP_F64) {
     set_error("unknown dtype");
     return NPP_ERR_INVALID_ARG;
   }

@@ -54,6 +54,11 @@ template <> struct RcOps<float> {
   using Acc = double;
   __device__ static float finish(double a) { return float(a); }
 };
+template <> struct RcOps<double> {
+  using S = double;
+  using Acc = double;
+  __device__ static double finish(double a) { return a; }
+};
 template <> struct RcOps<int32_t> {
   using S = unsigned;
   using Acc = unsigned;
@@ -308,9 +313,10 @@ cudaError_t launch_t(bool staged, const CUtensorMap& map, const RowsColsArgs& a,
 cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int grid, cudaStream_t st) {
   CUtensorMap map;
   std::memset(&map, 0, sizeof map);
-  const int esz = dtype == NPP_I64 ? 8 : 4;
+  const int esz = (dtype == NPP_I64 || dtype == NPP_F64) ? 8 : 4;
   const CUtensorMapDataType dt = dtype == NPP_F32   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                  : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
+                                 : dtype == NPP_F64 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64
                                                     : CU_TENSOR_MAP_DATA_TYPE_INT64;
   if (staged) {
     cudaError_t e = encode_2d(&map, a.m, dt, esz, a.R, a.C, unsigned(1024 / esz), unsigned(kTileRows));
@@ -319,6 +325,7 @@ cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int g
   switch (dtype) {
     case NPP_F32: return launch_t<float>(staged, map, a, grid, st);
     case NPP_I32: return launch_t<int32_t>(staged, map, a, grid, st);
+    case NPP_F64: return launch_t<double>(staged, map, a, grid, st);
     default: return launch_t<int64_t>(staged, map, a, grid, st);
   }
 }

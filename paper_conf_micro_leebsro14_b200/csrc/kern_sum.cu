@@ -35,6 +35,7 @@ template <typename T> struct AccOf;
 template <> struct AccOf<float> { using type = double; };
 template <> struct AccOf<int32_t> { using type = unsigned int; };
 template <> struct AccOf<int64_t> { using type = unsigned long long; };
+template <> struct AccOf<double> { using type = double; };
 
 constexpr int kUnroll = 8;
 
@@ -55,6 +56,9 @@ __device__ __forceinline__ void ldg_stream(const int64_t* p, Vec<int64_t, 2>& r)
   r.v[0] = a;
   r.v[1] = b;
 }
+__device__ __forceinline__ void ldg_stream(const double* p, Vec<double, 2>& r) {
+  asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(r.v[0]), "=d"(r.v[1]) : "l"(p));
+}
 template <typename T>
 __device__ __forceinline__ void ldg_stream(const T* p, Vec<T, 1>& r) { r.v[0] = __ldg(p); }
 
@@ -69,6 +73,15 @@ template <> struct Ops<float> {
   __device__ static Acc widen(Part p) { return double(p); }
   __device__ static Part from(float x) { return x; }
   __device__ static float finish(Acc a) { return float(a); }
+};
+template <> struct Ops<double> {
+  using Acc = double;
+  using Part = double;  // pairwise fp64 inside one batch, fp64 across
+  __device__ static Part mul(double a, double w) { return a * w; }
+  __device__ static Part add(Part a, Part b) { return a + b; }
+  __device__ static Acc widen(Part p) { return p; }
+  __device__ static Part from(double x) { return x; }
+  __device__ static double finish(Acc a) { return a; }
 };
 template <> struct Ops<int32_t> {
   using Acc = unsigned int;
@@ -363,6 +376,7 @@ cudaError_t launch_sum(int dtype, int kclass, int vec, bool weighted, const SumA
   switch (dtype) {
     case NPP_F32: return launch_v<float, 4>(kclass, vec, weighted, a, grid, block, smem, st);
     case NPP_I32: return launch_v<int32_t, 4>(kclass, vec, weighted, a, grid, block, smem, st);
+    case NPP_F64: return launch_v<double, 2>(kclass, vec, weighted, a, grid, block, smem, st);
     default: return launch_v<int64_t, 2>(kclass, vec, weighted, a, grid, block, smem, st);
   }
 }
@@ -471,6 +485,7 @@ cudaError_t launch_sum_temp(int dtype, int kclass, bool malloc_mode, const SumAr
   switch (dtype) {
     case NPP_F32: return launch_temp_t<float>(kclass, malloc_mode, a, grid, block, smem, st);
     case NPP_I32: return launch_temp_t<int32_t>(kclass, malloc_mode, a, grid, block, smem, st);
+    case NPP_F64: return launch_temp_t<double>(kclass, malloc_mode, a, grid, block, smem, st);
     default: return launch_temp_t<int64_t>(kclass, malloc_mode, a, grid, block, smem, st);
   }
 }
@@ -498,6 +513,10 @@ int sum_kernels_max_regs() {
   add_attr<int32_t, 1, true>(&regs);
   add_attr<int64_t, 2, true>(&regs);
   add_attr<int64_t, 1, true>(&regs);
+  add_attr<double, 2, false>(&regs);
+  add_attr<double, 1, false>(&regs);
+  add_attr<double, 2, true>(&regs);
+  add_attr<double, 1, true>(&regs);
   return regs;
 }
 

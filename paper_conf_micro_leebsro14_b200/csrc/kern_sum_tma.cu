@@ -66,6 +66,10 @@ template <> struct SOps<float> {
   using Acc = double;
   __device__ static float finish(double a) { return float(a); }
 };
+template <> struct SOps<double> {
+  using Acc = double;
+  __device__ static double finish(double a) { return a; }
+};
 template <> struct SOps<int32_t> {
   using Acc = unsigned int;
   __device__ static int32_t finish(unsigned a) { return int32_t(a); }
@@ -83,6 +87,7 @@ __device__ __forceinline__ unsigned vsum(const int4& v) {
 __device__ __forceinline__ unsigned long long vsum(const longlong2& v) {
   return (unsigned long long)v.x + (unsigned long long)v.y;
 }
+__device__ __forceinline__ double vsum(const double2& v) { return v.x + v.y; }
 // weighted: Σ of the 16-byte vector's products with the weights (fp32 pairwise; integers wrap)
 __device__ __forceinline__ float vdot(const float4& x, const float4& w) {
   return (x.x * w.x + x.y * w.y) + (x.z * w.z + x.w * w.w);
@@ -94,7 +99,9 @@ __device__ __forceinline__ unsigned vdot(const int4& x, const int4& w) {
 __device__ __forceinline__ unsigned long long vdot(const longlong2& x, const longlong2& w) {
   return (unsigned long long)x.x * (unsigned long long)w.x + (unsigned long long)x.y * (unsigned long long)w.y;
 }
+__device__ __forceinline__ double vdot(const double2& x, const double2& w) { return x.x * w.x + x.y * w.y; }
 __device__ __forceinline__ float vmul(float x, float w) { return x * w; }
+__device__ __forceinline__ double vmul(double x, double w) { return x * w; }
 __device__ __forceinline__ int32_t vmul(int32_t x, int32_t w) { return int32_t(unsigned(x) * unsigned(w)); }
 __device__ __forceinline__ int64_t vmul(int64_t x, int64_t w) {
   return int64_t((unsigned long long)x * (unsigned long long)w);
@@ -103,6 +110,7 @@ template <typename T> struct V16;
 template <> struct V16<float> { using type = float4; };
 template <> struct V16<int32_t> { using type = int4; };
 template <> struct V16<int64_t> { using type = longlong2; };
+template <> struct V16<double> { using type = double2; };
 
 template <typename A>
 __device__ __forceinline__ A warp_sum(A v) {
@@ -368,7 +376,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
             v[rr] = tt[(rg * kRowsPer + rr) * W + k * BC + col];
             if constexpr (WT) v[rr] = vmul(v[rr], reinterpret_cast<const T*>(vs)[rg * kRowsPer + rr]);
           }
-          if constexpr (std::is_same<T, float>::value) {  // fp32: pairwise tree inside the tile
+          if constexpr (std::is_floating_point<T>::value) {  // floats: pairwise tree inside the tile
 #pragma unroll
             for (int w = kRowsPer / 2; w >= 1; w /= 2)
 #pragma unroll
@@ -514,10 +522,11 @@ cudaError_t launch_dtype(bool rows, const CUtensorMap& map, const CUtensorMap& v
 
 cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedArgs& a, int grid, cudaStream_t st) {
   if (a.To * a.Ti >= 0x7fffffffll) return cudaErrorInvalidValue;  // 32-bit slot tags
-  const int esz = dtype == NPP_I64 ? 8 : 4;
+  const int esz = (dtype == NPP_I64 || dtype == NPP_F64) ? 8 : 4;
   const cuuint64_t bc = cuuint64_t(1024 / esz);
   const CUtensorMapDataType dt = dtype == NPP_F32   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                  : dtype == NPP_I32 ? CU_TENSOR_MAP_DATA_TYPE_INT32
+                                 : dtype == NPP_F64 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64
                                                     : CU_TENSOR_MAP_DATA_TYPE_INT64;
   CUtensorMap map;
   cudaError_t e;
@@ -539,6 +548,7 @@ cudaError_t launch_sum_staged(int dtype, bool rows, const void* m, const StagedA
   switch (dtype) {
     case NPP_F32: return launch_dtype<float>(rows, map, vmap, a, grid, st);
     case NPP_I32: return launch_dtype<int32_t>(rows, map, vmap, a, grid, st);
+    case NPP_F64: return launch_dtype<double>(rows, map, vmap, a, grid, st);
     default: return launch_dtype<int64_t>(rows, map, vmap, a, grid, st);
   }
 }

@@ -498,7 +498,7 @@ RcTiling rc_tiling(int64_t R, int64_t C, int dtype, int sm_count) {
   return best;
 }
 
-int dtype_size(int dtype) { return dtype == NPP_I64 ? 8 : 4; }
+int dtype_size(int dtype) { return (dtype == NPP_I64 || dtype == NPP_F64) ? 8 : 4; }
 
 bool is_rows_pattern(int p) { return p == NPP_SUM_ROWS || p == NPP_SUM_WEIGHTED_ROWS; }
 
@@ -860,7 +860,7 @@ extern "C" int npp_select(int pattern, const int64_t* shape, int ndim, int dtype
     set_error("out is NULL");
     return NPP_ERR_INVALID_ARG;
   }
-  if (dtype < NPP_F32 || dtype > NPP_I64) {
+  if (dtype < NPP_F32 || dtype > NPP_F64) {
     set_error("unknown dtype");
     return NPP_ERR_INVALID_ARG;
   }
@@ -885,7 +885,7 @@ extern "C" int64_t npp_enumerate(int pattern, const int64_t* shape, int ndim, in
     set_error("out is NULL or cap < 0");
     return NPP_ERR_INVALID_ARG;
   }
-  if (dtype < NPP_F32 || dtype > NPP_I64) {
+  if (dtype < NPP_F32 || dtype > NPP_F64) {
     set_error("unknown dtype");
     return NPP_ERR_INVALID_ARG;
   }

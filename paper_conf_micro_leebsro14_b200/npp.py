@@ -16,8 +16,8 @@ LIB_PATH = os.environ.get("NPP_LIB_PATH") or os.path.join(_PKG, "libnpp.so")  # 
 
 # enums (include/npp.h)
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_ALIGNMENT, ERR_WORKSPACE, ERR_NO_FEASIBLE, ERR_CUDA = 0, -1, -2, -3, -4, -5, -6
-DTYPES = {"f32": 0, "i32": 1, "i64": 2}
-TORCH_DTYPES = {"f32": torch.float32, "i32": torch.int32, "i64": torch.int64}
+DTYPES = {"f32": 0, "i32": 1, "i64": 2, "f64": 3}
+TORCH_DTYPES = {"f32": torch.float32, "i32": torch.int32, "i64": torch.int64, "f64": torch.float64}
 PATTERNS = {"SUM_ROWS": 0, "SUM_COLS": 1, "KMEANS_ASSIGN": 2, "LOGREG_GRAD": 3,
             "SUM_WEIGHTED_ROWS": 4, "SUM_WEIGHTED_COLS": 5, "SUM_ROWS_COLS": 6,
             "KMEANS_UPDATE": 7, "PAGERANK": 8}

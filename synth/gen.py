@@ -70,6 +70,16 @@ def uniform_f32(seed, shape, offset=0, device="cpu", lo=0.0, scale=1.0):
     return _fill(_empty(shape, torch.float32, device), offset, fn)
 
 
+def uniform_f64(seed, shape, offset=0, device="cpu", lo=0.0, scale=1.0):
+    """fp64 values lo + scale * u, u = (h1 >> 11 : h2) * 2^-53 from two hashes (53 random bits, exact)."""
+    def fn(i):
+        h1 = hash32(seed, i) >> 11                       # 21 bits
+        h2 = hash32(seed ^ 0x5bd1e995, i)                 # 32 bits
+        u = ((h1 << 32) | h2).to(torch.float64) * (2.0 ** -53)
+        return u * scale + lo
+    return _fill(_empty(shape, torch.float64, device), offset, fn)
+
+
 def exact_f32(seed, shape, offset=0, device="cpu"):
     """fp32 values k * 2^-8, k in [0, 256): sums of <= 65,536 of them are exact in fp32."""
     def fn(i):

@@ -6,7 +6,7 @@ by the GPU white-box trace tests (tests/test_gpu_trace.py). No method arithmetic
 from __future__ import annotations
 
 X = 0
-ESZ = {"f32": 4, "i32": 4, "i64": 8}
+ESZ = {"f32": 4, "i32": 4, "i64": 8, "f64": 8}
 
 
 def cdiv(a, b):

@@ -27,18 +27,20 @@ def npp(cuda_device):
 def _mat(dtype, shape, seed, dev):
     if dtype == "f32":
         return gen.uniform_f32(seed, shape, device=dev)
+    if dtype == "f64":
+        return gen.uniform_f64(seed, shape, lo=-1.0, scale=2.0, device=dev)
     if dtype == "i32":
         return gen.int_uniform(seed, shape, -1000, 1000, device=dev)
     return gen.int64_wide(seed, shape, device=dev)
 
 
 def _close(got, want, scale, dtype):
-    if dtype == "f32":
-        return np.all(np.abs(got.astype(np.float64) - want) <= 1e-5 * scale)
+    if dtype in ("f32", "f64"):
+        return np.all(np.abs(got.astype(np.float64) - want) <= (1e-5 if dtype == "f32" else 1e-12) * scale)
     return np.array_equal(got.astype(np.int64), want.astype(np.int64))
 
 
-@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64", "f64"])
 def test_random_sums_and_rows_cols(npp, cuda_device, dtype):
     for i, shape in enumerate(SUM_SHAPES):
         m = _mat(dtype, shape, 900 + i, cuda_device)

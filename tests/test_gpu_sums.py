@@ -1,7 +1,7 @@
 """GPU parity: the CUDA sum families (through the C-ABI) vs the fp64/int oracle, element by element.
 
 Integers: bit-exact. fp32: |gpu - oracle| <= 1e-5 * Σ|terms| per output (north_star tolerance; for the
-non-negative U[0,1) inputs this is 1e-5 relative).
+non-negative U[0,1) inputs this is 1e-5 relative). fp64: <= 1e-12 * Σ|terms|.
 """
 import numpy as np
 import pytest
@@ -27,6 +27,8 @@ def npp(cuda_device):
 def _make(dtype, shape, seed, device):
     if dtype == "f32":
         return gen.uniform_f32(seed, shape, device=device)
+    if dtype == "f64":
+        return gen.uniform_f64(seed, shape, lo=-1.0, scale=2.0, device=device)  # signed: cancellation
     if dtype == "i32":
         return gen.int_uniform(seed, shape, -1000, 1000, device=device)
     return gen.int64_wide(seed, shape, device=device)
@@ -44,8 +46,8 @@ def check(pattern, m, got, dtype):
     m_np = m.cpu().numpy()
     want = _oracle(pattern, m_np)
     g = got.cpu().numpy()
-    if dtype == "f32":
-        tol = 1e-5 * _abs_scale(pattern, m_np)
+    if dtype in ("f32", "f64"):
+        tol = (1e-5 if dtype == "f32" else 1e-12) * _abs_scale(pattern, m_np)
         err = np.abs(g.astype(np.float64) - want)
         bad = np.nonzero(err > tol)[0]
         assert bad.size == 0, f"{pattern} first bad {bad[:5]} got {g[bad[:5]]} want {want[bad[:5]]}"
@@ -54,7 +56,7 @@ def check(pattern, m, got, dtype):
 
 
 @pytest.mark.parametrize("pattern", ["SUM_ROWS", "SUM_COLS"])
-@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64", "f64"])
 @pytest.mark.parametrize("strategy", STRATS)
 def test_parity_small(npp, cuda_device, pattern, dtype, strategy):
     for i, shape in enumerate(SHAPES):
@@ -107,13 +109,13 @@ def test_paper_shapes_full(npp, cuda_device, shape):
             assert torch.all((out - out2).abs() <= out.abs() * 2.0 ** -23), "stale workspace"
 
 
-@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64", "f64"])
 def test_overlap_back_to_back(npp, cuda_device, dtype):
     # npp_execute_ex(NPP_EXEC_OVERLAP): programmatic dependent launches back to back on one stream —
     # the same plan (shared workspace: pool counter, tickets, accumulators) and different plans.
     # Results equal the oracle's and every workspace ends zero (S8 balance rule).
     shapes = [(65536, 1024), (1024, 65536), (4097, 300), (300, 4100), (33, 1 << 16)]
-    if dtype == "i64":
+    if dtype in ("i64", "f64"):
         shapes = [(s[0], s[1] // 2) if s[1] % 2 == 0 else s for s in shapes]
     plans = []
     for i, s in enumerate(shapes):
@@ -276,7 +278,7 @@ def _counters(p):
     return ws[part:part + -(-4 * m["levels"][0]["grid"] // 256) * 256]
 
 
-@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64", "f64"])
 def test_weighted(npp, cuda_device, dtype):
     # sumWeightedRows / sumWeightedCols (Fig 15): AUTO runs the staged TMA family with v staged per
     # tile (narrow and wide tiles, ragged edges), the literal / prior-work mappings the direct family
@@ -302,8 +304,9 @@ def test_weighted(npp, cuda_device, dtype):
                 torch.cuda.synchronize()
                 for o in (out, out2):
                     g = o.cpu().numpy()
-                    if dtype == "f32":
-                        assert np.all(np.abs(g - want) <= 1e-5 * scale), (pattern, shape, strategy)
+                    if dtype in ("f32", "f64"):
+                        tol = 1e-5 if dtype == "f32" else 1e-12
+                        assert np.all(np.abs(g - want) <= tol * scale), (pattern, shape, strategy)
                     else:
                         assert np.array_equal(g.astype(np.int64), want.astype(np.int64)), (pattern, shape, strategy)
                 if p.workspace is not None and p.mapping["temp"] == 0:  # S10 temp regions are scratch
@@ -370,7 +373,7 @@ def _check_rc(m, got, dtype):
     check("SUM_COLS", m, got[R:], dtype)
 
 
-@pytest.mark.parametrize("dtype", ["f32", "i32", "i64"])
+@pytest.mark.parametrize("dtype", ["f32", "i32", "i64", "f64"])
 def test_rows_cols_parity(npp, cuda_device, dtype):
     # one pass, both outputs: staged (16-B row pitch) and direct (ragged pitch) variants, regions cut
     # along rows only, columns only and both (tickets), ragged edge tiles; back-to-back executes

@@ -125,7 +125,7 @@ def test_sum_schedules(profile, pattern):
     for R, C in itertools.product(SIZES, SIZES):
         if R * C > (1 << 30):
             continue
-        for dtype in ("f32", "i32", "i64"):
+        for dtype in ("f32", "i32", "i64", "f64"):
             rec = _select(pattern, (R, C), dtype, lim)
             if rec is None:
                 continue
@@ -204,7 +204,7 @@ def test_kmeans_update_schedules(profile):
 def test_rowscols_schedules(profile):
     lim = PROFILES[profile]
     for R, C in itertools.product([1, 31, 33, 1000, 8192, 65536], [1, 4, 257, 1024, 8192, 65536]):
-        for dtype in ("f32", "i32", "i64"):
+        for dtype in ("f32", "i32", "i64", "f64"):
             rec = _select("SUM_ROWS_COLS", (R, C), dtype, lim)
             if rec is None:
                 continue

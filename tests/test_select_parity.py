@@ -42,7 +42,7 @@ def test_sums_exhaustive(profile, pattern):
     for R, C in itertools.product(SIZES, SIZES):
         if R * C > (1 << 34):
             continue
-        for dtype in ("f32", "i32", "i64"):
+        for dtype in ("f32", "i32", "i64", "f64"):
             for strat in SUM_STRATS:
                 _cmp(pattern, (R, C), dtype, lim, strat)
 

@@ -38,3 +38,14 @@ def test_kmeans_logreg_recipes():
     assert torch.equal(xi, xi.round()) and float(xi.abs().max()) <= 8
     X, y, w = gen.logreg_inputs(4, 8, 16)
     assert X.shape == (32, 16) and set(y.tolist()) <= {0.0, 1.0} and float(w.abs().max()) <= 1 / 16
+
+
+def test_uniform_f64_is_53_bit_and_counter_based():
+    # 53 random bits in [0, 1), identical for any offset split (shards regenerate the same values)
+    full = gen.uniform_f64(5, (4, 1000))
+    part = gen.uniform_f64(5, (2, 1000), offset=2000)
+    assert torch.equal(full[2:], part)
+    assert float(full.min()) >= 0.0 and float(full.max()) < 1.0
+    frac = (full * 2.0 ** 53)
+    assert torch.equal(frac, torch.floor(frac))
+    assert (frac % 2 == 1).any()  # the low bit is used
