@@ -460,6 +460,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
           if (mine[i]) static_cast<T*>(a.out)[oidx[i]] = SOps<T>::finish(val[i]);
         continue;
       }
+#ifdef NPP_SUM_NO_COMBINE  // measurement variant (wrong results): the cost of the fused Split combine
+      continue;
+#endif
       const int fi = int(nfl % kFlushRing);
       if (nfl >= kFlushRing) mbar_wait(fl_free + fi, unsigned(((nfl / kFlushRing) - 1) & 1));
 #pragma unroll
