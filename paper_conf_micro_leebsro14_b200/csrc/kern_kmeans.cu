@@ -376,11 +376,14 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #ifndef NPP_KM_MAXNREG_D128
 #define NPP_KM_MAXNREG_D128 48
 #endif
+#ifndef NPP_KM_MAXNREG_D64X
+#define NPP_KM_MAXNREG_D64X 80
+#endif
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
                                                                          KmeansArgs a) {
   kmeans_body<4, 8, 0>(&map, a);  // D <= 64: 256-point tiles
 }
-__global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64_exact(
+__global__ void __maxnreg__(NPP_KM_MAXNREG_D64X) npp_kmeans_tma_kernel_d64_exact(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
   kmeans_body<4, 8, 64>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
 }
