@@ -446,6 +446,12 @@ def cpu_baseline(items, budget_s=10.0):
 
 # ------------------------------------------------------------------------- timing plumbing
 
+def torchrun_cmd(gpus: int, port: int, argv) -> list:
+    """The command that runs this bench as `gpus` ranks of one node (rendezvous on 127.0.0.1)."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + list(argv)
+
+
 def self_launch(args) -> int:
     """`python bench.py --gpus N` outside torchrun: re-run this command as N ranks (one per GPU)."""
     import socket
@@ -454,9 +460,7 @@ def self_launch(args) -> int:
     s.bind(("127.0.0.1", 0))
     port = s.getsockname()[1]
     s.close()
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
-           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
-    return subprocess.call(cmd)
+    return subprocess.call(torchrun_cmd(args.gpus, port, sys.argv[1:]))
 
 
 def capture_step(torch, step, stream, world):

@@ -28,3 +28,21 @@ def test_reference_arm_other_ranks_exit_quietly():
                           "--warmup", "0"], capture_output=True, text=True, timeout=300, cwd=ROOT,
                          env=dict(os.environ, WORLD_SIZE="2", RANK="1"))
     assert out.returncode == 0 and out.stdout.strip() == ""
+
+
+def test_multi_gpu_self_launch_command():
+    # `bench.py --gpus N` outside torchrun re-runs itself as N ranks on one node over 127.0.0.1
+    sys.path.insert(0, ROOT)
+    import bench
+    cmd = bench.torchrun_cmd(8, 29511, ["--gpus", "8", "--steps", "5"])
+    assert cmd[1:4] == ["-m", "torch.distributed.run", "--nnodes=1"]
+    assert "--nproc-per-node=8" in cmd and cmd[cmd.index("--master-addr") + 1] == "127.0.0.1"
+    assert cmd[-4:] == ["--gpus", "8", "--steps", "5"] and cmd[-5].endswith("bench.py")
+
+
+def test_world_size_mismatch_is_an_error():
+    # under torchrun, --gpus must equal WORLD_SIZE (a silent one-rank measurement would mislabel N)
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--steps", "1",
+                          "--warmup", "0"], capture_output=True, text=True, timeout=300, cwd=ROOT,
+                         env=dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0"))
+    assert out.returncode != 0 and "WORLD_SIZE=2" in (out.stderr + out.stdout)
