@@ -615,7 +615,6 @@ int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, v
     s.pool = static_cast<unsigned*>(workspace);  // S9 staged workspace: [256 B pool][tickets][acc]
     s.tickets = reinterpret_cast<unsigned*>(static_cast<char*>(workspace) + 256);
     s.acc = static_cast<char*>(workspace) + 256 + ((t.To * 4 + 255) / 256) * 256;
-    s.ncopy = npp::staged_acc_copies(m.grid, t.To);
     cudaError_t e = npp::launch_sum_staged(plan->dtype, rows, ins[0], s, int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("staged kernel launch", e);
     return NPP_OK;

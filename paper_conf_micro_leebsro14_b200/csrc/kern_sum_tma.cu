@@ -162,7 +162,6 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long bid = blockIdx.x, G = gridDim.x;
   const long long total = a.To * a.Ti;
-  const long long O = a.O;  // outputs; accumulator copy cp lives at accg + cp * O
   // static range (MX-narrow: whole strips, so no strip is ever cut)
   const long long s0 = ALIGN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
   const long long s1 = ALIGN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
@@ -295,19 +294,15 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         for (int base = 0; base < OUT_PER_TILE; base += 32 * J) {
           Acc v[J];
 #pragma unroll
-          for (int q = 0; q < J; ++q) v[q] = Acc(0);
-          for (long long cp = 0; cp < a.ncopy; ++cp) {  // the copies in order 0..NC-1
-#pragma unroll
-            for (int q = 0; q < J; ++q) {
-              const long long o = o0 + base + lane + 32 * q;
-              if (base + lane + 32 * q < OUT_PER_TILE && o < oend) v[q] += __ldcg(accg + cp * O + o);
-            }
+          for (int q = 0; q < J; ++q) {
+            const long long o = o0 + base + lane + 32 * q;
+            v[q] = (base + lane + 32 * q < OUT_PER_TILE && o < oend) ? __ldcg(accg + o) : Acc(0);
           }
 #pragma unroll
           for (int q = 0; q < J; ++q) {
             const long long o = o0 + base + lane + 32 * q;
             if (base + lane + 32 * q < OUT_PER_TILE && o < oend) {
-              for (long long cp = 0; cp < a.ncopy; ++cp) __stcg(accg + cp * O + o, Acc(0));
+              __stcg(accg + o, Acc(0));
               static_cast<T*>(a.out)[o] = SOps<T>::finish(v[q]);
             }
           }
@@ -470,10 +465,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
 #endif
       const int fi = int(nfl % kFlushRing);
       if (nfl >= kFlushRing) mbar_wait(fl_free + fi, unsigned(((nfl / kFlushRing) - 1) & 1));
-      Acc* accb = accg + (bid % a.ncopy) * O;  // this block's accumulator copy
 #pragma unroll
       for (int i = 0; i < NV; ++i)
-        if (mine[i]) atomicAdd(accb + oidx[i], val[i]);
+        if (mine[i]) atomicAdd(accg + oidx[i], val[i]);
       __syncwarp();
       if (lane == 0) {
         if (warp == 0) {

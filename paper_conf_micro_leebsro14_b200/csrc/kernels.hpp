@@ -66,8 +66,7 @@ int sum_kernels_max_regs();
 struct StagedArgs {
   void* out;
   const void* v;        // weighted sums: v [C] (sumWeightedRows) or [R] (sumWeightedCols), else NULL
-  void* acc;           // [ncopy x O] accumulators (fp64 / u32 / u64), zero on entry and on exit
-  int64_t ncopy;       // accumulator copies (S8): block b adds into copy b % ncopy
+  void* acc;           // [O] accumulators (fp64 / u32 / u64), zero on entry and on exit
   unsigned* pool;      // [2]: pool claim counter, blocks-done ticket (zero on entry and on exit)
   unsigned* tickets;   // [To] tiles contributed per outer tile (partial contributors), zero on entry/exit
   int64_t O;           // outputs: R (sumRows) or C (sumCols)

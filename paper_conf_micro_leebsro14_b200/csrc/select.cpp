@@ -438,8 +438,6 @@ StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count) {
   return b;
 }
 
-int64_t staged_acc_copies(int64_t G, int64_t To) { return std::min<int64_t>(8, cdiv(G, To)); }
-
 StagedTiling staged_tiling(int pattern, int64_t R, int64_t C, int dtype) {
   StagedTiling t;
   const int64_t esz = dtype_size(dtype);
@@ -741,11 +739,10 @@ int record_from_choice(const Nest& n, int dtype, const npp_limits& lim, Choice c
     m.workspace_bytes = 256 * cdiv(4 * t.gr, 256) + 256 * cdiv(4 * t.gc, 256) + 256 * cdiv(n.N[0] * ab, 256) +
                         256 * cdiv(n.N[1] * ab, 256);
   } else if (is_sum_pattern(n.pattern) && c.staged) {
-    // pool counters (256 B) + tickets [To] + NC accumulator copies [NC x O] of the accumulator type
+    // pool counters (256 B) + tickets [To] + accumulators [O] of the accumulator type
     const StagedTiling t = staged_tiling(n.pattern, is_rows_pattern(n.pattern) ? n.N[0] : n.N[1], n.cols, dtype);
-    const int64_t nc = staged_acc_copies(m.grid, t.To);
     m.workspace_bytes =
-        256 + 256 * cdiv(4 * t.To, 256) + 256 * cdiv(nc * eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
+        256 + 256 * cdiv(4 * t.To, 256) + 256 * cdiv(eff(n.N[0]) * acc_bytes(n.pattern, dtype), 256);
   } else if (is_sum_pattern(n.pattern) && m.level[1].grid >= 2) {
     const int64_t part = m.level[1].grid * eff(n.N[0]) * acc_bytes(n.pattern, dtype);
     const int64_t tick = m.level[0].grid * 4;

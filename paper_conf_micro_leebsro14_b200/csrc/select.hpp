@@ -70,8 +70,6 @@ struct StagedBalance {
   int64_t G, U, Ts;  // persistent blocks, pool claim unit, statically split tiles
 };
 StagedBalance staged_balance(int64_t To, int64_t Ti, int sm_count);
-// S8: copies of a staged sum's accumulators, NC = min(8, ceil(G / To)); block b adds into copy b mod NC
-int64_t staged_acc_copies(int64_t G, int64_t To);
 
 // S8 RC (SUM_ROWS_COLS): the Tr x Tc grid of 32-row x 1 KB tiles is cut into gr x gc regions of cr row
 // bands x cc column tiles (cc <= kRcColTilesMax: a region's column accumulators fit shared memory);
