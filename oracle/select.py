@@ -392,12 +392,6 @@ def r2_staged(nest, dtype, lim):
     return blocks, spans, factors, vec, chunks, G, CL
 
 
-def acc_copies(G, To) -> int:
-    """DESIGN.md S8: NC = min(8, ceil(G / To)) copies of a staged sum's accumulators (block b adds into
-    copy b mod NC), so the final flushes of many blocks into few outer tiles spread over NC addresses."""
-    return min(8, cdiv(G, To))
-
-
 def r2_staged_static(nest, dtype, lim) -> int:
     """Ts of the balance rule for a staged sum: the tiles split statically (the rest is the pool)."""
     _, _, _, To, Ti = staged_tiles(nest, dtype)
@@ -605,12 +599,11 @@ def make_record(nest, dtype, lim, dims, blocks, spans, factors, vec, score_, chu
         B, C = _eff(nest["levels"][0][0]), _eff(nest["levels"][2][0])
         rec["workspace_bytes"] = 256 * cdiv(4 * B, 256) + 256 * cdiv(8 * B * C, 256)
     if nest["pattern"] in ("SUM_ROWS", "SUM_COLS", "SUM_WEIGHTED_ROWS", "SUM_WEIGHTED_COLS"):
-        if staged:  # pool counters (256 B) + tickets [To] + NC accumulator copies [NC x O] (S8)
+        if staged:  # pool counters (256 B) + tickets [To] + accumulators [O] (S8 staged)
             O = _eff(nest["levels"][0][0])
-            To = staged_tiles(nest, dtype)[3]   # tickets [To] u32, then accumulators [NC x O]
-            nc = acc_copies(grid, To)
+            To = staged_tiles(nest, dtype)[3]   # tickets [To] u32, then accumulators [O]
             rec["workspace_bytes"] = (256 + 256 * cdiv(4 * To, 256)
-                                      + 256 * cdiv(nc * O * acc_bytes(nest["pattern"], dtype), 256))
+                                      + 256 * cdiv(O * acc_bytes(nest["pattern"], dtype), 256))
         elif levels[1]["grid"] >= 2:
             O = _eff(nest["levels"][0][0])
             part = levels[1]["grid"] * O * acc_bytes(nest["pattern"], dtype)

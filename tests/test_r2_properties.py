@@ -83,12 +83,10 @@ def _check_staged_sum(pattern, shape, dtype, lim, rec):
         for o in range(s0 // Ti, cdiv(s1, Ti)):
             contrib[o] += max(0, min(s1, (o + 1) * Ti) - max(s0, o * Ti))
     assert contrib == [Ti] * To
-    # workspace: pool counters (256 B), tickets [To] u32, NC accumulator copies [NC x O] (fp64 / u32 / u64)
+    # workspace: pool counters (256 B), tickets [To] u32, accumulators [O] (fp64 / u32 / u64)
     O = R if rows else C
     ab = 4 if dtype == "i32" else 8
-    nc = min(8, cdiv(G, To))
-    assert 1 <= nc <= 8 and (nc == 1 or To < G)
-    need = 256 + 256 * cdiv(4 * To, 256) + nc * O * ab
+    need = 256 + 256 * cdiv(4 * To, 256) + O * ab
     assert rec["workspace_bytes"] >= need
     # the x level streams 16-byte vectors (RX) or one column per thread (MX)
     assert rec["vec"] == (16 // esz if rows else 1)
