@@ -286,17 +286,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
           float4 xv[PPT];
 #pragma unroll
           for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
-#if !defined(NPP_KM_NO_NORM) && !defined(NPP_KM_NORM_LOOP)
-          // the group's quarter of the dims: its share of ||x||² from the x already in registers (a
-          // warp-uniform branch, taken on kc == 0 for a quarter of the steps)
-          if (kc == 0 && d4 >= q0 && d4 < q1) {
-#pragma unroll
-            for (int i = 0; i < PPT; ++i) {
-              ffma2(n2[i], make_float2(xv[i].x, xv[i].y), make_float2(xv[i].x, xv[i].y));
-              ffma2(n2[i], make_float2(xv[i].z, xv[i].w), make_float2(xv[i].z, xv[i].w));
-            }
-          }
-#endif
 #pragma unroll
           for (int p = 0; p < CPT / 2; ++p) {
 #pragma unroll
@@ -321,7 +310,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         }
 #pragma unroll 2
         for (; j < jn; ++j) step(j, std::false_type{});
-#if defined(NPP_KM_NORM_LOOP)  // measurement variant: the norm share in a separate loop re-reading x
         if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
           const int lo = max(q0, 8 * bx), hi = min(q1, 8 * bx + jn);
           for (int d4 = lo; d4 < hi; ++d4) {
@@ -335,7 +323,6 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
             }
           }
         }
-#endif
         if (last_chunk) {  // the set is past this box of the slot: the last warp refills it (tile t + kStages)
           __syncwarp();
           if (lane == 0) {
