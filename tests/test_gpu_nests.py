@@ -368,7 +368,7 @@ def test_kmeans_literal_mapping_exact(npp, cuda_device, N, D, K):
     assert np.array_equal(a.cpu().numpy(), okm.assign(x.cpu().numpy(), c.cpu().numpy()))
 
 
-@pytest.mark.parametrize("N,D,K", [(300, 8, 5), (200, 64, 32)])
+@pytest.mark.parametrize("N,D,K", [(300, 8, 5), (4096, 32, 16)])
 def test_kmeans_every_enumerated_mapping(npp, cuda_device, N, D, K):
     # the Fig 17 space of the three-level nest: every hard-feasible Algorithm 1 candidate without Split
     # executes through npp_plan_with_mapping and returns the oracle's assignment; Split candidates are
@@ -389,4 +389,4 @@ def test_kmeans_every_enumerated_mapping(npp, cuda_device, N, D, K):
         torch.cuda.synchronize()
         assert np.array_equal(a.cpu().numpy(), want), rec["levels"]
         ran += 1
-    assert ran > 300
+    assert ran > 100
