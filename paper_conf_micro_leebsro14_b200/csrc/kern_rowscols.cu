@@ -222,10 +222,14 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int j = 0; j < WPG; ++j) s += rsum[(rb * kConsumerWarps + g * WPG + j) * 32 + li];
         const long long row = br * kTileRows + lane;
         if (row < a.R) {
+#ifdef NPP_RC_NO_COMBINE  // measurement variant (wrong results for cut bands): no cross-region combine
+          out[row] = RcOps<T>::finish(s);
+#else
           if (a.gc == 1)
             out[row] = RcOps<T>::finish(s);
           else
             atomicAdd(accR + row, s);  // completed by the row-region ticket at region end
+#endif
         }
       }
       rb ^= 1;
@@ -242,12 +246,20 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       const long long cg = c0 * BC + c;
       if (cg < a.C) {
+#ifdef NPP_RC_NO_COMBINE
+        out[a.R + cg] = RcOps<T>::finish(s);
+#else
         if (a.gr == 1)
           out[a.R + cg] = RcOps<T>::finish(s);
         else
           atomicAdd(accC + cg, s);
+#endif
       }
     }
+#ifdef NPP_RC_NO_COMBINE
+    consumers_sync();
+    continue;
+#endif
     // Split combine (fused): one fence and one ticket per region and direction. The gc
     // column regions of row region ri add their row partials (band ends above), the gr row regions of
     // column group cj their column partials; the last of each converts and re-zeroes.

@@ -8,7 +8,7 @@ for spec in "base:" "$@"; do
   name=${spec%%:*}; flags=${spec#*:}
   lib=build/variants/libnpp_$name.so
   python -m paper_conf_micro_leebsro14_b200.build $flags --out=$lib > /dev/null 2>&1 || { echo "$name build failed"; continue; }
-  NPP_LIB_PATH=$PWD/$lib timeout 300 python bench.py --steps 20 --no-cpu --no-e2e --no-per-config --no-mappings \
+  NPP_LIB_PATH=$PWD/$lib timeout 300 python bench.py --steps 20 --no-cpu --no-e2e --no-per-config --no-mappings ${BENCH_ARGS} \
     > "$O/bench_$name.json" 2> "$O/bench_$name.err"
   python - "$O/bench_$name.json" "$name" >> "$O/sum_variants.log" <<'PY'
 import json, sys
