@@ -265,37 +265,62 @@ __global__ void __launch_bounds__(kThreads, 1)
     // column group cj their column partials; the last of each converts and re-zeroes.
     if (a.gr > 1 || a.gc > 1) {
       consumers_sync();
-      if (threadIdx.x == 0) {  // acq_rel tickets: the release of every consumer's adds (barrier above)
-        bool last_r = false, last_c = false;
+      // acq_rel tickets (the release of every consumer's adds, ordered by the barrier above), the row and
+      // the column ticket taken by two warps at once (their round trips overlap)
+      if (threadIdx.x == 0) {
+        bool last_r = false;
         if (a.gc > 1) {
           last_r = ticket_add(a.tick_r + ri, 1u) + 1u == unsigned(a.gc);
           if (last_r) a.tick_r[ri] = 0u;
         }
+        flag[0] = last_r ? 1 : 0;
+      } else if (threadIdx.x == 32) {
+        bool last_c = false;
         if (a.gr > 1) {
           last_c = ticket_add(a.tick_c + cj, 1u) + 1u == unsigned(a.gr);
           if (last_c) a.tick_c[cj] = 0u;
         }
-        flag[0] = last_r ? 1 : 0;
         flag[1] = last_c ? 1 : 0;
       }
       consumers_sync();
       const bool last_r = flag[0] != 0, last_c = flag[1] != 0;
       if (last_r || last_c) __threadfence();
+      // the conversions issue all of a thread's loads before any store: one L2 round trip, not one per
+      // element (a region has <= 32 * 256 columns: <= 32 per thread; its rows <= kConsumers per pass)
       if (last_r) {
         const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
-        for (long long row = rlo + threadIdx.x; row < rhi; row += kConsumers) {
-          const Acc val = __ldcg(accR + row);
-          __stcg(accR + row, Acc(0));
-          out[row] = RcOps<T>::finish(val);
+        for (long long r0 = rlo; r0 < rhi; r0 += 8 * kConsumers) {
+          Acc val[8];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const long long row = r0 + threadIdx.x + q * kConsumers;
+            val[q] = row < rhi ? __ldcg(accR + row) : Acc(0);
+          }
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const long long row = r0 + threadIdx.x + q * kConsumers;
+            if (row < rhi) {
+              __stcg(accR + row, Acc(0));
+              out[row] = RcOps<T>::finish(val[q]);
+            }
+          }
         }
       }
       if (last_c) {
-        for (long long c = threadIdx.x; c < ncols; c += kConsumers) {
-          const long long cg = c0 * BC + c;
-          if (cg < a.C) {
-            const Acc val = __ldcg(accC + cg);
-            __stcg(accC + cg, Acc(0));
-            out[a.R + cg] = RcOps<T>::finish(val);
+        for (long long cb = 0; cb < ncols; cb += 8 * kConsumers) {
+          Acc val[8];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
+            val[q] = (c < ncols && cg < a.C) ? __ldcg(accC + cg) : Acc(0);
+          }
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
+            if (c < ncols && cg < a.C) {
+              __stcg(accC + cg, Acc(0));
+              out[a.R + cg] = RcOps<T>::finish(val[q]);
+            }
           }
         }
       }
