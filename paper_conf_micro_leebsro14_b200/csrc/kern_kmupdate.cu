@@ -228,12 +228,22 @@ __global__ void __launch_bounds__(kThreads, 1)
     flag[0] = last ? 1 : 0;
   }
   consumers_sync();
-  if (flag[0]) {
+  if (flag[0]) {  // every load of a thread issued before its stores: one L2 round trip per 9 elements
     __threadfence();
-    for (int i = threadIdx.x; i < KD1; i += kConsumers) {
-      const double v = __ldcg(a.acc + i);
-      __stcg(a.acc + i, 0.0);
-      a.out[i] = float(v);
+    constexpr int kQ = (kMaxKD + kMaxK + kConsumers - 1) / kConsumers;  // K*(D+1) <= 2304: <= 9 per thread
+    double v[kQ];
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) {
+      const int i = threadIdx.x + q * kConsumers;
+      v[q] = i < KD1 ? __ldcg(a.acc + i) : 0.0;
+    }
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) {
+      const int i = threadIdx.x + q * kConsumers;
+      if (i < KD1) {
+        __stcg(a.acc + i, 0.0);
+        a.out[i] = float(v[q]);
+      }
     }
   }
 }

@@ -10,7 +10,7 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw,temperature.gpu -
 for step in "$@"; do
   case "$step" in
     tests)
-      timeout 2400 python -m pytest ${PYTEST_PATHS:-tests} -m gpu -q ${PYTEST_ARGS} > "$O/pytest_gpu.log" 2>&1
+      eval "timeout 2400 python -m pytest ${PYTEST_PATHS:-tests} -m gpu -q ${PYTEST_ARGS}" > "$O/pytest_gpu.log" 2>&1
       echo "pytest rc=$?" >> "$O/pytest_gpu.log"; tail -3 "$O/pytest_gpu.log" ;;
     smoke)
       timeout 600 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > "$O/smoke.log" 2>&1
