@@ -222,7 +222,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int j = 0; j < WPG; ++j) s += rsum[(rb * kConsumerWarps + g * WPG + j) * 32 + li];
         const long long row = br * kTileRows + lane;
         if (row < a.R) {
-#ifdef NPP_RC_NO_COMBINE  // measurement variant (wrong results for cut bands): no cross-region combine
+#if defined(NPP_RC_NO_COMBINE) || defined(NPP_RC_NO_ROWRED)  // measurement variants (wrong results)
           out[row] = RcOps<T>::finish(s);
 #else
           if (a.gc == 1)
@@ -246,7 +246,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       const long long cg = c0 * BC + c;
       if (cg < a.C) {
-#ifdef NPP_RC_NO_COMBINE
+#if defined(NPP_RC_NO_COMBINE) || defined(NPP_RC_NO_COLRED)
         out[a.R + cg] = RcOps<T>::finish(s);
 #else
         if (a.gr == 1)
