@@ -283,8 +283,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         flag[1] = last_c ? 1 : 0;
       }
       consumers_sync();
+      // no further fence: the ticket atomics were acq_rel (the acquire of every other region's adds) and the
+      // barrier above orders this block's threads after them; the reads below go to L2 (ld.cg)
       const bool last_r = flag[0] != 0, last_c = flag[1] != 0;
-      if (last_r || last_c) __threadfence();
       // the conversions issue all of a thread's loads before any store: one L2 round trip, not one per
       // element (a region has <= 32 * 256 columns: <= 32 per thread; its rows <= kConsumers per pass)
       if (last_r) {
