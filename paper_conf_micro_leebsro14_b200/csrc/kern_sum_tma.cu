@@ -283,7 +283,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         last = prev + cnt == unsigned(a.Ti);
         if (last) a.tickets[ot] = 0u;
       }
-      if (__any_sync(0xffffffffu, last)) asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      // the lane whose acq_rel ticket completed a tile acquired every contributor's adds; __syncwarp orders
+      // the other lanes (which read the tile's accumulators from L2 below) after that acquire
+      __syncwarp();
       unsigned lasts = __ballot_sync(0xffffffffu, last);
       while (lasts) {  // every contribution to these outer tiles is in: read (L2), convert, re-zero
         const int j = __ffs(lasts) - 1;
