@@ -122,6 +122,17 @@ __device__ __forceinline__ A warp_sum(A v) {
 
 }  // namespace
 
+#ifdef NPP_SUM_STAMPS  // measurement variant: per-block globaltimer stamps of the last 32 launches
+// [launch % 32][block][entry, first tile, consumers' end, combiner's end]; tools/sum_stamps.py reads them
+__device__ unsigned long long g_sum_stamps[32][256][4];
+__device__ unsigned long long g_sum_blocks;
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#endif
+
 // WT: weighted sums (sumWeightedRows / sumWeightedCols, Fig 15) fused: the zipWith
 // product m·v is formed in registers from the staged tile and the tile's slice of v (staged by a 1-D
 // TMA box on the same mbarrier), so no inner allocation exists at all (§V-A taken to its limit).
@@ -166,6 +177,15 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   const long long s0 = ALIGN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
   const long long s1 = ALIGN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
   const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order, then single tiles
+#ifdef NPP_SUM_STAMPS
+  __shared__ unsigned long long* stamp_row;
+  if (threadIdx.x == 0) {
+    const unsigned long long t0 = gtimer();
+    const unsigned long long L = atomicAdd(&g_sum_blocks, 1ull) / (unsigned long long)G;
+    stamp_row = g_sum_stamps[L % 32][bid % 256];
+    stamp_row[0] = t0;
+  }
+#endif
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
@@ -315,6 +335,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       k += n;
       if (ends) break;
     }
+#ifdef NPP_SUM_STAMPS
+    if (lane == 0) stamp_row[3] = gtimer();
+#endif
   } else {
     // ------------------------------------------------------------ consumers
     constexpr int kGroups = ROWS ? 1 : 256 / W;   // MX row groups (1 / 2 for 4- / 8-byte; MX-narrow 4 / 8)
@@ -329,6 +352,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     for (long long t = 0;; ++t) {
       const int slot = int(t % kStages);
       mbar_wait(full + slot, unsigned((t / kStages) & 1));
+#ifdef NPP_SUM_STAMPS
+      if (t == 0 && threadIdx.x == 0) stamp_row[1] = gtimer();
+#endif
       unsigned tag_u = 0;
       if (lane == 0) tag_u = atomicAdd(slot_tile + slot, 0u);
       tag_u = __shfl_sync(0xffffffffu, tag_u, 0);
@@ -481,6 +507,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       ++nfl;
     }
     // end marker for the combiner
+#ifdef NPP_SUM_STAMPS
+    if (threadIdx.x == 0) stamp_row[2] = gtimer();
+#endif
     const int fi = int(nfl % kFlushRing);
     if (nfl >= kFlushRing) mbar_wait(fl_free + fi, unsigned(((nfl / kFlushRing) - 1) & 1));
     __syncwarp();
@@ -490,6 +519,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     }
   }
 }
+
+#ifdef NPP_SUM_STAMPS
+extern "C" __attribute__((visibility("default"))) int npp_debug_sum_stamps(unsigned long long* host) {
+  return int(cudaMemcpyFromSymbol(host, g_sum_stamps, sizeof(g_sum_stamps)));  // 32 x 256 x 4 stamps
+}
+#endif
 
 // ====================================================================================== host side
 namespace {

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--shapes", default="65536x1024,8192x8192,1024x65536")
     ap.add_argument("--patterns", default="SUM_ROWS,SUM_COLS")
     ap.add_argument("--dtype", default="f32")
+    ap.add_argument("--no-pdl", action="store_true", help="NPP_EXEC_NO_PDL launches (isolated kernel timing)")
     args = ap.parse_args()
     dev = torch.device("cuda:0")
     for sh in args.shapes.split(","):
@@ -36,13 +37,13 @@ def main():
             p = npp.Plan(pattern, (R, C), args.dtype, args.strategy)
             out = p.new_out()
             for i in range(3):
-                p.execute([bufs[i % args.nbuf]], out)
+                p.execute([bufs[i % args.nbuf]], out, pdl=not args.no_pdl)
             torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             t0 = time.perf_counter()
             a.record()
             for i in range(args.iters):
-                p.execute([bufs[i % args.nbuf]], out)
+                p.execute([bufs[i % args.nbuf]], out, pdl=not args.no_pdl)
             b.record()
             host_us = (time.perf_counter() - t0) * 1e6 / args.iters
             torch.cuda.synchronize()
@@ -54,7 +55,7 @@ def main():
             with torch.cuda.stream(s):
                 with torch.cuda.graph(g, stream=s):
                     for i in range(args.iters):
-                        p.execute([bufs[i % args.nbuf]], out, stream=s)
+                        p.execute([bufs[i % args.nbuf]], out, stream=s, pdl=not args.no_pdl)
             torch.cuda.synchronize()
             g.replay()
             torch.cuda.synchronize()
