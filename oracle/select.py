@@ -486,9 +486,26 @@ def r2_logreg(nest, lim, dims):
     return blocks, spans, factors, 4, chunks, G, P
 
 
+KM_REGS = 80                                      # DESIGN.md S8 KM: the kernels' register cap
+
+
+def km_sets(K: int, lim) -> int:
+    """DESIGN.md S8 KM: warp sets (256 threads each) taking tiles round robin — 3 when the centroids are
+    one 32-chunk (K <= 32) and a 768-thread block of KM_REGS registers fits, else 2."""
+    fits3 = lim["max_threads_per_block"] >= 768 and 768 * KM_REGS <= lim["regs_per_block"]
+    return 3 if cdiv(K, 32) == 1 and fits3 else 2
+
+
+def km_smem_bytes(K: int, D: int, S: int) -> int:
+    """DESIGN.md S8 KM shared memory: 1 KB alignment pad + 256 B barriers + ||c||² [32⌈K/32⌉] fp32 +
+    exchange words [S sets x (2 if S == 2 else 1) areas][4 groups][TP] x 8 B + a 3-deep ring of 64 KB."""
+    TP = 256 if D <= 64 else 128
+    return 1024 + 256 + 4 * 32 * cdiv(K, 32) + S * (2 if S == 2 else 1) * 4 * TP * 8 + 3 * 65536
+
+
 def r2_kmeans(nest, lim):
     """DESIGN.md S8, KMEANS_ASSIGN staged: TP-point tiles, TP/64 points per thread, 4 centroid groups,
-    two warp sets taking alternate tiles."""
+    km_sets(K) warp sets taking tiles round robin."""
     (N, _), (K, _), (D, _) = nest["levels"]
     if D % 4 != 0 or D < 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384:
         raise Unsupported("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128, K <= 256, Kpad*D <= 16384")
@@ -496,10 +513,14 @@ def r2_kmeans(nest, lim):
     T = cdiv(N, TP)
     P = cdiv(T, min(lim["sm_count"], T))
     G = cdiv(T, P)
-    blocks = (128, 4, 1)                         # two sets of 64 x 4 threads take alternate tiles
+    S = km_sets(K, lim)
+    if (256 * S > lim["max_threads_per_block"] or 256 * S * KM_REGS > lim["regs_per_block"]
+            or km_smem_bytes(K, D, S) > lim["smem_per_block"]):
+        raise Unsupported("KMEANS_ASSIGN AUTO needs a 512-thread block of 80 registers and its shared memory")
+    blocks = (64 * S, 4, 1)                      # S sets of 64 x 4 threads take tiles round robin
     spans = (SPAN_N, ALL, ALL)
     factors = (TP // 64, 1, 1)
-    chunks = (2 * TP, K, D)
+    chunks = (S * TP, K, D)
     return blocks, spans, factors, 4, chunks, G, P
 
 

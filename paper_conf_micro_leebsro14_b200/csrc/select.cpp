@@ -283,9 +283,16 @@ bool r2_kmeans(const Nest& n, const npp_limits& lim, Choice* c) {
   c->persistent_grid = cdiv(T, per_block);
   c->staged = 1;
   c->vec = 4;
-  // two sets of 64 x 4 threads take alternate tiles (ping-pong): y = 128, a block covers 2 tiles at once
-  c->blocks[0] = 128, c->blocks[1] = 4, c->blocks[2] = 1;
-  c->spans[0] = NPP_SPAN_N, c->factors[0] = TP / 64, c->chunks[0] = 2 * TP;
+  // S sets of 64 x 4 threads take tiles round robin: 3 when the centroids are one 32-chunk and a
+  // 768-thread block of kKmRegs registers fits, else 2; a block covers S tiles at once
+  constexpr int64_t kKmRegs = 80;
+  const bool fits3 = lim.max_threads_per_block >= 768 && 768 * kKmRegs <= lim.regs_per_block;
+  const int64_t S = cdiv(K, 32) == 1 && fits3 ? 3 : 2;
+  const int64_t km_smem = 1024 + 256 + 4 * 32 * cdiv(K, 32) + S * (S == 2 ? 2 : 1) * 4 * TP * 8 + 3 * 65536;
+  if (256 * S > lim.max_threads_per_block || 256 * S * kKmRegs > lim.regs_per_block || km_smem > lim.smem_per_block)
+    return false;
+  c->blocks[0] = int(64 * S), c->blocks[1] = 4, c->blocks[2] = 1;
+  c->spans[0] = NPP_SPAN_N, c->factors[0] = TP / 64, c->chunks[0] = S * TP;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = K;
   c->spans[2] = NPP_SPAN_ALL, c->factors[2] = 1, c->chunks[2] = D;
   return true;
@@ -824,7 +831,8 @@ int select_mapping(const Nest& n, int dtype, const npp_limits& lim, int strategy
   }
   if (n.pattern == NPP_KMEANS_ASSIGN) {
     if (!r2_kmeans(n, lim, &c)) {
-      set_error("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128 and K <= 256");
+      set_error("KMEANS_ASSIGN AUTO needs D % 4 == 0, 4 <= D <= 128, K <= 256, 32*ceil(K/32)*D <= 16384 and a "
+                "device that holds its 512-thread (80-register) block and shared memory");
       return NPP_ERR_UNSUPPORTED;
     }
     return record_from_choice(n, dtype, lim, c, sc, out);

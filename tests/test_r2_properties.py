@@ -179,13 +179,23 @@ def test_kmeans_schedules(profile):
     for N, D, K in [(1 << 22, 64, 32), (1000, 4, 1), (257, 64, 256), (4099, 128, 96), (20000, 64, 256),
                     (10, 128, 128), (1, 8, 3), (300000, 68, 33)]:
         rec = _select("KMEANS_ASSIGN", (N, D, K), "f32", lim)
-        if rec is None:  # unsupported shapes, or the hard constraints of a small profile (smem)
+        if rec is None:  # unsupported shapes, or a profile that cannot hold the block (threads, regs, smem)
             assert lim is not S.B200 or D % 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384
+            assert (D % 4 or D > 128 or K > 256 or 32 * cdiv(K, 32) * D > 16384 or lim["max_threads_per_block"] < 512
+                    or lim["smem_per_block"] < S.km_smem_bytes(K, D, 2))
             continue
         TP = 256 if D <= 64 else 128
         T, P, G = cdiv(N, TP), rec["claim_tiles"], rec["grid"]
         assert G <= lim["sm_count"] and G * P >= T > (G - 1) * P
         assert 32 * cdiv(K, 32) * D <= 16384  # the centroid pairs fit the 64 KB constant bank
+        # warp sets: three only when every set reads the same (single) 32-centroid chunk; a block of
+        # S sets x 256 threads covers S tiles at once (TP/64 points per thread)
+        S_ = 3 if K <= 32 and lim["max_threads_per_block"] >= 768 else 2
+        l0 = rec["levels"][0]
+        assert l0["block"] * rec["levels"][1]["block"] == 256 * S_
+        assert l0["chunk"] == S_ * TP == l0["block"] * l0["factor"]
+        assert 256 * S_ * 80 <= lim["regs_per_block"]  # the 80-register cap keeps the block resident
+        assert S.km_smem_bytes(K, D, S_) <= lim["smem_per_block"]
 
 
 @pytest.mark.parametrize("profile", list(PROFILES))
