@@ -519,6 +519,7 @@ int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, v
     k.D = plan->shape[1];
     k.K = plan->shape[2];
     k.per_block = m.claim_tiles;
+    k.sets = m.level[0].block / 64;
     k.trace = trace;
     cudaError_t e = npp::launch_kmeans(k, static_cast<const float*>(ins[0]), int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("kmeans kernel launch", e);

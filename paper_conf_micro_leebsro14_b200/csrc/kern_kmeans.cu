@@ -30,15 +30,19 @@ namespace {
 
 constexpr int kMaxStages = 3;
 constexpr int kBoxCols = 32;  // 128 B of floats: the 128-B swizzle span
-// ping-pong: kSets sets of 8 warps take alternate tiles, so one set's per-tile epilogue (argmin,
-// group combine, set barrier) overlaps the other set's FMA stream
-#ifndef NPP_KM_SETS
-#define NPP_KM_SETS 2
-#endif
-constexpr int kSets = NPP_KM_SETS;
+// ping-pong: SETS sets of 8 warps take tiles round robin, so one set's per-tile epilogue (argmin, group
+// combine, set barrier) overlaps the other sets' FMA streams. Three sets (24 warps, 768 threads at the
+// 80-register cap) when the centroids are one 32-chunk, which all sets read at once from the constant
+// cache; with more chunks the sets sit in different chunks and three of them overrun the constant
+// cache (K = 256: 3x slower), so two. Exchange areas per set: 2 (tile parity, one set barrier per tile)
+// with two sets; 1 with three (shared memory), plus a second set barrier before the words are rewritten.
+template <int SETS>
+struct KmSets {
+  static constexpr int kPar = SETS == 2 ? 2 : 1;
+  static constexpr int kThreads = SETS * 256;  // no producer warp: see the refill below
+};
 constexpr int kConsumerWarps = 8;                 // per set
 constexpr int kConsumers = kConsumerWarps * 32;   // per set
-constexpr int kThreads = kSets * kConsumers;      // no producer warp: see the refill below
 constexpr int kSmemHeader = 256;
 constexpr int kMaxBoxes = 4;  // D <= 128: four 32-float boxes per point row
 constexpr int kMaxStageBytes = 64 * 1024;
@@ -63,17 +67,17 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
 
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
-__host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp) {  // everything but the ring
-  // alignment pad + barriers (full, released) + ||c||² + exchange words
-  // [kSets x 2 parities][4 groups][tp]
-  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(kSets) * 2 * 4 * tp * 8;
+__host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp, int sets) {  // everything but the ring
+  // alignment pad + barriers (full, released) + ||c||² + exchange words [sets x parities][4 groups][tp]
+  const int par = sets == 2 ? 2 : 1;
+  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(sets) * par * 4 * tp * 8;
 }
 // ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
-__host__ __device__ inline int km_stages(int64_t K, int tp) {
-  return km_rest_bytes(K, tp) + 3 * int64_t(kMaxStageBytes) <= kSmemLimit ? 3 : 2;
+__host__ __device__ inline int km_stages(int64_t K, int tp, int sets) {
+  return km_rest_bytes(K, tp, sets) + 3 * int64_t(kMaxStageBytes) <= kSmemLimit ? 3 : 2;
 }
-inline size_t km_smem_bytes(int64_t K, int tp) {
-  return size_t(km_rest_bytes(K, tp) + int64_t(km_stages(K, tp)) * kMaxStageBytes);
+inline size_t km_smem_bytes(int64_t K, int tp, int sets) {
+  return size_t(km_rest_bytes(K, tp, sets) + int64_t(km_stages(K, tp, sets)) * kMaxStageBytes);
 }
 
 // x·c with even/odd dims in the two halves of an f32x2 accumulator
@@ -96,8 +100,9 @@ __device__ __forceinline__ float decode12(unsigned c) { return __uint_as_float(c
 // PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
 // groups; a tile is TP = PPT·256/G points. DT = D when it is known at compile time (the d loop is then
 // unrolled with immediate centroid offsets), 0 for any D.
-template <int PPT, int CPT, int DT>
+template <int PPT, int CPT, int DT, int SETS>
 __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const KmeansArgs& a) {
+  constexpr int kSets = SETS, kPar = KmSets<SETS>::kPar, kThreads = KmSets<SETS>::kThreads;
   const CUtensorMap& map = *mapp;
   constexpr int G = 32 / CPT;
   static_assert(G == 4, "the exchange word packs four centroid groups");
@@ -108,16 +113,16 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   extern __shared__ __align__(1024) unsigned char smem[];
   const int D = DT ? DT : int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
   const int nb = DT ? (DT + kBoxCols - 1) / kBoxCols : km_boxes(a.D);
-  const int kStages = km_stages(a.K, TP);  // ring depth (2 or 3)
+  const int kStages = km_stages(a.K, TP, SETS);  // ring depth (2 or 3)
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
   unsigned char* ring = smem + pad;
   float* cn = reinterpret_cast<float*>(ring + kStages * kMaxStageBytes);  // [Kp] ||c_k||², +inf padded
   // exchange words per (set, tile parity): each group's (best score, {k, margin code, norm code}) per point
-  uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kSets * 2][G][TP]
+  uint2* xch = reinterpret_cast<uint2*>(cn + Kp);  // [kSets * kPar][G][TP]
   // the ring is tracked per 32-float box of a slot, so a box is refilled as soon as the 8 warps of its set
   // are past it (a 64-dim tile frees its first half mid-tile: more lead for the next loads)
-  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * 2 * G * TP);  // [kMaxStages][kMaxBoxes]
+  uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * kPar * G * TP);  // [kMaxStages][kMaxBoxes]
   unsigned* released = reinterpret_cast<unsigned*>(full + kMaxStages * kMaxBoxes);  // [kMaxStages][kMaxBoxes]
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
@@ -353,7 +358,9 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     }
     // the words of tile t into area (set, tile parity); the set's barrier then lets every warp merge
     // its share of the tile (the area is rewritten two tiles later, after the next barrier)
-    const int ar = set * 2 + int((t / kSets) & 1);
+    const int ar = kPar == 2 ? set * 2 + int((t / kSets) & 1) : set;
+    if (kPar == 1 && t >= kSets)  // every warp of the set is done merging the previous words of this area
+      asm volatile("bar.sync %0, %1;" ::"r"(1 + set), "n"(kConsumers) : "memory");
     uint2* ex = xch + (ar * G + g) * TP;
 #pragma unroll
     for (int i = 0; i < PPT; ++i) {
@@ -379,17 +386,20 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #ifndef NPP_KM_MAXNREG_D64X
 #define NPP_KM_MAXNREG_D64X 80
 #endif
+template <int SETS>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
                                                                          KmeansArgs a) {
-  kmeans_body<4, 8, 0>(&map, a);  // D <= 64: 256-point tiles
+  kmeans_body<4, 8, 0, SETS>(&map, a);  // D <= 64: 256-point tiles
 }
+template <int SETS>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64X) npp_kmeans_tma_kernel_d64_exact(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
-  kmeans_body<4, 8, 64>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
+  kmeans_body<4, 8, 64, SETS>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
 }
+template <int SETS>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D128) npp_kmeans_tma_kernel_d128(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
-  kmeans_body<2, 8, 0>(&map, a);  // 64 < D <= 128: 128-point tiles
+  kmeans_body<2, 8, 0, SETS>(&map, a);  // 64 < D <= 128: 128-point tiles
 }
 
 
@@ -402,11 +412,11 @@ namespace {
 std::mutex g_km_mutex;
 cudaEvent_t g_km_done[64] = {};
 
-cudaError_t launch_tp(void (*kern)(const CUtensorMap, KmeansArgs), const CUtensorMap& map, const KmeansArgs& a,
-                      int grid, size_t smem, cudaStream_t st) {
+cudaError_t launch_tp(void (*kern)(const CUtensorMap, KmeansArgs), int threads, const CUtensorMap& map,
+                      const KmeansArgs& a, int grid, size_t smem, cudaStream_t st) {
   cudaError_t e = ensure_smem(kern, int(smem));
   if (e != cudaSuccess) return e;
-  kern<<<grid, kThreads, smem, st>>>(map, a);
+  kern<<<grid, threads, smem, st>>>(map, a);
   return cudaGetLastError();
 }
 
@@ -419,7 +429,9 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   // with 4 centroid groups of 8 (S8)
   const bool small = a.D <= 64;
   const int tp = small ? 256 : 128;
-  const size_t smem = km_smem_bytes(a.K, tp);
+  const int sets = a.sets;  // the record's warp sets (S8 KM): 3 or 2
+  if (sets != 2 && sets != 3) return cudaErrorInvalidValue;
+  const size_t smem = km_smem_bytes(a.K, tp, sets);
   if (km_kpad(a.K) * a.D > kConstFloats) return cudaErrorInvalidValue;  // S8 bound (constant bank)
   CUtensorMap map;
   cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(kBoxCols),
@@ -442,8 +454,13 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   if ((e = cudaGetSymbolAddress(&pack, km_pack_buf)) != cudaSuccess) return e;
   e = cudaMemcpyToSymbolAsync(km_pairs, pack, size_t(Kp) * D * 4, 0, cudaMemcpyDeviceToDevice, st);
   if (e != cudaSuccess) return e;
-  auto kern = a.D == 64 ? npp_kmeans_tma_kernel_d64_exact : small ? npp_kmeans_tma_kernel_d64 : npp_kmeans_tma_kernel_d128;
-  e = launch_tp(kern, map, a, grid, smem, st);
+  auto kern = sets == 3 ? (a.D == 64 ? npp_kmeans_tma_kernel_d64_exact<3>
+                           : small  ? npp_kmeans_tma_kernel_d64<3>
+                                    : npp_kmeans_tma_kernel_d128<3>)
+                        : (a.D == 64 ? npp_kmeans_tma_kernel_d64_exact<2>
+                           : small  ? npp_kmeans_tma_kernel_d64<2>
+                                    : npp_kmeans_tma_kernel_d128<2>);
+  e = launch_tp(kern, sets * 256, map, a, grid, smem, st);
   if (e != cudaSuccess) return e;
   if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);
   return e;

@@ -106,6 +106,7 @@ struct KmeansArgs {
   int* assign;         // [N]
   int64_t N, D, K;
   int64_t per_block;   // P: block b handles TP-point tiles [b*P, (b+1)*P)
+  int sets;            // warp sets of 256 threads taking the block's tiles round robin (record L0 block / 64)
   int* trace;          // npp_execute_traced: [2 x T] block of each tile, loads per tile (else NULL)
 };
 cudaError_t launch_kmeans(const KmeansArgs& a, const float* x, int grid, cudaStream_t st);
