@@ -44,7 +44,10 @@ constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
 constexpr int kMaxKD = 2048;               // DESIGN.md S8 KU: K*D <= 2048, K <= 256
 constexpr int kMaxK = 256;
-constexpr int kFlushTiles = 8;
+#ifndef NPP_KU_FLUSH_TILES  // measurement knob only: the fp32 error bound of DESIGN.md §5 assumes 8
+#define NPP_KU_FLUSH_TILES 8
+#endif
+constexpr int kFlushTiles = NPP_KU_FLUSH_TILES;
 constexpr int kSmemBytes = kHeader + kStages * (kXSlot + kASlot) + kConsumerWarps * kMaxKD * 4 +
                            kConsumerWarps * kMaxK * 4 + (kMaxKD + kMaxK) * 8;
 
@@ -156,6 +159,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     const float* xt = reinterpret_cast<const float*>(xring + slot * kXSlot);
     const int* at = reinterpret_cast<const int*>(aring + slot * kASlot);
     const int np = t + 1 < t1 || t1 * kTP <= a.N ? kTP : int(a.N - t * kTP);  // valid points (TMA zero-fills)
+#ifdef NPP_KU_NO_ACC  // measurement variant (wrong results): the stream without the accumulation
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + slot);
+    continue;
+#endif
     // the warp's 16 points of the tile are p = warp + 8j: lane j < 16 reads key j (-1: no group)
     int kl = -1;
     if (lane < kTP / kConsumerWarps && warp + kConsumerWarps * lane < np) {

@@ -220,7 +220,8 @@ def _check_update(u, x, a, K):
 
 
 @pytest.mark.parametrize("N,D,K", [(1, 4, 1), (127, 8, 3), (129, 64, 32), (3000, 64, 32), (10007, 60, 34),
-                                   (5000, 4, 256), (70000, 16, 128), (200000, 64, 32), (33, 32, 64)])
+                                   (5000, 4, 256), (70000, 16, 128), (200000, 64, 32), (33, 32, 64),
+                                   (100003, 32, 64), (65536, 64, 7), (300, 32, 9)])
 def test_kmeans_update_parity(npp, cuda_device, N, D, K):
     # random keys in [-1, K] (the out-of-range ones belong to no group), ragged last tile, every
     # warp-row / flush boundary; back-to-back executes (plain and PDL-overlapped) leave the workspace zero
@@ -234,6 +235,17 @@ def test_kmeans_update_parity(npp, cuda_device, N, D, K):
     for u in outs:
         _check_update(u, x, a, K)
     assert int(p.workspace.count_nonzero()) == 0
+
+
+@pytest.mark.parametrize("D,K", [(64, 32), (32, 64), (16, 128)])
+def test_kmeans_update_skewed_keys(npp, cuda_device, D, K):
+    # degenerate clusterings: every point in one group, then two groups of 1:1000 size (the key-owner
+    # path puts a whole tile on one warp)
+    N = 70001
+    x, _ = gen.kmeans_inputs(N, D, K, seed=42, device=cuda_device)
+    for a in (torch.full((N,), K - 1, dtype=torch.int32, device=cuda_device),
+              torch.where(gen.int_uniform(43, (N,), 0, 999, device=cuda_device) == 0, 3, K - 2).to(torch.int32)):
+        _check_update(npp.kmeans_update(x, a, K), x, a, K)
 
 
 def test_kmeans_update_integer_exact(npp, cuda_device):
