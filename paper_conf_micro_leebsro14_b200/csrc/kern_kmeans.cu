@@ -41,6 +41,10 @@ struct KmSets {
   static constexpr int kPar = SETS == 2 ? 2 : 1;
   static constexpr int kThreads = SETS * 256;  // no producer warp: see the refill below
 };
+#ifndef NPP_KM_JUNROLL
+#define NPP_KM_JUNROLL 2
+#endif
+constexpr int kJUnroll = NPP_KM_JUNROLL;          // 4-dim steps per iteration of the dims loop
 constexpr int kConsumerWarps = 8;                 // per set
 constexpr int kConsumers = kConsumerWarps * 32;   // per set
 constexpr int kSmemHeader = 256;
@@ -313,7 +317,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         if constexpr (DT != 0) {  // peeled first step (the generic-D path keeps the copies: its uniform
           if (bx == 0) step(j++, std::true_type{});  // datapath does not survive the peel)
         }
-#pragma unroll 2
+#pragma unroll kJUnroll
         for (; j < jn; ++j) step(j, std::false_type{});
         if (kc == 0) {  // the group's quarter of the dims inside this box: its share of ||x||²
           const int lo = max(q0, 8 * bx), hi = min(q1, 8 * bx + jn);
