@@ -36,11 +36,8 @@ constexpr int kBoxCols = 32;  // 128 B of floats: the 128-B swizzle span
 // cache; with more chunks the sets sit in different chunks and three of them overrun the constant
 // cache (K = 256: 3x slower), so two. Exchange areas per set: 2 (tile parity, one set barrier per tile)
 // with two sets; 1 with three (shared memory), plus a second set barrier before the words are rewritten.
-template <int SETS>
-struct KmSets {
-  static constexpr int kPar = SETS == 2 ? 2 : 1;
-  static constexpr int kThreads = SETS * 256;  // no producer warp: see the refill below
-};
+// exchange areas per set: 2 (tile parity) with two sets over several chunks, else 1
+__host__ __device__ constexpr int km_par(int sets, bool one) { return sets == 2 && !one ? 2 : 1; }
 #ifndef NPP_KM_JUNROLL
 #define NPP_KM_JUNROLL 2
 #endif
@@ -71,17 +68,36 @@ __global__ void npp_kmeans_pack_kernel(const float* __restrict__ c, int K, int K
 
 __host__ __device__ inline int64_t km_kpad(int64_t K) { return (K + 31) / 32 * 32; }
 __host__ __device__ inline int km_boxes(int64_t D) { return int((D + kBoxCols - 1) / kBoxCols); }
-__host__ __device__ inline int64_t km_rest_bytes(int64_t K, int tp, int sets) {  // everything but the ring
+// shared-memory pairs: LDSP of each thread's 4 pairs per 32-chunk come from a shared-memory copy
+// (csm[chunk][d][group][LS] float2, LS = LDSP rounded up to a power of two), the rest from the constant
+// bank, so the two operand paths share the load: in the bare dims loop the LDCU stream alone caps FFMA2
+// at ~0.63-0.69 of peak, the LDS broadcast alone at ~0.74, half and half at ~0.82 (profiles/r02/kmeans/
+// micro_inner.log). In the full kernels it pays only where registers are left for the extra operands:
+// the D > 64 kernel (2 pairs with three sets, 1 with two); the D <= 64 kernels at the 80-register cap
+// are fastest with every pair from the constant bank (profiles/r02/kmeans/lds_pairs.log).
+__host__ __device__ constexpr int km_ls(int ldsp) { return ldsp == 0 ? 0 : ldsp == 1 ? 1 : ldsp == 2 ? 2 : 4; }
+__host__ __device__ inline int64_t km_csm_bytes(int64_t K, int64_t D, int ldsp) {
+  return km_kpad(K) * D * km_ls(ldsp);  // (Kp/32) chunks x D x 4 groups x LS pairs x 8 B
+}
+__host__ __device__ inline int64_t km_rest_bytes(int64_t K, int64_t D, int tp, int sets, bool one, int ldsp) {
   // alignment pad + barriers (full, released) + ||c||² + exchange words [sets x parities][4 groups][tp]
-  const int par = sets == 2 ? 2 : 1;
-  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(sets) * par * 4 * tp * 8;
+  // + the shared-memory pairs
+  const int par = km_par(sets, one);
+  return 1024 + kSmemHeader + km_kpad(K) * 4 + int64_t(sets) * par * 4 * tp * 8 + km_csm_bytes(K, D, ldsp);
 }
-// ring depth: 3 x 64 KB tiles when they fit (always, with the centroids out of shared memory)
-__host__ __device__ inline int km_stages(int64_t K, int tp, int sets) {
-  return km_rest_bytes(K, tp, sets) + 3 * int64_t(kMaxStageBytes) <= kSmemLimit ? 3 : 2;
+// ring depth: 3 x 64 KB tiles when they fit
+__host__ __device__ inline int km_stages(int64_t K, int64_t D, int tp, int sets, bool one, int ldsp) {
+  return km_rest_bytes(K, D, tp, sets, one, ldsp) + 3 * int64_t(kMaxStageBytes) <= kSmemLimit ? 3 : 2;
 }
-inline size_t km_smem_bytes(int64_t K, int tp, int sets) {
-  return size_t(km_rest_bytes(K, tp, sets) + int64_t(km_stages(K, tp, sets)) * kMaxStageBytes);
+inline size_t km_smem_bytes(int64_t K, int64_t D, int tp, int sets, bool one, int ldsp) {
+  return size_t(km_rest_bytes(K, D, tp, sets, one, ldsp) +
+                int64_t(km_stages(K, D, tp, sets, one, ldsp)) * kMaxStageBytes);
+}
+// the shared-memory pairs of a launch: the kernel's choice where it leaves the 3-deep ring in place,
+// else none (every pair from the constant bank)
+inline int km_ldsp(int64_t K, int64_t D, int tp, int sets, bool one) {
+  const int want = D <= 64 ? 0 : sets == 3 ? 2 : 1;
+  return want > 0 && km_stages(K, D, tp, sets, one, want) == 3 ? want : 0;
 }
 
 // x·c with even/odd dims in the two halves of an f32x2 accumulator
@@ -104,9 +120,9 @@ __device__ __forceinline__ float decode12(unsigned c) { return __uint_as_float(c
 // PPT points per thread, CPT centroids per thread and 32-chunk; G = 32/CPT warp-uniform centroid
 // groups; a tile is TP = PPT·256/G points. DT = D when it is known at compile time (the d loop is then
 // unrolled with immediate centroid offsets), 0 for any D.
-template <int PPT, int CPT, int DT, int SETS>
+template <int PPT, int CPT, int DT, int SETS, int LDSP, bool ONE>
 __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const KmeansArgs& a) {
-  constexpr int kSets = SETS, kPar = KmSets<SETS>::kPar, kThreads = KmSets<SETS>::kThreads;
+  constexpr int kSets = SETS, kPar = km_par(SETS, ONE), kThreads = SETS * 256;  // no producer warp (refill below)
   const CUtensorMap& map = *mapp;
   constexpr int G = 32 / CPT;
   static_assert(G == 4, "the exchange word packs four centroid groups");
@@ -117,7 +133,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   extern __shared__ __align__(1024) unsigned char smem[];
   const int D = DT ? DT : int(a.D), K = int(a.K), Kp = int(km_kpad(a.K));
   const int nb = DT ? (DT + kBoxCols - 1) / kBoxCols : km_boxes(a.D);
-  const int kStages = km_stages(a.K, TP, SETS);  // ring depth (2 or 3)
+  constexpr int LS = km_ls(LDSP);
+  const int kStages = km_stages(a.K, D, TP, SETS, ONE, LDSP);  // ring depth (2 or 3)
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
   unsigned char* ring = smem + pad;
@@ -128,6 +145,8 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   // are past it (a 64-dim tile frees its first half mid-tile: more lead for the next loads)
   uint64_t* full = reinterpret_cast<uint64_t*>(xch + kSets * kPar * G * TP);  // [kMaxStages][kMaxBoxes]
   unsigned* released = reinterpret_cast<unsigned*>(full + kMaxStages * kMaxBoxes);  // [kMaxStages][kMaxBoxes]
+  // shared-memory pairs [Kp/32][D][4 groups][LS] (16-byte aligned: the header is 256 B)
+  float2* csm = reinterpret_cast<float2*>(reinterpret_cast<unsigned char*>(full) + kSmemHeader);
 
   // warp index broadcast from lane 0: ptxas then knows the split is warp-uniform and may use the
   // uniform datapath (LDCU) for the centroid reads after it
@@ -150,6 +169,15 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     if (k < K)
       for (int d = 0; d < D; ++d) s = fmaf(__ldg(a.c + k * D + d), __ldg(a.c + k * D + d), s);
     cn[k] = k < K ? s : __int_as_float(0x7f800000);
+  }
+  if constexpr (LDSP > 0) {  // pair m < LDSP of group g in chunk ch at dim d: pair (16 ch + 4 g + m) at d
+    const int n = Kp / 32 * D * 4 * LS;
+    for (int i = threadIdx.x; i < n; i += kThreads) {
+      const int m = i % LS, gg = (i / LS) % 4, d = (i / (4 * LS)) % D, ch = i / (4 * LS * D);
+      // from the launch's staging copy (the constant bank's source), not the bank: per-thread constant
+      // reads would leave the uniform datapath
+      csm[i] = m < LDSP ? km_pack_buf[(16 * ch + 4 * gg + m) * D + d] : make_float2(0.f, 0.f);
+    }
   }
   __syncthreads();
   // near-tie bound (DESIGN.md §5 k-means): every fp32 score s_k = fl(||c_k||² − 2 x·c_k) is within
@@ -267,8 +295,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
     int bk[PPT];
     float2 n2[PPT];  // the group's share of ||x||² (even / odd dims)
 #pragma unroll
-    for (int i = 0; i < PPT; ++i) bs[i] = s2[i] = __int_as_float(0x7f800000), bk[i] = 0, n2[i] = make_float2(0.f, 0.f);
-    for (int kc = 0; kc < Kp; kc += 32) {
+    for (int i = 0; i < PPT; ++i) n2[i] = make_float2(0.f, 0.f);
+    // ONE: the centroids are one 32-chunk (always with three sets, S8 KM): the chunk loop then
+    // runs once at compile time, and the argmin state is born after the dims loop (fewer live registers)
+    constexpr bool kOneChunk = ONE;
+    for (int kc = 0; kc < (kOneChunk ? 32 : Kp); kc += 32) {
       const int k0 = kc + g * CPT;  // the thread's first centroid of the chunk
       const bool last_chunk = kc + 32 >= Kp;
       float2 acc[PPT][CPT / 2];  // .x: centroid k0 + 2p, .y: k0 + 2p + 1; starts at (||c||², ||c'||²)
@@ -282,6 +313,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
           for (int p = 0; p < CPT / 2; ++p) acc[i][p] = nkp[p];
       }
       const float2* cq = km_pairs + (k0 >> 1) * D;  // pairs of −2c: the chain ends at the score
+      const float2* cs = csm + ((kc / 32) * D * 4 + g) * LS;  // + d·4·LS + m: the shared-memory pairs
 #pragma unroll 1
       for (int bx = 0; bx < nb; ++bx) {
         uint64_t* fb = full + slot * kMaxBoxes + bx;
@@ -296,10 +328,27 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #pragma unroll
           for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(xb + LP * 128 * i);
 #pragma unroll
-          for (int p = 0; p < CPT / 2; ++p) {
+          for (int q = 0; q < 4; ++q) {
+            float2 cvs[CPT / 2];  // warp-uniform: broadcast LDS for p < LDSP, LDCU for the rest
+            const float2* cd = cs + (4 * d4 + q) * 4 * LS;
+            if constexpr (LS == 1) {
+              cvs[0] = cd[0];
+            } else if constexpr (LS >= 2) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              const float2 cv = cq[p * D + 4 * d4 + q];  // warp-uniform
+              for (int m = 0; m < LDSP; m += 2) {
+                if (m + 1 < LDSP) {
+                  const float4 c4 = *reinterpret_cast<const float4*>(cd + m);
+                  cvs[m] = make_float2(c4.x, c4.y), cvs[m + 1] = make_float2(c4.z, c4.w);
+                } else {
+                  cvs[m] = cd[m];
+                }
+              }
+            }
+#pragma unroll
+            for (int p = LDSP; p < CPT / 2; ++p) cvs[p] = cq[p * D + 4 * d4 + q];
+#pragma unroll
+            for (int p = 0; p < CPT / 2; ++p) {
+              const float2 cv = cvs[p];
 #pragma unroll
               for (int i = 0; i < PPT; ++i) {
                 const float xs = q == 0 ? xv[i].x : q == 1 ? xv[i].y : q == 2 ? xv[i].z : xv[i].w;
@@ -346,6 +395,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
           }
         }
       }
+      if (kc == 0) {
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) bs[i] = s2[i] = __int_as_float(0x7f800000), bk[i] = 0;
+      }
 #pragma unroll
       for (int p = 0; p < CPT / 2; ++p) {  // increasing k within the thread: strict < keeps the first
 #pragma unroll
@@ -390,22 +443,21 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
 #ifndef NPP_KM_MAXNREG_D64X
 #define NPP_KM_MAXNREG_D64X 80
 #endif
-template <int SETS>
+template <int SETS, int LDSP>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64) npp_kmeans_tma_kernel_d64(const __grid_constant__ CUtensorMap map,
                                                                          KmeansArgs a) {
-  kmeans_body<4, 8, 0, SETS>(&map, a);  // D <= 64: 256-point tiles
+  kmeans_body<4, 8, 0, SETS, LDSP, SETS == 3>(&map, a);  // D <= 64: 256-point tiles
 }
-template <int SETS>
+template <int SETS, int LDSP>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D64X) npp_kmeans_tma_kernel_d64_exact(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
-  kmeans_body<4, 8, 64, SETS>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
+  kmeans_body<4, 8, 64, SETS, LDSP, SETS == 3>(&map, a);  // D = 64 (BASELINE.json config 4): immediate centroid offsets
 }
-template <int SETS>
+template <int SETS, int LDSP>
 __global__ void __maxnreg__(NPP_KM_MAXNREG_D128) npp_kmeans_tma_kernel_d128(
     const __grid_constant__ CUtensorMap map, KmeansArgs a) {
-  kmeans_body<2, 8, 0, SETS>(&map, a);  // 64 < D <= 128: 128-point tiles
+  kmeans_body<2, 8, 0, SETS, LDSP, SETS == 3>(&map, a);  // 64 < D <= 128: 128-point tiles
 }
-
 
 namespace {
 
@@ -435,7 +487,10 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   const int tp = small ? 256 : 128;
   const int sets = a.sets;  // the record's warp sets (S8 KM): 3 or 2
   if (sets != 2 && sets != 3) return cudaErrorInvalidValue;
-  const size_t smem = km_smem_bytes(a.K, tp, sets);
+  if (sets == 3 && km_kpad(a.K) != 32) return cudaErrorInvalidValue;  // three sets: one 32-chunk (S8 KM)
+  const bool one = sets == 3;  // the kernels' ONE (compile-time single chunk)
+  const int ldsp = km_ldsp(a.K, a.D, tp, sets, one);  // shared-memory pairs (D > 64 kernel only)
+  const size_t smem = km_smem_bytes(a.K, a.D, tp, sets, one, ldsp);
   if (km_kpad(a.K) * a.D > kConstFloats) return cudaErrorInvalidValue;  // S8 bound (constant bank)
   CUtensorMap map;
   cudaError_t e = tma::encode_2d(&map, x, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.N, a.D, unsigned(kBoxCols),
@@ -458,12 +513,10 @@ cudaError_t launch_kmeans(const KmeansArgs& args, const float* x, int grid, cuda
   if ((e = cudaGetSymbolAddress(&pack, km_pack_buf)) != cudaSuccess) return e;
   e = cudaMemcpyToSymbolAsync(km_pairs, pack, size_t(Kp) * D * 4, 0, cudaMemcpyDeviceToDevice, st);
   if (e != cudaSuccess) return e;
-  auto kern = sets == 3 ? (a.D == 64 ? npp_kmeans_tma_kernel_d64_exact<3>
-                           : small  ? npp_kmeans_tma_kernel_d64<3>
-                                    : npp_kmeans_tma_kernel_d128<3>)
-                        : (a.D == 64 ? npp_kmeans_tma_kernel_d64_exact<2>
-                           : small  ? npp_kmeans_tma_kernel_d64<2>
-                                    : npp_kmeans_tma_kernel_d128<2>);
+  auto kern = a.D == 64 ? (sets == 3 ? npp_kmeans_tma_kernel_d64_exact<3, 0> : npp_kmeans_tma_kernel_d64_exact<2, 0>)
+              : small    ? (sets == 3 ? npp_kmeans_tma_kernel_d64<3, 0> : npp_kmeans_tma_kernel_d64<2, 0>)
+              : sets == 3 ? (ldsp ? npp_kmeans_tma_kernel_d128<3, 2> : npp_kmeans_tma_kernel_d128<3, 0>)
+                          : (ldsp ? npp_kmeans_tma_kernel_d128<2, 1> : npp_kmeans_tma_kernel_d128<2, 0>);
   e = launch_tp(kern, sets * 256, map, a, grid, smem, st);
   if (e != cudaSuccess) return e;
   if (cap == cudaStreamCaptureStatusNone) e = cudaEventRecord(g_km_done[dev], st);

@@ -90,7 +90,8 @@ def test_kmeans_integer_data_exact(npp, cuda_device, N, D, K):
     assert a.cpu().numpy().tolist() == okm.assign(x.cpu().numpy(), c.cpu().numpy()).tolist()
 
 
-@pytest.mark.parametrize("N,D,K", [(50000, 64, 32), (3000, 16, 7), (20000, 128, 128), (7777, 4, 3)])
+@pytest.mark.parametrize("N,D,K", [(50000, 64, 32), (3000, 16, 7), (20000, 128, 128), (7777, 4, 3), (9000, 96, 32),
+                                   (4097, 72, 20), (6000, 100, 64)])
 def test_kmeans_random_data_exact(npp, cuda_device, N, D, K):
     x, c = gen.kmeans_inputs(N, D, K, device=cuda_device)
     p = npp.Plan("KMEANS_ASSIGN", (N, D, K), "f32", "AUTO")
