@@ -20,8 +20,10 @@ __device__ __forceinline__ void ffma2(float2& acc, const float2 a, const float2 
   acc = *reinterpret_cast<float2*>(&C);
 }
 
-template <int PPT, int CPT, int LP, int WARPS, int CSRC, int UNR>
-__global__ void __launch_bounds__(WARPS * 32) k_inner(float* out, int tiles) {
+// XW: x operands per point and load — 4 (one LDS.128 per 4-dim step, the kernel's form) or 1 / 2 (LDS.32 /
+// LDS.64 per dim / dim pair, fewer live x registers); MAXR: the register cap (255 = none)
+template <int PPT, int CPT, int LP, int WARPS, int CSRC, int UNR, int XW, int MAXR>
+__global__ void __maxnreg__(MAXR) k_inner(float* out, int tiles) {
   extern __shared__ __align__(1024) unsigned char smem[];
   constexpr int G = 32 / CPT, NP = CPT / 2, TP = PPT * LP;
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);
@@ -50,10 +52,27 @@ __global__ void __launch_bounds__(WARPS * 32) k_inner(float* out, int tiles) {
       for (int j = 0; j < 8; ++j) {
         const int d4 = 8 * bx + j;
         float4 xv[PPT];
+        if constexpr (XW == 4) {
 #pragma unroll
-        for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(tb + LP * 128 * i + ((unsigned(j) << 4) ^ key4));
+          for (int i = 0; i < PPT; ++i) xv[i] = *reinterpret_cast<const float4*>(tb + LP * 128 * i + ((unsigned(j) << 4) ^ key4));
+        }
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
+          if constexpr (XW == 1) {
+#pragma unroll
+            for (int i = 0; i < PPT; ++i) {
+              const float v = *reinterpret_cast<const float*>(tb + LP * 128 * i + ((unsigned(j) << 4) ^ key4) + 4 * q);
+              xv[i] = make_float4(v, v, v, v);
+            }
+          } else if constexpr (XW == 2) {
+            if ((q & 1) == 0) {
+#pragma unroll
+              for (int i = 0; i < PPT; ++i) {
+                const float2 v = *reinterpret_cast<const float2*>(tb + LP * 128 * i + ((unsigned(j) << 4) ^ key4) + 4 * q);
+                xv[i] = make_float4(v.x, v.y, v.x, v.y);
+              }
+            }
+          }
           float2 cv[NP];
           if constexpr (CSRC == 0) {
 #pragma unroll
@@ -94,9 +113,9 @@ __global__ void __launch_bounds__(WARPS * 32) k_inner(float* out, int tiles) {
   if (best == 1.2345f) out[0] = best;
 }
 
-template <int PPT, int CPT, int LP, int WARPS, int CSRC, int UNR = 2>
+template <int PPT, int CPT, int LP, int WARPS, int CSRC, int UNR = 2, int XW = 4, int MAXR = 255>
 void run(float* out, int sms, const char* name) {
-  auto kern = k_inner<PPT, CPT, LP, WARPS, CSRC, UNR>;
+  auto kern = k_inner<PPT, CPT, LP, WARPS, CSRC, UNR, XW, MAXR>;
   const int smem = PPT * LP * D * 4 + 16 * D * 8;
   cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   int per_sm = 0;
@@ -131,25 +150,18 @@ int main() {
   for (int i = 0; i < 16 * D; ++i) h[i] = make_float2(0.001f * (i % 31), -0.002f * (i % 17));
   cudaMemcpyToSymbol(cp, h, sizeof(h));
   for (int rep = 0; rep < 2; ++rep) {
+    // run 3 (profiles/r02/kmeans/micro_inner.log): thread tile and centroid source, no register cap
     run<4, 8, 64, 8, 0>(out, sms, "P4 C8 LP64 8w LDCU");
     run<4, 8, 64, 8, 2>(out, sms, "P4 C8 LP64 8w LDS");
     run<4, 8, 64, 8, 4>(out, sms, "P4 C8 LP64 8w hybrid");
     run<4, 8, 64, 8, 3>(out, sms, "P4 C8 LP64 8w regs");
-    run<4, 16, 64, 4, 0>(out, sms, "P4 C16 LP64 4w LDCU");
-    run<4, 16, 64, 4, 2>(out, sms, "P4 C16 LP64 4w LDS");
     run<4, 16, 64, 4, 4>(out, sms, "P4 C16 LP64 4w hybrid");
-    run<4, 16, 64, 4, 3>(out, sms, "P4 C16 LP64 4w regs");
-    run<4, 16, 32, 2, 2>(out, sms, "P4 C16 LP32 2w LDS");
-    run<4, 16, 32, 2, 4>(out, sms, "P4 C16 LP32 2w hybrid");
-    run<4, 16, 64, 8, 2>(out, sms, "P4 C16 LP64 8w(dup) LDS");
-    run<2, 16, 64, 8, 2>(out, sms, "P2 C16 LP64 8w(dup) LDS");
-    run<2, 16, 64, 8, 4>(out, sms, "P2 C16 LP64 8w(dup) hybrid");
-    run<8, 8, 32, 4, 2>(out, sms, "P8 C8 LP32 4w LDS");
-    run<8, 8, 32, 4, 4>(out, sms, "P8 C8 LP32 4w hybrid");
-    run<8, 16, 32, 2, 2>(out, sms, "P8 C16 LP32 2w LDS");
-    run<8, 16, 32, 2, 3>(out, sms, "P8 C16 LP32 2w regs");
-    run<4, 16, 64, 4, 2, 1>(out, sms, "P4 C16 LP64 4w LDS u1");
-    run<4, 16, 64, 4, 2, 4>(out, sms, "P4 C16 LP64 4w LDS u4");
+    // runs 4-5: 8 points per thread under a register cap (ptxas keeps LDCU), 24 and 12 warps per SM
+    run<4, 8, 64, 8, 0, 2, 4, 80>(out, sms, "P4 C8 LP64 8w LDCU cap80");
+    run<8, 8, 32, 8, 0, 2, 2, 80>(out, sms, "P8 C8 LP32 8w LDCU xw2 u2 cap80");
+    run<8, 8, 32, 8, 0, 1, 4, 80>(out, sms, "P8 C8 LP32 8w LDCU xw4 u1 cap80");
+    run<8, 8, 32, 4, 0, 2, 4, 96>(out, sms, "P8 C8 LP32 4w LDCU xw4 u2 cap96");
+    run<8, 8, 32, 4, 0, 4, 4, 128>(out, sms, "P8 C8 LP32 4w LDCU xw4 u4 cap128");
   }
   return 0;
 }
