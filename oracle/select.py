@@ -444,10 +444,15 @@ def r2_rowscols(nest, dtype, lim):
 
 
 def r2_pagerank(nest, lim):
-    """DESIGN.md S8 PR: V = min(32, pow2 >= ceil(ceil(E/N)/2)) lanes per row on x, 256/V row groups on y, rows
-    claimed by warps in chunks of 4*32/V; min(4*SMs, chunks) blocks. Returns (dims, blocks, spans, factors,
-    vec, chunks, G, chunk)."""
+    """DESIGN.md S8 PR: mean in-degree m = ceil(E/N). m >= 8 (segmented): warps claim chunks of 31 rows, the
+    chunk's edges split over 32 lanes (Split), min(8*SMs, chunks) blocks. m < 8 (row groups): V = min(32,
+    pow2 >= ceil(m/4)) lanes per row on x, 256/V row groups on y, warp claims of 4*32/V rows, min(4*SMs,
+    chunks) blocks. Returns (dims, blocks, spans, factors, vec, chunks, G, chunk)."""
     (N, _), (inner, _) = nest["levels"]
+    if inner >= 8:                                 # segmented: 8 warps x 32 lanes, 31 rows per claim
+        chunk = 31
+        G = min(8 * lim["sm_count"], cdiv(N, chunk))
+        return (Y, X), (8, 32), (SPAN_N, SPLIT), (chunk, 32), 1, (chunk, inner), G, chunk
     V = min(32, pow2ceil(cdiv(inner, 4)))          # four edges per lane for a row of average length
     RPB = 256 // V
     chunk = 4 * (32 // V)                          # a warp's claim: 4 rows per group

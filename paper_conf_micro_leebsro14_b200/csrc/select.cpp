@@ -391,16 +391,25 @@ bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
 // S8 PAGERANK (class PR): V = min(32, pow2 >= ceil(ceil(E/N)/2)) lanes per row on x, 256/V row groups on y,
 // rows claimed by warps in chunks of 4*32/V; min(4*SMs, chunks) blocks.
 void r2_pagerank(const Nest& n, const npp_limits& lim, Choice* c) {
-  const int64_t N = n.N[0], inner = n.N[1];
+  const int64_t N = n.N[0], inner = n.N[1];  // inner = mean in-degree ceil(E/N)
+  c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
+  c->vec = 1;
+  c->staged = 0;
+  if (inner >= 8) {  // segmented: warps claim 31 rows, the chunk's edges split over 32 lanes
+    const int64_t chunk = 31;
+    c->blocks[0] = 8, c->blocks[1] = 32;
+    c->spans[0] = NPP_SPAN_N, c->factors[0] = chunk, c->chunks[0] = chunk;
+    c->spans[1] = NPP_SPLIT_K, c->factors[1] = 32, c->chunks[1] = inner;
+    c->persistent_grid = std::min<int64_t>(8 * int64_t(lim.sm_count), cdiv(N, chunk));  // 8 x 256 threads per SM
+    c->claim_tiles = chunk;
+    return;
+  }
   const int64_t V = std::min<int64_t>(32, pow2ceil(cdiv(inner, 4)));  // four edges per lane on average
   const int64_t RPB = 256 / V, chunk = 4 * (32 / V);  // a warp's claim: 4 rows per group
   const int64_t units = cdiv(N, chunk);
-  c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
   c->blocks[0] = int(RPB), c->blocks[1] = int(V);
   c->spans[0] = NPP_SPAN_N, c->factors[0] = 4, c->chunks[0] = chunk;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = inner;
-  c->vec = 1;
-  c->staged = 0;
   c->persistent_grid = std::min<int64_t>(4 * int64_t(lim.sm_count), units);  // 4 x 256 threads per SM
   c->claim_tiles = chunk;
 }

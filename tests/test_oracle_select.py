@@ -246,12 +246,18 @@ def test_kmeans_update_record_by_hand():
 
 
 def test_pagerank_record_by_hand():
-    # mean in-degree ceil(63710769 / 4194304) = 16 -> V = pow2 >= 16/4 = 4 lanes per row, 64 row groups
-    # per block, warp claims of 4 rows x 8 groups = 32 rows, min(4 x 148, 131072) = 592 blocks;
-    # workspace = claim counter + contrib [4M] f32
+    # mean in-degree ceil(63710769 / 4194304) = 16 >= 8 -> segmented: 8 warps x 32 lanes, warp claims of 31
+    # rows (ceil(4M / 31) = 135301 chunks), the chunk's edges Split over 32 lanes, min(8 x 148, 135301) =
+    # 1184 blocks; workspace = claim counter + contrib [4M] f32
     rec = S.select("PAGERANK", (1 << 22, 63710769), "f32", S.B200, "AUTO")
     assert rec["kernel_class"] == S.PR and rec["staged"] == 0
-    assert [lv["block"] for lv in rec["levels"]] == [64, 4]
-    assert rec["levels"][0]["chunk"] == 32 and rec["levels"][0]["grid"] == (1 << 22) // 32
-    assert rec["grid"] == 592 and rec["levels"][1]["chunk"] == 16
+    assert [lv["block"] for lv in rec["levels"]] == [8, 32]
+    assert [lv["span"] for lv in rec["levels"]] == [S.SPAN_N, S.SPLIT]
+    assert rec["levels"][0]["chunk"] == 31 and rec["levels"][0]["grid"] == -(-(1 << 22) // 31)
+    assert rec["grid"] == 1184 and rec["claim_tiles"] == 31 and rec["levels"][1]["chunk"] == 16
     assert rec["workspace_bytes"] == 256 + 4 * (1 << 22)
+    # mean in-degree 4 < 8 -> row groups: V = pow2 >= 4/4 = 1 lane per row, 256 row groups per block,
+    # warp claims of 4 rows x 32 groups = 128 rows, min(4 x 148, 32768) = 592 blocks
+    rec = S.select("PAGERANK", (1 << 22, 16443020), "f32", S.B200, "AUTO")
+    assert [lv["block"] for lv in rec["levels"]] == [256, 1] and rec["levels"][1]["span"] == S.ALL
+    assert rec["levels"][0]["chunk"] == 128 and rec["grid"] == 592 and rec["claim_tiles"] == 128

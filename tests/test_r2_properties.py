@@ -242,7 +242,14 @@ def test_pagerank_schedules(profile):
         N = shape[0]
         V = rec["levels"][1]["block"]
         chunk = rec["claim_tiles"]
-        assert V & (V - 1) == 0 and 1 <= V <= 32 and chunk == 4 * (32 // V)
-        assert rec["grid"] <= 4 * lim["sm_count"] and rec["grid"] * chunk >= min(N, rec["grid"] * chunk)
+        m = rec["levels"][1]["chunk"]  # mean in-degree ceil(E/N)
+        if m >= 8:  # segmented: 32 lanes split a chunk of 31 rows' edges; lane i of a claim holds row i
+            assert rec["levels"][1]["span"] == S.SPLIT and V == 32 and rec["levels"][0]["block"] == 8
+            assert chunk == 31 and chunk < 32 and rec["grid"] <= 8 * lim["sm_count"]
+        else:
+            assert rec["levels"][1]["span"] == S.ALL
+            assert V & (V - 1) == 0 and 1 <= V <= 32 and chunk == 4 * (32 // V)
+            assert rec["grid"] <= 4 * lim["sm_count"]
+        assert rec["grid"] == min(rec["grid"], -(-N // chunk)) and (N == 0 or rec["grid"] >= 1)
         nodes = shape[2] if len(shape) == 3 else shape[0]
         assert rec["workspace_bytes"] >= 256 + 4 * nodes
