@@ -537,7 +537,8 @@ int execute_impl(npp_plan_t plan, const void* const* ins, int n_in, void* out, v
     r.N = plan->shape[0];
     r.Nnodes = plan->ndim == 3 ? plan->shape[2] : plan->shape[0];
     r.damp = 0.85f;
-    cudaError_t e = npp::launch_pagerank(r, m.level[1].block, int(m.grid), st);
+    const int seg = m.level[1].span == NPP_SPLIT_K ? int(m.claim_tiles) : 0;  // S8 PR: segmented or row groups
+    cudaError_t e = npp::launch_pagerank(r, m.level[1].block, seg, int(m.grid), st);
     if (e != cudaSuccess) return cuda_fail("PageRank kernel launch", e);
     return NPP_OK;
   }

@@ -174,6 +174,7 @@ struct PagerankArgs {
   int64_t Nnodes;   // nodes of the graph: length of pr / outdeg / contrib, and the N of (1-damp)/N
   float damp;
 };
-cudaError_t launch_pagerank(const PagerankArgs& a, int V, int grid, cudaStream_t st);
+// V: lanes per row (row-group mapping); seg_rows > 0: the segmented mapping with that many rows per claim
+cudaError_t launch_pagerank(const PagerankArgs& a, int V, int seg_rows, int grid, cudaStream_t st);
 
 }  // namespace npp

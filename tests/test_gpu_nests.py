@@ -349,6 +349,29 @@ def test_pagerank_edge_cases(npp, cuda_device):
         assert e.value.status == npp.ERR_UNSUPPORTED
 
 
+def test_pagerank_segmented_row_structure(npp, cuda_device):
+    # the segmented mapping (mean in-degree >= 8, S8 PR): empty rows between non-empty ones,
+    # rows ending exactly on a 32-edge batch boundary, rows longer than a claim's 8 batches, a claim whose
+    # rows are all empty, and a row count that is not a multiple of 31
+    degs = ([0, 0, 37, 1, 0, 64, 5, 0, 32, 31, 33, 1000, 0] * 40 + [0] * 31 + [2000, 1, 0, 95] * 3)[:611]
+    N = len(degs)
+    rowptr = torch.tensor([0] + list(np.cumsum(degs)), dtype=torch.int64, device=cuda_device)
+    E = int(rowptr[-1])
+    colidx = gen.int_uniform(11, (E,), 0, N - 1, device=cuda_device)
+    pr = gen.uniform_f32(12, (N,), device=cuda_device, lo=0.5)
+    outdeg = torch.bincount(colidx.long(), minlength=N).clamp(min=1).to(torch.int32)
+    p = npp.Plan("PAGERANK", (N, E))
+    assert p.mapping["levels"][1]["span"] == osel.SPLIT and p.mapping["claim_tiles"] == 31
+    out = p.execute([rowptr, colidx, pr, outdeg], p.new_out())
+    torch.cuda.synchronize()
+    _check_pr(out, rowptr, colidx, pr, outdeg)
+    assert int(p.workspace[:256].count_nonzero()) == 0
+    # mean in-degree < 8: the row-group mapping
+    rowptr, colidx, pr, outdeg = gen.pagerank_inputs(5000, avg_deg=3, seed=3, max_deg=64, device=cuda_device)
+    p = npp.Plan("PAGERANK", (5000, colidx.numel()))
+    assert p.mapping["levels"][1]["span"] == osel.ALL
+
+
 def test_pagerank_full_size(npp, cuda_device):
     # the bench workload: 4M nodes, power-law in-degrees (mean ~16, cap 1024), ~63M edges
     rowptr, colidx, pr, outdeg = gen.pagerank_inputs(1 << 22, avg_deg=16, seed=7, max_deg=1024, device=cuda_device)
