@@ -461,18 +461,21 @@ def r2_pagerank(nest, lim):
 
 
 def r2_kmupdate(nest, lim):
-    """DESIGN.md S8 KU: 128-point tiles, contiguous ranges of P tiles, 8 warps x 32 lanes (2 dims per lane).
+    """DESIGN.md S8 KU: 96-point tiles, contiguous ranges of P tiles, 12 warps x 32 lanes (2 dims per lane).
     Returns (dims, blocks, spans, factors, vec, chunks, G, P)."""
     (N, _), (D, _) = nest["levels"]
     K = nest["K"]
     if D % 4 != 0 or D < 4 or D > 64 or K < 1 or K > 256 or K * D > 2048:
         raise Unsupported("KMEANS_UPDATE AUTO needs D % 4 == 0, 4 <= D <= 64, 1 <= K <= 256, K*D <= 2048")
-    T = cdiv(N, 128)
+    T = cdiv(N, KU_TILE)
     P = cdiv(T, min(lim["sm_count"], T))
     G = cdiv(T, P)
     spans = (SPLIT if G > 1 else ALL, ALL)
-    chunks = (128 * P if G > 1 else N, D)
-    return (Y, X), (8, 32), spans, (G, 1), 2, chunks, G, P
+    chunks = (KU_TILE * P if G > 1 else N, D)
+    return (Y, X), (12, 32), spans, (G, 1), 2, chunks, G, P
+
+
+KU_TILE = 96                                      # DESIGN.md S8 KU: points per tile (8 per consumer warp)
 
 
 def r2_logreg(nest, lim, dims):

@@ -369,19 +369,20 @@ void r2_rowscols(const Nest& n, int dtype, const npp_limits& lim, Choice* c) {
   c->claim_tiles = t.cr * t.cc;
 }
 
-// S8 KMEANS_UPDATE (class KU): 128-point tiles, contiguous ranges of P tiles, 8 warps one point at a
+// S8 KMEANS_UPDATE (class KU): 96-point tiles, contiguous ranges of P tiles, 12 warps one point at a
 // time with 2 dims per lane on x.
+constexpr int64_t kKuTile = 96;  // S8 KU: points per tile (8 per consumer warp, 12 warps)
 bool r2_kmupdate(const Nest& n, const npp_limits& lim, Choice* c) {
   const int64_t N = n.N[0], D = n.N[1], K = n.K;
   if (D % 4 != 0 || D < 4 || D > 64 || K < 1 || K > 256 || K * D > 2048) return false;
-  const int64_t T = cdiv(N, 128);
+  const int64_t T = cdiv(N, kKuTile);
   const int64_t P = cdiv(T, std::min<int64_t>(lim.sm_count, T));
   c->dims[0] = NPP_DIM_Y, c->dims[1] = NPP_DIM_X;
-  c->blocks[0] = 8, c->blocks[1] = 32;
+  c->blocks[0] = 12, c->blocks[1] = 32;
   c->persistent_grid = cdiv(T, P);
   c->claim_tiles = P;
   c->spans[0] = c->persistent_grid > 1 ? NPP_SPLIT_K : NPP_SPAN_ALL, c->factors[0] = c->persistent_grid;
-  c->chunks[0] = c->persistent_grid > 1 ? 128 * P : N;
+  c->chunks[0] = c->persistent_grid > 1 ? kKuTile * P : N;
   c->spans[1] = NPP_SPAN_ALL, c->factors[1] = 1, c->chunks[1] = D;
   c->vec = 2;
   c->staged = 1;

@@ -237,11 +237,12 @@ def test_rowscols_regions_by_hand():
 
 
 def test_kmeans_update_record_by_hand():
-    # 4M points / 128 = 32768 tiles over 148 SMs: P = 222 tiles per block, G = ceil(32768/222) = 148;
+    # 4M points / 96 = 43691 tiles over 148 SMs: P = 296 tiles per block, G = ceil(43691/296) = 148;
     # workspace = 256-B ticket + 32 x 65 fp64 accumulators rounded up to 256 B
     rec = S.select("KMEANS_UPDATE", (1 << 22, 64, 32), "f32", S.B200, "AUTO")
-    assert rec["kernel_class"] == S.KU and rec["grid"] == 148 and rec["claim_tiles"] == 222
-    assert rec["levels"][0]["chunk"] == 128 * 222 and rec["levels"][0]["factor"] == 148
+    assert rec["kernel_class"] == S.KU and rec["grid"] == 148 and rec["claim_tiles"] == 296
+    assert [lv["block"] for lv in rec["levels"]] == [12, 32]
+    assert rec["levels"][0]["chunk"] == 96 * 296 and rec["levels"][0]["factor"] == 148
     assert rec["workspace_bytes"] == 256 + 256 * -(-32 * 65 * 8 // 256)
 
 

@@ -204,10 +204,11 @@ def test_kmeans_update_schedules(profile):
     for N, D, K in [(1 << 22, 64, 32), (1000, 4, 1), (129, 64, 32), (5000, 16, 128), (1, 8, 8), (77777, 60, 34)]:
         rec = _select("KMEANS_UPDATE", (N, D, K), "f32", lim)
         assert rec is not None
-        T, P, G = cdiv(N, 128), rec["claim_tiles"], rec["grid"]
+        T, P, G = cdiv(N, 96), rec["claim_tiles"], rec["grid"]
         assert G <= lim["sm_count"] and G * P >= T > (G - 1) * P
         assert rec["workspace_bytes"] >= 256 + 8 * K * (D + 1)
-        assert K * D <= 2048  # eight warp-private fp32 [K x D] copies in 64 KB of shared memory
+        assert [lv["block"] for lv in rec["levels"]] == [12, 32]  # 12 consumer warps, 8 points each per tile
+        assert K * D <= 2048  # twelve warp-private fp32 [K x D] copies in 96 KB of shared memory
 
 
 @pytest.mark.parametrize("profile", list(PROFILES))
