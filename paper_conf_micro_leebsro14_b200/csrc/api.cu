@@ -688,7 +688,7 @@ int64_t npp_plan_tiles(npp_plan_t plan) {
     case NPP_CLASS_KMEANS:
       if (!m.staged) return 0;
       return (s[0] + (s[1] <= 64 ? 255 : 127)) / (s[1] <= 64 ? 256 : 128);
-    case NPP_CLASS_KMUPDATE: return (s[0] + 127) / 128;
+    case NPP_CLASS_KMUPDATE: return (s[0] + 95) / 96;  // S8 KU tiles
     case NPP_CLASS_RC: return m.level[0].grid * m.level[1].grid;
     default: return 0;
   }

@@ -2,24 +2,26 @@
 // NEXT 4), Table I's groupBy followed by a Reduce per group:
 //     points groupBy { i => a_i } map { g => ((g map x) reduce +, g.size) }
 //     U[k, d] = Σ_{i: a_i = k} x[i, d],  U[k, D] = |{i : a_i = k}|     (a_i outside [0, K): no group)
-// The path is HBM-bound (4·D + 4 bytes per point, D adds): tiles of 128 points (x: 2-D TMA box of
-// 128 rows x D floats; a: 1-D box of 128 ints) stream through a 4-deep mbarrier ring, one block per
-// SM, contiguous tile ranges. The data-dependent key is why this is not a sum family: the reduction
-// target of a point is only known when its a_i arrives.
-//   Consumer warp w adds points w, w+8, ... of each tile: lane l owns dims 2l, 2l+1 (float2), so a
-//   point is one conflict-free 8-byte read of the tile plus a read-modify-write of the warp's OWN
-//   fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are CAS loops on
-//   sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are independent and
-//   overlap (the serial load-add-store chain per point was the limit: ncu short-scoreboard stalls,
-//   405 -> 235 µs); counts come from one match.any per tile (the lowest lane of each key group adds
-//   its size). Measured and dropped: 8 points per step with repeated keys merged first (331 µs: the
-//   merge tests cost more than the overlap gains), half-warp points with float4 lanes one step
-//   (279 µs) or two steps (280 µs) at a time, counts updated by lane 0 next to each row update
-//   instead of the match.any (306 µs: divergent lane-0 branches). Every 8 tiles (<= 128 points per warp accumulator, so the
-//   fp32 error stays below 127u·Σ|x|) the 8 warp copies are folded into one fp64 block accumulator;
-//   at the end each block adds it to the fp64 workspace accumulators with RED atomics and a ticket
-//   elects the last block, which converts to f32 and re-zeroes (the Split combine of P:L880-883,
-//   fused).
+// The path is HBM-bound (4·D + 4 bytes per point, D adds): tiles of 96 points (x: 2-D TMA box of
+// 96 rows x D floats; a: 1-D box of 96 ints) stream through a 4-deep mbarrier ring, one block per
+// SM, contiguous tile ranges (S8 KU). The data-dependent key is why this is not a sum family:
+// the reduction target of a point is only known when its a_i arrives.
+//   Consumer warp w of 12 adds points w, w+12, ... of each tile (8 per tile): lane l owns dims 2l, 2l+1
+//   (float2), so a point is one conflict-free 8-byte read of the tile plus a read-modify-write of the
+//   warp's OWN fp32 accumulator row k in shared memory (no atomics: shared-memory float atomics are
+//   CAS loops on sm_100a). Points go 4 at a time: with distinct keys their 4 row updates are
+//   independent and overlap (the serial load-add-store chain per point was the limit: ncu
+//   short-scoreboard stalls, 405 -> 235 µs); counts come from one match.any per tile (the lowest lane
+//   of each key group adds its size). The kernel stays bound by those read-modify-write chains, so
+//   more warps hide more of them: 12 warps (96 KB of copies, 96-point tiles) 198 µs vs 8 warps with
+//   128-point tiles 221 µs (profiles/r02/kmeans_update/). Measured and dropped: 8 points per step with
+//   repeated keys merged first (331 µs: the merge tests cost more than the overlap gains), half-warp
+//   points with float4 lanes one step (279 µs) or two steps (280 µs) at a time, counts updated by lane
+//   0 next to each row update instead of the match.any (306 µs: divergent lane-0 branches). Every
+//   128 / 8 = 16 tiles (<= 128 points per warp accumulator, so the fp32 error stays below 127u·Σ|x|)
+//   the 12 warp copies are folded into one fp64 block accumulator; at the end each block adds it to the
+//   fp64 workspace accumulators with RED atomics and a ticket elects the last block, which converts to
+//   f32 and re-zeroes (the Split combine of P:L880-883, fused).
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -34,18 +36,29 @@ namespace {
 
 using namespace tma;
 
-constexpr int kStages = 4;
-constexpr int kTP = 128;                  // points per tile
-constexpr int kXSlot = 32 * 1024;         // kTP * D * 4 <= 32 KB (D <= 64)
-constexpr int kASlot = kTP * 4;           // 512 B of keys
-constexpr int kConsumerWarps = 8;
+#ifndef NPP_KU_STAGES
+#define NPP_KU_STAGES 4
+#endif
+#ifndef NPP_KU_TP  // DESIGN.md S8 KU: 96-point tiles, 12 consumer warps (8 points each per tile)
+#define NPP_KU_TP 96
+#endif
+#ifndef NPP_KU_WARPS
+#define NPP_KU_WARPS 12
+#endif
+constexpr int kStages = NPP_KU_STAGES;
+constexpr int kTP = NPP_KU_TP;            // points per tile
+constexpr int kXSlot = kTP * 256;         // kTP * D * 4 <= kTP * 256 B (D <= 64)
+constexpr int kASlot = (kTP * 4 + 127) / 128 * 128;  // keys (TMA destinations stay 128-B aligned)
+constexpr int kConsumerWarps = NPP_KU_WARPS;
+constexpr int kPPW = kTP / kConsumerWarps;  // points of a tile per warp
+static_assert(kTP % kConsumerWarps == 0 && kPPW % 4 == 0 && kPPW <= 32, "whole 4-point batches per warp");
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kThreads = kConsumers + 32;  // + producer warp
 constexpr int kHeader = 1024;
 constexpr int kMaxKD = 2048;               // DESIGN.md S8 KU: K*D <= 2048, K <= 256
 constexpr int kMaxK = 256;
-#ifndef NPP_KU_FLUSH_TILES  // measurement knob only: the fp32 error bound of DESIGN.md §5 assumes 8
-#define NPP_KU_FLUSH_TILES 8
+#ifndef NPP_KU_FLUSH_TILES  // measurement knob only: the fp32 error bound of DESIGN.md §5 assumes <= 128
+#define NPP_KU_FLUSH_TILES (128 / (NPP_KU_TP / NPP_KU_WARPS))  // points per warp copy between flushes
 #endif
 constexpr int kFlushTiles = NPP_KU_FLUSH_TILES;
 constexpr int kSmemBytes = kHeader + kStages * (kXSlot + kASlot) + kConsumerWarps * kMaxKD * 4 +
@@ -117,13 +130,14 @@ __global__ void __launch_bounds__(kThreads, 1)
   float* myacc = accw + warp * KD;
   unsigned* mycnt = cntw + warp * K;
   const bool dim_lane = 2 * lane < D;
-  int krow[kMaxKD / kConsumers];  // flush: accumulator row of element tid + 256 r (no division per flush)
+  constexpr int kFR = (kMaxKD + kConsumers - 1) / kConsumers;  // flush elements per thread
+  int krow[kFR];  // flush: accumulator row of element tid + kConsumers r (no division per flush)
 #pragma unroll
-  for (int r = 0; r < kMaxKD / kConsumers; ++r) krow[r] = (int(threadIdx.x) + kConsumers * r) / D;
+  for (int r = 0; r < kFR; ++r) krow[r] = (int(threadIdx.x) + kConsumers * r) / D;
   auto flush = [&]() {  // fold the 8 warp copies into the fp64 block accumulator, zero the copies
     consumers_sync();
 #pragma unroll
-    for (int r = 0; r < kMaxKD / kConsumers; ++r) {
+    for (int r = 0; r < kFR; ++r) {
       const int i = int(threadIdx.x) + kConsumers * r;
       if (i >= KD) break;
       // the 8 warp copies meet in an fp32 pairwise tree (error <= 3u on top of the copies' <= 127u), then
@@ -135,9 +149,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         accw[w * KD + i] = 0.f;
       }
 #pragma unroll
-      for (int h = kConsumerWarps / 2; h >= 1; h /= 2)
+      for (int h = 1; h < kConsumerWarps; h *= 2)  // pairwise tree (any copy count)
 #pragma unroll
-        for (int w = 0; w < h; ++w) v[w] += v[w + h];
+        for (int w = 0; w + h < kConsumerWarps; w += 2 * h) v[w] += v[w + h];
       bacc[i + krow[r]] += double(v[0]);  // row k of [K x (D+1)]
     }
     for (int k = threadIdx.x; k < K; k += kConsumers) {
@@ -164,9 +178,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane == 0) mbar_arrive(empty + slot);
     continue;
 #endif
-    // the warp's 16 points of the tile are p = warp + 8j: lane j < 16 reads key j (-1: no group)
+    // the warp's kPPW points of the tile are p = warp + W·j: lane j < kPPW reads key j (-1: no group)
     int kl = -1;
-    if (lane < kTP / kConsumerWarps && warp + kConsumerWarps * lane < np) {
+    if (lane < kPPW && warp + kConsumerWarps * lane < np) {
       kl = at[warp + kConsumerWarps * lane];
       if (unsigned(kl) >= unsigned(K)) kl = -1;
     }
@@ -175,7 +189,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const unsigned same = __match_any_sync(0xffffffffu, kl);
     // sums: 4 points at a time
 #pragma unroll
-    for (int j0 = 0; j0 < kTP / kConsumerWarps; j0 += 4) {
+    for (int j0 = 0; j0 < kPPW; j0 += 4) {
       int k[4];
       float2 xv[4];
 #pragma unroll
@@ -264,7 +278,13 @@ cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* ke
   if (e != cudaSuccess) return e;
   if ((e = encode_1d(&amap, keys, CU_TENSOR_MAP_DATA_TYPE_INT32, a.N, unsigned(kTP))) != cudaSuccess) return e;
   if ((e = ensure_smem(npp_kmupdate_kernel, kSmemBytes)) != cudaSuccess) return e;
+#if NPP_KU_TP != 96  // measurement variants: the record's ranges are in 96-point tiles
+  KmUpdateArgs b = a;
+  b.per_block = ((a.N + kTP - 1) / kTP + grid - 1) / grid;
+  return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, a.pdl != 0, xmap, amap, b);
+#else
   return launch_pdl(npp_kmupdate_kernel, grid, kThreads, kSmemBytes, st, a.pdl != 0, xmap, amap, a);
+#endif
 }
 
 }  // namespace npp

@@ -148,7 +148,7 @@ struct RowsColsArgs {
 cudaError_t launch_rowscols(int dtype, bool staged, const RowsColsArgs& a, int grid, cudaStream_t st);
 
 // k-means centroid update (class KU, S8 KU): x [N x D] fp32, keys [N] int32 ->
-// out [K x (D+1)] fp32 = per group (Σ x, count). Block b takes 128-point tiles [b*P, (b+1)*P).
+// out [K x (D+1)] fp32 = per group (Σ x, count). Block b takes 96-point tiles [b*P, (b+1)*P) (S8 KU).
 struct KmUpdateArgs {
   float* out;          // [K x (D+1)]
   double* acc;         // [K x (D+1)] fp64 accumulators (zero on entry and on exit)
@@ -157,7 +157,7 @@ struct KmUpdateArgs {
   int64_t per_block;   // P
   int early_reads;     // NPP_EXEC_OVERLAP
   int pdl;             // programmatic dependent launch (not NPP_EXEC_NO_PDL)
-  int* trace;          // npp_execute_traced: [2 x T] block of each 128-point tile, loads per tile (else NULL)
+  int* trace;          // npp_execute_traced: [2 x T] block of each 96-point tile, loads per tile (else NULL)
 };
 cudaError_t launch_kmupdate(const KmUpdateArgs& a, const float* x, const int* keys, int grid, cudaStream_t st);
 

@@ -117,7 +117,7 @@ def test_kmeans_update_schedule(npp, cuda_device):
         x, c = gen.kmeans_inputs(N, D, K, device=cuda_device, integer=True)
         keys = gen.int_uniform(9, (N,), 0, K - 1, dtype=torch.int32, device=cuda_device)
         p = npp.Plan("KMEANS_UPDATE", (N, D, K), "f32", "AUTO")
-        T = -(-N // 128)
+        T = -(-N // 96)  # DESIGN.md S8 KU: 96-point tiles
         assert p.tiles == T
         out = p.new_out()
         blk, cnt = p.execute_traced([x, keys], out)
