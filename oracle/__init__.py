@@ -12,6 +12,7 @@ Modules
   kmeans  — k-means assignment (argmin of squared distances)            (BASELINE.json config 4)
   logreg  — batched logistic-regression gradient                        (BASELINE.json config 5)
 
-Parity unpinned: the soft-constraint intrinsic weights, the tie-break key and the R2
-runtime rule are pinned only by DESIGN.md, not by printed values in the paper.
+Readings of points the paper leaves open: the soft-constraint intrinsic weights and the
+tie-break key are pinned by invariance (every reading consistent with L674-676 / L741 gives the same
+records on the BASELINE workloads); the R2 runtime rule by schedule properties (tests/test_r2_properties.py).
 """

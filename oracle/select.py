@@ -11,7 +11,7 @@ Follows PAPER.md §IV step by step, with the readings of DESIGN.md §2/§3 where
   runtime parameter step (AUTO)              L810-817                                         (S8)
 Written as plain nested loops over the whole candidate space (no pruning, no memoisation).
 
-Parity unpinned vs the paper: W_C/W_B, the tie-break key and R2.
+W_C/W_B and the tie-break key are readings pinned by invariance, R2 by schedule properties.
 """
 from __future__ import annotations
 
