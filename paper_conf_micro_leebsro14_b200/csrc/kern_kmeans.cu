@@ -135,6 +135,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const int nb = DT ? (DT + kBoxCols - 1) / kBoxCols : km_boxes(a.D);
   constexpr int LS = km_ls(LDSP);
   const int kStages = km_stages(a.K, D, TP, SETS, ONE, LDSP);  // ring depth (2 or 3)
+  constexpr bool kBarrierRelease = DT == 0 || SETS == 2;  // see the box release below
   // the 128-byte swizzle is a function of smem address bits [7:9]: boxes must be 1 KB aligned
   const unsigned pad = (1024u - (tma::smem_u32(smem) & 1023u)) & 1023u;
   unsigned char* ring = smem + pad;
@@ -381,7 +382,11 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
             }
           }
         }
-        if (last_chunk) {  // the set is past this box of the slot: the last warp refills it (tile t + kStages)
+        // the set is past this box of the slot: the last warp refills it (tile t + kStages). In the
+        // generic-D kernels the last box of a multi-box tile is refilled after the set barrier instead
+        // (every warp is past it there), so only the earlier boxes pay the release atomics (D = 96: 373 ->
+        // 362 us; in the three-set D = 64 kernel the extra code pushes ptxas off the uniform datapath)
+        if (last_chunk && !(kBarrierRelease && nb > 1 && bx == nb - 1)) {
           __syncwarp();
           if (lane == 0) {
             __threadfence_block();
@@ -426,6 +431,10 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
                                                                code_up(__fadd_ru(n2[i].x, n2[i].y)));
     }
     asm volatile("bar.sync %0, %1;" ::"r"(1 + set), "n"(kConsumers) : "memory");  // this set only
+    if (kBarrierRelease && nb > 1 && wis == kConsumerWarps - 1 && lane == 0 && t + kStages < n_tiles) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // the set's reads of the box, then TMA
+      issue_box(t + kStages, slot, nb - 1);
+    }
     merge_share(t, ar);
     for (slot += kSets; slot >= kStages; slot -= kStages) ++round;
   }
