@@ -16,6 +16,11 @@
 //   minimum in increasing k; with G = 2 the two groups meet in shared memory (lower k on ties).
 //   x·c runs on the packed FP32 pipe (FFMA2, fma.rn.f32x2): even and odd dims accumulate in the two
 //   halves of a float2.
+//   The dims loop's ceiling is the uniform constant path, not the FMA pipe: one LDCU.64 per 4 FFMA2
+//   caps it at ~0.65 of the FFMA2 peak (tools/micro_km_inner.cu). The D > 64 kernel therefore takes 1-2
+//   of each thread's 4 pairs per chunk from a broadcast shared-memory copy; the D <= 64 kernels (80-register
+//   cap) keep all of them in the constant bank, and with three sets (one 32-chunk) the chunk loop is a
+//   compile-time single pass, so the argmin state is born after the dims loop.
 // The path is FP32-FMA-bound: 2·N·K·D flops against 4·D bytes of x per point.
 #include <cstdint>
 #include <mutex>
