@@ -174,8 +174,20 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   const long long bid = blockIdx.x, G = gridDim.x;
   const long long total = a.To * a.Ti;
   // static range (MX-narrow: whole strips, so no strip is ever cut)
-  const long long s0 = ALIGN ? (bid * (a.static_tiles / a.Ti) / G) * a.Ti : bid * a.static_tiles / G;
-  const long long s1 = ALIGN ? ((bid + 1) * (a.static_tiles / a.Ti) / G) * a.Ti : (bid + 1) * a.static_tiles / G;
+#ifndef NPP_SUM_FAST_DIV
+#define NPP_SUM_FAST_DIV 1
+#endif
+  // static range (MX-narrow: whole strips, so no strip is ever cut). Tile ids are < 2^31 (the launch
+  // checks), so the producer's divisions run in 32 bits, and floor(b·S/G) with b·S < 2^40 in double:
+  // exact, since a quotient's fraction is at most 1 − 1/G, far from the 2^-13 rounding error — the 64-bit
+  // integer divisions sat in front of the first TMA issue of every launch
+  auto fdiv = [](long long num, long long den) -> long long {
+    return NPP_SUM_FAST_DIV ? (long long)floor(double(num) / double(den)) : num / den;
+  };
+  const long long so = NPP_SUM_FAST_DIV ? (long long)(unsigned(a.static_tiles) / unsigned(a.Ti)) : a.static_tiles / a.Ti;
+  const long long s0 = ALIGN ? (fdiv(bid * so, G)) * a.Ti : fdiv(bid * a.static_tiles, G);
+  const long long s1 = ALIGN ? (fdiv((bid + 1) * so, G)) * a.Ti
+                             : fdiv((bid + 1) * a.static_tiles, G);
   const long long U = a.unit;  // pool: units of U tiles from static_tiles on, claimed in order, then single tiles
 #ifdef NPP_SUM_STAMPS
   __shared__ unsigned long long* stamp_row;
@@ -239,7 +251,9 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       long long t = 0;
       for (; cur >= 0; ++t) {
         const long long nxt = next_tile();  // claimed one ahead: its latency hides behind the slot wait
-        const bool flush = nxt < 0 || (nxt / a.Ti) != (cur / a.Ti);
+        const unsigned uTi = unsigned(a.Ti);  // tile ids and Ti < 2^31: 32-bit divisions
+        const long long ot = NPP_SUM_FAST_DIV ? (long long)(unsigned(cur) / uTi) : cur / a.Ti;
+        const bool flush = nxt < 0 || (NPP_SUM_FAST_DIV ? (long long)(unsigned(nxt) / uTi) : nxt / a.Ti) != ot;
         const int slot = int(t % kStages);
         if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
         // the tag travels through shared memory ordered by the slot's mbarriers; it is written and
@@ -252,7 +266,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         }
         constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
         mbar_expect_tx(full + slot, kTileBytes + kVBytes);
-        const long long ot = cur / a.Ti, it = cur - ot * a.Ti;
+        const long long it = cur - ot * a.Ti;
         const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
         const int y = int(ROWS ? ot * RT : it * RT);     // first row
         if constexpr (WT) {  // v over the tile's columns (RX) or rows (MX); zero-filled past the end
@@ -426,7 +440,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         asm volatile("griddepcontrol.wait;" ::: "memory");
         waited = true;
       }
-      const long long ot = (tag & ~kFlush) / a.Ti;
+      const long long ot = NPP_SUM_FAST_DIV ? (long long)((tag & ~kFlush) / unsigned(a.Ti)) : (tag & ~kFlush) / a.Ti;
       const bool whole = n_acc == unsigned(a.Ti);  // this block added every tile of ot
       long long oidx[4];
       Acc val[4];
