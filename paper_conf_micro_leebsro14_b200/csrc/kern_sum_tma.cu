@@ -199,6 +199,48 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
   }
 #endif
 
+  // stream tile cur into ring slot t % kStages (nxt: the block's next tile, -1 = none, for the flush tag)
+  auto issue = [&](long long t, long long cur, long long nxt) {
+    const unsigned uTi = unsigned(a.Ti);  // tile ids and Ti < 2^31: 32-bit divisions
+    const long long ot = NPP_SUM_FAST_DIV ? (long long)(unsigned(cur) / uTi) : cur / a.Ti;
+    const bool flush = nxt < 0 || (NPP_SUM_FAST_DIV ? (long long)(unsigned(nxt) / uTi) : nxt / a.Ti) != ot;
+    const int slot = int(t % kStages);
+    if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
+    // the tag travels through shared memory ordered by the slot's mbarriers; it is written and
+    // read with (relaxed) shared atomics so compute-sanitizer's racecheck, which does not model
+    // mbarrier ordering, sees no plain-access race
+    atomicExch(slot_tile + slot, static_cast<unsigned>(cur) | (flush ? kFlush : 0u));
+    if (a.trace) {  // white-box schedule trace (npp_execute_traced): who streamed tile cur
+      a.trace[cur] = int(bid);
+      atomicAdd(a.trace + total + cur, 1);
+    }
+    constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
+    mbar_expect_tx(full + slot, kTileBytes + kVBytes);
+    const long long it = cur - ot * a.Ti;
+    const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
+    const int y = int(ROWS ? ot * RT : it * RT);     // first row
+    if constexpr (WT) {  // v over the tile's columns (RX) or rows (MX); zero-filled past the end
+      if constexpr (ROWS) {
+#pragma unroll
+        for (int q = 0; q < NCH; ++q)
+          tma::load_1d(vslots + slot * kVSlot + q * 1024, &vmap, (ch + q) * BC, full + slot);
+      } else {
+        tma::load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
+      }
+    }
+    if constexpr (WIDE && ROWS)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
+      tma::load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
+    else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
+      tma::load_2d(tiles + slot * kTileBytes, &map, MXN ? int(ot * W) : ch * BC, y, full + slot);
+  };
+#ifndef NPP_SUM_EARLY_ISSUE
+#define NPP_SUM_EARLY_ISSUE 1
+#endif
+  // the first tiles of the static range are issued by the thread that initialises the barriers, before
+  // the block-wide barrier (the producer warp then continues after them): the first loads leave ~a
+  // barrier and a warp hand-off earlier
+  const long long early = NPP_SUM_EARLY_ISSUE ? (s1 - s0 - 1 < kStages ? (s1 - s0 - 1 > 0 ? s1 - s0 - 1 : 0)
+                                                                        : kStages) : 0;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(full + i, 1);
@@ -209,6 +251,11 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
       mbar_init(fl_free + i, 1);
     }
     tma::mbar_fence_init();
+    if (early > 0) {
+      tma::prefetch_map(&map);
+      if (a.early_reads == 0) asm volatile("griddepcontrol.wait;" ::: "memory");
+      for (long long j = 0; j < early; ++j) issue(j, s0 + j, s0 + j + 1);  // nxt stays inside the range
+    }
   }
   __syncthreads();
 
@@ -247,41 +294,12 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
         }
         return u_cur++;
       };
+      sn = s0 + early;  // the first `early` tiles of the static range are already in flight
       long long cur = next_tile();
-      long long t = 0;
+      long long t = early;
       for (; cur >= 0; ++t) {
         const long long nxt = next_tile();  // claimed one ahead: its latency hides behind the slot wait
-        const unsigned uTi = unsigned(a.Ti);  // tile ids and Ti < 2^31: 32-bit divisions
-        const long long ot = NPP_SUM_FAST_DIV ? (long long)(unsigned(cur) / uTi) : cur / a.Ti;
-        const bool flush = nxt < 0 || (NPP_SUM_FAST_DIV ? (long long)(unsigned(nxt) / uTi) : nxt / a.Ti) != ot;
-        const int slot = int(t % kStages);
-        if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
-        // the tag travels through shared memory ordered by the slot's mbarriers; it is written and
-        // read with (relaxed) shared atomics so compute-sanitizer's racecheck, which does not model
-        // mbarrier ordering, sees no plain-access race
-        atomicExch(slot_tile + slot, static_cast<unsigned>(cur) | (flush ? kFlush : 0u));
-        if (a.trace) {  // white-box schedule trace (npp_execute_traced): who streamed tile cur
-          a.trace[cur] = int(bid);
-          atomicAdd(a.trace + total + cur, 1);
-        }
-        constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
-        mbar_expect_tx(full + slot, kTileBytes + kVBytes);
-        const long long it = cur - ot * a.Ti;
-        const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
-        const int y = int(ROWS ? ot * RT : it * RT);     // first row
-        if constexpr (WT) {  // v over the tile's columns (RX) or rows (MX); zero-filled past the end
-          if constexpr (ROWS) {
-#pragma unroll
-            for (int q = 0; q < NCH; ++q)
-              tma::load_1d(vslots + slot * kVSlot + q * 1024, &vmap, (ch + q) * BC, full + slot);
-          } else {
-            tma::load_1d(vslots + slot * kVSlot, &vmap, y, full + slot);
-          }
-        }
-        if constexpr (WIDE && ROWS)  // 3-D map {BC, C/BC, R}: box {BC, 4, 8} = 8 rows x 4 KB
-          tma::load_3d(tiles + slot * kTileBytes, &map, 0, ch, y, full + slot);
-        else  // 2-D map {C, R}: box {BC, 32} = 32 rows x 1 KB
-          tma::load_2d(tiles + slot * kTileBytes, &map, MXN ? int(ot * W) : ch * BC, y, full + slot);
+        issue(t, cur, nxt);
         cur = nxt;
       }
       const int slot = int(t % kStages);  // end marker: an arrival without bytes
