@@ -162,12 +162,32 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const long long P = a.per_block;
   const long long r0 = bid * P, r1 = (T < r0 + P) ? T : r0 + P;
 
+#ifndef NPP_KM_EARLY
+#define NPP_KM_EARLY 2  // 2: the D = 64 kernels (config 4 341.6 -> 339.7 us; the generic-D kernels lose with it)
+#endif
+  constexpr bool kEarlyIssue = NPP_KM_EARLY == 1 || (NPP_KM_EARLY == 2 && DT != 0);
+  const long long n_tiles = r1 - r0;
+  auto issue_box = [&](long long t, int slot, int bx) {  // box bx of tile t of the range into slot t % kStages
+    if (a.trace && bx == 0) {  // white-box schedule trace (npp_execute_traced)
+      a.trace[r0 + t] = int(bid);
+      atomicAdd(a.trace + T + r0 + t, 1);
+    }
+    tma::mbar_expect_tx(full + slot * kMaxBoxes + bx, unsigned(TP * 128));
+    tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
+                 full + slot * kMaxBoxes + bx);
+  };
   if (threadIdx.x == 0) {
     for (int i = 0; i < kMaxStages * kMaxBoxes; ++i) {
       tma::mbar_init(full + i, 1);
       released[i] = 0;
     }
     tma::mbar_fence_init();
+    // the ring's first tiles load while the block computes ||c||² and the shared-memory pairs below
+    if (kEarlyIssue) {
+      tma::prefetch_map(&map);
+      for (int t = 0; t < kStages && t < n_tiles; ++t)
+        for (int bx = 0; bx < nb; ++bx) issue_box(t, t, bx);
+    }
   }
   // ||c_k||² (fp32 FMA chain over d); padded rows get +inf and are never selected
   for (int k = threadIdx.x; k < Kp; k += kThreads) {
@@ -197,17 +217,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
   const float g2d = float(2 * D + 2) * 5.9604645e-8f;  // (2D+2) u, u = 2^-24
   const float coef = 4.04f * (g2d / (1.f - g2d) + float(D + 3) * 1.1102230e-16f);
 
-  const long long n_tiles = r1 - r0;
-  auto issue_box = [&](long long t, int slot, int bx) {  // box bx of tile t of the range into slot t % kStages
-    if (a.trace && bx == 0) {  // white-box schedule trace (npp_execute_traced)
-      a.trace[r0 + t] = int(bid);
-      atomicAdd(a.trace + T + r0 + t, 1);
-    }
-    tma::mbar_expect_tx(full + slot * kMaxBoxes + bx, unsigned(TP * 128));
-    tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
-                 full + slot * kMaxBoxes + bx);
-  };
-  if (threadIdx.x == 0) {
+  if (!kEarlyIssue && threadIdx.x == 0) {
     tma::prefetch_map(&map);
     for (int t = 0; t < kStages && t < n_tiles; ++t)
       for (int bx = 0; bx < nb; ++bx) issue_box(t, t, bx);
