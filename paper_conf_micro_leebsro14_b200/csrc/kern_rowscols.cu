@@ -133,13 +133,38 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long bid = blockIdx.x, G = gridDim.x;
   const long long q0 = bid * a.nreg / G, q1 = (bid + 1) * a.nreg / G;
-
-  if (threadIdx.x == 0) {
+#ifndef NPP_RC_EARLY_ISSUE
+#define NPP_RC_EARLY_ISSUE 1
+#endif
+  // the producer lane initialises the ring and issues its first kStages tiles before the block barrier,
+  // so they load while the consumers zero the column accumulators
+  constexpr bool kEarly = STAGED && NPP_RC_EARLY_ISSUE;
+  const int init_thread = kEarly ? kConsumers : 0;
+  auto tile_rc = [&](long long q, long long* b0, long long* b1, long long* c0, long long* c1) {
+    const long long ri = q / a.gc, cj = q - ri * a.gc;
+    *b0 = ri * a.cr, *b1 = *b0 + a.cr < a.Tr ? *b0 + a.cr : a.Tr;
+    *c0 = cj * a.cc, *c1 = *c0 + a.cc < a.Tc ? *c0 + a.cc : a.Tc;
+  };
+  long long early = 0;
+  if (threadIdx.x == init_thread) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(full + i, 1);
       mbar_init(empty + i, kConsumerWarps);
     }
     mbar_fence_init();
+    if (kEarly) {
+      prefetch_map(&map);
+      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
+      for (long long q = q0; q < q1 && early < kStages; ++q) {
+        long long b0, b1, c0, c1;
+        tile_rc(q, &b0, &b1, &c0, &c1);
+        for (long long br = b0; br < b1 && early < kStages; ++br)
+          for (long long ct = c0; ct < c1 && early < kStages; ++ct, ++early) {
+            mbar_expect_tx(full + early, kTileBytes);
+            load_2d(tiles + early * kTileBytes, &map, int(ct * BC), int(br * kTileRows), full + early);
+          }
+      }
+    }
   }
   if (threadIdx.x < kConsumers)
     for (int i = threadIdx.x; i < NRG * CAP; i += kConsumers) colacc[i] = Acc(0);
@@ -148,15 +173,17 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (warp == kConsumerWarps) {
     // ------------------------------------------------------------ producer: one elected lane
     if (STAGED && lane == 0) {
-      prefetch_map(&map);
-      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
+      if (!kEarly) {
+        prefetch_map(&map);
+        if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
+      }
       long long t = 0;
       for (long long q = q0; q < q1; ++q) {
-        const long long ri = q / a.gc, cj = q - ri * a.gc;
-        const long long b0 = ri * a.cr, b1 = b0 + a.cr < a.Tr ? b0 + a.cr : a.Tr;
-        const long long c0 = cj * a.cc, c1 = c0 + a.cc < a.Tc ? c0 + a.cc : a.Tc;
+        long long b0, b1, c0, c1;
+        tile_rc(q, &b0, &b1, &c0, &c1);
         for (long long br = b0; br < b1; ++br)
           for (long long ct = c0; ct < c1; ++ct, ++t) {
+            if (t < early) continue;  // issued before the block barrier
             const int slot = int(t % kStages);
             if (t >= kStages) mbar_wait(empty + slot, unsigned((t / kStages) & 1) ^ 1u);
             mbar_expect_tx(full + slot, kTileBytes);
