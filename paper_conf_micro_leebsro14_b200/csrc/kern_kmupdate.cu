@@ -89,12 +89,32 @@ __global__ void __launch_bounds__(kThreads, 1)
   const long long t0 = blockIdx.x * a.per_block;
   const long long t1 = t0 + a.per_block < T ? t0 + a.per_block : T;
 
-  if (threadIdx.x == 0) {
+  // the producer lane initialises the ring and issues its first kStages tiles before the block barrier,
+  // so they load while the consumers zero their accumulator copies
+  const unsigned bytes = unsigned(kTP * D * 4 + kTP * 4);  // x box + key box
+  long long early = 0;
+  auto issue = [&](long long t) {
+    const long long i = t - t0;
+    const int slot = int(i % kStages);
+    if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
+    mbar_expect_tx(full + slot, bytes);
+    load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
+    load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
+    if (a.trace) {
+      a.trace[t] = int(blockIdx.x);
+      atomicAdd(a.trace + T + t, 1);
+    }
+  };
+  if (threadIdx.x == kConsumers) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(full + i, 1);
       mbar_init(empty + i, kConsumerWarps);
     }
     mbar_fence_init();
+    prefetch_map(&xmap);
+    prefetch_map(&amap);
+    if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
+    for (; early < kStages && t0 + early < t1; ++early) issue(t0 + early);
   }
   if (threadIdx.x < kConsumers) {
     for (int i = threadIdx.x; i < kConsumerWarps * KD; i += kConsumers) accw[i] = 0.f;
@@ -105,24 +125,8 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp == kConsumerWarps) {
     // ------------------------------------------------------------ producer: one elected lane
-    if (lane == 0) {
-      prefetch_map(&xmap);
-      prefetch_map(&amap);
-      if (!a.early_reads) asm volatile("griddepcontrol.wait;" ::: "memory");
-      const unsigned bytes = unsigned(kTP * D * 4 + kASlot);
-      for (long long t = t0; t < t1; ++t) {
-        const long long i = t - t0;
-        const int slot = int(i % kStages);
-        if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
-        mbar_expect_tx(full + slot, bytes);
-        load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
-        load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
-        if (a.trace) {
-          a.trace[t] = int(blockIdx.x);
-          atomicAdd(a.trace + T + t, 1);
-        }
-      }
-    }
+    if (lane == 0)
+      for (long long t = t0 + early; t < t1; ++t) issue(t);
     return;
   }
 
