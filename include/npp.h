@@ -71,7 +71,9 @@ typedef enum { NPP_F32 = 0, NPP_I32 = 1, NPP_I64 = 2, NPP_F64 = 3 } npp_dtype;
  *                      out[N] f32 = (1-0.85)/N + 0.85 * Σ_{j=rowptr[n]}^{rowptr[n+1]-1} pr[w_j]/outdeg[w_j], w_j = colidx[j]
  *                      one PageRank step (Fig 5) over the CSR of IN-neighbours; the caller
  *                      guarantees 0 <= rowptr[n] <= rowptr[n+1] <= E, 0 <= colidx < N and outdeg >= 1 for
- *                      every id in colidx (no device-side checks). AUTO only; E < 2^31. */
+ *                      every id in colidx (no device-side checks). AUTO only; E < 2^31. The record's inner
+ *                      level is Split (segmented: warps claim 31 rows, their edges over 32 lanes) when
+ *                      ceil(E/N) >= 8, else Span(all) over V lanes per row (S8 PR). */
 typedef enum {
   NPP_SUM_ROWS = 0,
   NPP_SUM_COLS = 1,
@@ -257,7 +259,7 @@ NPP_API int npp_execute_host(npp_plan_t plan, const void* const* host_ins, int n
 
 /* Tiles of the plan's schedule (white-box tests of the runtime rule, S8): To*Ti for a staged
  * sum (outer-major tile order), B*ceil(Rb/32) for LOGREG_GRAD, ceil(N/TP) for KMEANS_ASSIGN (TP = 256 if
- * D <= 64 else 128), ceil(N/128) for KMEANS_UPDATE, the number of regions for SUM_ROWS_COLS; 0 for plans
+ * D <= 64 else 128), ceil(N/96) for KMEANS_UPDATE, the number of regions for SUM_ROWS_COLS; 0 for plans
  * without a tile schedule (direct-load families, PAGERANK, empty plans). */
 NPP_API int64_t npp_plan_tiles(npp_plan_t plan);
 
