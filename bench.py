@@ -748,7 +748,11 @@ def roofline(item, us, gbs, peak, peak_src, traffic, flops, wavefronts=None):
         return dict(base, bound="alu", achieved=round(achieved, 2), peak=round(alu_peak, 2), unit="TFLOP/s",
                     frac=round(achieved / alu_peak, 4),
                     peak_source="derived: 148 SM x 128 FP32 FMA/clk x 2 x 1965 MHz (guide unit counts)",
-                    algorithmic_flops=flops)
+                    algorithmic_flops=flops,
+                    # measured context (profiles/r02/kmeans/micro_inner.log): the kernel's dims loop alone, with
+                    # its 4-point x 8-centroid thread tile, reaches 0.63-0.69 of this peak — one uniform
+                    # constant-bank load per 4 packed FMAs, not the FMA pipe, sets that ceiling
+                    operand_path_ceiling_frac=[0.63, 0.69])
     return dict(base, bound="hbm", achieved=round(gbs, 1), peak=peak, peak_source=peak_src, unit="GB/s",
                 frac=round(gbs / peak, 4))
 
