@@ -172,6 +172,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
       a.trace[r0 + t] = int(bid);
       atomicAdd(a.trace + T + r0 + t, 1);
     }
+    NPP_CHECK(t >= 0 && t < n_tiles && r0 + t < T && bx < nb && slot < kStages);
     tma::mbar_expect_tx(full + slot * kMaxBoxes + bx, unsigned(TP * 128));
     tma::load_2d(ring + slot * kMaxStageBytes + bx * (TP * 128), &map, bx * kBoxCols, int((r0 + t) * TP),
                  full + slot * kMaxBoxes + bx);
@@ -298,6 +299,7 @@ __device__ __forceinline__ void kmeans_body(const CUtensorMap* mapp, const Kmean
         const int ok = __shfl_xor_sync(0xffffffffu, bestk, off);
         if (ob < best || (ob == best && ok < bestk)) best = ob, bestk = ok;
       }
+      NPP_CHECK(gs < a.N && bestk < K);
       if (lane == 0) a.assign[gs] = bestk;
     }
   };

@@ -97,6 +97,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const long long i = t - t0;
     const int slot = int(i % kStages);
     if (i >= kStages) mbar_wait(empty + slot, unsigned((i / kStages) & 1) ^ 1u);
+    NPP_CHECK(t >= t0 && t < t1 && t * kTP < a.N);
     mbar_expect_tx(full + slot, bytes);
     load_2d(xring + slot * kXSlot, &xmap, 0, int(t * kTP), full + slot);
     load_1d(aring + slot * kASlot, &amap, int(t * kTP), full + slot);
@@ -204,6 +205,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           xv[q] = *reinterpret_cast<const float2*>(xt + (warp + kConsumerWarps * (j0 + q)) * D + 2 * lane);
       }
       if (!dim_lane) continue;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) NPP_CHECK(k[q] < K);
       // a repeated key adds its point into the first point of that key (branch-free selects), so
       // the remaining row updates are distinct and their loads may all issue before the stores;
       // with no branches the compiler interleaves consecutive batches

@@ -160,6 +160,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         tile_rc(q, &b0, &b1, &c0, &c1);
         for (long long br = b0; br < b1 && early < kStages; ++br)
           for (long long ct = c0; ct < c1 && early < kStages; ++ct, ++early) {
+            NPP_CHECK(br < a.Tr && ct < a.Tc && q < a.nreg);
             mbar_expect_tx(full + early, kTileBytes);
             load_2d(tiles + early * kTileBytes, &map, int(ct * BC), int(br * kTileRows), full + early);
           }

@@ -217,6 +217,7 @@ __global__ void __launch_bounds__(kThreads, 1) npp_sum_tma_kernel(const __grid_c
     constexpr unsigned kVBytes = WT ? (ROWS ? NCH * 1024 : RT * unsigned(sizeof(T))) : 0;
     mbar_expect_tx(full + slot, kTileBytes + kVBytes);
     const long long it = cur - ot * a.Ti;
+    NPP_CHECK(cur >= 0 && cur < total && ot < a.To && it >= 0 && it < a.Ti && (nxt < 0 || nxt < total));
     const int ch = int(ROWS ? it * NCH : ot * NCH);  // first 1 KB chunk of the tile's rows
     const int y = int(ROWS ? ot * RT : it * RT);     // first row
     if constexpr (WT) {  // v over the tile's columns (RX) or rows (MX); zero-filled past the end

@@ -8,6 +8,20 @@
 
 #include "npp.h"
 
+// Device-side bounds checks (measurement / validation builds only: -DNPP_DEVICE_CHECKS). A failed check
+// traps the kernel, so a parity run against such a build proves the checked indices stayed in range —
+// the stand-in for compute-sanitizer where the pool has it closed (profiles/r02/device_checks/).
+#ifdef NPP_DEVICE_CHECKS
+#define NPP_CHECK(cond) \
+  do {                  \
+    if (!(cond)) __trap(); \
+  } while (0)
+#else
+#define NPP_CHECK(cond) \
+  do {                  \
+  } while (0)
+#endif
+
 namespace npp {
 
 // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is per device: set it once per (kernel, device) under a
