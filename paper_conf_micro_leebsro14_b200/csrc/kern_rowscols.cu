@@ -316,40 +316,33 @@ __global__ void __launch_bounds__(kThreads, 1)
       const bool last_r = flag[0] != 0, last_c = flag[1] != 0;
       // the conversions issue all of a thread's loads before any store: one L2 round trip, not one per
       // element (a region has <= 32 * 256 columns: <= 32 per thread; its rows <= kConsumers per pass)
-      if (last_r) {
-        const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
-        for (long long r0 = rlo; r0 < rhi; r0 += 8 * kConsumers) {
-          Acc val[8];
+      // a block may complete both its row region and its column group: both conversions issue their
+      // first chunk's loads before any store (one L2 round trip for the pair); further chunks (regions
+      // taller than 8 x 256 rows or wider than 8 x 256 columns) follow one round trip each
+      const long long rlo = b0 * kTileRows, rhi = b1 * kTileRows < a.R ? b1 * kTileRows : a.R;
+      for (long long k = 0;; ++k) {
+        const long long r0 = rlo + k * 8 * kConsumers, cb = k * 8 * kConsumers;
+        const bool do_r = last_r && r0 < rhi, do_c = last_c && cb < ncols;
+        if (!do_r && !do_c) break;
+        Acc vr[8], vc[8];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const long long row = r0 + threadIdx.x + q * kConsumers;
-            val[q] = row < rhi ? __ldcg(accR + row) : Acc(0);
-          }
-#pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const long long row = r0 + threadIdx.x + q * kConsumers;
-            if (row < rhi) {
-              __stcg(accR + row, Acc(0));
-              out[row] = RcOps<T>::finish(val[q]);
-            }
-          }
+        for (int q = 0; q < 8; ++q) {
+          const long long row = r0 + threadIdx.x + q * kConsumers;
+          vr[q] = do_r && row < rhi ? __ldcg(accR + row) : Acc(0);
+          const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
+          vc[q] = do_c && c < ncols && cg < a.C ? __ldcg(accC + cg) : Acc(0);
         }
-      }
-      if (last_c) {
-        for (long long cb = 0; cb < ncols; cb += 8 * kConsumers) {
-          Acc val[8];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
-            val[q] = (c < ncols && cg < a.C) ? __ldcg(accC + cg) : Acc(0);
+        for (int q = 0; q < 8; ++q) {
+          const long long row = r0 + threadIdx.x + q * kConsumers;
+          if (do_r && row < rhi) {
+            __stcg(accR + row, Acc(0));
+            out[row] = RcOps<T>::finish(vr[q]);
           }
-#pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
-            if (c < ncols && cg < a.C) {
-              __stcg(accC + cg, Acc(0));
-              out[a.R + cg] = RcOps<T>::finish(val[q]);
-            }
+          const long long c = cb + threadIdx.x + q * kConsumers, cg = c0 * BC + c;
+          if (do_c && c < ncols && cg < a.C) {
+            __stcg(accC + cg, Acc(0));
+            out[a.R + cg] = RcOps<T>::finish(vc[q]);
           }
         }
       }
