@@ -752,7 +752,7 @@ def roofline(item, us, gbs, peak, peak_src, traffic, flops, wavefronts=None):
                     # measured context (profiles/r02/kmeans/micro_inner.log): the kernel's dims loop alone, with
                     # its 4-point x 8-centroid thread tile, reaches 0.63-0.69 of this peak — one uniform
                     # constant-bank load per 4 packed FMAs, not the FMA pipe, sets that ceiling
-                    operand_path_ceiling_frac=[0.63, 0.69])
+                    dims_loop_alone_frac=[0.63, 0.69])
     return dict(base, bound="hbm", achieved=round(gbs, 1), peak=peak, peak_source=peak_src, unit="GB/s",
                 frac=round(gbs / peak, 4))
 
